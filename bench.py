@@ -1,0 +1,423 @@
+#!/usr/bin/env python
+"""bench.py -- effective TFLOPS of the fused Winograd F(2x2,3x3) path on B200.
+
+Metric (BASELINE.json): effective TFLOPS = 2*N*K*C*H*W*9 / t (direct-conv
+equivalent) and % of FP32 peak, per ResNet 3x3 layer, at 1/2/4/8 GPUs.
+
+One *step* = one pass of the whole hot path (FTF kernel + fused
+ITF/GEMM/OTF kernel) over every layer of the workload.  The default workload is
+all four ResNet 3x3 layers (BASELINE configs[1..4]: conv5_x N=32, conv4_x N=64,
+conv3_x N=128, conv2_x N=256) at their global batch; with --gpus P each rank
+takes a contiguous N/P batch shard of every layer (strong scaling: total work
+fixed), the transformed filter is broadcast once from rank 0 with NCCL at setup,
+and there is no collective on the conv path.  Time = max over ranks of CUDA-event
+device time; L2 is flushed (512 MiB write) before every timed step, outside the
+events.
+
+Prints ONE JSON line (rank 0).  `--impl reference` times the CPU fp64 oracle
+(test infrastructure) on a bounded sample of the same workload instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+import torch.distributed as dist  # noqa: E402
+
+from synth_inputs import CONFIGS, RESNET_LAYERS, SEED_W, SEED_X, make_inputs, shard_range  # noqa: E402
+
+FP32_PEAK_NOTE = "derived: 148 SMs x 128 FP32 lanes x 2 flop x sm_max_mhz (B200_PROFILING.md SM count, clocks.max.sm)"
+L2_FLUSH_BYTES = 512 << 20
+METRIC = "effective TFLOPS & % of FP32 peak per ResNet 3x3 layer at 1/2/4/8 B200"
+
+
+def _peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    sm_mhz, src = 1965.0, "fallback clocks.max.sm 1965 MHz (B200_PROFILING.md)"
+    hbm = 6650.0
+    if os.path.exists(path):
+        with open(path) as f:
+            mp = json.load(f)
+        sm_mhz = float(mp.get("sm_max_mhz", sm_mhz))
+        hbm = float(mp.get("hbm_gbs", hbm))
+        src = "MEASURED_PEAKS.json sm_max_mhz"
+    fp32_tflops = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
+    return fp32_tflops, hbm, src
+
+
+def _workload(name):
+    if name == "resnet_3x3":
+        return [CONFIGS[n] for n in ("conv5_x", "conv4_x", "conv3_x", "conv2_x")]
+    return [CONFIGS[name]]
+
+
+class ClockSampler:
+    """nvidia-smi sampling of SM clock and throttle reasons DURING the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+        self._t = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.dev}", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except (FileNotFoundError, OSError):
+            self.proc = None
+            return
+        self._t = threading.Thread(target=self._read, daemon=True)
+        self._t.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        if self._t:
+            self._t.join(timeout=1)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def _init_dist():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1 and not dist.is_initialized():
+        backend = "nccl" if torch.cuda.is_available() else "gloo"
+        if torch.cuda.is_available():
+            torch.cuda.set_device(local)
+        dist.init_process_group(backend=backend)
+    return rank, world, local
+
+
+def _max_over_ranks(v: float, world: int, device) -> float:
+    if world == 1:
+        return v
+    t = torch.tensor([v], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def _oracle_sample(layers, target_s_per_layer: float):
+    """Time the fp64 oracle's direct conv (Eq. 4) on a K-slice of every layer, the slice
+    sized for about target_s_per_layer seconds; returns (flops, seconds, description)."""
+    import oracle
+    total_flops, total_s, desc = 0, 0.0, []
+    for cfg in layers:
+        x, w = make_inputs(cfg)
+        per_k = 18 * cfg.N * cfg.C * cfg.H * cfg.W
+        t0 = time.perf_counter()
+        oracle.direct_conv(x, w[..., :1].contiguous())
+        t1 = time.perf_counter() - t0
+        ks = int(max(1, min(cfg.K, target_s_per_layer / max(t1, 1e-6))))
+        t0 = time.perf_counter()
+        oracle.direct_conv(x, w[..., :ks].contiguous())
+        dt = time.perf_counter() - t0
+        total_flops += per_k * ks
+        total_s += dt
+        desc.append(f"{cfg.name}: k 0..{ks - 1} of {cfg.K}")
+    return total_flops, total_s, "; ".join(desc)
+
+
+def run_reference(args, layers, rank, world):
+    """--impl reference: the CPU fp64 oracle, as it stands, on a bounded sample."""
+    if rank != 0:
+        return None
+    import oracle
+    cores = oracle.num_threads()
+    # calibrate the per-layer K-slice once, then time warmup + steps with that slice
+    slices = []
+    for cfg in layers:
+        x, w = make_inputs(cfg)
+        t0 = time.perf_counter()
+        oracle.direct_conv(x, w[..., :1].contiguous())
+        t1 = time.perf_counter() - t0
+        slices.append((cfg, x, w[..., :int(max(1, min(cfg.K, args.ref_step_s / len(layers) / max(t1, 1e-6))))]
+                       .contiguous()))
+    flops_step = sum(18 * c.N * c.C * c.H * c.W * wk.shape[3] for c, _, wk in slices)
+    for _ in range(args.warmup):
+        for c, x, wk in slices:
+            oracle.direct_conv(x, wk)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        for c, x, wk in slices:
+            oracle.direct_conv(x, wk)
+    dt = time.perf_counter() - t0
+    value = flops_step * args.steps / dt / 1e12
+    sample = "; ".join(f"{c.name}: k 0..{wk.shape[3] - 1} of {c.K} (direct fp64, Eq. 4)" for c, _, wk in slices)
+    return {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "TFLOPS", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": _config(args, layers, world),
+        "cpu_baseline": {"value": value, "unit": "TFLOPS", "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": "TFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+
+
+def _config(args, layers, world):
+    return {
+        "workload": args.workload if args.workload != "resnet_3x3" else "resnet_3x3 (conv5_x,conv4_x,conv3_x,conv2_x)",
+        "layers": {c.name: {"N": c.N, "C": c.C, "K": c.K, "H": c.H, "W": c.W, "pad": 1, "stride": 1} for c in layers},
+        "global_batch": {c.name: c.N for c in layers},
+        "parallelism": f"dp{world} (batch-sharded, strong scaling)",
+        "variant": args.variant,
+        "inputs": f"uniform[-1,1) fp32, torch seeds x={SEED_X} w={SEED_W}",
+        "l2": "flushed by a 512 MiB write before every timed step (outside the events)",
+        "step": "per layer: FTF kernel + fused ITF/16xGEMM/OTF kernel",
+    }
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", default="resnet_3x3", choices=["resnet_3x3", *RESNET_LAYERS, "tiny"])
+    ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-baseline-s", type=float, default=3.0, help="oracle seconds per layer")
+    ap.add_argument("--ref-step-s", type=float, default=4.0, help="oracle seconds per reference step")
+    ap.add_argument("--out", default=None)
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "ours":
+        print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
+        args.warmup = 3
+
+    rank, world, local = _init_dist()
+    layers = _workload(args.workload)
+
+    if args.impl == "reference":
+        res = run_reference(args, layers, rank, world)
+        if rank == 0:
+            print(json.dumps(res), flush=True)
+        if world > 1 and dist.is_initialized():
+            dist.destroy_process_group()
+        return
+
+    import paper_conf_ppopp_yanwc20_b200 as wino
+
+    dev = torch.device(f"cuda:{local}")
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream(dev)
+    fp32_peak, hbm_peak, peak_src = _peaks()
+
+    # ---- setup: inputs (host, full N, seeded) -> this rank's shard on device ----
+    per = []
+    for cfg in layers:
+        lo, hi = shard_range(cfg.N, rank, world)
+        x, w = make_inputs(cfg)
+        xs = x[..., lo:hi].contiguous()
+        n_loc = hi - lo
+        d = {"cfg": cfg, "n": n_loc, "x": xs.to(dev), "w": w.to(dev),
+             "u": torch.empty((cfg.C, 4, 4, cfg.K), dtype=torch.float32, device=dev),
+             "y": torch.empty((cfg.K, cfg.H, cfg.W, max(n_loc, 1)), dtype=torch.float32, device=dev)}
+        # transformed filter: computed on rank 0, broadcast once over NVLink (NCCL)
+        if rank == 0:
+            wino.filter_transform(d["w"], out=d["u"])
+        if world > 1:
+            dist.broadcast(d["u"], src=0)
+        if args.impl == "ours" and not args.no_e2e:
+            d["x_h"] = xs.pin_memory()
+            d["w_h"] = w.pin_memory()
+            d["y_h"] = torch.empty((cfg.K, cfg.H, cfg.W, max(n_loc, 1)), dtype=torch.float32).pin_memory()
+            d["ws"] = torch.empty(wino.host_workspace_bytes(max(n_loc, 1), cfg.C, cfg.H, cfg.W, cfg.K),
+                                  dtype=torch.uint8, device=dev)
+        per.append(d)
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
+    launches_per_step = 0
+    for d in per:
+        if d["n"] > 0:
+            c = d["cfg"]
+            launches_per_step += 1 + wino.plan(d["n"], c.C, c.H, c.W, c.K).launches
+
+    def step(ev_layer=None):
+        for i, d in enumerate(per):
+            if d["n"] == 0:
+                continue
+            c = d["cfg"]
+            if ev_layer is not None:
+                ev_layer[i][0].record(stream)
+            wino.filter_transform(d["w"], out=d["u"])
+            if ev_layer is not None:
+                ev_layer[i][1].record(stream)
+            wino.conv2d(d["x"], d["u"], out=d["y"], variant=args.variant)
+            if ev_layer is not None:
+                ev_layer[i][2].record(stream)
+
+    for _ in range(args.warmup):
+        flush.fill_(1.0)
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(local) if rank == 0 else None
+    if sampler:
+        sampler.start()
+        time.sleep(0.3)
+    mk = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    step_ev = [(mk(), mk()) for _ in range(args.steps)]
+    lay_ev = [[[mk(), mk(), mk()] for _ in per] for _ in range(args.steps)]
+    t_wall0 = time.perf_counter()
+    for s in range(args.steps):
+        flush.fill_(float(s))
+        step_ev[s][0].record(stream)
+        step(lay_ev[s])
+        step_ev[s][1].record(stream)
+    torch.cuda.synchronize()
+    wall = time.perf_counter() - t_wall0
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = sampler.stop() if sampler else None
+
+    ms_step = sum(a.elapsed_time(b) for a, b in step_ev) / args.steps
+    ftf_ms, conv_ms = [0.0] * len(per), [0.0] * len(per)
+    for s in range(args.steps):
+        for i, d in enumerate(per):
+            if d["n"] == 0:
+                continue
+            e0, e1, e2 = lay_ev[s][i]
+            ftf_ms[i] += e0.elapsed_time(e1) / args.steps
+            conv_ms[i] += e1.elapsed_time(e2) / args.steps
+    ms_step = _max_over_ranks(ms_step, world, dev)
+    conv_ms = [_max_over_ranks(v, world, dev) for v in conv_ms]
+    ftf_ms = [_max_over_ranks(v, world, dev) for v in ftf_ms]
+
+    # ---- e2e: the public C-ABI host entry point, host buffers, copies in the timed region ----
+    e2e = None
+    if not args.no_e2e:
+        for _ in range(2):
+            for d in per:
+                if d["n"]:
+                    wino.conv2d_host(d["x_h"], d["w_h"], d["y_h"], d["ws"])
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        e_steps = max(1, min(args.steps, 5))
+        e0, e1 = mk(), mk()
+        e0.record(stream)
+        for _ in range(e_steps):
+            for d in per:
+                if d["n"]:
+                    wino.conv2d_host(d["x_h"], d["w_h"], d["y_h"], d["ws"])
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e_ms = _max_over_ranks(e0.elapsed_time(e1) / e_steps, world, dev)
+        h2d = sum(d["x_h"].numel() * 4 + d["w_h"].numel() * 4 for d in per if d["n"]) * world
+        d2h = sum(d["y_h"].numel() * 4 for d in per if d["n"]) * world
+        total_flops = sum(c.eff_flops for c in layers)
+        e2e = {"value": total_flops / (e_ms * 1e-3) / 1e12, "unit": "TFLOPS", "ms_per_step": e_ms,
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "api": "wino_conv2d_f2x3_fwd_host (pinned host x,w -> device FTF+fused conv -> host y)"}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    total_eff = sum(c.eff_flops for c in layers)
+    value = total_eff / (ms_step * 1e-3) / 1e12
+    layer_rep = {}
+    ewmm_flops, conv_total_ms = 0, 0.0
+    for i, d in enumerate(per):
+        c = d["cfg"]
+        eff = c.eff_flops / (conv_ms[i] * 1e-3) / 1e12
+        ew = 32 * c.K * c.C * c.N * c.tiles
+        ewmm_flops += ew
+        conv_total_ms += conv_ms[i]
+        layer_rep[c.name] = {
+            "conv_us": conv_ms[i] * 1e3, "ftf_us": ftf_ms[i] * 1e3,
+            "eff_tflops": eff, "pct_fp32_peak_eff": 100 * eff / fp32_peak,
+            "ffma_pipe_pct": 100 * ew / (conv_ms[i] * 1e-3) / 1e12 / fp32_peak,
+            "eff_tflops_incl_ftf": c.eff_flops / ((conv_ms[i] + ftf_ms[i]) * 1e-3) / 1e12,
+        }
+    achieved = ewmm_flops / (conv_total_ms * 1e-3) / 1e12
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        try:
+            with open(tpath) as f:
+                tj = json.load(f)
+            key = f"{args.workload}:{args.variant}:dp{world}"
+            traffic = tj.get(key)
+        except (OSError, ValueError):
+            traffic = None
+
+    res = {
+        "metric": METRIC, "value": value, "unit": "TFLOPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic", "config": _config(args, layers, world),
+        "pct_fp32_peak_eff": 100 * value / fp32_peak,
+        "fp32_peak_tflops": fp32_peak, "fp32_peak_source": f"{FP32_PEAK_NOTE}; {peak_src}",
+        "layers": layer_rep,
+        "roofline": {"bound": "alu", "kernel": f"wino fused_{args.variant}", "achieved": achieved,
+                     "peak": fp32_peak, "unit": "TFLOP/s", "frac": achieved / fp32_peak, "traffic": traffic,
+                     "achieved_def": "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) per launch summed over layers / "
+                                     "summed CUDA-event conv durations",
+                     "peak_def": FP32_PEAK_NOTE},
+        "gpu_launches": launches_per_step * args.steps,
+        "clocks": clocks, "wall_s_timed_region": wall,
+    }
+    if e2e:
+        res["e2e"] = e2e
+    if world == 1 and not args.no_cpu_baseline:
+        import oracle
+        fl, sec, sample = _oracle_sample(layers, args.cpu_baseline_s)
+        res["cpu_baseline"] = {"value": fl / sec / 1e12, "unit": "TFLOPS", "cores": oracle.num_threads(),
+                               "kind": "oracle", "sample": f"direct fp64 conv (Eq. 4) on {sample}; {sec:.1f} s"}
+    line = json.dumps(res)
+    print(line, flush=True)
+    if args.out:
+        with open(args.out, "w") as f:
+            f.write(line + "\n")
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

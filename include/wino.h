@@ -1,0 +1,159 @@
+/*
+ * include/wino.h -- C ABI of libwino.so: fused batched Winograd F(2x2,3x3)
+ * forward convolution for NVIDIA B200 (sm_100a).
+ *
+ * Method: Yan, Wang & Chu, "Optimizing Batched Winograd Convolution on GPUs"
+ * (PPoPP'20).  Citations "L<n>" are lines of the paper text with the
+ * section / equation they fall in; DESIGN.md lists every reading taken where
+ * the text is silent or garbled.
+ *
+ * Conventions shared by every entry point
+ * ---------------------------------------
+ *  * Pointers named *_dev are caller-owned DEVICE pointers (cudaMalloc'd or
+ *    equivalent) to dense, row-major fp32 tensors, 16-byte aligned; pointers
+ *    named *_host are caller-owned HOST pointers (pinned memory recommended).
+ *    The library never allocates, frees or retains caller memory, and keeps no
+ *    state across calls other than per-device capability / attribute caches,
+ *    so calls are thread-safe.
+ *  * All calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy
+ *    default stream).  The return value reports argument validation and
+ *    launch errors only; device faults surface at the caller's next
+ *    synchronisation, as usual in CUDA.
+ *  * Tensor layouts are the paper's (Table 4):
+ *        x  (C,H,W,N)  "CHWN"     input,  N contiguous
+ *        w  (C,3,3,K)  "CRSK"     filter, K contiguous
+ *        u  (C,4,4,K)  "CR'S'K"   transformed filter; element (r',s') of
+ *                                 G*w*G^T at [c][r'][s'][k] (reading R6)
+ *        y  (K,H,W,N)  "KHWN"     output
+ *  * Only pad = 1, stride = 1 are supported (ResNet 3x3 layers, Table 1):
+ *    other values return WINO_ERR_UNSUPPORTED.  Any N, C, K, H, W >= 1 is
+ *    accepted (L1281 states peak speed at N%32 = 0, K%64 = 0, C%8 = 0; other
+ *    shapes take generic load paths, never a CPU fallback).
+ *  * Errors: NULL pointer or dimension <= 0 -> WINO_ERR_INVALID_ARG;
+ *    y overlapping x or u -> WINO_ERR_INVALID_ARG; a tensor of >= 2^31
+ *    elements -> WINO_ERR_TOO_LARGE; a device pointer not 16-byte aligned ->
+ *    WINO_ERR_MISALIGNED; current device not sm_100 -> WINO_ERR_UNSUPPORTED;
+ *    a CUDA runtime failure -> WINO_ERR_CUDA (see wino_last_cuda_error()).
+ *  * Output is deterministic: no atomics; split-C partial sums are reduced in
+ *    a fixed order.
+ */
+#ifndef WINO_H_
+#define WINO_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* wino_stream_t; /* identical to cudaStream_t */
+
+typedef enum {
+    WINO_OK = 0,
+    WINO_ERR_INVALID_ARG = 1,
+    WINO_ERR_UNSUPPORTED = 2,
+    WINO_ERR_MISALIGNED = 3,
+    WINO_ERR_TOO_LARGE = 4,
+    WINO_ERR_CUDA = 5
+} wino_status_t;
+
+typedef enum {
+    WINO_TC_TF32 = 0,   /* operands rounded to TF32 (cvt.rna), FP32 accumulate    */
+    WINO_TC_3XTF32 = 1  /* big*big + big*small + small*big, ~FP32 accuracy        */
+} wino_tc_mode_t;
+
+/* Library ABI version (major*10000 + minor*100 + patch). */
+int wino_version(void);
+
+/* Human-readable name of a status code; never NULL. */
+const char* wino_status_string(wino_status_t s);
+
+/* The cudaError_t of the most recent WINO_ERR_CUDA on the calling thread (0 if none). */
+int wino_last_cuda_error(void);
+
+/*
+ * Size in bytes of the transformed-filter workspace u: 16*C*K floats
+ * (L993, Sec. 7.3: "16KC transformed filter data (0.25MB for Conv2, 1MB for
+ * Conv3, 4MB for Conv4 and 16MB for Conv5)").  Returns 0 if C or K <= 0.
+ * Pure host computation; needs no GPU.
+ */
+size_t wino_filter_workspace_bytes(int C, int K);
+
+/*
+ * Filter transform (FTF), Eq. 5 (L191), "separate kernel" of Sec. 3.1 (L209)
+ * and Sec. 4.1 (L345):  u[c,:,:,k] = G * w[c,:,:,k] * G^T with
+ * G = [[1,0,0],[1/2,1/2,1/2],[1/2,-1/2,1/2],[0,0,1]] (Eq. 3; reading R1).
+ *   w_dev : (C,3,3,K) fp32, read-only
+ *   u_dev : (C,4,4,K) fp32, written (wino_filter_workspace_bytes(C,K) bytes)
+ * Run once per weight set; the result is consumed by wino_conv2d_f2x3_fwd*.
+ */
+wino_status_t wino_filter_transform(const float* w_dev, float* u_dev, int C, int K,
+                                    wino_stream_t stream);
+
+/*
+ * Fused forward convolution on FP32 CUDA cores (FFMA), Sec. 3-4 and
+ * Algorithm 1 (L351-355): for every 4x4 input tile the input transform
+ * V = B^T d B (Eq. 6), the 16 Winograd-domain batched GEMMs
+ * M^(xi) = sum_c U^(xi)[c,k] V^(xi)[c,nu] (Eq. 7/9/10, L197-203, L373-395) and
+ * the output transform Y = A^T M A (Eq. 8) in ONE kernel; implicit zero
+ * padding (Sec. 3.5); odd H/W compute and discard the extra row/column
+ * (L1155).  Computes y[k,i,j,n] = sum_{c,r,s} x[c,i+r-1,j+s-1,n] * w[c,r,s,k]
+ * (Eq. 4; zero outside the image).
+ *   x_dev : (C,H,W,N) fp32          u_dev : (C,4,4,K) from wino_filter_transform
+ *   y_dev : (K,H,W,N) fp32, fully overwritten; must not overlap x_dev or u_dev
+ *   pad, stride : must both be 1
+ */
+wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float* y_dev,
+                                   int N, int C, int H, int W, int K, int pad, int stride,
+                                   wino_stream_t stream);
+
+/*
+ * Same computation with the Winograd-domain GEMM (Eq. 7) on the 5th-generation
+ * tensor cores (tcgen05.mma kind::tf32, accumulators in TMEM).  The paper has
+ * no tensor-core path ("the data layout needs a redesign", Sec. 8.3);
+ * this variant is the B200 redesign named in BASELINE.json's north_star.
+ * mode selects TF32 (accuracy ~5e-4 relative) or 3xTF32 (~FP32 accuracy).
+ * Arguments and errors as wino_conv2d_f2x3_fwd, plus WINO_ERR_INVALID_ARG for
+ * an unknown mode.
+ */
+wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_dev, float* y_dev,
+                                      int N, int C, int H, int W, int K, int pad, int stride,
+                                      wino_tc_mode_t mode, wino_stream_t stream);
+
+/*
+ * End-to-end call on HOST buffers: copies w_host and x_host to the device,
+ * runs the filter transform and the fused FP32 convolution, and copies y back
+ * to y_host, all enqueued on `stream` (so the call returns before the copies
+ * finish; synchronise the stream before reading y_host).
+ *   x_host (C,H,W,N), w_host (C,3,3,K) : read;  y_host (K,H,W,N) : written
+ *   ws_dev / ws_bytes : caller-owned device workspace of at least
+ *                       wino_host_workspace_bytes(N,C,H,W,K) bytes
+ * Host buffers should be page-locked for the copies to be asynchronous.
+ */
+size_t wino_host_workspace_bytes(int N, int C, int H, int W, int K);
+wino_status_t wino_conv2d_f2x3_fwd_host(const float* x_host, const float* w_host, float* y_host,
+                                        int N, int C, int H, int W, int K, int pad, int stride,
+                                        void* ws_dev, size_t ws_bytes, wino_stream_t stream);
+
+/*
+ * Launch plan the library would use for a shape (host only, needs no GPU);
+ * used by tests and by bench.py to count launches and report tiling.
+ */
+typedef struct {
+    int variant;        /* 0 = FP32 FFMA fused kernel, 1 = tcgen05 TF32 / 3xTF32   */
+    int bk, bn, bc;     /* filters, tiles and channels per CTA step (Sec. 3.3)      */
+    int vec_x, vec_u;   /* global-load vector width for x and u (1 or 4 floats)     */
+    int split_c;        /* channel split factor (1 = none)                          */
+    int64_t ctas;       /* CTAs of the main kernel                                  */
+    int threads;        /* threads per CTA                                          */
+    int smem_bytes;     /* dynamic shared memory per CTA                            */
+    int launches;       /* kernels launched by one wino_conv2d_f2x3_fwd* call       */
+} wino_plan_t;
+
+wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_plan_t* plan);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* WINO_H_ */

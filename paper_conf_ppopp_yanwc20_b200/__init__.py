@@ -1,0 +1,212 @@
+"""Python binding of libwino.so -- fused batched Winograd F(2x2,3x3) on B200.
+
+Yan, Wang & Chu, "Optimizing Batched Winograd Convolution on GPUs" (PPoPP'20),
+re-designed for sm_100a.  This module only marshals arguments: it checks
+dtype / device / contiguity / shape of torch tensors, passes raw pointers and
+the current CUDA stream to the C ABI declared in include/wino.h, and raises on
+any non-OK status.  Every step of the computation runs in the CUDA kernels of
+libwino.so; if the library is missing the import of any op raises -- there is
+no CPU or PyTorch fallback.
+
+Layouts (Table 4): x (C,H,W,N), w (C,3,3,K), u (C,4,4,K), y (K,H,W,N).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import torch
+
+__all__ = [
+    "WinoError", "lib", "version", "filter_workspace_bytes", "filter_transform", "conv2d",
+    "conv2d_host", "host_workspace_bytes", "plan", "Plan", "TC_TF32", "TC_3XTF32",
+]
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_PKG, "libwino.so")
+_lib = None
+
+TC_TF32 = 0
+TC_3XTF32 = 1
+_STATUS = {0: "WINO_OK", 1: "WINO_ERR_INVALID_ARG", 2: "WINO_ERR_UNSUPPORTED",
+           3: "WINO_ERR_MISALIGNED", 4: "WINO_ERR_TOO_LARGE", 5: "WINO_ERR_CUDA"}
+
+
+class WinoError(RuntimeError):
+    def __init__(self, status: int, where: str, cuda_error: int = 0):
+        self.status = status
+        self.cuda_error = cuda_error
+        msg = f"{where}: {_STATUS.get(status, status)}"
+        if status == 5:
+            msg += f" (cudaError {cuda_error})"
+        super().__init__(msg)
+
+
+class _Plan(ctypes.Structure):
+    _fields_ = [("variant", ctypes.c_int), ("bk", ctypes.c_int), ("bn", ctypes.c_int),
+                ("bc", ctypes.c_int), ("vec_x", ctypes.c_int), ("vec_u", ctypes.c_int),
+                ("split_c", ctypes.c_int), ("ctas", ctypes.c_int64), ("threads", ctypes.c_int),
+                ("smem_bytes", ctypes.c_int), ("launches", ctypes.c_int)]
+
+
+@dataclass(frozen=True)
+class Plan:
+    variant: int
+    bk: int
+    bn: int
+    bc: int
+    vec_x: int
+    vec_u: int
+    split_c: int
+    ctas: int
+    threads: int
+    smem_bytes: int
+    launches: int
+
+
+def lib() -> ctypes.CDLL:
+    """Load libwino.so (built in-tree by __graft_entry__.build()); raise if absent."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_LIB_PATH):
+        raise ImportError(f"libwino.so not built at {_LIB_PATH}; run __graft_entry__.build() "
+                          "(there is no CPU fallback)")
+    L = ctypes.CDLL(_LIB_PATH)
+    vp, i, st = ctypes.c_void_p, ctypes.c_int, ctypes.c_size_t
+    L.wino_version.restype = i
+    L.wino_version.argtypes = []
+    L.wino_status_string.restype = ctypes.c_char_p
+    L.wino_status_string.argtypes = [i]
+    L.wino_last_cuda_error.restype = i
+    L.wino_last_cuda_error.argtypes = []
+    L.wino_filter_workspace_bytes.restype = st
+    L.wino_filter_workspace_bytes.argtypes = [i, i]
+    L.wino_filter_transform.restype = i
+    L.wino_filter_transform.argtypes = [vp, vp, i, i, vp]
+    L.wino_conv2d_f2x3_fwd.restype = i
+    L.wino_conv2d_f2x3_fwd.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
+    L.wino_conv2d_f2x3_fwd_tc.restype = i
+    L.wino_conv2d_f2x3_fwd_tc.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
+    L.wino_host_workspace_bytes.restype = st
+    L.wino_host_workspace_bytes.argtypes = [i, i, i, i, i]
+    L.wino_conv2d_f2x3_fwd_host.restype = i
+    L.wino_conv2d_f2x3_fwd_host.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp, st, vp]
+    L.wino_plan.restype = i
+    L.wino_plan.argtypes = [i, i, i, i, i, i, ctypes.POINTER(_Plan)]
+    _lib = L
+    return L
+
+
+def _check(status: int, where: str):
+    if status != 0:
+        raise WinoError(status, where, lib().wino_last_cuda_error() if status == 5 else 0)
+
+
+def version() -> int:
+    return lib().wino_version()
+
+
+def _stream_ptr(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _need_cuda_f32(t: torch.Tensor, name: str, ndim: int):
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{name} must be a torch.Tensor")
+    if t.dtype != torch.float32:
+        raise TypeError(f"{name} must be float32, got {t.dtype}")
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor (no CPU fallback)")
+    if t.dim() != ndim:
+        raise ValueError(f"{name} must have {ndim} dims, got shape {tuple(t.shape)}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+
+
+def filter_workspace_bytes(C: int, K: int) -> int:
+    """16*C*K*4 bytes (L993)."""
+    return int(lib().wino_filter_workspace_bytes(C, K))
+
+
+def host_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
+    return int(lib().wino_host_workspace_bytes(N, C, H, W, K))
+
+
+def plan(N: int, C: int, H: int, W: int, K: int, variant: int = 0) -> Plan:
+    p = _Plan()
+    _check(lib().wino_plan(N, C, H, W, K, variant, ctypes.byref(p)), "wino_plan")
+    return Plan(**{f: getattr(p, f) for f, _ in _Plan._fields_})
+
+
+def filter_transform(w: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """FTF, Eq. 5 (L191): w (C,3,3,K) -> u (C,4,4,K) on the GPU."""
+    _need_cuda_f32(w, "w", 4)
+    C, r, s, K = w.shape
+    if (r, s) != (3, 3):
+        raise ValueError(f"w must be (C,3,3,K), got {tuple(w.shape)}")
+    if out is None:
+        out = torch.empty((C, 4, 4, K), dtype=torch.float32, device=w.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (C, 4, 4, K):
+        raise ValueError("out must be (C,4,4,K)")
+    with torch.cuda.device(w.device):
+        _check(lib().wino_filter_transform(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                           C, K, _stream_ptr(stream)), "wino_filter_transform")
+    return out
+
+
+def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, variant: str = "fp32",
+           stream=None) -> torch.Tensor:
+    """Fused Winograd forward conv, pad 1 stride 1: x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N).
+
+    variant: "fp32" (FFMA kernel), "tf32" or "3xtf32" (tcgen05 kernel).
+    """
+    _need_cuda_f32(x, "x", 4)
+    _need_cuda_f32(u, "u", 4)
+    C, H, W, N = x.shape
+    if u.shape[0] != C or tuple(u.shape[1:3]) != (4, 4):
+        raise ValueError(f"u must be (C,4,4,K) with C={C}, got {tuple(u.shape)}")
+    if u.device != x.device:
+        raise ValueError("x and u must be on the same device")
+    K = u.shape[3]
+    if out is None:
+        out = torch.empty((K, H, W, N), dtype=torch.float32, device=x.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (K, H, W, N):
+        raise ValueError("out must be (K,H,W,N)")
+    args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+            N, C, H, W, K, 1, 1)
+    with torch.cuda.device(x.device):
+        if variant == "fp32":
+            _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
+        elif variant in ("tf32", "3xtf32"):
+            mode = TC_TF32 if variant == "tf32" else TC_3XTF32
+            _check(lib().wino_conv2d_f2x3_fwd_tc(*args, mode, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc")
+        else:
+            raise ValueError(f"unknown variant {variant!r}")
+    return out
+
+
+def conv2d_host(x_host: torch.Tensor, w_host: torch.Tensor, y_host: torch.Tensor, ws: torch.Tensor,
+                stream=None) -> None:
+    """End-to-end call on host buffers (x (C,H,W,N), w (C,3,3,K) -> y (K,H,W,N), pinned CPU
+    fp32) through ``wino_conv2d_f2x3_fwd_host``; ``ws`` is a CUDA byte buffer of at least
+    host_workspace_bytes().  Asynchronous on the stream."""
+    for t, n in ((x_host, "x_host"), (w_host, "w_host"), (y_host, "y_host")):
+        if t.is_cuda or t.dtype != torch.float32 or not t.is_contiguous() or t.dim() != 4:
+            raise ValueError(f"{n} must be a contiguous 4-d float32 CPU tensor")
+    if not ws.is_cuda:
+        raise ValueError("ws must be a CUDA tensor")
+    C, H, W, N = x_host.shape
+    K = w_host.shape[3]
+    if tuple(y_host.shape) != (K, H, W, N) or tuple(w_host.shape) != (C, 3, 3, K):
+        raise ValueError("shape mismatch")
+    nbytes = ws.numel() * ws.element_size()
+    with torch.cuda.device(ws.device):
+        _check(lib().wino_conv2d_f2x3_fwd_host(
+            ctypes.c_void_p(x_host.data_ptr()), ctypes.c_void_p(w_host.data_ptr()),
+            ctypes.c_void_p(y_host.data_ptr()), N, C, H, W, K, 1, 1,
+            ctypes.c_void_p(ws.data_ptr()), nbytes, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_host")

@@ -1,0 +1,29 @@
+// ftf.cuh -- filter-transform kernel (FTF), the separate kernel of Sec. 3.1
+// (L209) / Sec. 4.1 (L345): u[c,:,:,k] = G w[c,:,:,k] G^T (Eq. 5).
+//
+// HBM-bound (Fig. 2): 36 B read + 64 B written per (c,k).  One thread
+// per (c,k) with k fastest, so each of the 9 loads and 16 stores is a fully
+// coalesced warp access along K (the "CR'S'K" layout of Table 4).
+#pragma once
+#include "wino_transforms.cuh"
+
+namespace wino {
+
+constexpr int FTF_THREADS = 256;
+
+__global__ void __launch_bounds__(FTF_THREADS) ftf_kernel(const float* __restrict__ w,
+                                                          float* __restrict__ u, int C, int K) {
+    const long idx = (long)blockIdx.x * FTF_THREADS + threadIdx.x;
+    if (idx >= (long)C * K) return;
+    const int c = (int)(idx / K), k = (int)(idx - (long)c * K);
+    const float* wc = w + (size_t)c * 9 * K + k;
+    float g[9], t[16];
+#pragma unroll
+    for (int e = 0; e < 9; ++e) g[e] = __ldg(wc + (size_t)e * K);
+    ftf_4x4(g, t);
+    float* uc = u + (size_t)c * 16 * K + k;
+#pragma unroll
+    for (int e = 0; e < 16; ++e) uc[(size_t)e * K] = t[e];
+}
+
+}  // namespace wino

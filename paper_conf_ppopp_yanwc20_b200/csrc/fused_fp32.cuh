@@ -1,0 +1,238 @@
+// fused_fp32.cuh -- fused ITF + 16-batched GEMM (FFMA) + OTF kernel for sm_100a.
+//
+// Yan, Wang & Chu (PPoPP'20): workflow Sec. 3.1 (L209), cache blocking
+// Sec. 3.2-3.3 (L211-217, bk=64, bn=32, bc=8), software pipelining Sec. 3.4
+// (L323-333), implicit zero padding Sec. 3.5 (L335), thread-block workload and
+// Algorithm 1 (L339-355), ITF Sec. 4.2 (L357-359), batched GEMM and lane
+// arrangement Sec. 4.3 / Fig. 3 (L361-439), OTF through shared memory Sec. 4.4
+// (L479-503).
+//
+// B200 redesign:
+//  * nu = (tile, n) is flattened with n fastest, so any N works (the paper
+//    assumes 32 consecutive n per CTA, L357) and small per-rank batches still
+//    fill CTAs;
+//  * global->shared staging is a STAGES-deep cp.async ring with hardware zero
+//    fill (src-size 0) instead of predicated LDG into 48 prefetch registers
+//    (Table 5) -- the padding masks live in a per-CTA shared table computed
+//    once (the paper's P2R-packed mask, L337, is not expressible in PTX);
+//  * B200's 227 KB of shared memory holds all 128 KB of accumulators at once,
+//    so the OTF transpose runs in ONE round instead of the paper's 4 (L499).
+#pragma once
+#include <cstdint>
+
+#include "wino_ptx.cuh"
+#include "wino_transforms.cuh"
+
+namespace wino {
+namespace fp32 {
+
+constexpr int BK = 64;   // filters per CTA   (Sec. 3.3)
+constexpr int BN = 32;   // tiles*images per CTA
+constexpr int BC = 8;    // channels per pipeline step
+constexpr int NT = 256;  // threads per CTA   (Sec. 4)
+constexpr int US_FLOATS = BC * 16 * BK;  // transformed-filter stage [c][xi][k]
+constexpr int XS_FLOATS = BC * 16 * BN;  // raw-input stage        [c][pos][nu]
+constexpr int STAGE_FLOATS = US_FLOATS + XS_FLOATS;
+constexpr int VS_FLOATS = 16 * BC * BN;  // transformed input      [xi][c][nu] (Table 4 (16,bc,bn))
+constexpr int EP_LD = BN + 4;            // padded row of the OTF transpose buffer
+constexpr int EP_FLOATS = 16 * BK * EP_LD;
+constexpr int TAB_INTS = 16 * BN;        // per-CTA gather/padding table
+
+template <int S>
+struct Smem {
+    static constexpr int main_floats = S * STAGE_FLOATS + 2 * VS_FLOATS;
+    static_assert(EP_FLOATS <= main_floats, "OTF buffer must fit in the pipeline buffers");
+    static constexpr int bytes = (main_floats + TAB_INTS) * 4;
+};
+
+struct Params {
+    const float* __restrict__ x;  // (C,H,W,N)
+    const float* __restrict__ u;  // (C,4,4,K)
+    float* __restrict__ y;        // (K,H,W,N)
+    int N, C, H, W, K;
+    int TW;      // ceil(W/2)
+    int NV;      // N * ceil(H/2) * ceil(W/2)
+    int num_kb;  // ceil(K/BK)
+    int num_it;  // ceil(C/BC)
+};
+
+template <int VX, int VU, int S>
+__global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const Params p) {
+    extern __shared__ __align__(1024) float smem[];
+    float* const vs = smem + S * STAGE_FLOATS;
+    int* const xtab = reinterpret_cast<int*>(vs + 2 * VS_FLOATS);
+
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // k-block fastest: the CTAs resident at once share input tiles through L2
+    const int kb = blockIdx.x % p.num_kb;
+    const int nb = blockIdx.x / p.num_kb;
+    const int k0 = kb * BK, nu0 = nb * BN;
+    const size_t HWN = (size_t)p.H * p.W * p.N;
+
+    // Spatial gather offsets (h*W+w)*N+n of the 4x4 window element `pos` of
+    // local tile nu, or -1 where the window leaves the image (zero padding).
+    for (int e = tid; e < TAB_INTS; e += NT) {
+        const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
+        int off = -1;
+        if (nu < p.NV) {
+            const int t = nu / p.N, n = nu - t * p.N;
+            const int th = t / p.TW, tw = t - th * p.TW;
+            const int h = 2 * th - 1 + (pos >> 2), w = 2 * tw - 1 + (pos & 3);
+            if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
+        }
+        xtab[e] = off;
+    }
+    __syncthreads();
+
+    // ---- producer: one pipeline stage = BC channels of u and raw x ----------
+    auto load_stage = [&](int it, int slot) {
+        const int c0 = it * BC;
+        float* us = smem + slot * STAGE_FLOATS;
+        float* xs = us + US_FLOATS;
+        constexpr int UV_ROW = BK / VU;
+        constexpr int U_PER_THREAD = BC * 16 * UV_ROW / NT;
+#pragma unroll
+        for (int j = 0; j < U_PER_THREAD; ++j) {
+            const int idx = tid + j * NT;
+            const int row = idx / UV_ROW, col = (idx % UV_ROW) * VU;
+            const int c = c0 + row / 16, k = k0 + col;
+            const bool ok = (c < p.C) && (k < p.K);
+            const float* src = ok ? p.u + ((size_t)c * 16 + (row & 15)) * p.K + k : p.u;
+            const uint32_t dst = smem_u32(us + row * BK + col);
+            if constexpr (VU == 4) cp_async16(dst, src, ok);
+            else cp_async4(dst, src, ok);
+        }
+        constexpr int XV_C = 16 * BN / VX;
+        constexpr int X_PER_THREAD = BC * XV_C / NT;
+#pragma unroll
+        for (int j = 0; j < X_PER_THREAD; ++j) {
+            const int idx = tid + j * NT;
+            const int cl = idx / XV_C, e = (idx % XV_C) * VX;
+            const int c = c0 + cl;
+            const int off = xtab[e];
+            const bool ok = (c < p.C) && (off >= 0);
+            const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
+            const uint32_t dst = smem_u32(xs + cl * 16 * BN + e);
+            if constexpr (VX == 4) cp_async16(dst, src, ok);
+            else cp_async4(dst, src, ok);
+        }
+    };
+
+    // ---- ITF (Sec. 4.2): one (c, nu) tile per thread, raw [c][pos][nu] ->
+    //      V [xi][c][nu]; lanes run along nu so both sides are conflict-free.
+    auto itf_stage = [&](int slot, int vbuf) {
+        const float* xs = smem + slot * STAGE_FLOATS + US_FLOATS;
+        float* v = vs + vbuf * VS_FLOATS;
+        const int cl = tid >> 5, nl = tid & 31;
+        float d[16], t[16];
+#pragma unroll
+        for (int e = 0; e < 16; ++e) d[e] = xs[(cl * 16 + e) * BN + nl];
+        itf_4x4(d, t);
+#pragma unroll
+        for (int e = 0; e < 16; ++e) v[(e * BC + cl) * BN + nl] = t[e];
+    };
+
+    // ---- EWMM as 16-batched GEMM (Sec. 4.3): warp w owns xi = 2w, 2w+1; the
+    //      lane owns an 8(k) x 8(nu) block of each, Fig. 3 lane arrangement.
+    const int fo = 4 * ((lane & 15) >> 1);             // k offset: fo..fo+3, fo+32..fo+35
+    const int io = 4 * ((lane & 1) + 2 * (lane >> 4));  // nu offset: io..io+3, io+16..io+19
+    const int xi0 = 2 * warp;
+    float acc[2][8][8];
+#pragma unroll
+    for (int q = 0; q < 2; ++q)
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+            for (int j = 0; j < 8; ++j) acc[q][i][j] = 0.f;
+
+    auto gemm_stage = [&](int slot, int vbuf) {
+        const float* us = smem + slot * STAGE_FLOATS + xi0 * BK + fo;
+        const float* v = vs + vbuf * VS_FLOATS + xi0 * BC * BN + io;
+#pragma unroll
+        for (int c = 0; c < BC; ++c) {
+            float f[2][8], g[2][8];
+#pragma unroll
+            for (int q = 0; q < 2; ++q) {
+                const float4 a = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK);
+                const float4 b = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK + 32);
+                const float4 va = *reinterpret_cast<const float4*>(v + (q * BC + c) * BN);
+                const float4 vb = *reinterpret_cast<const float4*>(v + (q * BC + c) * BN + 16);
+                f[q][0] = a.x; f[q][1] = a.y; f[q][2] = a.z; f[q][3] = a.w;
+                f[q][4] = b.x; f[q][5] = b.y; f[q][6] = b.z; f[q][7] = b.w;
+                g[q][0] = va.x; g[q][1] = va.y; g[q][2] = va.z; g[q][3] = va.w;
+                g[q][4] = vb.x; g[q][5] = vb.y; g[q][6] = vb.z; g[q][7] = vb.w;
+            }
+#pragma unroll
+            for (int q = 0; q < 2; ++q)
+#pragma unroll
+                for (int i = 0; i < 8; ++i)
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) acc[q][i][j] = fmaf(f[q][i], g[q][j], acc[q][i][j]);
+        }
+    };
+
+    // ---- main loop (Algorithm 1 lines 6-16) with an S-stage cp.async ring --
+    const int NIT = p.num_it;
+#pragma unroll
+    for (int s = 0; s < S - 1; ++s) {
+        if (s < NIT) load_stage(s, s);
+        cp_async_commit();
+    }
+    cp_async_wait<S - 2>();  // stage 0 landed
+    __syncthreads();
+    itf_stage(0, 0);
+
+    for (int it = 0; it < NIT; ++it) {
+        cp_async_wait<S - 3>();  // stage it+1 landed (if issued)
+        __syncthreads();         // V[it&1] complete; slot (it-1)%S free
+        const int nxt = it + S - 1;
+        if (nxt < NIT) load_stage(nxt, nxt % S);
+        cp_async_commit();
+        if (it + 1 < NIT) itf_stage((it + 1) % S, (it + 1) & 1);
+        gemm_stage(it % S, it & 1);
+    }
+    cp_async_wait<0>();
+    __syncthreads();
+
+    // ---- OTF (Sec. 4.4): accumulators -> smem [xi][k][nu] in one round ------
+    float* ep = smem;
+#pragma unroll
+    for (int q = 0; q < 2; ++q)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int kl = fo + (i & 3) + (i >> 2) * 32;
+            float* row = ep + ((xi0 + q) * BK + kl) * EP_LD + io;
+            *reinterpret_cast<float4*>(row) =
+                make_float4(acc[q][i][0], acc[q][i][1], acc[q][i][2], acc[q][i][3]);
+            *reinterpret_cast<float4*>(row + 16) =
+                make_float4(acc[q][i][4], acc[q][i][5], acc[q][i][6], acc[q][i][7]);
+        }
+    __syncthreads();
+
+    const int nu = nu0 + lane;
+    if (nu < p.NV) {
+        const int t = nu / p.N, n = nu - t * p.N;
+        const int th = t / p.TW, tw = t - th * p.TW;
+        const int i0 = 2 * th, j0 = 2 * tw;
+        const bool okr = i0 + 1 < p.H, okc = j0 + 1 < p.W;  // odd H/W: drop extra outputs (L1155)
+        const size_t base = ((size_t)i0 * p.W + j0) * p.N + n;
+        const size_t dW = (size_t)p.W * p.N;
+#pragma unroll 2
+        for (int r = 0; r < BK / 8; ++r) {
+            const int kl = warp + 8 * r, k = k0 + kl;
+            if (k >= p.K) break;
+            float m[16], o[4];
+#pragma unroll
+            for (int e = 0; e < 16; ++e) m[e] = ep[(e * BK + kl) * EP_LD + lane];
+            otf_2x2(m, o);
+            float* yk = p.y + (size_t)k * HWN + base;
+            yk[0] = o[0];
+            if (okc) yk[p.N] = o[1];
+            if (okr) yk[dW] = o[2];
+            if (okr && okc) yk[dW + p.N] = o[3];
+        }
+    }
+}
+
+}  // namespace fp32
+}  // namespace wino

@@ -1,0 +1,258 @@
+// wino_api.cu -- the C ABI of libwino.so (declared in include/wino.h).
+//
+// Argument validation, shape -> kernel-variant dispatch, launches.  Every step
+// of the computation runs in the CUDA kernels included below; there is no host
+// or CPU fallback anywhere in this library.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+
+#include "../../include/wino.h"
+#include "ftf.cuh"
+#include "fused_fp32.cuh"
+
+namespace {
+
+thread_local int g_last_cuda_error = 0;
+
+constexpr int kMaxDevices = 64;
+constexpr int kStages = 3;  // cp.async ring depth of the FP32 kernel
+
+wino_status_t cuda_fail(cudaError_t e) {
+    g_last_cuda_error = static_cast<int>(e);
+    return WINO_ERR_CUDA;
+}
+
+// Per-device capability cache: 0 unknown, 1 sm_100, 2 other.
+std::atomic<int> g_dev_cap[kMaxDevices];
+
+wino_status_t check_device(int* dev_out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e);
+    if (dev < 0 || dev >= kMaxDevices) return WINO_ERR_UNSUPPORTED;
+    int cap = g_dev_cap[dev].load(std::memory_order_acquire);
+    if (cap == 0) {
+        int major = 0, minor = 0;
+        if ((e = cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev)) != cudaSuccess)
+            return cuda_fail(e);
+        if ((e = cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev)) != cudaSuccess)
+            return cuda_fail(e);
+        cap = (major == 10 && minor == 0) ? 1 : 2;
+        g_dev_cap[dev].store(cap, std::memory_order_release);
+    }
+    *dev_out = dev;
+    return cap == 1 ? WINO_OK : WINO_ERR_UNSUPPORTED;
+}
+
+// Opt-in to >48 KB dynamic shared memory once per (device, kernel instance).
+std::mutex g_attr_mu;
+template <typename Kern>
+wino_status_t ensure_smem_attr(Kern kern, int dev, int bytes, std::atomic<uint64_t>& done_mask) {
+    const uint64_t bit = 1ull << dev;
+    if (done_mask.load(std::memory_order_acquire) & bit) return WINO_OK;
+    std::lock_guard<std::mutex> lk(g_attr_mu);
+    if (done_mask.load(std::memory_order_relaxed) & bit) return WINO_OK;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e != cudaSuccess) return cuda_fail(e);
+    done_mask.fetch_or(bit, std::memory_order_release);
+    return WINO_OK;
+}
+
+bool overlaps(const void* a, size_t na, const void* b, size_t nb) {
+    const uintptr_t pa = reinterpret_cast<uintptr_t>(a), pb = reinterpret_cast<uintptr_t>(b);
+    return pa < pb + nb && pb < pa + na;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+constexpr int64_t kMaxElems = (int64_t(1) << 31) - 1;
+
+// Shape checks common to every conv entry point.
+wino_status_t check_shape(int N, int C, int H, int W, int K, int pad, int stride) {
+    if (N <= 0 || C <= 0 || H <= 0 || W <= 0 || K <= 0) return WINO_ERR_INVALID_ARG;
+    if (pad != 1 || stride != 1) return WINO_ERR_UNSUPPORTED;
+    const int64_t hw = int64_t(H) * W;
+    const int64_t xe = int64_t(C) * hw * N, ye = int64_t(K) * hw * N, ue = int64_t(16) * C * K;
+    const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
+    if (xe > kMaxElems || ye > kMaxElems || ue > kMaxElems || nv > kMaxElems) return WINO_ERR_TOO_LARGE;
+    return WINO_OK;
+}
+
+struct Fp32Plan {
+    int vec_x, vec_u;
+    int64_t ctas;
+    int smem;
+};
+
+Fp32Plan plan_fp32(int N, int C, int H, int W, int K) {
+    Fp32Plan p;
+    p.vec_x = (N % 4 == 0) ? 4 : 1;
+    p.vec_u = (K % 4 == 0) ? 4 : 1;
+    const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
+    const int64_t nb = (nv + wino::fp32::BN - 1) / wino::fp32::BN;
+    const int64_t kb = (K + wino::fp32::BK - 1) / wino::fp32::BK;
+    p.ctas = nb * kb;
+    p.smem = wino::fp32::Smem<kStages>::bytes;
+    (void)C;
+    return p;
+}
+
+std::atomic<uint64_t> g_attr_fp32[4];
+
+template <int VX, int VU>
+wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem, int dev,
+                          cudaStream_t st, std::atomic<uint64_t>& done) {
+    auto kern = wino::fp32::fused_fp32_kernel<VX, VU, kStages>;
+    wino_status_t s = ensure_smem_attr(kern, dev, smem, done);
+    if (s != WINO_OK) return s;
+    kern<<<dim3(static_cast<unsigned>(ctas)), wino::fp32::NT, smem, st>>>(prm);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
+}  // namespace
+
+extern "C" {
+
+int wino_version(void) { return 100; }  // 0.1.0
+
+const char* wino_status_string(wino_status_t s) {
+    switch (s) {
+        case WINO_OK: return "WINO_OK";
+        case WINO_ERR_INVALID_ARG: return "WINO_ERR_INVALID_ARG";
+        case WINO_ERR_UNSUPPORTED: return "WINO_ERR_UNSUPPORTED";
+        case WINO_ERR_MISALIGNED: return "WINO_ERR_MISALIGNED";
+        case WINO_ERR_TOO_LARGE: return "WINO_ERR_TOO_LARGE";
+        case WINO_ERR_CUDA: return "WINO_ERR_CUDA";
+    }
+    return "WINO_ERR_UNKNOWN";
+}
+
+int wino_last_cuda_error(void) { return g_last_cuda_error; }
+
+size_t wino_filter_workspace_bytes(int C, int K) {
+    if (C <= 0 || K <= 0) return 0;
+    return size_t(16) * size_t(C) * size_t(K) * sizeof(float);
+}
+
+wino_status_t wino_filter_transform(const float* w_dev, float* u_dev, int C, int K, wino_stream_t stream) {
+    if (!w_dev || !u_dev || C <= 0 || K <= 0) return WINO_ERR_INVALID_ARG;
+    if (int64_t(16) * C * K > kMaxElems) return WINO_ERR_TOO_LARGE;
+    if (!aligned16(w_dev) || !aligned16(u_dev)) return WINO_ERR_MISALIGNED;
+    if (overlaps(w_dev, size_t(9) * C * K * 4, u_dev, size_t(16) * C * K * 4)) return WINO_ERR_INVALID_ARG;
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    const int64_t n = int64_t(C) * K;
+    const unsigned blocks = static_cast<unsigned>((n + wino::FTF_THREADS - 1) / wino::FTF_THREADS);
+    wino::ftf_kernel<<<blocks, wino::FTF_THREADS, 0, reinterpret_cast<cudaStream_t>(stream)>>>(w_dev, u_dev, C, K);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
+wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_plan_t* plan) {
+    if (!plan) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, 1, 1);
+    if (s != WINO_OK) return s;
+    std::memset(plan, 0, sizeof(*plan));
+    if (variant != 0) return WINO_ERR_UNSUPPORTED;
+    Fp32Plan p = plan_fp32(N, C, H, W, K);
+    plan->variant = 0;
+    plan->bk = wino::fp32::BK;
+    plan->bn = wino::fp32::BN;
+    plan->bc = wino::fp32::BC;
+    plan->vec_x = p.vec_x;
+    plan->vec_u = p.vec_u;
+    plan->split_c = 1;
+    plan->ctas = p.ctas;
+    plan->threads = wino::fp32::NT;
+    plan->smem_bytes = p.smem;
+    plan->launches = 1;
+    return WINO_OK;
+}
+
+wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H,
+                                   int W, int K, int pad, int stride, wino_stream_t stream) {
+    if (!x_dev || !u_dev || !y_dev) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (!aligned16(x_dev) || !aligned16(u_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t yb = size_t(K) * hwn * 4;
+    if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) || overlaps(y_dev, yb, u_dev, size_t(16) * C * K * 4))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+
+    Fp32Plan pl = plan_fp32(N, C, H, W, K);
+    wino::fp32::Params prm;
+    prm.x = x_dev;
+    prm.u = u_dev;
+    prm.y = y_dev;
+    prm.N = N;
+    prm.C = C;
+    prm.H = H;
+    prm.W = W;
+    prm.K = K;
+    prm.TW = (W + 1) / 2;
+    prm.NV = N * ((H + 1) / 2) * prm.TW;
+    prm.num_kb = (K + wino::fp32::BK - 1) / wino::fp32::BK;
+    prm.num_it = (C + wino::fp32::BC - 1) / wino::fp32::BC;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (pl.vec_x == 4 && pl.vec_u == 4) return launch_fp32<4, 4>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[0]);
+    if (pl.vec_x == 4) return launch_fp32<4, 1>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[1]);
+    if (pl.vec_u == 4) return launch_fp32<1, 4>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[2]);
+    return launch_fp32<1, 1>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[3]);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H,
+                                      int W, int K, int pad, int stride, wino_tc_mode_t mode,
+                                      wino_stream_t stream) {
+    if (!x_dev || !u_dev || !y_dev) return WINO_ERR_INVALID_ARG;
+    if (mode != WINO_TC_TF32 && mode != WINO_TC_3XTF32) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    (void)stream;
+    return WINO_ERR_UNSUPPORTED;  // tcgen05 variant not built yet
+}
+
+static size_t round_up256(size_t b) { return (b + 255) & ~size_t(255); }
+
+size_t wino_host_workspace_bytes(int N, int C, int H, int W, int K) {
+    if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
+    const size_t hwn = size_t(H) * W * N;
+    return round_up256(size_t(C) * hwn * 4) + round_up256(size_t(9) * C * K * 4) +
+           round_up256(size_t(16) * C * K * 4) + round_up256(size_t(K) * hwn * 4);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_host(const float* x_host, const float* w_host, float* y_host, int N, int C,
+                                        int H, int W, int K, int pad, int stride, void* ws_dev, size_t ws_bytes,
+                                        wino_stream_t stream) {
+    if (!x_host || !w_host || !y_host || !ws_dev) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (ws_bytes < wino_host_workspace_bytes(N, C, H, W, K)) return WINO_ERR_INVALID_ARG;
+    if (!aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t xb = size_t(C) * hwn * 4, wb = size_t(9) * C * K * 4, ub = size_t(16) * C * K * 4,
+                 yb = size_t(K) * hwn * 4;
+    char* base = static_cast<char*>(ws_dev);
+    float* x_dev = reinterpret_cast<float*>(base);
+    float* w_dev = reinterpret_cast<float*>(base + round_up256(xb));
+    float* u_dev = reinterpret_cast<float*>(base + round_up256(xb) + round_up256(wb));
+    float* y_dev = reinterpret_cast<float*>(base + round_up256(xb) + round_up256(wb) + round_up256(ub));
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    cudaError_t e;
+    if ((e = cudaMemcpyAsync(w_dev, w_host, wb, cudaMemcpyHostToDevice, st)) != cudaSuccess) return cuda_fail(e);
+    if ((s = wino_filter_transform(w_dev, u_dev, C, K, stream)) != WINO_OK) return s;
+    if ((e = cudaMemcpyAsync(x_dev, x_host, xb, cudaMemcpyHostToDevice, st)) != cudaSuccess) return cuda_fail(e);
+    if ((s = wino_conv2d_f2x3_fwd(x_dev, u_dev, y_dev, N, C, H, W, K, pad, stride, stream)) != WINO_OK) return s;
+    if ((e = cudaMemcpyAsync(y_host, y_dev, yb, cudaMemcpyDeviceToHost, st)) != cudaSuccess) return cuda_fail(e);
+    return WINO_OK;
+}
+
+}  // extern "C"

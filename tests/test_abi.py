@@ -1,0 +1,126 @@
+"""C-ABI checks that need no GPU: the library loads, exports every symbol that
+include/wino.h declares, and its host-only logic (status strings, workspace
+sizes, launch plans, argument validation that precedes any device access)
+behaves as the header documents."""
+import ctypes
+import json
+import os
+import re
+
+import pytest
+
+import paper_conf_ppopp_yanwc20_b200 as wino
+from synth_inputs import CONFIGS
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "wino.h")
+
+
+def _declared_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(wino_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    L = wino.lib()
+    names = _declared_functions()
+    assert len(names) >= 10, names
+    for n in names:
+        assert hasattr(L, n), f"libwino.so does not export {n}"
+
+
+def test_status_strings_and_version():
+    L = wino.lib()
+    assert wino.version() >= 100
+    for code, name in [(0, b"WINO_OK"), (1, b"WINO_ERR_INVALID_ARG"), (2, b"WINO_ERR_UNSUPPORTED"),
+                       (3, b"WINO_ERR_MISALIGNED"), (4, b"WINO_ERR_TOO_LARGE"), (5, b"WINO_ERR_CUDA")]:
+        assert L.wino_status_string(code) == name
+    assert L.wino_status_string(99) == b"WINO_ERR_UNKNOWN"
+
+
+def test_filter_workspace_bytes_matches_paper():
+    """L993: 16KC floats = 0.25 / 1 / 4 / 16 MB for Conv2..Conv5."""
+    with open(os.path.join(ROOT, "tests", "golden", "paper_constants.json")) as f:
+        mb = json.load(f)["workspace_MB"]["value"]
+    for name, v in mb.items():
+        cfg = CONFIGS[name]
+        assert wino.filter_workspace_bytes(cfg.C, cfg.K) == int(v * 2 ** 20)
+    assert wino.filter_workspace_bytes(0, 5) == 0
+    assert wino.filter_workspace_bytes(3, -1) == 0
+
+
+def test_host_workspace_bytes():
+    n = wino.host_workspace_bytes(2, 3, 5, 5, 4)
+    need = 3 * 25 * 2 * 4 + 9 * 3 * 4 * 4 + 16 * 3 * 4 * 4 + 4 * 25 * 2 * 4
+    assert need <= n <= need + 4 * 256
+    assert wino.host_workspace_bytes(0, 3, 5, 5, 4) == 0
+
+
+@pytest.mark.parametrize("name", list(CONFIGS))
+def test_plan_shapes(name):
+    c = CONFIGS[name]
+    p = wino.plan(c.N, c.C, c.H, c.W, c.K)
+    assert p.variant == 0 and (p.bk, p.bn, p.bc) == (64, 32, 8)
+    nv = c.N * c.tiles
+    assert p.ctas == -(-nv // p.bn) * -(-c.K // p.bk) * p.split_c
+    assert p.threads == 256 and 0 < p.smem_bytes <= 232448
+    assert p.vec_x == (4 if c.N % 4 == 0 else 1) and p.vec_u == (4 if c.K % 4 == 0 else 1)
+    assert p.launches >= 1
+
+
+def test_plan_rejects_bad_shapes():
+    with pytest.raises(wino.WinoError) as e:
+        wino.plan(0, 1, 1, 1, 1)
+    assert e.value.status == 1
+    with pytest.raises(wino.WinoError) as e:
+        wino.plan(1 << 16, 1 << 10, 64, 64, 1)  # x has 2^42 elements
+    assert e.value.status == 4
+
+
+# Validation that happens before any device access (so it runs here without a GPU).
+def _fwd(x, u, y, N=2, C=3, H=4, W=4, K=5, pad=1, stride=1):
+    L = wino.lib()
+    return L.wino_conv2d_f2x3_fwd(ctypes.c_void_p(x), ctypes.c_void_p(u), ctypes.c_void_p(y),
+                                  N, C, H, W, K, pad, stride, None)
+
+
+def test_fwd_argument_validation_host_side():
+    X, U, Y = 0x100000, 0x200000, 0x300000  # fake, never dereferenced on these paths
+    assert _fwd(0, U, Y) == 1                      # NULL
+    assert _fwd(X, U, Y, N=0) == 1                 # dim <= 0
+    assert _fwd(X, U, Y, K=-3) == 1
+    assert _fwd(X, U, Y, pad=0) == 2               # pad != 1
+    assert _fwd(X, U, Y, stride=2) == 2            # stride != 1
+    assert _fwd(X + 4, U, Y) == 3                  # misaligned
+    assert _fwd(X, U, Y + 8) == 3
+    assert _fwd(X, U, X) == 1                      # y aliases x
+    assert _fwd(X, U, U + 16) == 1                 # y overlaps u
+    assert _fwd(X, U, Y, N=1 << 14, C=1 << 10, H=16, W=16) == 4  # too large
+    L = wino.lib()
+    assert L.wino_filter_transform(None, ctypes.c_void_p(U), 3, 5, None) == 1
+    assert L.wino_filter_transform(ctypes.c_void_p(X + 4), ctypes.c_void_p(U), 3, 5, None) == 3
+    assert L.wino_conv2d_f2x3_fwd_tc(ctypes.c_void_p(X), ctypes.c_void_p(U), ctypes.c_void_p(Y),
+                                     2, 3, 4, 4, 5, 1, 1, 7, None) == 1  # unknown mode
+
+
+def test_python_layer_refuses_cpu_tensors():
+    import torch
+    x = torch.zeros(3, 4, 4, 2)
+    with pytest.raises(ValueError):
+        wino.conv2d(x, torch.zeros(3, 4, 4, 5))
+    with pytest.raises(ValueError):
+        wino.filter_transform(torch.zeros(3, 3, 3, 5))
+    with pytest.raises(TypeError):
+        wino.conv2d(x.double(), torch.zeros(3, 4, 4, 5))
+
+
+def test_product_package_never_imports_oracle():
+    """The product path must not route through the oracle (no CPU fallback)."""
+    pkg = os.path.join(ROOT, "paper_conf_ppopp_yanwc20_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                src = open(os.path.join(dirpath, f), errors="ignore").read()
+                assert not re.search(r"^\s*(import|from)\s+oracle\b", src, re.M), f
+                assert "wino_oracle" not in src and "liboracle" not in src, f

@@ -1,0 +1,160 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Bars (BASELINE.json north_star / SURVEY 8(c)):
+* small-integer inputs: bit-exact vs the direct definition (Eq. 4) -- every FP32
+  intermediate is a small dyadic rational;
+* random inputs: max|y - y_ref| / max|y_ref| <= 1e-4 (FP32 kernel);
+* transformed filter u vs oracle U: bit-exact on small integers, <= 1e-6 random.
+Full-size configs are checked on sampled outputs computed one by one by the
+oracle (Eq. 4 at each point), in the launch configuration bench.py times.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth_inputs import CONFIGS, Conv3x3Config, make_inputs, sample_points
+
+pytestmark = pytest.mark.gpu
+
+FP32_TOL = 1e-4
+FTF_TOL = 1e-6
+
+
+@pytest.fixture(scope="module")
+def wino():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ppopp_yanwc20_b200 as w
+    w.lib()
+    return w
+
+
+DEV = "cuda:0"
+
+
+def _run(wino, x, w, variant="fp32"):
+    u = wino.filter_transform(w.to(DEV))
+    y = wino.conv2d(x.to(DEV), u, variant=variant)
+    torch.cuda.synchronize()
+    return u.cpu(), y.cpu()
+
+
+# Shapes spanning several k-blocks / nu-blocks / channel steps with ragged tails,
+# odd and tiny planes, N%4 != 0 and K%4 != 0 (generic load paths), C%8 != 0.
+EDGE = [
+    (1, 1, 1, 1, 1), (1, 8, 8, 8, 8), (3, 7, 5, 5, 5), (2, 9, 65, 7, 7), (33, 8, 64, 3, 3),
+    (4, 20, 70, 13, 9), (5, 17, 130, 6, 10), (64, 16, 128, 2, 2), (1, 3, 3, 1, 17),
+    (6, 12, 3, 14, 1), (32, 24, 96, 4, 6), (2, 64, 64, 16, 16), (7, 40, 72, 11, 12),
+]
+
+
+@pytest.mark.parametrize("shape", EDGE, ids=[str(s) for s in EDGE])
+def test_edge_shapes_small_int_bit_exact(wino, shape):
+    N, C, K, H, W = shape
+    cfg = Conv3x3Config("edge", N, C, K, H, W)
+    x, w = make_inputs(cfg, kind="smallint")
+    u, y = _run(wino, x, w)
+    assert np.array_equal(u.double().numpy(), oracle.filter_transform(w))
+    assert np.array_equal(y.double().numpy(), oracle.direct_conv(x, w))
+
+
+@pytest.mark.parametrize("shape", EDGE, ids=[str(s) for s in EDGE])
+def test_edge_shapes_random(wino, shape):
+    N, C, K, H, W = shape
+    cfg = Conv3x3Config("edge", N, C, K, H, W)
+    x, w = make_inputs(cfg, kind="uniform", seed_x=11, seed_w=12)
+    u, y = _run(wino, x, w)
+    assert oracle.max_rel_err(u.double().numpy(), oracle.filter_transform(w)) <= FTF_TOL
+    assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= FP32_TOL
+
+
+@pytest.mark.parametrize("name", ["tiny", "conv5_x", "conv4_x", "conv3_x", "conv2_x"])
+@pytest.mark.parametrize("kind", ["smallint", "uniform", "resnet"])
+def test_full_configs_sampled(wino, name, kind):
+    """BASELINE configs at full size: FTF checked element by element; outputs on
+    a seeded sample of points (always including all corners / first / last k, n)."""
+    cfg = CONFIGS[name]
+    x, w = make_inputs(cfg, kind=kind)
+    u, y = _run(wino, x, w)
+    u_ref = oracle.filter_transform(w)
+    idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 4000 if name != "tiny" else 200)
+    ref = oracle.direct_sample(x, w, idx)
+    ii = idx.numpy()
+    got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
+    if kind == "smallint":
+        assert np.array_equal(u.double().numpy(), u_ref)
+        assert np.array_equal(got, ref)
+    else:
+        assert oracle.max_rel_err(u.double().numpy(), u_ref) <= FTF_TOL
+        # normalise by the max of the full output (all GPU values are checked finite)
+        assert np.isfinite(y.numpy()).all()
+        den = max(float(np.max(np.abs(ref))), 1e-30)
+        assert float(np.max(np.abs(got - ref))) / den <= FP32_TOL
+
+
+def test_tiny_full_oracle_both_forms(wino):
+    """Tiny config (the one the oracle runs in full): y vs direct AND vs naive Winograd."""
+    cfg = CONFIGS["tiny"]
+    x, w = make_inputs(cfg)
+    _, y = _run(wino, x, w)
+    yd = y.double().numpy()
+    assert oracle.max_rel_err(yd, oracle.direct_conv(x, w)) <= FP32_TOL
+    assert oracle.max_rel_err(yd, oracle.winograd_conv(x, w)) <= FP32_TOL
+
+
+def test_deterministic_and_batch_shard_consistent(wino):
+    """Same output on repeated runs, and conv of a contiguous batch shard equals the
+    shard of the full output bit for bit (per-output arithmetic does not depend on
+    which CTA computes it) -- the property batch-sharded dispatch relies on."""
+    cfg = CONFIGS["conv3_x"].with_batch(16)
+    x, w = make_inputs(cfg)
+    u = wino.filter_transform(w.to(DEV))
+    xd = x.to(DEV)
+    y1 = wino.conv2d(xd, u)
+    y2 = wino.conv2d(xd, u)
+    torch.cuda.synchronize()
+    assert torch.equal(y1, y2)
+    for lo, hi in [(0, 8), (8, 16), (3, 10), (15, 16)]:
+        ys = wino.conv2d(xd[..., lo:hi].contiguous(), u)
+        torch.cuda.synchronize()
+        assert torch.equal(ys, y1[..., lo:hi])
+
+
+def test_host_entry_point_matches_device_path(wino):
+    cfg = Conv3x3Config("host", 8, 24, 40, 10, 9)
+    x, w = make_inputs(cfg)
+    u, y = _run(wino, x, w)
+    xh, wh = x.pin_memory(), w.pin_memory()
+    yh = torch.empty((cfg.K, cfg.H, cfg.W, cfg.N), dtype=torch.float32).pin_memory()
+    ws = torch.empty(wino.host_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
+                     device=DEV)
+    wino.conv2d_host(xh, wh, yh, ws)
+    torch.cuda.synchronize()
+    assert torch.equal(yh, y)
+
+
+def test_output_fully_overwritten(wino):
+    cfg = Conv3x3Config("ow", 3, 5, 6, 7, 5)
+    x, w = make_inputs(cfg)
+    u = wino.filter_transform(w.to(DEV))
+    out = torch.full((cfg.K, cfg.H, cfg.W, cfg.N), float("nan"), device=DEV)
+    wino.conv2d(x.to(DEV), u, out=out)
+    torch.cuda.synchronize()
+    assert torch.isfinite(out).all()
+    assert oracle.max_rel_err(out.cpu().double().numpy(), oracle.direct_conv(x, w)) <= FP32_TOL
+
+
+def test_device_side_errors(wino):
+    base = torch.zeros(3 * 4 * 4 * 4 + 1, device=DEV)
+    x_mis = base[1:].view(3, 4, 4, 4)  # contiguous but 4-byte aligned only
+    u = torch.zeros(3, 4, 4, 5, device=DEV)
+    with pytest.raises(wino.WinoError) as e:
+        wino.conv2d(x_mis, u)
+    assert e.value.status == 3  # WINO_ERR_MISALIGNED
+    big = torch.zeros(16 * 3 * 5 + 5 * 4 * 4 * 4, device=DEV)
+    u2 = big[:240].view(3, 4, 4, 5)
+    y_alias = big[:320].view(5, 4, 4, 4)  # overlaps u2
+    with pytest.raises(wino.WinoError) as e:
+        wino.conv2d(torch.zeros(3, 4, 4, 4, device=DEV), u2, out=y_alias)
+    assert e.value.status == 1  # WINO_ERR_INVALID_ARG (aliasing)
