@@ -143,7 +143,8 @@ wino_status_t wino_conv2d_f2x3_fwd_host(const float* x_host, const float* w_host
 typedef struct {
     int variant;        /* 0 = FP32 FFMA fused kernel, 1 = tcgen05 TF32 / 3xTF32   */
     int bk, bn, bc;     /* filters, tiles and channels per CTA step (Sec. 3.3)      */
-    int vec_x, vec_u;   /* global-load vector width for x and u (1 or 4 floats)     */
+    int load_x, load_u; /* how x / u reach shared memory: 0 = cp.async 4 B,         */
+                        /* 1 = cp.async 16 B, 2 = TMA tiled box (cp.async.bulk.tensor) */
     int split_c;        /* channel split factor (1 = none)                          */
     int64_t ctas;       /* CTAs of the main kernel                                  */
     int threads;        /* threads per CTA                                          */

@@ -45,7 +45,7 @@ class WinoError(RuntimeError):
 
 class _Plan(ctypes.Structure):
     _fields_ = [("variant", ctypes.c_int), ("bk", ctypes.c_int), ("bn", ctypes.c_int),
-                ("bc", ctypes.c_int), ("vec_x", ctypes.c_int), ("vec_u", ctypes.c_int),
+                ("bc", ctypes.c_int), ("load_x", ctypes.c_int), ("load_u", ctypes.c_int),
                 ("split_c", ctypes.c_int), ("ctas", ctypes.c_int64), ("threads", ctypes.c_int),
                 ("smem_bytes", ctypes.c_int), ("launches", ctypes.c_int)]
 
@@ -56,8 +56,8 @@ class Plan:
     bk: int
     bn: int
     bc: int
-    vec_x: int
-    vec_u: int
+    load_x: int  # 0 cp.async 4 B, 1 cp.async 16 B, 2 TMA
+    load_u: int
     split_c: int
     ctas: int
     threads: int

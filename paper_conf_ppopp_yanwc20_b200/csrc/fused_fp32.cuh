@@ -3,21 +3,27 @@
 // Yan, Wang & Chu (PPoPP'20): workflow Sec. 3.1 (L209), cache blocking
 // Sec. 3.2-3.3 (L211-217, bk=64, bn=32, bc=8), software pipelining Sec. 3.4
 // (L323-333), implicit zero padding Sec. 3.5 (L335), thread-block workload and
-// Algorithm 1 (L339-355), ITF Sec. 4.2 (L357-359), batched GEMM and lane
-// arrangement Sec. 4.3 / Fig. 3 (L361-439), OTF through shared memory Sec. 4.4
-// (L479-503).
+// Algorithm 1 (L339-355), ITF Sec. 4.2 (L357-359), batched GEMM, lane
+// arrangement and register-bank-aware FFMA order Sec. 4.3 / Fig. 3-4
+// (L361-477), OTF through shared memory Sec. 4.4 (L479-503).
 //
 // B200 redesign:
-//  * nu = (tile, n) is flattened with n fastest, so any N works (the paper
-//    assumes 32 consecutive n per CTA, L357) and small per-rank batches still
-//    fill CTAs;
-//  * global->shared staging is a STAGES-deep cp.async ring with hardware zero
-//    fill (src-size 0) instead of predicated LDG into 48 prefetch registers
-//    (Table 5) -- the padding masks live in a per-CTA shared table computed
-//    once (the paper's P2R-packed mask, L337, is not expressible in PTX);
+//  * global->shared staging is an S-deep ring filled by TMA tiled loads
+//    (cp.async.bulk.tensor, completion on an mbarrier): one elected thread moves
+//    a (k:64, xi:16, c:8) box of u and a (n:32, w:4, h:4, c:8) box of raw x per
+//    stage; TMA's out-of-bounds zero fill IS the implicit padding of Sec. 3.5
+//    (negative / past-the-end h, w coordinates) and also pads the C and K tails.
+//    This removes the paper's 48 prefetch registers and predicate masks
+//    (Table 5).  Shapes TMA cannot express (N % 32 != 0 for x,
+//    K % 4 != 0 for u) fall back to cp.async with src-size-0 zero fill and a
+//    per-CTA gather table -- still on the GPU, never on the host;
+//  * nu = (tile, n) is flattened with n fastest, so any N works and small
+//    per-rank batches still fill CTAs (the paper assumes 32 consecutive n);
 //  * B200's 227 KB of shared memory holds all 128 KB of accumulators at once,
 //    so the OTF transpose runs in ONE round instead of the paper's 4 (L499).
 #pragma once
+#include <cuda.h>
+
 #include <cstdint>
 
 #include "wino_ptx.cuh"
@@ -36,16 +42,22 @@ constexpr int STAGE_FLOATS = US_FLOATS + XS_FLOATS;
 constexpr int VS_FLOATS = 16 * BC * BN;  // transformed input      [xi][c][nu] (Table 4 (16,bc,bn))
 constexpr int EP_LD = BN + 4;            // padded row of the OTF transpose buffer
 constexpr int EP_FLOATS = 16 * BK * EP_LD;
-constexpr int TAB_INTS = 16 * BN;        // per-CTA gather/padding table
+constexpr int TAB_INTS = 16 * BN;        // per-CTA gather/padding table (cp.async x path)
+
+// how a stage's operand reaches shared memory
+enum LoadMode : int { LD_CP4B = 0, LD_CP16B = 1, LD_TMA = 2 };
 
 template <int S>
 struct Smem {
     static constexpr int main_floats = S * STAGE_FLOATS + 2 * VS_FLOATS;
     static_assert(EP_FLOATS <= main_floats, "OTF buffer must fit in the pipeline buffers");
-    static constexpr int bytes = (main_floats + TAB_INTS) * 4;
+    static constexpr int bar_offset = (main_floats + TAB_INTS) * 4;
+    static constexpr int bytes = bar_offset + S * 8;
 };
 
-struct Params {
+struct __align__(64) Params {
+    CUtensorMap tmx;  // x (C,H,W,N) as 4-d (N, W, H, C), box (32, 4, 4, BC)   [LD_TMA only]
+    CUtensorMap tmu;  // u (C,16,K)  as 3-d (K, 16, C),   box (BK, 16, BC)      [LD_TMA only]
     const float* __restrict__ x;  // (C,H,W,N)
     const float* __restrict__ u;  // (C,4,4,K)
     float* __restrict__ y;        // (K,H,W,N)
@@ -56,11 +68,14 @@ struct Params {
     int num_it;  // ceil(C/BC)
 };
 
-template <int VX, int VU, int S>
-__global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const Params p) {
+template <int XM, int UM, int S>
+__global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant__ Params p) {
+    constexpr bool kTma = (XM == LD_TMA) || (UM == LD_TMA);
+    constexpr uint32_t kTmaBytes = (XM == LD_TMA ? XS_FLOATS * 4 : 0) + (UM == LD_TMA ? US_FLOATS * 4 : 0);
     extern __shared__ __align__(1024) float smem[];
     float* const vs = smem + S * STAGE_FLOATS;
     int* const xtab = reinterpret_cast<int*>(vs + 2 * VS_FLOATS);
+    uint64_t* const bar = reinterpret_cast<uint64_t*>(reinterpret_cast<char*>(smem) + Smem<S>::bar_offset);
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     // k-block fastest: the CTAs resident at once share input tiles through L2
@@ -69,53 +84,89 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const Params p) {
     const int k0 = kb * BK, nu0 = nb * BN;
     const size_t HWN = (size_t)p.H * p.W * p.N;
 
-    // Spatial gather offsets (h*W+w)*N+n of the 4x4 window element `pos` of
-    // local tile nu, or -1 where the window leaves the image (zero padding).
-    for (int e = tid; e < TAB_INTS; e += NT) {
-        const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
-        int off = -1;
-        if (nu < p.NV) {
-            const int t = nu / p.N, n = nu - t * p.N;
-            const int th = t / p.TW, tw = t - th * p.TW;
-            const int h = 2 * th - 1 + (pos >> 2), w = 2 * tw - 1 + (pos & 3);
-            if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
+    if constexpr (kTma) {
+        if (tid == 0) {
+            if constexpr (XM == LD_TMA) tma_prefetch_desc(&p.tmx);
+            if constexpr (UM == LD_TMA) tma_prefetch_desc(&p.tmu);
+#pragma unroll
+            for (int s = 0; s < S; ++s) mbar_init(&bar[s], 1);
+            fence_mbar_init();
         }
-        xtab[e] = off;
+    }
+    // TMA x box origin: N % 32 == 0, so the CTA's 32 nu are 32 consecutive n of one tile
+    int tma_n0 = 0, tma_w0 = 0, tma_h0 = 0;
+    if constexpr (XM == LD_TMA) {
+        const int t = nu0 / p.N;
+        tma_n0 = nu0 - t * p.N;
+        const int th = t / p.TW, tw = t - th * p.TW;
+        tma_w0 = 2 * tw - 1;  // may be -1: TMA zero-fills (implicit padding, Sec. 3.5)
+        tma_h0 = 2 * th - 1;
+    } else {
+        // Spatial gather offsets (h*W+w)*N+n of the 4x4 window element `pos` of
+        // local tile nu, or -1 where the window leaves the image (zero padding).
+        for (int e = tid; e < TAB_INTS; e += NT) {
+            const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
+            int off = -1;
+            if (nu < p.NV) {
+                const int t = nu / p.N, n = nu - t * p.N;
+                const int th = t / p.TW, tw = t - th * p.TW;
+                const int h = 2 * th - 1 + (pos >> 2), w = 2 * tw - 1 + (pos & 3);
+                if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
+            }
+            xtab[e] = off;
+        }
     }
     __syncthreads();
 
     // ---- producer: one pipeline stage = BC channels of u and raw x ----------
-    auto load_stage = [&](int it, int slot) {
+    auto issue_stage = [&](int it, int slot) {
         const int c0 = it * BC;
         float* us = smem + slot * STAGE_FLOATS;
         float* xs = us + US_FLOATS;
-        constexpr int UV_ROW = BK / VU;
-        constexpr int U_PER_THREAD = BC * 16 * UV_ROW / NT;
-#pragma unroll
-        for (int j = 0; j < U_PER_THREAD; ++j) {
-            const int idx = tid + j * NT;
-            const int row = idx / UV_ROW, col = (idx % UV_ROW) * VU;
-            const int c = c0 + row / 16, k = k0 + col;
-            const bool ok = (c < p.C) && (k < p.K);
-            const float* src = ok ? p.u + ((size_t)c * 16 + (row & 15)) * p.K + k : p.u;
-            const uint32_t dst = smem_u32(us + row * BK + col);
-            if constexpr (VU == 4) cp_async16(dst, src, ok);
-            else cp_async4(dst, src, ok);
+        if constexpr (kTma) {
+            if (tid == 0) {
+                fence_proxy_async_smem();  // prior generic reads of this slot before async writes
+                mbar_arrive_expect_tx(&bar[slot], kTmaBytes);
+                if constexpr (UM == LD_TMA) tma_load_3d(us, &p.tmu, &bar[slot], k0, 0, c0);
+                if constexpr (XM == LD_TMA) tma_load_4d(xs, &p.tmx, &bar[slot], tma_n0, tma_w0, tma_h0, c0);
+            }
         }
-        constexpr int XV_C = 16 * BN / VX;
-        constexpr int X_PER_THREAD = BC * XV_C / NT;
+        if constexpr (UM != LD_TMA) {
+            constexpr int VU = UM == LD_CP16B ? 4 : 1;
+            constexpr int UV_ROW = BK / VU;
+            constexpr int U_PER_THREAD = BC * 16 * UV_ROW / NT;
 #pragma unroll
-        for (int j = 0; j < X_PER_THREAD; ++j) {
-            const int idx = tid + j * NT;
-            const int cl = idx / XV_C, e = (idx % XV_C) * VX;
-            const int c = c0 + cl;
-            const int off = xtab[e];
-            const bool ok = (c < p.C) && (off >= 0);
-            const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
-            const uint32_t dst = smem_u32(xs + cl * 16 * BN + e);
-            if constexpr (VX == 4) cp_async16(dst, src, ok);
-            else cp_async4(dst, src, ok);
+            for (int j = 0; j < U_PER_THREAD; ++j) {
+                const int idx = tid + j * NT;
+                const int row = idx / UV_ROW, col = (idx % UV_ROW) * VU;
+                const int c = c0 + row / 16, k = k0 + col;
+                const bool ok = (c < p.C) && (k < p.K);
+                const float* src = ok ? p.u + ((size_t)c * 16 + (row & 15)) * p.K + k : p.u;
+                const uint32_t dst = smem_u32(us + row * BK + col);
+                if constexpr (VU == 4) cp_async16(dst, src, ok);
+                else cp_async4(dst, src, ok);
+            }
         }
+        if constexpr (XM != LD_TMA) {
+            constexpr int VX = XM == LD_CP16B ? 4 : 1;
+            constexpr int XV_C = 16 * BN / VX;
+            constexpr int X_PER_THREAD = BC * XV_C / NT;
+#pragma unroll
+            for (int j = 0; j < X_PER_THREAD; ++j) {
+                const int idx = tid + j * NT;
+                const int cl = idx / XV_C, e = (idx % XV_C) * VX;
+                const int c = c0 + cl;
+                const int off = xtab[e];
+                const bool ok = (c < p.C) && (off >= 0);
+                const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
+                const uint32_t dst = smem_u32(xs + cl * 16 * BN + e);
+                if constexpr (VX == 4) cp_async16(dst, src, ok);
+                else cp_async4(dst, src, ok);
+            }
+        }
+    };
+    auto wait_tma = [&](int it) {
+        if constexpr (kTma) mbar_wait(&bar[it % S], (it / S) & 1);
     };
 
     // ---- ITF (Sec. 4.2): one (c, nu) tile per thread, raw [c][pos][nu] ->
@@ -162,31 +213,42 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const Params p) {
                 g[q][0] = va.x; g[q][1] = va.y; g[q][2] = va.z; g[q][3] = va.w;
                 g[q][4] = vb.x; g[q][5] = vb.y; g[q][6] = vb.z; g[q][7] = vb.w;
             }
+            // Register-bank-aware FFMA order (the paper's Fig. 4 rule, L469-477,
+            // re-derived for sm_100: an FFMA costs max(#even, #odd) register
+            // reads among operands not served by the reuse cache).  f[i] is
+            // reused along a row; acc[i][j] is packed with parity opposite to
+            // g[j] (see the swapped float4 packing in the OTF store) and rows
+            // snake so the row change reuses g[j_end] instead of f[i].
 #pragma unroll
             for (int q = 0; q < 2; ++q)
 #pragma unroll
                 for (int i = 0; i < 8; ++i)
 #pragma unroll
-                    for (int j = 0; j < 8; ++j) acc[q][i][j] = fmaf(f[q][i], g[q][j], acc[q][i][j]);
+                    for (int jj = 0; jj < 8; ++jj) {
+                        const int j = (i & 1) ? 7 - jj : jj;
+                        acc[q][i][j] = fmaf(f[q][i], g[q][j], acc[q][i][j]);
+                    }
         }
     };
 
-    // ---- main loop (Algorithm 1 lines 6-16) with an S-stage cp.async ring --
+    // ---- main loop (Algorithm 1 lines 6-16) with an S-stage ring -----------
     const int NIT = p.num_it;
 #pragma unroll
     for (int s = 0; s < S - 1; ++s) {
-        if (s < NIT) load_stage(s, s);
+        if (s < NIT) issue_stage(s, s);
         cp_async_commit();
     }
-    cp_async_wait<S - 2>();  // stage 0 landed
+    cp_async_wait<S - 2>();
+    wait_tma(0);
     __syncthreads();
     itf_stage(0, 0);
 
     for (int it = 0; it < NIT; ++it) {
-        cp_async_wait<S - 3>();  // stage it+1 landed (if issued)
-        __syncthreads();         // V[it&1] complete; slot (it-1)%S free
+        cp_async_wait<S - 3>();
+        if (it + 1 < NIT) wait_tma(it + 1);  // stage it+1 landed
+        __syncthreads();                      // V[it&1] complete; slot (it-1)%S free
         const int nxt = it + S - 1;
-        if (nxt < NIT) load_stage(nxt, nxt % S);
+        if (nxt < NIT) issue_stage(nxt, nxt % S);
         cp_async_commit();
         if (it + 1 < NIT) itf_stage((it + 1) % S, (it + 1) & 1);
         gemm_stage(it % S, it & 1);
@@ -195,6 +257,8 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const Params p) {
     __syncthreads();
 
     // ---- OTF (Sec. 4.4): accumulators -> smem [xi][k][nu] in one round ------
+    // Columns are stored pair-swapped (nu^1), matching the register packing
+    // chosen for bank-conflict-free FFMAs; the reader undoes it.
     float* ep = smem;
 #pragma unroll
     for (int q = 0; q < 2; ++q)
@@ -203,9 +267,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const Params p) {
             const int kl = fo + (i & 3) + (i >> 2) * 32;
             float* row = ep + ((xi0 + q) * BK + kl) * EP_LD + io;
             *reinterpret_cast<float4*>(row) =
-                make_float4(acc[q][i][0], acc[q][i][1], acc[q][i][2], acc[q][i][3]);
+                make_float4(acc[q][i][1], acc[q][i][0], acc[q][i][3], acc[q][i][2]);
             *reinterpret_cast<float4*>(row + 16) =
-                make_float4(acc[q][i][4], acc[q][i][5], acc[q][i][6], acc[q][i][7]);
+                make_float4(acc[q][i][5], acc[q][i][4], acc[q][i][7], acc[q][i][6]);
         }
     __syncthreads();
 
@@ -223,7 +287,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const Params p) {
             if (k >= p.K) break;
             float m[16], o[4];
 #pragma unroll
-            for (int e = 0; e < 16; ++e) m[e] = ep[(e * BK + kl) * EP_LD + lane];
+            for (int e = 0; e < 16; ++e) m[e] = ep[(e * BK + kl) * EP_LD + (lane ^ 1)];
             otf_2x2(m, o);
             float* yk = p.y + (size_t)k * HWN + base;
             yk[0] = o[0];

@@ -3,7 +3,9 @@
 // Argument validation, shape -> kernel-variant dispatch, launches.  Every step
 // of the computation runs in the CUDA kernels included below; there is no host
 // or CPU fallback anywhere in this library.
+#include <cuda.h>
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 
 #include <atomic>
 #include <cstdint>
@@ -83,31 +85,62 @@ wino_status_t check_shape(int N, int C, int H, int W, int K, int pad, int stride
 }
 
 struct Fp32Plan {
-    int vec_x, vec_u;
+    int load_x, load_u;  // wino::fp32::LoadMode
     int64_t ctas;
     int smem;
 };
 
 Fp32Plan plan_fp32(int N, int C, int H, int W, int K) {
+    using namespace wino::fp32;
     Fp32Plan p;
-    p.vec_x = (N % 4 == 0) ? 4 : 1;
-    p.vec_u = (K % 4 == 0) ? 4 : 1;
+    p.load_x = (N % 32 == 0) ? LD_TMA : (N % 4 == 0 ? LD_CP16B : LD_CP4B);
+    p.load_u = (K % 4 == 0) ? LD_TMA : LD_CP4B;
     const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
-    const int64_t nb = (nv + wino::fp32::BN - 1) / wino::fp32::BN;
-    const int64_t kb = (K + wino::fp32::BK - 1) / wino::fp32::BK;
+    const int64_t nb = (nv + BN - 1) / BN;
+    const int64_t kb = (K + BK - 1) / BK;
     p.ctas = nb * kb;
-    p.smem = wino::fp32::Smem<kStages>::bytes;
+    p.smem = Smem<kStages>::bytes;
     (void)C;
     return p;
 }
 
-std::atomic<uint64_t> g_attr_fp32[4];
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda).
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+    static std::atomic<void*> fn{nullptr};
+    void* f = fn.load(std::memory_order_acquire);
+    if (!f) {
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            return nullptr;
+        fn.store(f, std::memory_order_release);
+    }
+    return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+}
 
-template <int VX, int VU>
-wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem, int dev,
-                          cudaStream_t st, std::atomic<uint64_t>& done) {
-    auto kern = wino::fp32::fused_fp32_kernel<VX, VU, kStages>;
-    wino_status_t s = ensure_smem_attr(kern, dev, smem, done);
+// fp32 tensor map over a dense row-major array, dims innermost first.
+bool encode_map(CUtensorMap* m, const float* base, int rank, const cuuint64_t* dims, const cuuint32_t* box) {
+    auto enc = tensor_map_encoder();
+    if (!enc) return false;
+    cuuint64_t strides[4];
+    cuuint64_t acc = 4;
+    for (int i = 0; i < rank - 1; ++i) {
+        acc *= dims[i];
+        strides[i] = acc;
+    }
+    cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, rank, const_cast<float*>(base), dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);  // OOB elements read as zero
+    return r == CUDA_SUCCESS;
+}
+
+std::atomic<uint64_t> g_attr_fp32[3][3];
+
+template <int XM, int UM>
+wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem, int dev, cudaStream_t st) {
+    auto kern = wino::fp32::fused_fp32_kernel<XM, UM, kStages>;
+    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_fp32[XM][UM]);
     if (s != WINO_OK) return s;
     kern<<<dim3(static_cast<unsigned>(ctas)), wino::fp32::NT, smem, st>>>(prm);
     cudaError_t e = cudaGetLastError();
@@ -165,8 +198,8 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
     plan->bk = wino::fp32::BK;
     plan->bn = wino::fp32::BN;
     plan->bc = wino::fp32::BC;
-    plan->vec_x = p.vec_x;
-    plan->vec_u = p.vec_u;
+    plan->load_x = p.load_x;
+    plan->load_u = p.load_u;
     plan->split_c = 1;
     plan->ctas = p.ctas;
     plan->threads = wino::fp32::NT;
@@ -188,8 +221,10 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
     int dev;
     if ((s = check_device(&dev)) != WINO_OK) return s;
 
+    using namespace wino::fp32;
     Fp32Plan pl = plan_fp32(N, C, H, W, K);
-    wino::fp32::Params prm;
+    Params prm;
+    std::memset(&prm, 0, sizeof(prm));
     prm.x = x_dev;
     prm.u = u_dev;
     prm.y = y_dev;
@@ -200,13 +235,29 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
     prm.K = K;
     prm.TW = (W + 1) / 2;
     prm.NV = N * ((H + 1) / 2) * prm.TW;
-    prm.num_kb = (K + wino::fp32::BK - 1) / wino::fp32::BK;
-    prm.num_it = (C + wino::fp32::BC - 1) / wino::fp32::BC;
+    prm.num_kb = (K + BK - 1) / BK;
+    prm.num_it = (C + BC - 1) / BC;
+    if (pl.load_x == LD_TMA) {
+        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
+        const cuuint32_t box[4] = {BN, 4, 4, BC};
+        if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    if (pl.load_u == LD_TMA) {
+        const cuuint64_t dims[3] = {cuuint64_t(K), 16, cuuint64_t(C)};
+        const cuuint32_t box[3] = {BK, 16, BC};
+        if (!encode_map(&prm.tmu, u_dev, 3, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+    }
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    if (pl.vec_x == 4 && pl.vec_u == 4) return launch_fp32<4, 4>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[0]);
-    if (pl.vec_x == 4) return launch_fp32<4, 1>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[1]);
-    if (pl.vec_u == 4) return launch_fp32<1, 4>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[2]);
-    return launch_fp32<1, 1>(prm, pl.ctas, pl.smem, dev, st, g_attr_fp32[3]);
+    const int64_t g = pl.ctas;
+    const int sm = pl.smem;
+    switch (pl.load_x * 3 + pl.load_u) {
+        case LD_TMA * 3 + LD_TMA: return launch_fp32<LD_TMA, LD_TMA>(prm, g, sm, dev, st);
+        case LD_TMA * 3 + LD_CP4B: return launch_fp32<LD_TMA, LD_CP4B>(prm, g, sm, dev, st);
+        case LD_CP16B * 3 + LD_TMA: return launch_fp32<LD_CP16B, LD_TMA>(prm, g, sm, dev, st);
+        case LD_CP16B * 3 + LD_CP4B: return launch_fp32<LD_CP16B, LD_CP4B>(prm, g, sm, dev, st);
+        case LD_CP4B * 3 + LD_TMA: return launch_fp32<LD_CP4B, LD_TMA>(prm, g, sm, dev, st);
+        default: return launch_fp32<LD_CP4B, LD_CP4B>(prm, g, sm, dev, st);
+    }
 }
 
 wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H,

@@ -78,17 +78,6 @@ def make_inputs(cfg: Conv3x3Config, kind: str = "uniform", seed_x: int = SEED_X,
     return x.contiguous(), w.contiguous()
 
 
-def shard_range(n_total: int, rank: int, world: int):
-    """Contiguous batch shard [lo, hi) of rank r out of `world`.
-
-    Remainders go to the lowest ranks so every rank gets floor or ceil of N/P.
-    """
-    base, rem = divmod(n_total, world)
-    lo = rank * base + min(rank, rem)
-    hi = lo + base + (1 if rank < rem else 0)
-    return lo, hi
-
-
 def sample_points(K: int, H: int, W: int, N: int, n_pts: int, seed: int = 7):
     """Seeded output sample (n_pts, 4) of (k, i, j, n) that always includes the
     four corners / borders of the output plane and the first and last k, n."""

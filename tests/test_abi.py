@@ -65,7 +65,8 @@ def test_plan_shapes(name):
     nv = c.N * c.tiles
     assert p.ctas == -(-nv // p.bn) * -(-c.K // p.bk) * p.split_c
     assert p.threads == 256 and 0 < p.smem_bytes <= 232448
-    assert p.vec_x == (4 if c.N % 4 == 0 else 1) and p.vec_u == (4 if c.K % 4 == 0 else 1)
+    assert p.load_x == (2 if c.N % 32 == 0 else (1 if c.N % 4 == 0 else 0))
+    assert p.load_u == (2 if c.K % 4 == 0 else 0)
     assert p.launches >= 1
 
 
