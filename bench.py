@@ -205,7 +205,7 @@ def _config(args, layers, world):
         "variant": args.variant,
         "inputs": f"uniform[-1,1) fp32, torch seeds x={SEED_X} w={SEED_W}",
         "l2": "flushed before every timed step by a 512 MiB write + 256 MiB read (outside the events)",
-        "step": "per layer: FTF kernel + fused ITF/16xGEMM/OTF kernel",
+        "step": "per layer: FTF kernel + fused ITF/16xGEMM/OTF kernel; the whole step replayed from one CUDA graph",
     }
 
 
@@ -281,23 +281,38 @@ def main():
             c = d["cfg"]
             launches_per_step += 1 + wino.plan(d["n"], c.C, c.H, c.W, c.K).launches
 
-    def step(ev_layer=None):
-        for i, d in enumerate(per):
-            if d["n"] == 0:
-                continue
-            c = d["cfg"]
-            if ev_layer is not None:
-                ev_layer[i][0].record(stream)
+    def run_layer(d, ftf=True, conv=True):
+        if d["n"] == 0:
+            return
+        if ftf:
             wino.filter_transform(d["w"], out=d["u"])
-            if ev_layer is not None:
-                ev_layer[i][1].record(stream)
+        if conv:
             wino.conv2d(d["x"], d["u"], out=d["y"], variant=args.variant)
-            if ev_layer is not None:
-                ev_layer[i][2].record(stream)
+
+    def step():
+        for d in per:
+            run_layer(d)
 
     for _ in range(args.warmup):
         flush_l2(1.0)
         step()
+    torch.cuda.synchronize()
+    # The timed step is replayed from a CUDA graph (captured once, after warm-up):
+    # host launch latency stays out of the device timeline, as in a serving loop.
+    g_step = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g_step):
+        step()
+    g_layer = []
+    for d in per:
+        gf, gc = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
+        with torch.cuda.graph(gf):
+            run_layer(d, conv=False)
+        with torch.cuda.graph(gc):
+            run_layer(d, ftf=False)
+        g_layer.append((gf, gc))
+    for _ in range(2):
+        flush_l2(2.0)
+        g_step.replay()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -309,12 +324,11 @@ def main():
         time.sleep(0.3)
     mk = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
     step_ev = [(mk(), mk()) for _ in range(args.steps)]
-    lay_ev = [[[mk(), mk(), mk()] for _ in per] for _ in range(args.steps)]
     t_wall0 = time.perf_counter()
     for s in range(args.steps):
         flush_l2(float(s))
         step_ev[s][0].record(stream)
-        step(lay_ev[s])
+        g_step.replay()
         step_ev[s][1].record(stream)
     torch.cuda.synchronize()
     wall = time.perf_counter() - t_wall0
@@ -322,8 +336,20 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     clocks = sampler.stop() if sampler else None
-
     ms_step = sum(a.elapsed_time(b) for a, b in step_ev) / args.steps
+
+    # per-layer breakdown (same graphs split per kernel, L2 flushed before each layer)
+    lay_ev = [[[mk(), mk(), mk()] for _ in per] for _ in range(args.steps)]
+    for s in range(args.steps):
+        for i, (gf, gc) in enumerate(g_layer):
+            flush_l2(float(s))
+            e0, e1, e2 = lay_ev[s][i]
+            e0.record(stream)
+            gf.replay()
+            e1.record(stream)
+            gc.replay()
+            e2.record(stream)
+    torch.cuda.synchronize()
     ftf_ms, conv_ms = [0.0] * len(per), [0.0] * len(per)
     for s in range(args.steps):
         for i, d in enumerate(per):

@@ -171,16 +171,20 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
 
     // ---- ITF (Sec. 4.2): one (c, nu) tile per thread, raw [c][pos][nu] ->
     //      V [xi][c][nu]; lanes run along nu so both sides are conflict-free.
-    auto itf_stage = [&](int slot, int vbuf) {
-        const float* xs = smem + slot * STAGE_FLOATS + US_FLOATS;
-        float* v = vs + vbuf * VS_FLOATS;
-        const int cl = tid >> 5, nl = tid & 31;
-        float d[16], t[16];
+    //      Split into load / transform+store halves so the main loop can
+    //      interleave them with the FFMA stream of the previous stage.
+    const int itf_c = tid >> 5, itf_n = tid & 31;
+    auto itf_load = [&](int slot, float d[16]) {
+        const float* xs = smem + slot * STAGE_FLOATS + US_FLOATS + itf_c * 16 * BN + itf_n;
 #pragma unroll
-        for (int e = 0; e < 16; ++e) d[e] = xs[(cl * 16 + e) * BN + nl];
+        for (int e = 0; e < 16; ++e) d[e] = xs[e * BN];
+    };
+    auto itf_store = [&](int vbuf, const float d[16]) {
+        float t[16];
         itf_4x4(d, t);
+        float* v = vs + vbuf * VS_FLOATS + itf_c * BN + itf_n;
 #pragma unroll
-        for (int e = 0; e < 16; ++e) v[(e * BC + cl) * BN + nl] = t[e];
+        for (int e = 0; e < 16; ++e) v[e * BC * BN] = t[e];
     };
 
     // ---- EWMM as 16-batched GEMM (Sec. 4.3): warp w owns xi = 2w, 2w+1; the
@@ -196,38 +200,54 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
 #pragma unroll
             for (int j = 0; j < 8; ++j) acc[q][i][j] = 0.f;
 
-    auto gemm_stage = [&](int slot, int vbuf) {
+    // fragments of one channel c: f = u[c][xi][k-block], g = V[xi][c][nu-block]
+    auto load_frag = [&](const float* us, const float* v, int c, float f[2][8], float g[2][8]) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            const float4 a = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK);
+            const float4 b = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK + 32);
+            const float4 va = *reinterpret_cast<const float4*>(v + (q * BC + c) * BN);
+            const float4 vb = *reinterpret_cast<const float4*>(v + (q * BC + c) * BN + 16);
+            f[q][0] = a.x; f[q][1] = a.y; f[q][2] = a.z; f[q][3] = a.w;
+            f[q][4] = b.x; f[q][5] = b.y; f[q][6] = b.z; f[q][7] = b.w;
+            g[q][0] = va.x; g[q][1] = va.y; g[q][2] = va.z; g[q][3] = va.w;
+            g[q][4] = vb.x; g[q][5] = vb.y; g[q][6] = vb.z; g[q][7] = vb.w;
+        }
+    };
+    // Register-bank-aware FFMA order (the paper's Fig. 4 rule, L469-477,
+    // re-derived for sm_100: an FFMA costs max(#even, #odd) register reads
+    // among operands not served by the reuse cache).  f[i] is reused along a
+    // row; acc[i][j] is packed with parity opposite to g[j] (see the swapped
+    // float4 packing in the OTF store) and rows snake so the row change reuses
+    // g[j_end] instead of f[i].
+    auto ffma_block = [&](const float f[2][8], const float g[2][8]) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q)
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+#pragma unroll
+                for (int jj = 0; jj < 8; ++jj) {
+                    const int j = (i & 1) ? 7 - jj : jj;
+                    acc[q][i][j] = fmaf(f[q][i], g[q][j], acc[q][i][j]);
+                }
+    };
+    // One pipeline step: GEMM over the BC channels of stage `slot` / V buffer
+    // `vbuf`, with fragments double-buffered in registers (Sec. 3.4:
+    // "hide the latency of LDS with software pipelining") and, when do_itf,
+    // the ITF of the next stage woven into the FFMA stream.
+    auto gemm_stage = [&](int slot, int vbuf, bool do_itf, int itf_slot, int itf_vbuf) {
         const float* us = smem + slot * STAGE_FLOATS + xi0 * BK + fo;
         const float* v = vs + vbuf * VS_FLOATS + xi0 * BC * BN + io;
+        float fa[2][8], ga[2][8], fb[2][8], gb[2][8], d[16];
+        load_frag(us, v, 0, fa, ga);
+        if (do_itf) itf_load(itf_slot, d);
 #pragma unroll
-        for (int c = 0; c < BC; ++c) {
-            float f[2][8], g[2][8];
-#pragma unroll
-            for (int q = 0; q < 2; ++q) {
-                const float4 a = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK);
-                const float4 b = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK + 32);
-                const float4 va = *reinterpret_cast<const float4*>(v + (q * BC + c) * BN);
-                const float4 vb = *reinterpret_cast<const float4*>(v + (q * BC + c) * BN + 16);
-                f[q][0] = a.x; f[q][1] = a.y; f[q][2] = a.z; f[q][3] = a.w;
-                f[q][4] = b.x; f[q][5] = b.y; f[q][6] = b.z; f[q][7] = b.w;
-                g[q][0] = va.x; g[q][1] = va.y; g[q][2] = va.z; g[q][3] = va.w;
-                g[q][4] = vb.x; g[q][5] = vb.y; g[q][6] = vb.z; g[q][7] = vb.w;
-            }
-            // Register-bank-aware FFMA order (the paper's Fig. 4 rule, L469-477,
-            // re-derived for sm_100: an FFMA costs max(#even, #odd) register
-            // reads among operands not served by the reuse cache).  f[i] is
-            // reused along a row; acc[i][j] is packed with parity opposite to
-            // g[j] (see the swapped float4 packing in the OTF store) and rows
-            // snake so the row change reuses g[j_end] instead of f[i].
-#pragma unroll
-            for (int q = 0; q < 2; ++q)
-#pragma unroll
-                for (int i = 0; i < 8; ++i)
-#pragma unroll
-                    for (int jj = 0; jj < 8; ++jj) {
-                        const int j = (i & 1) ? 7 - jj : jj;
-                        acc[q][i][j] = fmaf(f[q][i], g[q][j], acc[q][i][j]);
-                    }
+        for (int c = 0; c < BC; c += 2) {
+            load_frag(us, v, c + 1, fb, gb);
+            ffma_block(fa, ga);
+            if (c == 0 && do_itf) itf_store(itf_vbuf, d);
+            if (c + 2 < BC) load_frag(us, v, c + 2, fa, ga);
+            ffma_block(fb, gb);
         }
     };
 
@@ -241,7 +261,11 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
     cp_async_wait<S - 2>();
     wait_tma(0);
     __syncthreads();
-    itf_stage(0, 0);
+    {
+        float d[16];
+        itf_load(0, d);
+        itf_store(0, d);
+    }
 
     for (int it = 0; it < NIT; ++it) {
         cp_async_wait<S - 3>();
@@ -250,8 +274,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
         const int nxt = it + S - 1;
         if (nxt < NIT) issue_stage(nxt, nxt % S);
         cp_async_commit();
-        if (it + 1 < NIT) itf_stage((it + 1) % S, (it + 1) & 1);
-        gemm_stage(it % S, it & 1);
+        gemm_stage(it % S, it & 1, it + 1 < NIT, (it + 1) % S, (it + 1) & 1);
     }
     cp_async_wait<0>();
     __syncthreads();
