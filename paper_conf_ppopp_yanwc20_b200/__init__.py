@@ -24,7 +24,7 @@ __all__ = [
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_PKG, "libwino.so")
+_LIB_PATH = os.environ.get("WINO_LIB_PATH") or os.path.join(_PKG, "libwino.so")  # override: A/B builds
 _lib = None
 
 TC_TF32 = 0

@@ -35,7 +35,6 @@ namespace fp32 {
 constexpr int BK = 64;   // filters per CTA   (Sec. 3.3)
 constexpr int BN = 32;   // tiles*images per CTA
 constexpr int BC = 8;    // channels per pipeline step
-constexpr int NT = 256;  // threads per CTA   (Sec. 4)
 constexpr int US_FLOATS = BC * 16 * BK;  // transformed-filter stage [c][xi][k]
 constexpr int XS_FLOATS = BC * 16 * BN;  // raw-input stage        [c][pos][nu]
 constexpr int STAGE_FLOATS = US_FLOATS + XS_FLOATS;
@@ -68,8 +67,17 @@ struct __align__(64) Params {
     int num_it;  // ceil(C/BC)
 };
 
-template <int XM, int UM, int S>
-__global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant__ Params p) {
+// XPW = Winograd elements xi per warp: 2 -> 8 warps / 256 threads (the paper's
+// Sec. 4 / Alg. 1 shape, 2 x 64 accumulators per thread); 1 -> 16 warps / 512
+// threads with 64 accumulators each (same CTA tile, twice the warps per
+// scheduler to hide LDS / barrier latency).
+template <int XPW>
+__host__ __device__ constexpr int threads_for() { return 512 / XPW; }
+
+template <int XM, int UM, int S, int XPW>
+__global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const __grid_constant__ Params p) {
+    constexpr int NT = threads_for<XPW>();
+    constexpr int NWARP = NT / 32;
     constexpr bool kTma = (XM == LD_TMA) || (UM == LD_TMA);
     constexpr uint32_t kTmaBytes = (XM == LD_TMA ? XS_FLOATS * 4 : 0) + (UM == LD_TMA ? US_FLOATS * 4 : 0);
     extern __shared__ __align__(1024) float smem[];
@@ -187,23 +195,23 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
         for (int e = 0; e < 16; ++e) v[e * BC * BN] = t[e];
     };
 
-    // ---- EWMM as 16-batched GEMM (Sec. 4.3): warp w owns xi = 2w, 2w+1; the
-    //      lane owns an 8(k) x 8(nu) block of each, Fig. 3 lane arrangement.
+    // ---- EWMM as 16-batched GEMM (Sec. 4.3): warp w owns xi = XPW*w .. +XPW-1;
+    //      the lane owns an 8(k) x 8(nu) block of each, Fig. 3 lane arrangement.
     const int fo = 4 * ((lane & 15) >> 1);             // k offset: fo..fo+3, fo+32..fo+35
     const int io = 4 * ((lane & 1) + 2 * (lane >> 4));  // nu offset: io..io+3, io+16..io+19
-    const int xi0 = 2 * warp;
-    float acc[2][8][8];
+    const int xi0 = XPW * warp;
+    float acc[XPW][8][8];
 #pragma unroll
-    for (int q = 0; q < 2; ++q)
+    for (int q = 0; q < XPW; ++q)
 #pragma unroll
         for (int i = 0; i < 8; ++i)
 #pragma unroll
             for (int j = 0; j < 8; ++j) acc[q][i][j] = 0.f;
 
     // fragments of one channel c: f = u[c][xi][k-block], g = V[xi][c][nu-block]
-    auto load_frag = [&](const float* us, const float* v, int c, float f[2][8], float g[2][8]) {
+    auto load_frag = [&](const float* us, const float* v, int c, float f[XPW][8], float g[XPW][8]) {
 #pragma unroll
-        for (int q = 0; q < 2; ++q) {
+        for (int q = 0; q < XPW; ++q) {
             const float4 a = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK);
             const float4 b = *reinterpret_cast<const float4*>(us + (c * 16 + q) * BK + 32);
             const float4 va = *reinterpret_cast<const float4*>(v + (q * BC + c) * BN);
@@ -220,9 +228,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
     // row; acc[i][j] is packed with parity opposite to g[j] (see the swapped
     // float4 packing in the OTF store) and rows snake so the row change reuses
     // g[j_end] instead of f[i].
-    auto ffma_block = [&](const float f[2][8], const float g[2][8]) {
+    auto ffma_block = [&](const float f[XPW][8], const float g[XPW][8]) {
 #pragma unroll
-        for (int q = 0; q < 2; ++q)
+        for (int q = 0; q < XPW; ++q)
 #pragma unroll
             for (int i = 0; i < 8; ++i)
 #pragma unroll
@@ -238,7 +246,8 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
     auto gemm_stage = [&](int slot, int vbuf, bool do_itf, int itf_slot, int itf_vbuf) {
         const float* us = smem + slot * STAGE_FLOATS + xi0 * BK + fo;
         const float* v = vs + vbuf * VS_FLOATS + xi0 * BC * BN + io;
-        float fa[2][8], ga[2][8], fb[2][8], gb[2][8], d[16];
+        float fa[XPW][8], ga[XPW][8], fb[XPW][8], gb[XPW][8], d[16];
+        do_itf = do_itf && (tid < BC * BN);  // warp-uniform: one (c, nu) tile per thread
         load_frag(us, v, 0, fa, ga);
         if (do_itf) itf_load(itf_slot, d);
 #pragma unroll
@@ -261,7 +270,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
     cp_async_wait<S - 2>();
     wait_tma(0);
     __syncthreads();
-    {
+    if (tid < BC * BN) {
         float d[16];
         itf_load(0, d);
         itf_store(0, d);
@@ -284,7 +293,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
     // chosen for bank-conflict-free FFMAs; the reader undoes it.
     float* ep = smem;
 #pragma unroll
-    for (int q = 0; q < 2; ++q)
+    for (int q = 0; q < XPW; ++q)
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
             const int kl = fo + (i & 3) + (i >> 2) * 32;
@@ -305,8 +314,8 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_kernel(const __grid_constant
         const size_t base = ((size_t)i0 * p.W + j0) * p.N + n;
         const size_t dW = (size_t)p.W * p.N;
 #pragma unroll 2
-        for (int r = 0; r < BK / 8; ++r) {
-            const int kl = warp + 8 * r, k = k0 + kl;
+        for (int r = 0; r < BK / NWARP; ++r) {
+            const int kl = warp + NWARP * r, k = k0 + kl;
             if (k >= p.K) break;
             float m[16], o[4];
 #pragma unroll

@@ -21,7 +21,11 @@ namespace {
 thread_local int g_last_cuda_error = 0;
 
 constexpr int kMaxDevices = 64;
-constexpr int kStages = 3;  // cp.async ring depth of the FP32 kernel
+constexpr int kStages = 3;  // smem ring depth of the FP32 kernel
+#ifndef WINO_XPW
+#define WINO_XPW 2
+#endif
+constexpr int kXpw = WINO_XPW;  // Winograd elements per warp (2: 256 threads, 1: 512 threads)
 
 wino_status_t cuda_fail(cudaError_t e) {
     g_last_cuda_error = static_cast<int>(e);
@@ -139,10 +143,10 @@ std::atomic<uint64_t> g_attr_fp32[3][3];
 
 template <int XM, int UM>
 wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem, int dev, cudaStream_t st) {
-    auto kern = wino::fp32::fused_fp32_kernel<XM, UM, kStages>;
+    auto kern = wino::fp32::fused_fp32_kernel<XM, UM, kStages, kXpw>;
     wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_fp32[XM][UM]);
     if (s != WINO_OK) return s;
-    kern<<<dim3(static_cast<unsigned>(ctas)), wino::fp32::NT, smem, st>>>(prm);
+    kern<<<dim3(static_cast<unsigned>(ctas)), wino::fp32::threads_for<kXpw>(), smem, st>>>(prm);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
@@ -202,7 +206,7 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
     plan->load_u = p.load_u;
     plan->split_c = 1;
     plan->ctas = p.ctas;
-    plan->threads = wino::fp32::NT;
+    plan->threads = wino::fp32::threads_for<kXpw>();
     plan->smem_bytes = p.smem;
     plan->launches = 1;
     return WINO_OK;
