@@ -279,15 +279,29 @@ def main():
     for d in per:
         if d["n"] > 0:
             c = d["cfg"]
-            launches_per_step += 1 + wino.plan(d["n"], c.C, c.H, c.W, c.K).launches
+            vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[args.variant]
+            launches_per_step += 1 + wino.plan(d["n"], c.C, c.H, c.W, c.K, variant=vid).launches
+
+    tc = args.variant != "fp32"
+    if tc:  # tensor-core operand layout of the transformed filter, same broadcast-once scheme
+        for d in per:
+            d["u"] = wino.filter_transform_tc(d["w"], args.variant)
+            if world > 1:
+                dist.broadcast(d["u"].data, src=0)
 
     def run_layer(d, ftf=True, conv=True):
         if d["n"] == 0:
             return
         if ftf:
-            wino.filter_transform(d["w"], out=d["u"])
+            if tc:
+                wino.filter_transform_tc(d["w"], args.variant, out=d["u"])
+            else:
+                wino.filter_transform(d["w"], out=d["u"])
         if conv:
-            wino.conv2d(d["x"], d["u"], out=d["y"], variant=args.variant)
+            if tc:
+                wino.conv2d_tc(d["x"], d["u"], out=d["y"])
+            else:
+                wino.conv2d(d["x"], d["u"], out=d["y"])
 
     def step():
         for d in per:

@@ -109,15 +109,24 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
                                    wino_stream_t stream);
 
 /*
- * Same computation with the Winograd-domain GEMM (Eq. 7) on the 5th-generation
- * tensor cores (tcgen05.mma kind::tf32, accumulators in TMEM).  The paper has
- * no tensor-core path ("the data layout needs a redesign", Sec. 8.3);
- * this variant is the B200 redesign named in BASELINE.json's north_star.
- * mode selects TF32 (accuracy ~5e-4 relative) or 3xTF32 (~FP32 accuracy).
- * Arguments and errors as wino_conv2d_f2x3_fwd, plus WINO_ERR_INVALID_ARG for
- * an unknown mode.
+ * Tensor-core variant (a5' of SURVEY 8(a)): the Winograd-domain GEMM (Eq. 7)
+ * on the 5th-generation tensor cores (tcgen05.mma kind::tf32, accumulators in
+ * TMEM).  The paper has no tensor-core path ("the data layout needs a
+ * redesign", Sec. 8.3); this is the B200 redesign named in
+ * BASELINE.json's north_star.  mode selects TF32 (operands rounded to TF32,
+ * ~5e-4 relative) or 3xTF32 (big*big + big*small + small*big, ~FP32 accuracy).
+ *
+ * Its filter transform writes the transformed filter straight into the tensor
+ * core's operand layout (TF32-rounded; 3xTF32 adds the residual plane):
+ *   u_tc : wino_filter_workspace_bytes_tc(C,K,mode) bytes, opaque layout
+ *          [ceil(C/8)][ceil(K/128)][16][planes][128 x 8 K-major tile], zero padded.
+ * Arguments and errors otherwise as the FP32 entry points, plus
+ * WINO_ERR_INVALID_ARG for an unknown mode.
  */
-wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_dev, float* y_dev,
+size_t wino_filter_workspace_bytes_tc(int C, int K, wino_tc_mode_t mode);
+wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int C, int K,
+                                       wino_tc_mode_t mode, wino_stream_t stream);
+wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev, float* y_dev,
                                       int N, int C, int H, int W, int K, int pad, int stride,
                                       wino_tc_mode_t mode, wino_stream_t stream);
 

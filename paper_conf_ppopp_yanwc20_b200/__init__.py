@@ -21,6 +21,7 @@ import torch
 __all__ = [
     "WinoError", "lib", "version", "filter_workspace_bytes", "filter_transform", "conv2d",
     "conv2d_host", "host_workspace_bytes", "plan", "Plan", "TC_TF32", "TC_3XTF32",
+    "TcFilter", "filter_workspace_bytes_tc", "filter_transform_tc", "conv2d_tc",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -89,6 +90,10 @@ def lib() -> ctypes.CDLL:
     L.wino_conv2d_f2x3_fwd.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
     L.wino_conv2d_f2x3_fwd_tc.restype = i
     L.wino_conv2d_f2x3_fwd_tc.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
+    L.wino_filter_workspace_bytes_tc.restype = st
+    L.wino_filter_workspace_bytes_tc.argtypes = [i, i, i]
+    L.wino_filter_transform_tc.restype = i
+    L.wino_filter_transform_tc.argtypes = [vp, vp, i, i, i, vp]
     L.wino_host_workspace_bytes.restype = st
     L.wino_host_workspace_bytes.argtypes = [i, i, i, i, i]
     L.wino_conv2d_f2x3_fwd_host.restype = i
@@ -158,12 +163,68 @@ def filter_transform(w: torch.Tensor, out: torch.Tensor | None = None, stream=No
     return out
 
 
+@dataclass
+class TcFilter:
+    """Transformed filter in the tensor-core operand layout (wino_filter_transform_tc)."""
+    data: torch.Tensor  # flat float32 CUDA tensor, wino_filter_workspace_bytes_tc bytes
+    C: int
+    K: int
+    mode: int  # TC_TF32 or TC_3XTF32
+
+
+def _tc_mode(variant) -> int:
+    if variant in ("tf32", TC_TF32):
+        return TC_TF32
+    if variant in ("3xtf32", TC_3XTF32):
+        return TC_3XTF32
+    raise ValueError(f"unknown tensor-core variant {variant!r}")
+
+
+def filter_workspace_bytes_tc(C: int, K: int, variant="tf32") -> int:
+    return int(lib().wino_filter_workspace_bytes_tc(C, K, _tc_mode(variant)))
+
+
+def filter_transform_tc(w: torch.Tensor, variant="tf32", out: TcFilter | None = None, stream=None) -> TcFilter:
+    """FTF (Eq. 5) into the tcgen05 operand layout, TF32-rounded (3xTF32: + residual plane)."""
+    _need_cuda_f32(w, "w", 4)
+    C, r, s_, K = w.shape
+    if (r, s_) != (3, 3):
+        raise ValueError(f"w must be (C,3,3,K), got {tuple(w.shape)}")
+    mode = _tc_mode(variant)
+    nbytes = filter_workspace_bytes_tc(C, K, mode)
+    if out is None:
+        out = TcFilter(torch.empty(nbytes // 4, dtype=torch.float32, device=w.device), C, K, mode)
+    if (out.C, out.K, out.mode) != (C, K, mode) or out.data.numel() * 4 < nbytes:
+        raise ValueError("out TcFilter does not match w / variant")
+    with torch.cuda.device(w.device):
+        _check(lib().wino_filter_transform_tc(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data.data_ptr()),
+                                              C, K, mode, _stream_ptr(stream)), "wino_filter_transform_tc")
+    return out
+
+
+def conv2d_tc(x: torch.Tensor, u_tc: TcFilter, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Fused Winograd conv with the Winograd-domain GEMM on tcgen05 (TF32 / 3xTF32)."""
+    _need_cuda_f32(x, "x", 4)
+    C, H, W, N = x.shape
+    if u_tc.C != C:
+        raise ValueError(f"u_tc was built for C={u_tc.C}, x has C={C}")
+    K = u_tc.K
+    if out is None:
+        out = torch.empty((K, H, W, N), dtype=torch.float32, device=x.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (K, H, W, N):
+        raise ValueError("out must be (K,H,W,N)")
+    with torch.cuda.device(x.device):
+        _check(lib().wino_conv2d_f2x3_fwd_tc(
+            ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_tc.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+            N, C, H, W, K, 1, 1, u_tc.mode, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc")
+    return out
+
+
 def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, variant: str = "fp32",
            stream=None) -> torch.Tensor:
-    """Fused Winograd forward conv, pad 1 stride 1: x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N).
-
-    variant: "fp32" (FFMA kernel), "tf32" or "3xtf32" (tcgen05 kernel).
-    """
+    """Fused Winograd forward conv on FP32 CUDA cores, pad 1 stride 1:
+    x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N)."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u, "u", 4)
     C, H, W, N = x.shape
@@ -180,13 +241,9 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
     args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(out.data_ptr()),
             N, C, H, W, K, 1, 1)
     with torch.cuda.device(x.device):
-        if variant == "fp32":
-            _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
-        elif variant in ("tf32", "3xtf32"):
-            mode = TC_TF32 if variant == "tf32" else TC_3XTF32
-            _check(lib().wino_conv2d_f2x3_fwd_tc(*args, mode, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc")
-        else:
-            raise ValueError(f"unknown variant {variant!r}")
+        if variant != "fp32":
+            raise ValueError(f"conv2d runs the FP32 kernel; use conv2d_tc for {variant!r}")
+        _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
     return out
 
 

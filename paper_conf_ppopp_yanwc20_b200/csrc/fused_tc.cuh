@@ -1,0 +1,341 @@
+// fused_tc.cuh -- fused Winograd F(2x2,3x3) with the Winograd-domain GEMM on
+// tcgen05 tensor cores (TF32 or 3xTF32), accumulators in TMEM.
+//
+// Paper: same method and steps as the FP32 kernel (Eq. 5-8;
+// Alg. 1); the paper has no tensor-core path and notes that "the data
+// layout needs a redesign" for one (Sec. 8.3).  This is that redesign.
+//
+// CTA tile: 128 filters (UMMA M) x 32 tiles*images nu (UMMA N) x all 16 xi.
+// TMEM: 16 accumulators D(xi) of 128 lanes x 32 columns = all 512 columns.
+// Per channel block cb (8 channels = one tf32 UMMA K step):
+//   * producer warp: TMA box of raw x (n:32, w:4, h:4, c:8) (zero fill = padding)
+//     and two bulk copies of the pre-arranged transformed filter (8 xi each);
+//   * 8 ITF warps: V = B^T d B (Eq. 6) for the 8 x 32 (c, nu) tiles, rounded to
+//     TF32 (3xTF32: big + small planes), stored as the K-major UMMA B operand;
+//   * MMA warp (one thread): per xi, D(xi) += U(xi) * V(xi) (3xTF32: big*big +
+//     big*small + small*big), tcgen05.commit frees the smem slots;
+//   * epilogue (8 warps): tcgen05.ld the 16 accumulators, OTF (Eq. 8), store.
+// Warp-specialised, mbarrier-synchronised; no __syncthreads in the main loop.
+#pragma once
+#include <cuda.h>
+
+#include <cstdint>
+
+#include "wino_ptx.cuh"
+#include "wino_transforms.cuh"
+
+namespace wino {
+namespace tc {
+
+constexpr int BM = 128;        // filters per CTA (UMMA M)
+constexpr int BN = 32;         // nu per CTA (UMMA N)
+constexpr int BC = 8;          // channels per block (UMMA K for tf32)
+constexpr int ITF_WARPS = 8;   // warps 0..7: ITF + epilogue
+constexpr int PROD_WARP = 8;   // TMA / bulk-copy producer
+constexpr int MMA_WARP = 9;    // tcgen05.mma issuer
+constexpr int NT = 320;
+constexpr int A_TILE = BM * BC * 4;  // one (xi, plane) A operand: 4 KB
+constexpr int B_TILE = BN * BC * 4;  // one (xi, plane) B operand: 1 KB
+constexpr int XS_BYTES = BC * 16 * BN * 4;  // raw x box: 16 KB
+constexpr int XI_PER_UNIT = 8;              // U ring unit = 8 xi of one channel block
+
+// u_tc layout (written by tc_filter_kernel, read with bulk copies):
+//   [cb = C/8][kb = K/128][xi 16][plane P][m/8 16][c/4 2][m%8 8][c%4 4]  fp32
+// i.e. per (cb, kb, xi, plane) one 4 KB K-major SWIZZLE_NONE UMMA A tile
+// (LBO = 128 B between the two 16 B K-chunks, SBO = 256 B between 8-row groups).
+__host__ __device__ inline size_t u_tc_floats(int C, int K, int planes) {
+    return size_t((C + BC - 1) / BC) * ((K + BM - 1) / BM) * 16 * planes * (BM * BC);
+}
+
+// FTF (Eq. 5) straight into the tensor-core operand layout, rounded to TF32
+// (reading R8; 3xTF32 also stores small = rna(u - big)).  Pads K and C with zeros.
+template <int P>
+__global__ void __launch_bounds__(256) tc_filter_kernel(const float* __restrict__ w, float* __restrict__ u_tc,
+                                                        int C, int K) {
+    const int Kp = ((K + BM - 1) / BM) * BM, Cp = ((C + BC - 1) / BC) * BC;
+    const long idx = (long)blockIdx.x * 256 + threadIdx.x;
+    if (idx >= (long)Cp * Kp) return;
+    const int c = (int)(idx / Kp), k = (int)(idx - (long)c * Kp);
+    float g[9], t[16];
+    if (c < C && k < K) {
+        const float* wc = w + (size_t)c * 9 * K + k;
+#pragma unroll
+        for (int e = 0; e < 9; ++e) g[e] = __ldg(wc + (size_t)e * K);
+        ftf_4x4(g, t);
+    } else {
+#pragma unroll
+        for (int e = 0; e < 16; ++e) t[e] = 0.f;
+    }
+    const int cb = c / BC, cl = c % BC, kb = k / BM, m = k % BM;
+    const int nkb = Kp / BM;
+    const size_t inner = size_t((m >> 3) * 64 + (cl >> 2) * 32 + (m & 7) * 4 + (cl & 3));
+#pragma unroll
+    for (int xi = 0; xi < 16; ++xi) {
+        const size_t base = ((((size_t)cb * nkb + kb) * 16 + xi) * P) * (BM * BC);
+        const float big = to_tf32(t[xi]);
+        u_tc[base + inner] = big;
+        if (P == 2) u_tc[base + (BM * BC) + inner] = to_tf32(t[xi] - big);
+    }
+}
+
+struct __align__(64) Params {
+    CUtensorMap tmx;  // x (C,H,W,N) as (N, W, H, C), box (32, 4, 4, 8)   [TMA x path]
+    const float* __restrict__ x;
+    const float* __restrict__ u_tc;
+    float* __restrict__ y;
+    int N, C, H, W, K;
+    int TW, NV;
+    int num_kb;  // ceil(K/128)
+    int num_cb;  // ceil(C/8)
+};
+
+template <int P>
+struct Cfg {
+    static constexpr int UNIT = XI_PER_UNIT * P * A_TILE;       // 32 KB (tf32) / 64 KB (3x)
+    static constexpr int U_SLOTS = (P == 1) ? 4 : 2;           // 128 KB of U ring either way
+    static constexpr int V_SLOT = 16 * P * B_TILE;             // 16 / 32 KB
+    static constexpr int OFF_U = 0;
+    static constexpr int OFF_X = OFF_U + U_SLOTS * UNIT;
+    static constexpr int OFF_V = OFF_X + 2 * XS_BYTES;
+    static constexpr int OFF_TAB = OFF_V + 2 * V_SLOT;          // cp.async gather table (16*32 ints)
+    static constexpr int OFF_BAR = OFF_TAB + 16 * BN * 4;
+    // barriers: u_full[U_SLOTS], u_empty[U_SLOTS], x_full[2], x_empty[2], v_full[2], v_empty[2], acc
+    static constexpr int NBAR = 2 * U_SLOTS + 9;
+    static constexpr int OFF_TMEM = OFF_BAR + NBAR * 8;
+    static constexpr int BYTES = OFF_TMEM + 16;
+};
+
+// XM: 2 = TMA x box (N % 32 == 0), 1 = cp.async 16 B gather, 0 = cp.async 4 B gather
+template <int P, int XM>
+__global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__ Params p) {
+    using G = Cfg<P>;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t* const su = smem + G::OFF_U;
+    float* const sx = reinterpret_cast<float*>(smem + G::OFF_X);
+    uint8_t* const sv = smem + G::OFF_V;
+    int* const xtab = reinterpret_cast<int*>(smem + G::OFF_TAB);
+    uint64_t* const bars = reinterpret_cast<uint64_t*>(smem + G::OFF_BAR);
+    uint64_t* const u_full = bars;
+    uint64_t* const u_empty = bars + G::U_SLOTS;
+    uint64_t* const x_full = bars + 2 * G::U_SLOTS;
+    uint64_t* const x_empty = x_full + 2;
+    uint64_t* const v_full = x_full + 4;
+    uint64_t* const v_empty = x_full + 6;
+    uint64_t* const acc_full = x_full + 8;
+    uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + G::OFF_TMEM);
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int kb = blockIdx.x % p.num_kb;
+    const int nb = blockIdx.x / p.num_kb;
+    const int k0 = kb * BM, nu0 = nb * BN;
+    const int NCB = p.num_cb;
+
+    if (tid == 0) {
+        for (int s = 0; s < G::U_SLOTS; ++s) {
+            mbar_init(&u_full[s], 1);
+            mbar_init(&u_empty[s], 1);
+        }
+        for (int s = 0; s < 2; ++s) {
+            mbar_init(&x_full[s], 1);
+            mbar_init(&x_empty[s], ITF_WARPS);
+            mbar_init(&v_full[s], ITF_WARPS);
+            mbar_init(&v_empty[s], 1);
+        }
+        mbar_init(acc_full, 1);
+        fence_mbar_init();
+        if constexpr (XM == 2) tma_prefetch_desc(&p.tmx);
+    }
+    if constexpr (XM != 2) {
+        for (int e = tid; e < 16 * BN; e += NT) {
+            const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
+            int off = -1;
+            if (nu < p.NV) {
+                const int t = nu / p.N, n = nu - t * p.N;
+                const int th = t / p.TW, tw = t - th * p.TW;
+                const int h = 2 * th - 1 + (pos >> 2), w = 2 * tw - 1 + (pos & 3);
+                if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
+            }
+            xtab[e] = off;
+        }
+    }
+    if (warp == 0) tmem_alloc(tmem_slot, 512);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == PROD_WARP) {
+        // ------------------------------ producer ------------------------------
+        int tma_n0 = 0, tma_w0 = 0, tma_h0 = 0;
+        if constexpr (XM == 2) {
+            const int t = nu0 / p.N;
+            tma_n0 = nu0 - t * p.N;
+            const int th = t / p.TW, tw = t - th * p.TW;
+            tma_w0 = 2 * tw - 1;
+            tma_h0 = 2 * th - 1;
+        }
+        const size_t HWN = (size_t)p.H * p.W * p.N;
+        int unit = 0;
+        for (int cb = 0; cb < NCB; ++cb) {
+            const int xs = cb & 1;
+            if (cb >= 2) mbar_wait(&x_empty[xs], ((cb >> 1) - 1) & 1);
+            float* xdst = sx + xs * (XS_BYTES / 4);
+            if constexpr (XM == 2) {
+                if (lane == 0) {
+                    mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
+                    tma_load_4d(xdst, &p.tmx, &x_full[xs], tma_n0, tma_w0, tma_h0, cb * BC);
+                }
+            } else {
+                constexpr int VX = XM == 1 ? 4 : 1;
+                for (int e = lane; e < BC * 16 * BN / VX; e += 32) {
+                    const int cl = e / (16 * BN / VX), r = (e % (16 * BN / VX)) * VX;
+                    const int c = cb * BC + cl;
+                    const int off = xtab[r];
+                    const bool ok = (c < p.C) && (off >= 0);
+                    const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
+                    const uint32_t dst = smem_u32(xdst + cl * 16 * BN + r);
+                    if constexpr (VX == 4) cp_async16(dst, src, ok);
+                    else cp_async4(dst, src, ok);
+                }
+                cp_async_wait_all();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&x_full[xs]);
+            }
+            for (int half = 0; half < 2; ++half, ++unit) {
+                const int us = unit % G::U_SLOTS;
+                if (unit >= G::U_SLOTS) mbar_wait(&u_empty[us], ((unit / G::U_SLOTS) - 1) & 1);
+                if (lane == 0) {
+                    const float* src = p.u_tc + ((((size_t)cb * p.num_kb + kb) * 16 + half * XI_PER_UNIT) * P) *
+                                                    (BM * BC);
+                    mbar_arrive_expect_tx(&u_full[us], G::UNIT);
+                    bulk_load(su + us * G::UNIT, src, G::UNIT, &u_full[us]);
+                }
+            }
+        }
+    } else if (warp == MMA_WARP) {
+        // ------------------------------ MMA issuer ----------------------------
+        constexpr uint32_t IDESC = umma_idesc_tf32(BM, BN);
+        int unit = 0;
+        for (int cb = 0; cb < NCB; ++cb) {
+            const int vs = cb & 1;
+            mbar_wait(&v_full[vs], (cb >> 1) & 1);
+            for (int half = 0; half < 2; ++half, ++unit) {
+                const int us = unit % G::U_SLOTS;
+                mbar_wait(&u_full[us], (unit / G::U_SLOTS) & 1);
+                tc_fence_after();
+                if (lane == 0) {
+                    const uint32_t ubase = smem_u32(su + us * G::UNIT);
+                    const uint32_t vbase = smem_u32(sv + vs * G::V_SLOT);
+#pragma unroll
+                    for (int q = 0; q < XI_PER_UNIT; ++q) {
+                        const int xi = half * XI_PER_UNIT + q;
+                        const uint32_t d = tmem + xi * BN;
+                        const uint32_t a0 = ubase + (q * P) * A_TILE, b0 = vbase + (xi * P) * B_TILE;
+                        const uint64_t ab = umma_desc(a0, 128, 256), bb = umma_desc(b0, 128, 256);
+                        umma_tf32(d, ab, bb, IDESC, cb > 0 ? 1u : 0u);
+                        if constexpr (P == 2) {
+                            const uint64_t as = umma_desc(a0 + A_TILE, 128, 256);
+                            const uint64_t bs = umma_desc(b0 + B_TILE, 128, 256);
+                            umma_tf32(d, ab, bs, IDESC, 1u);
+                            umma_tf32(d, as, bb, IDESC, 1u);
+                        }
+                    }
+                    umma_commit(&u_empty[us]);
+                    if (half == 1) umma_commit(&v_empty[vs]);
+                }
+                __syncwarp();
+            }
+        }
+        if (lane == 0) umma_commit(acc_full);
+        __syncwarp();
+    } else {
+        // ------------------------------ ITF warps -----------------------------
+        // thread -> (c, nu) with lanes over (nu%8, c%4): conflict-free K-major stores
+        const int nl = (warp & 3) * 8 + (lane >> 2);
+        const int cl = (warp >> 2) * 4 + (lane & 3);
+        const uint32_t voff = (nl >> 3) * 256 + (cl >> 2) * 128 + (nl & 7) * 16 + (cl & 3) * 4;
+        for (int cb = 0; cb < NCB; ++cb) {
+            const int xs = cb & 1, vs = cb & 1;
+            mbar_wait(&x_full[xs], (cb >> 1) & 1);
+            if (cb >= 2) mbar_wait(&v_empty[vs], ((cb >> 1) - 1) & 1);
+            const float* xsrc = sx + xs * (XS_BYTES / 4) + cl * 16 * BN + nl;
+            float d[16], t[16];
+#pragma unroll
+            for (int e = 0; e < 16; ++e) d[e] = xsrc[e * BN];
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&x_empty[xs]);
+            itf_4x4(d, t);
+            uint8_t* vdst = sv + vs * G::V_SLOT + voff;
+#pragma unroll
+            for (int xi = 0; xi < 16; ++xi) {
+                const float big = to_tf32(t[xi]);
+                *reinterpret_cast<float*>(vdst + (xi * P) * B_TILE) = big;
+                if constexpr (P == 2) *reinterpret_cast<float*>(vdst + (xi * P + 1) * B_TILE) = to_tf32(t[xi] - big);
+            }
+            fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&v_full[vs]);
+        }
+
+        // ------------------------------ epilogue ------------------------------
+        mbar_wait(acc_full, 0);
+        tc_fence_after();
+        const int kl = (warp & 3) * 32 + lane;  // TMEM lane = filter within the tile
+        const int k = k0 + kl;
+        const uint32_t trow = tmem + ((uint32_t)((warp & 3) * 32) << 16);
+        const size_t HWN = (size_t)p.H * p.W * p.N;
+        const size_t dW = (size_t)p.W * p.N;
+        for (int ch = 0; ch < 2; ++ch) {
+            const int nb0 = (warp >> 2) * 16 + ch * 8;  // 8 nu per chunk
+            float m[16][8];
+#pragma unroll
+            for (int xi = 0; xi < 16; ++xi) tmem_ld8(trow + xi * BN + nb0, m[xi]);
+            tmem_ld_wait();
+            if (k >= p.K) continue;
+            float o[8][4];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                float mm[16];
+#pragma unroll
+                for (int xi = 0; xi < 16; ++xi) mm[xi] = m[xi][j];
+                otf_2x2(mm, o[j]);
+            }
+            const int nu_first = nu0 + nb0;
+            if constexpr (XM == 2) {
+                // N % 32 == 0: the 8 nu are 8 consecutive n of one tile -> 2 x float4 per output pixel
+                const int t = nu_first / p.N, n = nu_first - t * p.N;
+                const int th = t / p.TW, tw = t - th * p.TW;
+                const int i0 = 2 * th, j0 = 2 * tw;
+                float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int a = q >> 1, b = q & 1;
+                    if (i0 + a >= p.H || j0 + b >= p.W) continue;  // odd H/W (L1155)
+                    float* dst = yk + a * dW + b * p.N;
+                    *reinterpret_cast<float4*>(dst) = make_float4(o[0][q], o[1][q], o[2][q], o[3][q]);
+                    *reinterpret_cast<float4*>(dst + 4) = make_float4(o[4][q], o[5][q], o[6][q], o[7][q]);
+                }
+            } else {
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    const int nu = nu_first + j;
+                    if (nu >= p.NV) break;
+                    const int t = nu / p.N, n = nu - t * p.N;
+                    const int th = t / p.TW, tw = t - th * p.TW;
+                    const int i0 = 2 * th, j0 = 2 * tw;
+                    float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+                    yk[0] = o[j][0];
+                    if (j0 + 1 < p.W) yk[p.N] = o[j][1];
+                    if (i0 + 1 < p.H) yk[dW] = o[j][2];
+                    if (i0 + 1 < p.H && j0 + 1 < p.W) yk[dW + p.N] = o[j][3];
+                }
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) tmem_dealloc(tmem, 512);
+}
+
+}  // namespace tc
+}  // namespace wino

@@ -15,6 +15,7 @@
 #include "../../include/wino.h"
 #include "ftf.cuh"
 #include "fused_fp32.cuh"
+#include "fused_tc.cuh"
 
 namespace {
 
@@ -153,6 +154,20 @@ wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem,
 
 }  // namespace
 
+namespace {
+std::atomic<uint64_t> g_attr_tc[2][3];
+template <int P, int XM>
+wino_status_t launch_tc(const wino::tc::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
+    auto kern = wino::tc::fused_tc_kernel<P, XM>;
+    const int smem = wino::tc::Cfg<P>::BYTES;
+    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc[P - 1][XM]);
+    if (s != WINO_OK) return s;
+    kern<<<dim3(static_cast<unsigned>(ctas)), wino::tc::NT, smem, st>>>(prm);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+}  // namespace
+
 extern "C" {
 
 int wino_version(void) { return 100; }  // 0.1.0
@@ -196,6 +211,22 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
     wino_status_t s = check_shape(N, C, H, W, K, 1, 1);
     if (s != WINO_OK) return s;
     std::memset(plan, 0, sizeof(*plan));
+    if (variant == 1 || variant == 2) {  // tcgen05 TF32 (1) / 3xTF32 (2)
+        using namespace wino::tc;
+        const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
+        plan->variant = variant;
+        plan->bk = BM;
+        plan->bn = BN;
+        plan->bc = BC;
+        plan->load_x = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
+        plan->load_u = 3;  // bulk copy of the pre-arranged operand tiles
+        plan->split_c = 1;
+        plan->ctas = ((nv + BN - 1) / BN) * ((K + BM - 1) / BM);
+        plan->threads = NT;
+        plan->smem_bytes = variant == 1 ? Cfg<1>::BYTES : Cfg<2>::BYTES;
+        plan->launches = 1;
+        return WINO_OK;
+    }
     if (variant != 0) return WINO_ERR_UNSUPPORTED;
     Fp32Plan p = plan_fp32(N, C, H, W, K);
     plan->variant = 0;
@@ -264,15 +295,79 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
     }
 }
 
-wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H,
+size_t wino_filter_workspace_bytes_tc(int C, int K, wino_tc_mode_t mode) {
+    if (C <= 0 || K <= 0 || (mode != WINO_TC_TF32 && mode != WINO_TC_3XTF32)) return 0;
+    return wino::tc::u_tc_floats(C, K, mode == WINO_TC_3XTF32 ? 2 : 1) * sizeof(float);
+}
+
+wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int C, int K, wino_tc_mode_t mode,
+                                       wino_stream_t stream) {
+    if (!w_dev || !u_tc_dev || C <= 0 || K <= 0) return WINO_ERR_INVALID_ARG;
+    if (mode != WINO_TC_TF32 && mode != WINO_TC_3XTF32) return WINO_ERR_INVALID_ARG;
+    const size_t ub = wino_filter_workspace_bytes_tc(C, K, mode);
+    if (ub / 4 > size_t(kMaxElems)) return WINO_ERR_TOO_LARGE;
+    if (!aligned16(w_dev) || !aligned16(u_tc_dev)) return WINO_ERR_MISALIGNED;
+    if (overlaps(w_dev, size_t(9) * C * K * 4, u_tc_dev, ub)) return WINO_ERR_INVALID_ARG;
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    const int64_t Kp = ((K + wino::tc::BM - 1) / wino::tc::BM) * wino::tc::BM;
+    const int64_t Cp = ((C + wino::tc::BC - 1) / wino::tc::BC) * wino::tc::BC;
+    const unsigned blocks = static_cast<unsigned>((Cp * Kp + 255) / 256);
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (mode == WINO_TC_TF32) wino::tc::tc_filter_kernel<1><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
+    else wino::tc::tc_filter_kernel<2><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
+
+wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, int N, int C, int H,
                                       int W, int K, int pad, int stride, wino_tc_mode_t mode,
                                       wino_stream_t stream) {
-    if (!x_dev || !u_dev || !y_dev) return WINO_ERR_INVALID_ARG;
+    if (!x_dev || !u_tc_dev || !y_dev) return WINO_ERR_INVALID_ARG;
     if (mode != WINO_TC_TF32 && mode != WINO_TC_3XTF32) return WINO_ERR_INVALID_ARG;
     wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
     if (s != WINO_OK) return s;
-    (void)stream;
-    return WINO_ERR_UNSUPPORTED;  // tcgen05 variant not built yet
+    if (!aligned16(x_dev) || !aligned16(u_tc_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t yb = size_t(K) * hwn * 4;
+    if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) ||
+        overlaps(y_dev, yb, u_tc_dev, wino_filter_workspace_bytes_tc(C, K, mode)))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    using namespace wino::tc;
+    Params prm;
+    std::memset(&prm, 0, sizeof(prm));
+    prm.x = x_dev;
+    prm.u_tc = u_tc_dev;
+    prm.y = y_dev;
+    prm.N = N;
+    prm.C = C;
+    prm.H = H;
+    prm.W = W;
+    prm.K = K;
+    prm.TW = (W + 1) / 2;
+    prm.NV = N * ((H + 1) / 2) * prm.TW;
+    prm.num_kb = (K + BM - 1) / BM;
+    prm.num_cb = (C + BC - 1) / BC;
+    const int xm = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
+    if (xm == 2) {
+        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
+        const cuuint32_t box[4] = {BN, 4, 4, BC};
+        if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    const int64_t ctas = int64_t((prm.NV + BN - 1) / BN) * prm.num_kb;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (mode == WINO_TC_TF32) {
+        if (xm == 2) return launch_tc<1, 2>(prm, ctas, dev, st);
+        if (xm == 1) return launch_tc<1, 1>(prm, ctas, dev, st);
+        return launch_tc<1, 0>(prm, ctas, dev, st);
+    }
+    if (xm == 2) return launch_tc<2, 2>(prm, ctas, dev, st);
+    if (xm == 1) return launch_tc<2, 1>(prm, ctas, dev, st);
+    return launch_tc<2, 0>(prm, ctas, dev, st);
 }
 
 static size_t round_up256(size_t b) { return (b + 255) & ~size_t(255); }

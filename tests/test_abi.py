@@ -103,6 +103,23 @@ def test_fwd_argument_validation_host_side():
     assert L.wino_filter_transform(ctypes.c_void_p(X + 4), ctypes.c_void_p(U), 3, 5, None) == 3
     assert L.wino_conv2d_f2x3_fwd_tc(ctypes.c_void_p(X), ctypes.c_void_p(U), ctypes.c_void_p(Y),
                                      2, 3, 4, 4, 5, 1, 1, 7, None) == 1  # unknown mode
+    assert L.wino_filter_transform_tc(ctypes.c_void_p(X), ctypes.c_void_p(U), 3, 5, 7, None) == 1
+    assert L.wino_conv2d_f2x3_fwd_tc(ctypes.c_void_p(X), ctypes.c_void_p(U), ctypes.c_void_p(Y),
+                                     2, 3, 4, 4, 5, 2, 1, 0, None) == 2  # pad != 1
+
+
+def test_tc_workspace_and_plan():
+    # [ceil(C/8)][ceil(K/128)][16 xi][planes][128 x 8] floats
+    for (C, K) in [(1, 1), (8, 128), (9, 129), (512, 512), (64, 64)]:
+        for mode, planes in [("tf32", 1), ("3xtf32", 2)]:
+            want = -(-C // 8) * -(-K // 128) * 16 * planes * 128 * 8 * 4
+            assert wino.filter_workspace_bytes_tc(C, K, mode) == want
+    assert wino.lib().wino_filter_workspace_bytes_tc(8, 8, 5) == 0
+    c = CONFIGS["conv3_x"]
+    p = wino.plan(c.N, c.C, c.H, c.W, c.K, variant=1)
+    assert (p.bk, p.bn, p.bc, p.threads) == (128, 32, 8, 320)
+    assert p.ctas == -(-(c.N * c.tiles) // 32) * -(-c.K // 128)
+    assert p.smem_bytes <= 232448 and wino.plan(c.N, c.C, c.H, c.W, c.K, variant=2).smem_bytes <= 232448
 
 
 def test_python_layer_refuses_cpu_tensors():

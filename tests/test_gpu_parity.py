@@ -158,3 +158,52 @@ def test_device_side_errors(wino):
     with pytest.raises(wino.WinoError) as e:
         wino.conv2d(torch.zeros(3, 4, 4, 4, device=DEV), u2, out=y_alias)
     assert e.value.status == 1  # WINO_ERR_INVALID_ARG (aliasing)
+
+
+# ---------------------------------------------------------------------------
+# tcgen05 variant (a5'): TF32 <= 5e-3, 3xTF32 <= 1e-4 (BASELINE / SURVEY 8(c))
+# ---------------------------------------------------------------------------
+TC_TOL = {"tf32": 5e-3, "3xtf32": 1e-4}
+
+
+def _run_tc(wino, x, w, variant):
+    u = wino.filter_transform_tc(w.to(DEV), variant)
+    y = wino.conv2d_tc(x.to(DEV), u)
+    torch.cuda.synchronize()
+    return y.cpu()
+
+
+@pytest.mark.parametrize("variant", ["tf32", "3xtf32"])
+@pytest.mark.parametrize("shape", EDGE, ids=[str(s) for s in EDGE])
+def test_tc_edge_shapes_random(wino, shape, variant):
+    N, C, K, H, W = shape
+    cfg = Conv3x3Config("edge", N, C, K, H, W)
+    x, w = make_inputs(cfg, kind="uniform", seed_x=11, seed_w=12)
+    y = _run_tc(wino, x, w, variant)
+    assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= TC_TOL[variant]
+
+
+@pytest.mark.parametrize("variant", ["tf32", "3xtf32"])
+@pytest.mark.parametrize("shape", EDGE[:8], ids=[str(s) for s in EDGE[:8]])
+def test_tc_edge_shapes_small_int(wino, shape, variant):
+    """Small integers are exact in TF32 (|V| <= 12, 4|U| <= 27), so the tensor-core
+    path must reproduce the definition exactly if it accumulates in >= FP32."""
+    N, C, K, H, W = shape
+    cfg = Conv3x3Config("edge", N, C, K, H, W)
+    x, w = make_inputs(cfg, kind="smallint")
+    y = _run_tc(wino, x, w, variant)
+    assert np.array_equal(y.double().numpy(), oracle.direct_conv(x, w))
+
+
+@pytest.mark.parametrize("variant", ["tf32", "3xtf32"])
+@pytest.mark.parametrize("name", ["tiny", "conv5_x", "conv4_x", "conv3_x", "conv2_x"])
+def test_tc_full_configs_sampled(wino, name, variant):
+    cfg = CONFIGS[name]
+    x, w = make_inputs(cfg, kind="uniform")
+    y = _run_tc(wino, x, w, variant)
+    idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 4000 if name != "tiny" else 200)
+    ref = oracle.direct_sample(x, w, idx)
+    ii = idx.numpy()
+    got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
+    assert np.isfinite(y.numpy()).all()
+    assert float(np.max(np.abs(got - ref))) / float(np.max(np.abs(ref))) <= TC_TOL[variant]
