@@ -8,14 +8,16 @@
 // CTA tile: 128 filters (UMMA M) x 32 tiles*images nu (UMMA N) x all 16 xi.
 // TMEM: 16 accumulators D(xi) of 128 lanes x 32 columns = all 512 columns.
 // Per channel block cb (8 channels = one tf32 UMMA K step):
-//   * producer warp: TMA box of raw x (n:32, w:4, h:4, c:8) (zero fill = padding)
-//     and two bulk copies of the pre-arranged transformed filter (8 xi each);
+//   * x producer warp: TMA box of raw x (n:32, w:4, h:4, c:8) (zero fill = padding);
+//   * U producer warp: 64 KB bulk copies of the pre-arranged transformed filter
+//     into a ring decoupled from x;
 //   * 8 ITF warps: V = B^T d B (Eq. 6) for the 8 x 32 (c, nu) tiles, rounded to
 //     TF32 (3xTF32: big + small planes), stored as the K-major UMMA B operand;
 //   * MMA warp (one thread): per xi, D(xi) += U(xi) * V(xi) (3xTF32: big*big +
 //     big*small + small*big), tcgen05.commit frees the smem slots;
 //   * epilogue (8 warps): tcgen05.ld the 16 accumulators, OTF (Eq. 8), store.
-// Warp-specialised, mbarrier-synchronised; no __syncthreads in the main loop.
+// Warp-specialised (separate producers for x and U so neither ring stalls the
+// other), mbarrier-synchronised; no __syncthreads in the main loop.
 #pragma once
 #include <cuda.h>
 
@@ -27,17 +29,39 @@
 namespace wino {
 namespace tc {
 
+#ifdef WINO_TC_TRACE
+// Debug-only event trace (CTA 0): [event][cb] = clock64 at the event.
+constexpr int TRACE_EVENTS = 8, TRACE_CB = 128;
+__device__ unsigned long long g_trace[TRACE_EVENTS * TRACE_CB];
+#define TC_TRACE(ev, cb)                                                                         \
+    do {                                                                                         \
+        if (blockIdx.x == 0 && (cb) < TRACE_CB) g_trace[(ev) * TRACE_CB + (cb)] = clock64();    \
+    } while (0)
+#else
+#define TC_TRACE(ev, cb) \
+    do {                 \
+    } while (0)
+#endif
+
 constexpr int BM = 128;        // filters per CTA (UMMA M)
 constexpr int BN = 32;         // nu per CTA (UMMA N)
 constexpr int BC = 8;          // channels per block (UMMA K for tf32)
 constexpr int ITF_WARPS = 8;   // warps 0..7: ITF + epilogue
-constexpr int PROD_WARP = 8;   // TMA / bulk-copy producer
+constexpr int PROD_WARP = 8;   // bulk-copy producer of the transformed filter U
 constexpr int MMA_WARP = 9;    // tcgen05.mma issuer
-constexpr int NT = 320;
+constexpr int XPROD_WARP = 10; // TMA / cp.async producer of raw x (decoupled from U)
+constexpr int NT = 352;
 constexpr int A_TILE = BM * BC * 4;  // one (xi, plane) A operand: 4 KB
 constexpr int B_TILE = BN * BC * 4;  // one (xi, plane) B operand: 1 KB
 constexpr int XS_BYTES = BC * 16 * BN * 4;  // raw x box: 16 KB
-constexpr int XI_PER_UNIT = 8;              // U ring unit = 8 xi of one channel block
+constexpr int X_PREFETCH = 6;               // channel blocks of x prefetched into L2 ahead
+// U ring unit: 64 KB = all 16 xi (TF32) or 8 xi x 2 planes (3xTF32) of one channel
+// block.  A bulk copy occupies the SM's copy engine for ~360 cycles whatever its
+// size up to 32 KB (scripts/microbench/bulk_bw.cu: 11 / 23 / 45 / 90 B/clk/SM for
+// 4 / 8 / 16 / 32 KB copies, ~110 B/clk for 64 KB), so the ring uses the largest
+// copies that still leave two slots in flight.
+template <int P>
+constexpr int xi_per_unit() { return P == 1 ? 16 : 8; }
 
 // u_tc layout (written by tc_filter_kernel, read with bulk copies):
 //   [cb = C/8][kb = K/128][xi 16][plane P][m/8 16][c/4 2][m%8 8][c%4 4]  fp32
@@ -91,16 +115,19 @@ struct __align__(64) Params {
 
 template <int P>
 struct Cfg {
-    static constexpr int UNIT = XI_PER_UNIT * P * A_TILE;       // 32 KB (tf32) / 64 KB (3x)
-    static constexpr int U_SLOTS = (P == 1) ? 4 : 2;           // 128 KB of U ring either way
+    static constexpr int XPU = xi_per_unit<P>();
+    static constexpr int UNITS_PER_CB = 16 / XPU;
+    static constexpr int UNIT = XPU * P * A_TILE;               // 64 KB
+    static constexpr int U_SLOTS = 2;                           // 128 KB of U in flight
+    static constexpr int X_SLOTS = 2;                           // raw x boxes in flight (L2-prefetched)
     static constexpr int V_SLOT = 16 * P * B_TILE;             // 16 / 32 KB
     static constexpr int OFF_U = 0;
     static constexpr int OFF_X = OFF_U + U_SLOTS * UNIT;
-    static constexpr int OFF_V = OFF_X + 2 * XS_BYTES;
+    static constexpr int OFF_V = OFF_X + X_SLOTS * XS_BYTES;
     static constexpr int OFF_TAB = OFF_V + 2 * V_SLOT;          // cp.async gather table (16*32 ints)
     static constexpr int OFF_BAR = OFF_TAB + 16 * BN * 4;
-    // barriers: u_full[U_SLOTS], u_empty[U_SLOTS], x_full[2], x_empty[2], v_full[2], v_empty[2], acc
-    static constexpr int NBAR = 2 * U_SLOTS + 9;
+    // barriers: u_full/u_empty[U_SLOTS], x_full/x_empty[X_SLOTS], v_full[2], v_empty[2], acc
+    static constexpr int NBAR = 2 * U_SLOTS + 2 * X_SLOTS + 5;
     static constexpr int OFF_TMEM = OFF_BAR + NBAR * 8;
     static constexpr int BYTES = OFF_TMEM + 16;
 };
@@ -118,10 +145,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     uint64_t* const u_full = bars;
     uint64_t* const u_empty = bars + G::U_SLOTS;
     uint64_t* const x_full = bars + 2 * G::U_SLOTS;
-    uint64_t* const x_empty = x_full + 2;
-    uint64_t* const v_full = x_full + 4;
-    uint64_t* const v_empty = x_full + 6;
-    uint64_t* const acc_full = x_full + 8;
+    uint64_t* const x_empty = x_full + G::X_SLOTS;
+    uint64_t* const v_full = x_empty + G::X_SLOTS;
+    uint64_t* const v_empty = v_full + 2;
+    uint64_t* const acc_full = v_full + 4;
     uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + G::OFF_TMEM);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -135,9 +162,11 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             mbar_init(&u_full[s], 1);
             mbar_init(&u_empty[s], 1);
         }
-        for (int s = 0; s < 2; ++s) {
+        for (int s = 0; s < G::X_SLOTS; ++s) {
             mbar_init(&x_full[s], 1);
             mbar_init(&x_empty[s], ITF_WARPS);
+        }
+        for (int s = 0; s < 2; ++s) {
             mbar_init(&v_full[s], ITF_WARPS);
             mbar_init(&v_empty[s], 1);
         }
@@ -164,22 +193,33 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
 
-    if (warp == PROD_WARP) {
-        // ------------------------------ producer ------------------------------
+    if (warp == XPROD_WARP) {
+        // --------------------------- raw-x producer ---------------------------
         int tma_n0 = 0, tma_w0 = 0, tma_h0 = 0;
         if constexpr (XM == 2) {
             const int t = nu0 / p.N;
             tma_n0 = nu0 - t * p.N;
             const int th = t / p.TW, tw = t - th * p.TW;
-            tma_w0 = 2 * tw - 1;
+            tma_w0 = 2 * tw - 1;  // may be -1: TMA zero fill = implicit padding (Sec. 3.5)
             tma_h0 = 2 * th - 1;
         }
         const size_t HWN = (size_t)p.H * p.W * p.N;
-        int unit = 0;
+        // x streams from HBM (first touch); warm L2 X_PREFETCH blocks ahead so the
+        // shared-memory ring only has to cover the L2 latency
+        if constexpr (XM == 2) {
+            if (lane == 0)
+                for (int cb = 0; cb < X_PREFETCH && cb < NCB; ++cb)
+                    tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, cb * BC);
+        }
         for (int cb = 0; cb < NCB; ++cb) {
-            const int xs = cb & 1;
-            if (cb >= 2) mbar_wait(&x_empty[xs], ((cb >> 1) - 1) & 1);
+            const int xs = cb % G::X_SLOTS;
+            if constexpr (XM == 2) {
+                if (lane == 0 && cb + X_PREFETCH < NCB)
+                    tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, (cb + X_PREFETCH) * BC);
+            }
+            if (cb >= G::X_SLOTS) mbar_wait(&x_empty[xs], ((cb / G::X_SLOTS) - 1) & 1);
             float* xdst = sx + xs * (XS_BYTES / 4);
+            if (lane == 0) TC_TRACE(0, cb);
             if constexpr (XM == 2) {
                 if (lane == 0) {
                     mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
@@ -201,11 +241,17 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&x_full[xs]);
             }
-            for (int half = 0; half < 2; ++half, ++unit) {
+        }
+    } else if (warp == PROD_WARP) {
+        // ------------------------ transformed-filter producer -----------------
+        int unit = 0;
+        for (int cb = 0; cb < NCB; ++cb) {
+            for (int h = 0; h < G::UNITS_PER_CB; ++h, ++unit) {
                 const int us = unit % G::U_SLOTS;
                 if (unit >= G::U_SLOTS) mbar_wait(&u_empty[us], ((unit / G::U_SLOTS) - 1) & 1);
                 if (lane == 0) {
-                    const float* src = p.u_tc + ((((size_t)cb * p.num_kb + kb) * 16 + half * XI_PER_UNIT) * P) *
+                    if (h == 0) TC_TRACE(1, cb);
+                    const float* src = p.u_tc + ((((size_t)cb * p.num_kb + kb) * 16 + h * G::XPU) * P) *
                                                     (BM * BC);
                     mbar_arrive_expect_tx(&u_full[us], G::UNIT);
                     bulk_load(su + us * G::UNIT, src, G::UNIT, &u_full[us]);
@@ -219,7 +265,8 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         for (int cb = 0; cb < NCB; ++cb) {
             const int vs = cb & 1;
             mbar_wait(&v_full[vs], (cb >> 1) & 1);
-            for (int half = 0; half < 2; ++half, ++unit) {
+            if (lane == 0) TC_TRACE(4, cb);
+            for (int half = 0; half < G::UNITS_PER_CB; ++half, ++unit) {
                 const int us = unit % G::U_SLOTS;
                 mbar_wait(&u_full[us], (unit / G::U_SLOTS) & 1);
                 tc_fence_after();
@@ -227,8 +274,8 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                     const uint32_t ubase = smem_u32(su + us * G::UNIT);
                     const uint32_t vbase = smem_u32(sv + vs * G::V_SLOT);
 #pragma unroll
-                    for (int q = 0; q < XI_PER_UNIT; ++q) {
-                        const int xi = half * XI_PER_UNIT + q;
+                    for (int q = 0; q < G::XPU; ++q) {
+                        const int xi = half * G::XPU + q;
                         const uint32_t d = tmem + xi * BN;
                         const uint32_t a0 = ubase + (q * P) * A_TILE, b0 = vbase + (xi * P) * B_TILE;
                         const uint64_t ab = umma_desc(a0, 128, 256), bb = umma_desc(b0, 128, 256);
@@ -241,7 +288,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                         }
                     }
                     umma_commit(&u_empty[us]);
-                    if (half == 1) umma_commit(&v_empty[vs]);
+                    if (half == G::UNITS_PER_CB - 1) {
+                        umma_commit(&v_empty[vs]);
+                        TC_TRACE(5, cb);
+                    }
                 }
                 __syncwarp();
             }
@@ -255,16 +305,17 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         const int cl = (warp >> 2) * 4 + (lane & 3);
         const uint32_t voff = (nl >> 3) * 256 + (cl >> 2) * 128 + (nl & 7) * 16 + (cl & 3) * 4;
         for (int cb = 0; cb < NCB; ++cb) {
-            const int xs = cb & 1, vs = cb & 1;
-            mbar_wait(&x_full[xs], (cb >> 1) & 1);
-            if (cb >= 2) mbar_wait(&v_empty[vs], ((cb >> 1) - 1) & 1);
+            const int xs = cb % G::X_SLOTS, vs = cb & 1;
+            mbar_wait(&x_full[xs], (cb / G::X_SLOTS) & 1);
+            if (tid == 0) TC_TRACE(2, cb);
             const float* xsrc = sx + xs * (XS_BYTES / 4) + cl * 16 * BN + nl;
             float d[16], t[16];
 #pragma unroll
             for (int e = 0; e < 16; ++e) d[e] = xsrc[e * BN];
+            itf_4x4(d, t);  // consumes the loads: the x slot can be released
             __syncwarp();
             if (lane == 0) mbar_arrive(&x_empty[xs]);
-            itf_4x4(d, t);
+            if (cb >= 2) mbar_wait(&v_empty[vs], ((cb >> 1) - 1) & 1);
             uint8_t* vdst = sv + vs * G::V_SLOT + voff;
 #pragma unroll
             for (int xi = 0; xi < 16; ++xi) {
@@ -275,10 +326,12 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
             __syncwarp();
             if (lane == 0) mbar_arrive(&v_full[vs]);
+            if (tid == 0) TC_TRACE(3, cb);
         }
 
         // ------------------------------ epilogue ------------------------------
         mbar_wait(acc_full, 0);
+        if (tid == 0) TC_TRACE(6, 0);
         tc_fence_after();
         const int kl = (warp & 3) * 32 + lane;  // TMEM lane = filter within the tile
         const int k = k0 + kl;
@@ -334,6 +387,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     }
     tc_fence_before();
     __syncthreads();
+    if (tid == 0) TC_TRACE(7, 0);
     if (warp == 0) tmem_dealloc(tmem, 512);
 }
 

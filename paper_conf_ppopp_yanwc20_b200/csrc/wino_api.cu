@@ -186,6 +186,13 @@ const char* wino_status_string(wino_status_t s) {
 
 int wino_last_cuda_error(void) { return g_last_cuda_error; }
 
+#ifdef WINO_TC_TRACE
+// debug builds only: copy the tcgen05 kernel's CTA-0 event trace to the host
+int wino_debug_tc_trace(unsigned long long* host, int n) {
+    return (int)cudaMemcpyFromSymbol(host, wino::tc::g_trace, sizeof(unsigned long long) * n);
+}
+#endif
+
 size_t wino_filter_workspace_bytes(int C, int K) {
     if (C <= 0 || K <= 0) return 0;
     return size_t(16) * size_t(C) * size_t(K) * sizeof(float);

@@ -159,3 +159,13 @@ __device__ __forceinline__ float to_tf32(float x) {
 }
 
 }  // namespace wino
+
+namespace wino {
+// L2 prefetch of a TMA box (no shared-memory destination, no completion)
+__device__ __forceinline__ void tma_prefetch_l2_4d(const void* map, int c0, int c1, int c2, int c3) {
+    asm volatile("cp.async.bulk.prefetch.tensor.4d.L2.global.tile [%0, {%1, %2, %3, %4}];\n" ::"l"(
+                     reinterpret_cast<uint64_t>(map)),
+                 "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+                 : "memory");
+}
+}  // namespace wino

@@ -8,11 +8,15 @@ from collections import defaultdict
 
 path = sys.argv[1]
 top = int(sys.argv[2]) if len(sys.argv) > 2 else 25
+section = int(sys.argv[3]) if len(sys.argv) > 3 else 0  # which profiled launch
 raw = subprocess.run(["ncu", "-i", path, "--page", "source", "--csv", "--print-source", "sass"],
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(raw)))
-h = rows[1]
-data = [r for r in rows[2:] if len(r) == len(h)]
+starts = [i for i, r in enumerate(rows) if r and r[0] == "Address"]
+st = starts[min(section, len(starts) - 1)]
+end = starts[starts.index(st) + 1] - 1 if starts.index(st) + 1 < len(starts) else len(rows)
+h = rows[st]
+data = [r for r in rows[st + 1:end] if len(r) == len(h) and r[0] != "Address"]
 idx = {n: i for i, n in enumerate(h)}
 stalls = [n for n in h if n.startswith("stall_") and "Not Issued" not in n]
 T = sum(int(r[idx[s]] or 0) for r in data for s in stalls)

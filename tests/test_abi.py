@@ -117,7 +117,7 @@ def test_tc_workspace_and_plan():
     assert wino.lib().wino_filter_workspace_bytes_tc(8, 8, 5) == 0
     c = CONFIGS["conv3_x"]
     p = wino.plan(c.N, c.C, c.H, c.W, c.K, variant=1)
-    assert (p.bk, p.bn, p.bc, p.threads) == (128, 32, 8, 320)
+    assert (p.bk, p.bn, p.bc, p.threads) == (128, 32, 8, 352)
     assert p.ctas == -(-(c.N * c.tiles) // 32) * -(-c.K // 128)
     assert p.smem_bytes <= 232448 and wino.plan(c.N, c.C, c.H, c.W, c.K, variant=2).smem_bytes <= 232448
 
