@@ -55,6 +55,15 @@ def _peaks():
     return fp32_tflops, hbm, src
 
 
+def _tf32_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    bf16 = 1590.0
+    if os.path.exists(path):
+        with open(path) as f:
+            bf16 = float(json.load(f).get("bf16_tflops", bf16))
+    return 0.5 * bf16
+
+
 def _workload(name):
     if name == "resnet_3x3":
         return [CONFIGS[n] for n in ("conv5_x", "conv4_x", "conv3_x", "conv2_x")]
@@ -119,12 +128,16 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def _init_dist():
+def _init_dist(backend="nccl"):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1 and torch.cuda.is_available():
+        # one process per GPU; with --dist-backend gloo several ranks may share a GPU (tests)
+        local = local % torch.cuda.device_count()
     if world > 1 and not dist.is_initialized():
-        backend = "nccl" if torch.cuda.is_available() else "gloo"
+        if not torch.cuda.is_available():
+            backend = "gloo"
         if torch.cuda.is_available():
             torch.cuda.set_device(local)
         dist.init_process_group(backend=backend)
@@ -218,6 +231,9 @@ def main():
     ap.add_argument("--workload", default="resnet_3x3", choices=["resnet_3x3", *RESNET_LAYERS, "tiny"])
     ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32"])
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo only to exercise the multi-rank logic with several ranks on one GPU")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-baseline-s", type=float, default=3.0, help="oracle seconds per layer")
     ap.add_argument("--ref-step-s", type=float, default=4.0, help="oracle seconds per reference step")
@@ -227,7 +243,7 @@ def main():
         print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
         args.warmup = 3
 
-    rank, world, local = _init_dist()
+    rank, world, local = _init_dist(args.dist_backend)
     layers = _workload(args.workload)
 
     if args.impl == "reference":
@@ -253,13 +269,7 @@ def main():
         xs = x[..., lo:hi].contiguous()
         n_loc = hi - lo
         d = {"cfg": cfg, "n": n_loc, "x": xs.to(dev), "w": w.to(dev),
-             "u": torch.empty((cfg.C, 4, 4, cfg.K), dtype=torch.float32, device=dev),
              "y": torch.empty((cfg.K, cfg.H, cfg.W, max(n_loc, 1)), dtype=torch.float32, device=dev)}
-        # transformed filter: computed on rank 0, broadcast once over NVLink (NCCL)
-        if rank == 0:
-            wino.filter_transform(d["w"], out=d["u"])
-        if world > 1:
-            dist.broadcast(d["u"], src=0)
         if args.impl == "ours" and not args.no_e2e:
             d["x_h"] = xs.pin_memory()
             d["w_h"] = w.pin_memory()
@@ -275,106 +285,123 @@ def main():
         # back here, outside the timed events, instead of inside the first timed kernel
         flush.fill_(v)
         flush_rd.sum()
-    launches_per_step = 0
-    for d in per:
-        if d["n"] > 0:
-            c = d["cfg"]
-            vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[args.variant]
-            launches_per_step += 1 + wino.plan(d["n"], c.C, c.H, c.W, c.K, variant=vid).launches
-
-    tc = args.variant != "fp32"
-    if tc:  # tensor-core operand layout of the transformed filter, same broadcast-once scheme
-        for d in per:
-            d["u"] = wino.filter_transform_tc(d["w"], args.variant)
-            if world > 1:
-                dist.broadcast(d["u"].data, src=0)
-
-    def run_layer(d, ftf=True, conv=True):
-        if d["n"] == 0:
-            return
-        if ftf:
-            if tc:
-                wino.filter_transform_tc(d["w"], args.variant, out=d["u"])
-            else:
-                wino.filter_transform(d["w"], out=d["u"])
-        if conv:
-            if tc:
-                wino.conv2d_tc(d["x"], d["u"], out=d["y"])
-            else:
-                wino.conv2d(d["x"], d["u"], out=d["y"])
-
-    def step():
-        for d in per:
-            run_layer(d)
-
-    for _ in range(args.warmup):
-        flush_l2(1.0)
-        step()
-    torch.cuda.synchronize()
-    # The timed step is replayed from a CUDA graph (captured once, after warm-up):
-    # host launch latency stays out of the device timeline, as in a serving loop.
-    g_step = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(g_step):
-        step()
-    g_layer = []
-    for d in per:
-        gf, gc = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
-        with torch.cuda.graph(gf):
-            run_layer(d, conv=False)
-        with torch.cuda.graph(gc):
-            run_layer(d, ftf=False)
-        g_layer.append((gf, gc))
-    for _ in range(2):
-        flush_l2(2.0)
-        g_step.replay()
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-
-    sampler = ClockSampler(local) if rank == 0 else None
-    if sampler:
-        sampler.start()
-        time.sleep(0.3)
     mk = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
-    step_ev = [(mk(), mk()) for _ in range(args.steps)]
-    t_wall0 = time.perf_counter()
-    for s in range(args.steps):
-        flush_l2(float(s))
-        step_ev[s][0].record(stream)
-        g_step.replay()
-        step_ev[s][1].record(stream)
-    torch.cuda.synchronize()
-    wall = time.perf_counter() - t_wall0
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    clocks = sampler.stop() if sampler else None
-    ms_step = sum(a.elapsed_time(b) for a, b in step_ev) / args.steps
 
-    # per-layer breakdown (same graphs split per kernel, L2 flushed before each layer)
-    lay_ev = [[[mk(), mk(), mk()] for _ in per] for _ in range(args.steps)]
-    for s in range(args.steps):
-        for i, (gf, gc) in enumerate(g_layer):
-            flush_l2(float(s))
-            e0, e1, e2 = lay_ev[s][i]
-            e0.record(stream)
-            gf.replay()
-            e1.record(stream)
-            gc.replay()
-            e2.record(stream)
-    torch.cuda.synchronize()
-    ftf_ms, conv_ms = [0.0] * len(per), [0.0] * len(per)
-    for s in range(args.steps):
-        for i, d in enumerate(per):
+    def measure(variant, sample_clocks):
+        """Warm up, capture the step in a CUDA graph, time args.steps replays (L2 flushed
+        before each, outside the events), then a per-layer breakdown.  Max over ranks."""
+        tc = variant != "fp32"
+        vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[variant]
+        launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=vid).launches
+                       for d in per if d["n"] > 0)
+        for d in per:
+            # transformed filter: computed on rank 0, broadcast once over NVLink (NCCL)
+            if tc:
+                d["u"] = wino.filter_transform_tc(d["w"], variant)
+                if world > 1:
+                    dist.broadcast(d["u"].data, src=0)
+            else:
+                d["u"] = torch.empty((d["cfg"].C, 4, 4, d["cfg"].K), dtype=torch.float32, device=dev)
+                if rank == 0:
+                    wino.filter_transform(d["w"], out=d["u"])
+                if world > 1:
+                    dist.broadcast(d["u"], src=0)
+
+        def run_layer(d, ftf=True, conv=True):
             if d["n"] == 0:
-                continue
-            e0, e1, e2 = lay_ev[s][i]
-            ftf_ms[i] += e0.elapsed_time(e1) / args.steps
-            conv_ms[i] += e1.elapsed_time(e2) / args.steps
-    ms_step = _max_over_ranks(ms_step, world, dev)
-    conv_ms = [_max_over_ranks(v, world, dev) for v in conv_ms]
-    ftf_ms = [_max_over_ranks(v, world, dev) for v in ftf_ms]
+                return
+            if ftf:
+                if tc:
+                    wino.filter_transform_tc(d["w"], variant, out=d["u"])
+                else:
+                    wino.filter_transform(d["w"], out=d["u"])
+            if conv:
+                if tc:
+                    wino.conv2d_tc(d["x"], d["u"], out=d["y"])
+                else:
+                    wino.conv2d(d["x"], d["u"], out=d["y"])
+
+        def step():
+            for d in per:
+                run_layer(d)
+
+        for _ in range(args.warmup):
+            flush_l2(1.0)
+            step()
+        torch.cuda.synchronize()
+        # The timed step is replayed from a CUDA graph (captured once, after warm-up):
+        # host launch latency stays out of the device timeline, as in a serving loop.
+        g_step = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g_step):
+            step()
+        g_layer = []
+        for d in per:
+            gf, gc = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gf):
+                run_layer(d, conv=False)
+            with torch.cuda.graph(gc):
+                run_layer(d, ftf=False)
+            g_layer.append((gf, gc))
+        for _ in range(2):
+            flush_l2(2.0)
+            g_step.replay()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+        sampler = ClockSampler(local) if (rank == 0 and sample_clocks) else None
+        if sampler:
+            sampler.start()
+            time.sleep(0.3)
+        step_ev = [(mk(), mk()) for _ in range(args.steps)]
+        t_wall0 = time.perf_counter()
+        for s in range(args.steps):
+            flush_l2(float(s))
+            step_ev[s][0].record(stream)
+            g_step.replay()
+            step_ev[s][1].record(stream)
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - t_wall0
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        clocks = sampler.stop() if sampler else None
+        ms_step = sum(a.elapsed_time(b) for a, b in step_ev) / args.steps
+
+        # per-layer breakdown (same graphs split per kernel, L2 flushed before each layer)
+        lay_ev = [[[mk(), mk(), mk()] for _ in per] for _ in range(args.steps)]
+        for s in range(args.steps):
+            for i, (gf, gc) in enumerate(g_layer):
+                flush_l2(float(s))
+                e0, e1, e2 = lay_ev[s][i]
+                e0.record(stream)
+                gf.replay()
+                e1.record(stream)
+                gc.replay()
+                e2.record(stream)
+        torch.cuda.synchronize()
+        ftf_ms, conv_ms = [0.0] * len(per), [0.0] * len(per)
+        for s in range(args.steps):
+            for i, d in enumerate(per):
+                if d["n"] == 0:
+                    continue
+                e0, e1, e2 = lay_ev[s][i]
+                ftf_ms[i] += e0.elapsed_time(e1) / args.steps
+                conv_ms[i] += e1.elapsed_time(e2) / args.steps
+        return {"ms_step": _max_over_ranks(ms_step, world, dev),
+                "conv_ms": [_max_over_ranks(v, world, dev) for v in conv_ms],
+                "ftf_ms": [_max_over_ranks(v, world, dev) for v in ftf_ms],
+                "launches": launches, "wall": wall, "clocks": clocks}
+
+    main_m = measure(args.variant, sample_clocks=True)
+    others = {}
+    if not args.no_variants:
+        for v in ("fp32", "tf32", "3xtf32"):
+            if v != args.variant:
+                others[v] = measure(v, sample_clocks=False)
+    ms_step, conv_ms, ftf_ms = main_m["ms_step"], main_m["conv_ms"], main_m["ftf_ms"]
+    launches_per_step, wall, clocks = main_m["launches"], main_m["wall"], main_m["clocks"]
 
     # ---- e2e: the public C-ABI host entry point, host buffers, copies in the timed region ----
     e2e = None
@@ -453,6 +480,23 @@ def main():
     }
     if e2e:
         res["e2e"] = e2e
+    tf32_peak = _tf32_peak()
+    vrep = {}
+    for v, m in others.items():
+        val = total_eff / (m["ms_step"] * 1e-3) / 1e12
+        vrep[v] = {"value": val, "ms_per_step": m["ms_step"], "pct_fp32_peak_eff": 100 * val / fp32_peak,
+                   "layers_eff_tflops": {d["cfg"].name: d["cfg"].eff_flops / (m["conv_ms"][i] * 1e-3) / 1e12
+                                         for i, d in enumerate(per) if d["n"]},
+                   "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4}[v]}
+        if v != "fp32":
+            ach = ewmm_flops / (sum(m["conv_ms"]) * 1e-3) / 1e12
+            mult = 3 if v == "3xtf32" else 1
+            vrep[v]["roofline"] = {"bound": "tensor", "achieved": ach * mult, "peak": tf32_peak,
+                                   "unit": "TFLOP/s", "frac": ach * mult / tf32_peak,
+                                   "achieved_def": f"{mult} x EWMM flops (tcgen05 kind::tf32 work) / conv time",
+                                   "peak_def": "MEASURED_PEAKS bf16_tflops x 0.5 (nominal tf32:bf16 dense ratio)"}
+    if vrep:
+        res["variants"] = vrep
     if world == 1 and not args.no_cpu_baseline:
         import oracle
         fl, sec, sample = _oracle_sample(layers, args.cpu_baseline_s)
