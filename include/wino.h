@@ -146,6 +146,29 @@ wino_status_t wino_conv2d_f2x3_fwd_host(const float* x_host, const float* w_host
                                         void* ws_dev, size_t ws_bytes, wino_stream_t stream);
 
 /*
+ * Multi-layer end-to-end call on HOST buffers with copy/compute overlap: for
+ * each layer the weights and input are copied in on a library-owned copy-in
+ * stream, the FTF + fused FP32 convolution run on `stream`, and the output is
+ * copied back on a library-owned copy-out stream in K-slices (or batch slices
+ * when K < 128), so H2D of layer l+1, compute of layer l and D2H of layer l-1
+ * proceed concurrently over PCIe.  `stream` is joined before returning-order
+ * completion: work enqueued on `stream` after this call sees all outputs.
+ * The two helper streams are created once per device (cached, like the
+ * attribute caches); events are created and released per call.
+ *   layers[i] : host pointers and shape of layer i (pad 1, stride 1)
+ *   ws_dev    : device workspace of >= wino_host_multi_workspace_bytes() bytes
+ */
+typedef struct {
+    const float* x_host; /* (C,H,W,N) */
+    const float* w_host; /* (C,3,3,K) */
+    float* y_host;       /* (K,H,W,N) */
+    int N, C, H, W, K;
+} wino_host_layer_t;
+size_t wino_host_multi_workspace_bytes(const wino_host_layer_t* layers, int n_layers);
+wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, int n_layers, void* ws_dev,
+                                              size_t ws_bytes, wino_stream_t stream);
+
+/*
  * Launch plan the library would use for a shape (host only, needs no GPU);
  * used by tests and by bench.py to count launches and report tiling.
  */

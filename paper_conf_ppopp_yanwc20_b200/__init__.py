@@ -22,6 +22,7 @@ __all__ = [
     "WinoError", "lib", "version", "filter_workspace_bytes", "filter_transform", "conv2d",
     "conv2d_host", "host_workspace_bytes", "plan", "Plan", "TC_TF32", "TC_3XTF32",
     "TcFilter", "filter_workspace_bytes_tc", "filter_transform_tc", "conv2d_tc",
+    "host_multi_workspace_bytes", "conv2d_host_multi",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -49,6 +50,12 @@ class _Plan(ctypes.Structure):
                 ("bc", ctypes.c_int), ("load_x", ctypes.c_int), ("load_u", ctypes.c_int),
                 ("split_c", ctypes.c_int), ("ctas", ctypes.c_int64), ("threads", ctypes.c_int),
                 ("smem_bytes", ctypes.c_int), ("launches", ctypes.c_int)]
+
+
+class _HostLayer(ctypes.Structure):
+    _fields_ = [("x_host", ctypes.c_void_p), ("w_host", ctypes.c_void_p), ("y_host", ctypes.c_void_p),
+                ("N", ctypes.c_int), ("C", ctypes.c_int), ("H", ctypes.c_int), ("W", ctypes.c_int),
+                ("K", ctypes.c_int)]
 
 
 @dataclass(frozen=True)
@@ -98,6 +105,10 @@ def lib() -> ctypes.CDLL:
     L.wino_host_workspace_bytes.argtypes = [i, i, i, i, i]
     L.wino_conv2d_f2x3_fwd_host.restype = i
     L.wino_conv2d_f2x3_fwd_host.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp, st, vp]
+    L.wino_host_multi_workspace_bytes.restype = st
+    L.wino_host_multi_workspace_bytes.argtypes = [ctypes.POINTER(_HostLayer), i]
+    L.wino_conv2d_f2x3_fwd_host_multi.restype = i
+    L.wino_conv2d_f2x3_fwd_host_multi.argtypes = [ctypes.POINTER(_HostLayer), i, vp, st, vp]
     L.wino_plan.restype = i
     L.wino_plan.argtypes = [i, i, i, i, i, i, ctypes.POINTER(_Plan)]
     _lib = L
@@ -267,3 +278,34 @@ def conv2d_host(x_host: torch.Tensor, w_host: torch.Tensor, y_host: torch.Tensor
             ctypes.c_void_p(x_host.data_ptr()), ctypes.c_void_p(w_host.data_ptr()),
             ctypes.c_void_p(y_host.data_ptr()), N, C, H, W, K, 1, 1,
             ctypes.c_void_p(ws.data_ptr()), nbytes, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_host")
+
+
+def _host_layers(layers):
+    arr = (_HostLayer * len(layers))()
+    for i, (xh, wh, yh) in enumerate(layers):
+        for t, n in ((xh, "x_host"), (wh, "w_host"), (yh, "y_host")):
+            if t.is_cuda or t.dtype != torch.float32 or not t.is_contiguous() or t.dim() != 4:
+                raise ValueError(f"layer {i}: {n} must be a contiguous 4-d float32 CPU tensor")
+        C, H, W, N = xh.shape
+        K = wh.shape[3]
+        if tuple(wh.shape) != (C, 3, 3, K) or tuple(yh.shape) != (K, H, W, N):
+            raise ValueError(f"layer {i}: shape mismatch")
+        arr[i] = _HostLayer(xh.data_ptr(), wh.data_ptr(), yh.data_ptr(), N, C, H, W, K)
+    return arr
+
+
+def host_multi_workspace_bytes(layers) -> int:
+    """Device workspace for conv2d_host_multi over [(x_host, w_host, y_host), ...]."""
+    return int(lib().wino_host_multi_workspace_bytes(_host_layers(layers), len(layers)))
+
+
+def conv2d_host_multi(layers, ws: torch.Tensor, stream=None) -> None:
+    """End-to-end multi-layer call on pinned host buffers with H2D / compute / D2H overlap
+    (``wino_conv2d_f2x3_fwd_host_multi``); asynchronous on the stream."""
+    arr = _host_layers(layers)
+    if not ws.is_cuda:
+        raise ValueError("ws must be a CUDA tensor")
+    with torch.cuda.device(ws.device):
+        _check(lib().wino_conv2d_f2x3_fwd_host_multi(arr, len(layers), ctypes.c_void_p(ws.data_ptr()),
+                                                     ws.numel() * ws.element_size(), _stream_ptr(stream)),
+               "wino_conv2d_f2x3_fwd_host_multi")

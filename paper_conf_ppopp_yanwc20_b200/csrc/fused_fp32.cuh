@@ -56,11 +56,12 @@ struct Smem {
 
 struct __align__(64) Params {
     CUtensorMap tmx;  // x (C,H,W,N) as 4-d (N, W, H, C), box (32, 4, 4, BC)   [LD_TMA only]
-    CUtensorMap tmu;  // u (C,16,K)  as 3-d (K, 16, C),   box (BK, 16, BC)      [LD_TMA only]
+    CUtensorMap tmu;  // u (C,16,ldu) as 3-d (K, 16, C),  box (BK, 16, BC)      [LD_TMA only]
     const float* __restrict__ x;  // (C,H,W,N)
     const float* __restrict__ u;  // (C,4,4,K)
     float* __restrict__ y;        // (K,H,W,N)
     int N, C, H, W, K;
+    int ldu;     // row stride of u in elements (>= K; > K when u is a K-slice)
     int TW;      // ceil(W/2)
     int NV;      // N * ceil(H/2) * ceil(W/2)
     int num_kb;  // ceil(K/BK)
@@ -149,7 +150,7 @@ __global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const
                 const int row = idx / UV_ROW, col = (idx % UV_ROW) * VU;
                 const int c = c0 + row / 16, k = k0 + col;
                 const bool ok = (c < p.C) && (k < p.K);
-                const float* src = ok ? p.u + ((size_t)c * 16 + (row & 15)) * p.K + k : p.u;
+                const float* src = ok ? p.u + ((size_t)c * 16 + (row & 15)) * p.ldu + k : p.u;
                 const uint32_t dst = smem_u32(us + row * BK + col);
                 if constexpr (VU == 4) cp_async16(dst, src, ok);
                 else cp_async4(dst, src, ok);

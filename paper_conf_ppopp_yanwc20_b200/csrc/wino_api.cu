@@ -123,15 +123,16 @@ PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
     return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
 }
 
-// fp32 tensor map over a dense row-major array, dims innermost first.
-bool encode_map(CUtensorMap* m, const float* base, int rank, const cuuint64_t* dims, const cuuint32_t* box) {
+// fp32 tensor map, dims innermost first; strides (bytes, dims 1..rank-1) default to dense.
+bool encode_map(CUtensorMap* m, const float* base, int rank, const cuuint64_t* dims, const cuuint32_t* box,
+                const cuuint64_t* strides_in = nullptr) {
     auto enc = tensor_map_encoder();
     if (!enc) return false;
     cuuint64_t strides[4];
     cuuint64_t acc = 4;
     for (int i = 0; i < rank - 1; ++i) {
         acc *= dims[i];
-        strides[i] = acc;
+        strides[i] = strides_in ? strides_in[i] : acc;
     }
     cuuint32_t estr[5] = {1, 1, 1, 1, 1};
     CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, rank, const_cast<float*>(base), dims, strides, box, estr,
@@ -167,6 +168,85 @@ wino_status_t launch_tc(const wino::tc::Params& prm, int64_t ctas, int dev, cuda
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 }  // namespace
+
+// FP32 fused conv on validated arguments; u may be a K-slice of a wider (C,4,4,ldu) array.
+wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, float* y_dev, int N, int C, int H,
+                              int W, int K, int dev, cudaStream_t st) {
+    using namespace wino::fp32;
+    Fp32Plan pl = plan_fp32(N, C, H, W, K);
+    if (ldu % 4 != 0 || !aligned16(u_dev)) pl.load_u = LD_CP4B;
+    Params prm;
+    std::memset(&prm, 0, sizeof(prm));
+    prm.x = x_dev;
+    prm.u = u_dev;
+    prm.y = y_dev;
+    prm.N = N;
+    prm.C = C;
+    prm.H = H;
+    prm.W = W;
+    prm.K = K;
+    prm.ldu = ldu;
+    prm.TW = (W + 1) / 2;
+    prm.NV = N * ((H + 1) / 2) * prm.TW;
+    prm.num_kb = (K + BK - 1) / BK;
+    prm.num_it = (C + BC - 1) / BC;
+    if (pl.load_x == LD_TMA) {
+        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
+        const cuuint32_t box[4] = {BN, 4, 4, BC};
+        if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    if (pl.load_u == LD_TMA) {
+        const cuuint64_t dims[3] = {cuuint64_t(K), 16, cuuint64_t(C)};
+        const cuuint64_t strides[2] = {cuuint64_t(ldu) * 4, cuuint64_t(16) * ldu * 4};
+        const cuuint32_t box[3] = {BK, 16, BC};
+        if (!encode_map(&prm.tmu, u_dev, 3, dims, box, strides)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    const int64_t g = pl.ctas;
+    const int sm = pl.smem;
+    switch (pl.load_x * 3 + pl.load_u) {
+        case LD_TMA * 3 + LD_TMA: return launch_fp32<LD_TMA, LD_TMA>(prm, g, sm, dev, st);
+        case LD_TMA * 3 + LD_CP4B: return launch_fp32<LD_TMA, LD_CP4B>(prm, g, sm, dev, st);
+        case LD_CP16B * 3 + LD_TMA: return launch_fp32<LD_CP16B, LD_TMA>(prm, g, sm, dev, st);
+        case LD_CP16B * 3 + LD_CP4B: return launch_fp32<LD_CP16B, LD_CP4B>(prm, g, sm, dev, st);
+        case LD_CP4B * 3 + LD_TMA: return launch_fp32<LD_CP4B, LD_TMA>(prm, g, sm, dev, st);
+        default: return launch_fp32<LD_CP4B, LD_CP4B>(prm, g, sm, dev, st);
+    }
+}
+
+// Copy-in / copy-out helper streams of the multi-layer host path, one pair per
+// device, created on first use (non-blocking, so they never sync with stream 0).
+std::mutex g_stream_mu;
+cudaStream_t g_s_in[kMaxDevices], g_s_out[kMaxDevices];
+wino_status_t helper_streams(int dev, cudaStream_t* in, cudaStream_t* out) {
+    std::lock_guard<std::mutex> lk(g_stream_mu);
+    if (!g_s_in[dev]) {
+        cudaError_t e = cudaStreamCreateWithFlags(&g_s_in[dev], cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&g_s_out[dev], cudaStreamNonBlocking);
+        if (e != cudaSuccess) return cuda_fail(e);
+    }
+    *in = g_s_in[dev];
+    *out = g_s_out[dev];
+    return WINO_OK;
+}
+
+// Events used for cross-stream ordering within one call; destroyed at the end of
+// the call (CUDA releases them once the recorded work completes).
+struct EventPool {
+    cudaEvent_t ev[256];
+    int n = 0;
+    cudaEvent_t get() {
+        if (n == 256) return nullptr;
+        cudaEvent_t e;
+        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+        ev[n++] = e;
+        return e;
+    }
+    ~EventPool() {
+        for (int i = 0; i < n; ++i) cudaEventDestroy(ev[i]);
+    }
+};
+
+size_t round_up256(size_t b) { return (b + 255) & ~size_t(255); }
 
 extern "C" {
 
@@ -262,44 +342,7 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
         return WINO_ERR_INVALID_ARG;
     int dev;
     if ((s = check_device(&dev)) != WINO_OK) return s;
-
-    using namespace wino::fp32;
-    Fp32Plan pl = plan_fp32(N, C, H, W, K);
-    Params prm;
-    std::memset(&prm, 0, sizeof(prm));
-    prm.x = x_dev;
-    prm.u = u_dev;
-    prm.y = y_dev;
-    prm.N = N;
-    prm.C = C;
-    prm.H = H;
-    prm.W = W;
-    prm.K = K;
-    prm.TW = (W + 1) / 2;
-    prm.NV = N * ((H + 1) / 2) * prm.TW;
-    prm.num_kb = (K + BK - 1) / BK;
-    prm.num_it = (C + BC - 1) / BC;
-    if (pl.load_x == LD_TMA) {
-        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
-        const cuuint32_t box[4] = {BN, 4, 4, BC};
-        if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
-    }
-    if (pl.load_u == LD_TMA) {
-        const cuuint64_t dims[3] = {cuuint64_t(K), 16, cuuint64_t(C)};
-        const cuuint32_t box[3] = {BK, 16, BC};
-        if (!encode_map(&prm.tmu, u_dev, 3, dims, box)) return cuda_fail(cudaErrorInvalidValue);
-    }
-    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    const int64_t g = pl.ctas;
-    const int sm = pl.smem;
-    switch (pl.load_x * 3 + pl.load_u) {
-        case LD_TMA * 3 + LD_TMA: return launch_fp32<LD_TMA, LD_TMA>(prm, g, sm, dev, st);
-        case LD_TMA * 3 + LD_CP4B: return launch_fp32<LD_TMA, LD_CP4B>(prm, g, sm, dev, st);
-        case LD_CP16B * 3 + LD_TMA: return launch_fp32<LD_CP16B, LD_TMA>(prm, g, sm, dev, st);
-        case LD_CP16B * 3 + LD_CP4B: return launch_fp32<LD_CP16B, LD_CP4B>(prm, g, sm, dev, st);
-        case LD_CP4B * 3 + LD_TMA: return launch_fp32<LD_CP4B, LD_TMA>(prm, g, sm, dev, st);
-        default: return launch_fp32<LD_CP4B, LD_CP4B>(prm, g, sm, dev, st);
-    }
+    return launch_fwd_fp32(x_dev, u_dev, K, y_dev, N, C, H, W, K, dev, reinterpret_cast<cudaStream_t>(stream));
 }
 
 size_t wino_filter_workspace_bytes_tc(int C, int K, wino_tc_mode_t mode) {
@@ -377,7 +420,6 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
     return launch_tc<2, 0>(prm, ctas, dev, st);
 }
 
-static size_t round_up256(size_t b) { return (b + 255) & ~size_t(255); }
 
 size_t wino_host_workspace_bytes(int N, int C, int H, int W, int K) {
     if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
@@ -409,6 +451,116 @@ wino_status_t wino_conv2d_f2x3_fwd_host(const float* x_host, const float* w_host
     if ((e = cudaMemcpyAsync(x_dev, x_host, xb, cudaMemcpyHostToDevice, st)) != cudaSuccess) return cuda_fail(e);
     if ((s = wino_conv2d_f2x3_fwd(x_dev, u_dev, y_dev, N, C, H, W, K, pad, stride, stream)) != WINO_OK) return s;
     if ((e = cudaMemcpyAsync(y_host, y_dev, yb, cudaMemcpyDeviceToHost, st)) != cudaSuccess) return cuda_fail(e);
+    return WINO_OK;
+}
+
+size_t wino_host_multi_workspace_bytes(const wino_host_layer_t* layers, int n_layers) {
+    if (!layers || n_layers <= 0) return 0;
+    size_t total = 0;
+    for (int i = 0; i < n_layers; ++i) {
+        const wino_host_layer_t& L = layers[i];
+        const size_t b = wino_host_workspace_bytes(L.N, L.C, L.H, L.W, L.K);
+        if (b == 0) return 0;
+        total += b;
+    }
+    return total;
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, int n_layers, void* ws_dev,
+                                              size_t ws_bytes, wino_stream_t stream) {
+    if (!layers || n_layers <= 0 || !ws_dev) return WINO_ERR_INVALID_ARG;
+    for (int i = 0; i < n_layers; ++i) {
+        const wino_host_layer_t& L = layers[i];
+        if (!L.x_host || !L.w_host || !L.y_host) return WINO_ERR_INVALID_ARG;
+        wino_status_t s = check_shape(L.N, L.C, L.H, L.W, L.K, 1, 1);
+        if (s != WINO_OK) return s;
+    }
+    if (ws_bytes < wino_host_multi_workspace_bytes(layers, n_layers)) return WINO_ERR_INVALID_ARG;
+    if (!aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    cudaStream_t s_in, s_out;
+    if ((s = helper_streams(dev, &s_in, &s_out)) != WINO_OK) return s;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    EventPool ev;
+    cudaError_t e;
+#define WINO_TRY(expr)                            \
+    do {                                          \
+        if ((e = (expr)) != cudaSuccess) return cuda_fail(e); \
+    } while (0)
+    cudaEvent_t e0 = ev.get();
+    if (!e0) return cuda_fail(cudaErrorMemoryAllocation);
+    WINO_TRY(cudaEventRecord(e0, st));
+    WINO_TRY(cudaStreamWaitEvent(s_in, e0, 0));
+    WINO_TRY(cudaStreamWaitEvent(s_out, e0, 0));
+    char* base = static_cast<char*>(ws_dev);
+    for (int i = 0; i < n_layers; ++i) {
+        const wino_host_layer_t& L = layers[i];
+        const size_t hw = size_t(L.H) * L.W, hwn = hw * L.N;
+        const size_t xb = size_t(L.C) * hwn * 4, wb = size_t(9) * L.C * L.K * 4, ub = size_t(16) * L.C * L.K * 4,
+                     yb = size_t(L.K) * hwn * 4;
+        float* x_dev = reinterpret_cast<float*>(base);
+        float* w_dev = reinterpret_cast<float*>(base + round_up256(xb));
+        float* u_dev = reinterpret_cast<float*>(base + round_up256(xb) + round_up256(wb));
+        float* y_dev = reinterpret_cast<float*>(base + round_up256(xb) + round_up256(wb) + round_up256(ub));
+        base += round_up256(xb) + round_up256(wb) + round_up256(ub) + round_up256(yb);
+        // weights in, FTF on the compute stream
+        WINO_TRY(cudaMemcpyAsync(w_dev, L.w_host, wb, cudaMemcpyHostToDevice, s_in));
+        cudaEvent_t ew = ev.get();
+        if (!ew) return cuda_fail(cudaErrorMemoryAllocation);
+        WINO_TRY(cudaEventRecord(ew, s_in));
+        WINO_TRY(cudaStreamWaitEvent(st, ew, 0));
+        if ((s = wino_filter_transform(w_dev, u_dev, L.C, L.K, stream)) != WINO_OK) return s;
+        // slicing: along K (contiguous copies) when K >= 128, else along the batch (2-D copies)
+        const bool kslice = L.K >= 128;
+        const int nslice = kslice ? (L.K >= 256 ? 4 : 2) : (L.N >= 128 && L.N % 64 == 0 ? L.N / 64 : 1);
+        if (kslice || nslice == 1) {
+            WINO_TRY(cudaMemcpyAsync(x_dev, L.x_host, xb, cudaMemcpyHostToDevice, s_in));
+            cudaEvent_t ex = ev.get();
+            if (!ex) return cuda_fail(cudaErrorMemoryAllocation);
+            WINO_TRY(cudaEventRecord(ex, s_in));
+            WINO_TRY(cudaStreamWaitEvent(st, ex, 0));
+            const int kc = ((L.K + nslice - 1) / nslice + 63) / 64 * 64;
+            for (int k0 = 0; k0 < L.K; k0 += kc) {
+                const int k1 = k0 + kc < L.K ? k0 + kc : L.K;
+                if ((s = launch_fwd_fp32(x_dev, u_dev + k0, L.K, y_dev + size_t(k0) * hwn, L.N, L.C, L.H, L.W,
+                                         k1 - k0, dev, st)) != WINO_OK)
+                    return s;
+                cudaEvent_t ec = ev.get();
+                if (!ec) return cuda_fail(cudaErrorMemoryAllocation);
+                WINO_TRY(cudaEventRecord(ec, st));
+                WINO_TRY(cudaStreamWaitEvent(s_out, ec, 0));
+                WINO_TRY(cudaMemcpyAsync(L.y_host + size_t(k0) * hwn, y_dev + size_t(k0) * hwn,
+                                         size_t(k1 - k0) * hwn * 4, cudaMemcpyDeviceToHost, s_out));
+            }
+        } else {
+            const int nc = L.N / nslice;  // batch slice, rows of nc*4 = 256 B
+            const size_t xs_elems = size_t(L.C) * hw * nc, ys_elems = size_t(L.K) * hw * nc;
+            for (int j = 0; j < nslice; ++j) {
+                float* xj = x_dev + j * xs_elems;
+                float* yj = y_dev + j * ys_elems;
+                WINO_TRY(cudaMemcpy2DAsync(xj, size_t(nc) * 4, L.x_host + size_t(j) * nc, size_t(L.N) * 4,
+                                           size_t(nc) * 4, size_t(L.C) * hw, cudaMemcpyHostToDevice, s_in));
+                cudaEvent_t ex = ev.get();
+                if (!ex) return cuda_fail(cudaErrorMemoryAllocation);
+                WINO_TRY(cudaEventRecord(ex, s_in));
+                WINO_TRY(cudaStreamWaitEvent(st, ex, 0));
+                if ((s = launch_fwd_fp32(xj, u_dev, L.K, yj, nc, L.C, L.H, L.W, L.K, dev, st)) != WINO_OK) return s;
+                cudaEvent_t ec = ev.get();
+                if (!ec) return cuda_fail(cudaErrorMemoryAllocation);
+                WINO_TRY(cudaEventRecord(ec, st));
+                WINO_TRY(cudaStreamWaitEvent(s_out, ec, 0));
+                WINO_TRY(cudaMemcpy2DAsync(L.y_host + size_t(j) * nc, size_t(L.N) * 4, yj, size_t(nc) * 4,
+                                           size_t(nc) * 4, size_t(L.K) * hw, cudaMemcpyDeviceToHost, s_out));
+            }
+        }
+    }
+    cudaEvent_t eo = ev.get();
+    if (!eo) return cuda_fail(cudaErrorMemoryAllocation);
+    WINO_TRY(cudaEventRecord(eo, s_out));
+    WINO_TRY(cudaStreamWaitEvent(st, eo, 0));  // caller's stream completes after every copy
+#undef WINO_TRY
     return WINO_OK;
 }
 

@@ -134,6 +134,34 @@ def test_host_entry_point_matches_device_path(wino):
     assert torch.equal(yh, y)
 
 
+def test_host_multi_matches_device_path(wino):
+    """The pipelined multi-layer host call (K slices, batch slices with 2-D copies) is
+    bit-identical to the device path layer by layer."""
+    cfgs = [Conv3x3Config("a", 4, 16, 256, 7, 7), Conv3x3Config("b", 256, 8, 64, 6, 5),
+            Conv3x3Config("c", 3, 5, 130, 9, 4), Conv3x3Config("d", 2, 3, 7, 3, 3)]
+    layers, refs = [], []
+    for i, cfg in enumerate(cfgs):
+        x, w = make_inputs(cfg, seed_x=40 + i, seed_w=50 + i)
+        refs.append(_run(wino, x, w)[1])
+        layers.append((x.pin_memory(), w.pin_memory(),
+                       torch.full((cfg.K, cfg.H, cfg.W, cfg.N), float("nan")).pin_memory()))
+    ws = torch.empty(wino.host_multi_workspace_bytes(layers), dtype=torch.uint8, device=DEV)
+    wino.conv2d_host_multi(layers, ws)
+    torch.cuda.synchronize()
+    for (xh, wh, yh), ref in zip(layers, refs):
+        assert torch.equal(yh, ref)
+
+
+def test_k_slices_equal_full(wino):
+    """Slicing K (the library's host pipeline does) cannot change any output bit."""
+    cfg = Conv3x3Config("ks", 32, 24, 256, 10, 10)
+    x, w = make_inputs(cfg)
+    _, y = _run(wino, x, w)
+    for k0, k1 in [(0, 64), (64, 256), (128, 192)]:
+        _, ys = _run(wino, x, w[..., k0:k1].contiguous())
+        assert torch.equal(ys, y[k0:k1])
+
+
 def test_output_fully_overwritten(wino):
     cfg = Conv3x3Config("ow", 3, 5, 6, 7, 5)
     x, w = make_inputs(cfg)
