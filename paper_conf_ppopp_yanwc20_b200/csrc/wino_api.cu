@@ -15,6 +15,7 @@
 #include "../../include/wino.h"
 #include "ftf.cuh"
 #include "fused_fp32.cuh"
+#include "fused_fp32_ws.cuh"
 #include "fused_tc.cuh"
 
 namespace {
@@ -142,6 +143,7 @@ bool encode_map(CUtensorMap* m, const float* base, int rank, const cuuint64_t* d
 }
 
 std::atomic<uint64_t> g_attr_fp32[3][3];
+std::atomic<uint64_t> g_attr_ws;
 
 template <int XM, int UM>
 wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem, int dev, cudaStream_t st) {
@@ -203,6 +205,17 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
     }
     const int64_t g = pl.ctas;
     const int sm = pl.smem;
+#ifndef WINO_NO_WS
+    if (pl.load_x == LD_TMA && pl.load_u == LD_TMA) {  // warp-specialised kernel
+        auto kern = wino::fp32ws::fused_fp32_ws_kernel;
+        const int wsm = wino::fp32ws::Smem::bytes;
+        wino_status_t s = ensure_smem_attr(kern, dev, wsm, g_attr_ws);
+        if (s != WINO_OK) return s;
+        kern<<<dim3(static_cast<unsigned>(g)), wino::fp32ws::NT, wsm, st>>>(prm);
+        cudaError_t e = cudaGetLastError();
+        return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+    }
+#endif
     switch (pl.load_x * 3 + pl.load_u) {
         case LD_TMA * 3 + LD_TMA: return launch_fp32<LD_TMA, LD_TMA>(prm, g, sm, dev, st);
         case LD_TMA * 3 + LD_CP4B: return launch_fp32<LD_TMA, LD_CP4B>(prm, g, sm, dev, st);

@@ -169,3 +169,19 @@ __device__ __forceinline__ void tma_prefetch_l2_4d(const void* map, int c0, int 
                  : "memory");
 }
 }  // namespace wino
+
+namespace wino {
+// Register re-distribution between warpgroups (must be executed by all warps of a warpgroup).
+template <int N>
+__device__ __forceinline__ void setmaxnreg_inc() {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(N));
+}
+template <int N>
+__device__ __forceinline__ void setmaxnreg_dec() {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(N));
+}
+// Named barrier over `count` threads (id 1..15; id 0 is __syncthreads).
+__device__ __forceinline__ void named_bar_sync(int id, int count) {
+    asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(count) : "memory");
+}
+}  // namespace wino
