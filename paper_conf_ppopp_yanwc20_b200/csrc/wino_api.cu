@@ -56,6 +56,17 @@ wino_status_t check_device(int* dev_out) {
     return cap == 1 ? WINO_OK : WINO_ERR_UNSUPPORTED;
 }
 
+// SM count per device (cached).
+std::atomic<int> g_sm_count[kMaxDevices];
+int sm_count(int dev) {
+    int n = g_sm_count[dev].load(std::memory_order_relaxed);
+    if (n == 0) {
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+        g_sm_count[dev].store(n, std::memory_order_relaxed);
+    }
+    return n;
+}
+
 // Opt-in to >48 KB dynamic shared memory once per (device, kernel instance).
 std::mutex g_attr_mu;
 template <typename Kern>
@@ -211,7 +222,9 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
         const int wsm = wino::fp32ws::Smem::bytes;
         wino_status_t s = ensure_smem_attr(kern, dev, wsm, g_attr_ws);
         if (s != WINO_OK) return s;
-        kern<<<dim3(static_cast<unsigned>(g)), wino::fp32ws::NT, wsm, st>>>(prm);
+        const int sms = sm_count(dev);
+        const int64_t grid = g < sms ? g : sms;  // persistent: one CTA per SM
+        kern<<<dim3(static_cast<unsigned>(grid)), wino::fp32ws::NT, wsm, st>>>(prm, static_cast<int>(g));
         cudaError_t e = cudaGetLastError();
         return e == cudaSuccess ? WINO_OK : cuda_fail(e);
     }
