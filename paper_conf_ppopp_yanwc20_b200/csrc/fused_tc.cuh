@@ -5,19 +5,22 @@
 // Alg. 1); the paper has no tensor-core path and notes that "the data
 // layout needs a redesign" for one (Sec. 8.3).  This is that redesign.
 //
-// CTA tile: 128 filters (UMMA M) x 32 tiles*images nu (UMMA N) x all 16 xi.
+// Tile: 128 filters (UMMA M) x 32 tiles*images nu (UMMA N) x all 16 xi.
 // TMEM: 16 accumulators D(xi) of 128 lanes x 32 columns = all 512 columns.
-// Per channel block cb (8 channels = one tf32 UMMA K step):
-//   * x producer warp: TMA box of raw x (n:32, w:4, h:4, c:8) (zero fill = padding);
-//   * U producer warp: 64 KB bulk copies of the pre-arranged transformed filter
-//     into a ring decoupled from x;
-//   * 8 ITF warps: V = B^T d B (Eq. 6) for the 8 x 32 (c, nu) tiles, rounded to
-//     TF32 (3xTF32: big + small planes), stored as the K-major UMMA B operand;
-//   * MMA warp (one thread): per xi, D(xi) += U(xi) * V(xi) (3xTF32: big*big +
-//     big*small + small*big), tcgen05.commit frees the smem slots;
-//   * epilogue (8 warps): tcgen05.ld the 16 accumulators, OTF (Eq. 8), store.
-// Warp-specialised (separate producers for x and U so neither ring stalls the
-// other), mbarrier-synchronised; no __syncthreads in the main loop.
+// Persistent (one CTA per SM, tiles blockIdx.x, +gridDim.x, ...), warp-specialised:
+//   * warp 12 (U producer): 64 KB bulk copies of the pre-arranged transformed
+//     filter per channel block into a 2-slot ring;
+//   * warp 14 (x producer): TMA box of raw x (n:32, w:4, h:4, c:8) per channel
+//     block (zero fill = implicit padding, Sec. 3.5), L2 prefetch ahead;
+//   * warps 4-11 (ITF): V = B^T d B (Eq. 6) for the 8 x 32 (c, nu) tiles of a
+//     block, rounded to TF32 (3xTF32: big + small planes), stored as the
+//     K-major UMMA B operand;
+//   * warp 13 (MMA, one thread): per xi, D(xi) += U(xi) * V(xi) (3xTF32:
+//     big*big + big*small + small*big); tcgen05.commit frees smem slots;
+//   * warps 0-3 (epilogue): tcgen05.ld of the 16 accumulators of their 32 TMEM
+//     lanes, OTF (Eq. 8) into registers, release TMEM to the next tile's MMAs,
+//     then coalesced 128 B stores -- overlapping the next tile's main loop.
+// All hand-offs are mbarriers; the producers run ahead across tile boundaries.
 #pragma once
 #include <cuda.h>
 
@@ -43,14 +46,17 @@ __device__ unsigned long long g_trace[TRACE_EVENTS * TRACE_CB];
     } while (0)
 #endif
 
-constexpr int BM = 128;        // filters per CTA (UMMA M)
-constexpr int BN = 32;         // nu per CTA (UMMA N)
+constexpr int BM = 128;        // filters per tile (UMMA M)
+constexpr int BN = 32;         // nu per tile (UMMA N)
 constexpr int BC = 8;          // channels per block (UMMA K for tf32)
-constexpr int ITF_WARPS = 8;   // warps 0..7: ITF + epilogue
-constexpr int PROD_WARP = 8;   // bulk-copy producer of the transformed filter U
-constexpr int MMA_WARP = 9;    // tcgen05.mma issuer
-constexpr int XPROD_WARP = 10; // TMA / cp.async producer of raw x (decoupled from U)
-constexpr int NT = 352;
+constexpr int EPI_WARPS = 4;   // warps 0..3: epilogue (TMEM lane quadrants 0..3)
+constexpr int ITF_WARP0 = 4;   // warps 4..11: ITF
+constexpr int ITF_WARPS = 8;
+constexpr int PROD_WARP = 12;  // bulk-copy producer of the transformed filter U
+constexpr int MMA_WARP = 13;   // tcgen05.mma issuer
+constexpr int XPROD_WARP = 14; // TMA / cp.async producer of raw x
+constexpr int NT = 512;        // 16 warps (warp 15 idle; warpgroup-granular register split)
+constexpr int REG_EPI = 232, REG_ITF = 88, REG_PROD = 56;  // 128*232 + 256*88 + 128*56 = 59264
 constexpr int A_TILE = BM * BC * 4;  // one (xi, plane) A operand: 4 KB
 constexpr int B_TILE = BN * BC * 4;  // one (xi, plane) B operand: 1 KB
 constexpr int XS_BYTES = BC * 16 * BN * 4;  // raw x box: 16 KB
@@ -109,8 +115,9 @@ struct __align__(64) Params {
     float* __restrict__ y;
     int N, C, H, W, K;
     int TW, NV;
-    int num_kb;  // ceil(K/128)
-    int num_cb;  // ceil(C/8)
+    int num_kb;     // ceil(K/128)
+    int num_cb;     // ceil(C/8)
+    int num_tiles;  // ceil(NV/32) * num_kb
 };
 
 template <int P>
@@ -126,8 +133,8 @@ struct Cfg {
     static constexpr int OFF_V = OFF_X + X_SLOTS * XS_BYTES;
     static constexpr int OFF_TAB = OFF_V + 2 * V_SLOT;          // cp.async gather table (16*32 ints)
     static constexpr int OFF_BAR = OFF_TAB + 16 * BN * 4;
-    // barriers: u_full/u_empty[U_SLOTS], x_full/x_empty[X_SLOTS], v_full[2], v_empty[2], acc
-    static constexpr int NBAR = 2 * U_SLOTS + 2 * X_SLOTS + 5;
+    // u_full/u_empty[U_SLOTS], x_full/x_empty[X_SLOTS], v_full[2], v_empty[2], acc_full, acc_empty
+    static constexpr int NBAR = 2 * U_SLOTS + 2 * X_SLOTS + 6;
     static constexpr int OFF_TMEM = OFF_BAR + NBAR * 8;
     static constexpr int BYTES = OFF_TMEM + 16;
 };
@@ -149,12 +156,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     uint64_t* const v_full = x_empty + G::X_SLOTS;
     uint64_t* const v_empty = v_full + 2;
     uint64_t* const acc_full = v_full + 4;
+    uint64_t* const acc_empty = acc_full + 1;
     uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + G::OFF_TMEM);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int kb = blockIdx.x % p.num_kb;
-    const int nb = blockIdx.x / p.num_kb;
-    const int k0 = kb * BM, nu0 = nb * BN;
     const int NCB = p.num_cb;
 
     if (tid == 0) {
@@ -171,192 +176,208 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             mbar_init(&v_empty[s], 1);
         }
         mbar_init(acc_full, 1);
+        mbar_init(acc_empty, EPI_WARPS);
         fence_mbar_init();
         if constexpr (XM == 2) tma_prefetch_desc(&p.tmx);
-    }
-    if constexpr (XM != 2) {
-        for (int e = tid; e < 16 * BN; e += NT) {
-            const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
-            int off = -1;
-            if (nu < p.NV) {
-                const int t = nu / p.N, n = nu - t * p.N;
-                const int th = t / p.TW, tw = t - th * p.TW;
-                const int h = 2 * th - 1 + (pos >> 2), w = 2 * tw - 1 + (pos & 3);
-                if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
-            }
-            xtab[e] = off;
-        }
     }
     if (warp == 0) tmem_alloc(tmem_slot, 512);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    const size_t HWN = (size_t)p.H * p.W * p.N;
 
-    if (warp == XPROD_WARP) {
-        // --------------------------- raw-x producer ---------------------------
-        int tma_n0 = 0, tma_w0 = 0, tma_h0 = 0;
-        if constexpr (XM == 2) {
-            const int t = nu0 / p.N;
-            tma_n0 = nu0 - t * p.N;
-            const int th = t / p.TW, tw = t - th * p.TW;
-            tma_w0 = 2 * tw - 1;  // may be -1: TMA zero fill = implicit padding (Sec. 3.5)
-            tma_h0 = 2 * th - 1;
-        }
-        const size_t HWN = (size_t)p.H * p.W * p.N;
-        // x streams from HBM (first touch); warm L2 X_PREFETCH blocks ahead so the
-        // shared-memory ring only has to cover the L2 latency
-        if constexpr (XM == 2) {
-            if (lane == 0)
-                for (int cb = 0; cb < X_PREFETCH && cb < NCB; ++cb)
-                    tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, cb * BC);
-        }
-        for (int cb = 0; cb < NCB; ++cb) {
-            const int xs = cb % G::X_SLOTS;
-            if constexpr (XM == 2) {
-                if (lane == 0 && cb + X_PREFETCH < NCB)
-                    tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, (cb + X_PREFETCH) * BC);
-            }
-            if (cb >= G::X_SLOTS) mbar_wait(&x_empty[xs], ((cb / G::X_SLOTS) - 1) & 1);
-            float* xdst = sx + xs * (XS_BYTES / 4);
-            if (lane == 0) TC_TRACE(0, cb);
-            if constexpr (XM == 2) {
-                if (lane == 0) {
-                    mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
-                    tma_load_4d(xdst, &p.tmx, &x_full[xs], tma_n0, tma_w0, tma_h0, cb * BC);
+    if (warp >= PROD_WARP) {
+        setmaxnreg_dec<REG_PROD>();
+        if (warp == XPROD_WARP) {
+            // --------------------------- raw-x producer ---------------------------
+            int gcb = 0;  // channel blocks issued so far (all tiles)
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+                const int nu0 = (tile / p.num_kb) * BN;
+                int tma_n0 = 0, tma_w0 = 0, tma_h0 = 0;
+                if constexpr (XM == 2) {
+                    const int t = nu0 / p.N;
+                    tma_n0 = nu0 - t * p.N;
+                    const int th = t / p.TW, tw = t - th * p.TW;
+                    tma_w0 = 2 * tw - 1;  // may be -1: TMA zero fill = implicit padding (Sec. 3.5)
+                    tma_h0 = 2 * th - 1;
+                    // x streams from HBM (first touch): warm L2 a few blocks ahead
+                    if (lane == 0)
+                        for (int cb = 0; cb < X_PREFETCH && cb < NCB; ++cb)
+                            tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, cb * BC);
+                } else {
+                    // gather offsets (h*W+w)*N+n of the 4x4 window element pos of local nu (-1: padding)
+                    __syncwarp();
+                    for (int e = lane; e < 16 * BN; e += 32) {
+                        const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
+                        int off = -1;
+                        if (nu < p.NV) {
+                            const int t = nu / p.N, n = nu - t * p.N;
+                            const int th = t / p.TW, tw = t - th * p.TW;
+                            const int h = 2 * th - 1 + (pos >> 2), w = 2 * tw - 1 + (pos & 3);
+                            if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
+                        }
+                        xtab[e] = off;
+                    }
+                    __syncwarp();
                 }
-            } else {
-                constexpr int VX = XM == 1 ? 4 : 1;
-                for (int e = lane; e < BC * 16 * BN / VX; e += 32) {
-                    const int cl = e / (16 * BN / VX), r = (e % (16 * BN / VX)) * VX;
-                    const int c = cb * BC + cl;
-                    const int off = xtab[r];
-                    const bool ok = (c < p.C) && (off >= 0);
-                    const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
-                    const uint32_t dst = smem_u32(xdst + cl * 16 * BN + r);
-                    if constexpr (VX == 4) cp_async16(dst, src, ok);
-                    else cp_async4(dst, src, ok);
-                }
-                cp_async_wait_all();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&x_full[xs]);
-            }
-        }
-    } else if (warp == PROD_WARP) {
-        // ------------------------ transformed-filter producer -----------------
-        int unit = 0;
-        for (int cb = 0; cb < NCB; ++cb) {
-            for (int h = 0; h < G::UNITS_PER_CB; ++h, ++unit) {
-                const int us = unit % G::U_SLOTS;
-                if (unit >= G::U_SLOTS) mbar_wait(&u_empty[us], ((unit / G::U_SLOTS) - 1) & 1);
-                if (lane == 0) {
-                    if (h == 0) TC_TRACE(1, cb);
-                    const float* src = p.u_tc + ((((size_t)cb * p.num_kb + kb) * 16 + h * G::XPU) * P) *
-                                                    (BM * BC);
-                    mbar_arrive_expect_tx(&u_full[us], G::UNIT);
-                    bulk_load(su + us * G::UNIT, src, G::UNIT, &u_full[us]);
+                for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                    const int xs = gcb % G::X_SLOTS;
+                    if (gcb >= G::X_SLOTS) mbar_wait(&x_empty[xs], ((gcb / G::X_SLOTS) - 1) & 1);
+                    float* xdst = sx + xs * (XS_BYTES / 4);
+                    if constexpr (XM == 2) {
+                        if (lane == 0) {
+                            if (cb + X_PREFETCH < NCB)
+                                tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, (cb + X_PREFETCH) * BC);
+                            mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
+                            tma_load_4d(xdst, &p.tmx, &x_full[xs], tma_n0, tma_w0, tma_h0, cb * BC);
+                        }
+                    } else {
+                        constexpr int VX = XM == 1 ? 4 : 1;
+                        for (int e = lane; e < BC * 16 * BN / VX; e += 32) {
+                            const int cl = e / (16 * BN / VX), r = (e % (16 * BN / VX)) * VX;
+                            const int c = cb * BC + cl;
+                            const int off = xtab[r];
+                            const bool ok = (c < p.C) && (off >= 0);
+                            const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
+                            const uint32_t dst = smem_u32(xdst + cl * 16 * BN + r);
+                            if constexpr (VX == 4) cp_async16(dst, src, ok);
+                            else cp_async4(dst, src, ok);
+                        }
+                        cp_async_wait_all();
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&x_full[xs]);
+                    }
                 }
             }
-        }
-    } else if (warp == MMA_WARP) {
-        // ------------------------------ MMA issuer ----------------------------
-        constexpr uint32_t IDESC = umma_idesc_tf32(BM, BN);
-        int unit = 0;
-        for (int cb = 0; cb < NCB; ++cb) {
-            const int vs = cb & 1;
-            mbar_wait(&v_full[vs], (cb >> 1) & 1);
-            if (lane == 0) TC_TRACE(4, cb);
-            for (int half = 0; half < G::UNITS_PER_CB; ++half, ++unit) {
-                const int us = unit % G::U_SLOTS;
-                mbar_wait(&u_full[us], (unit / G::U_SLOTS) & 1);
-                tc_fence_after();
-                if (lane == 0) {
-                    const uint32_t ubase = smem_u32(su + us * G::UNIT);
-                    const uint32_t vbase = smem_u32(sv + vs * G::V_SLOT);
-#pragma unroll
-                    for (int q = 0; q < G::XPU; ++q) {
-                        const int xi = half * G::XPU + q;
-                        const uint32_t d = tmem + xi * BN;
-                        const uint32_t a0 = ubase + (q * P) * A_TILE, b0 = vbase + (xi * P) * B_TILE;
-                        const uint64_t ab = umma_desc(a0, 128, 256), bb = umma_desc(b0, 128, 256);
-                        umma_tf32(d, ab, bb, IDESC, cb > 0 ? 1u : 0u);
-                        if constexpr (P == 2) {
-                            const uint64_t as = umma_desc(a0 + A_TILE, 128, 256);
-                            const uint64_t bs = umma_desc(b0 + B_TILE, 128, 256);
-                            umma_tf32(d, ab, bs, IDESC, 1u);
-                            umma_tf32(d, as, bb, IDESC, 1u);
+        } else if (warp == PROD_WARP) {
+            // ------------------------ transformed-filter producer -----------------
+            int unit = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+                const int kb = tile % p.num_kb;
+                for (int cb = 0; cb < NCB; ++cb) {
+                    for (int h = 0; h < G::UNITS_PER_CB; ++h, ++unit) {
+                        const int us = unit % G::U_SLOTS;
+                        if (unit >= G::U_SLOTS) mbar_wait(&u_empty[us], ((unit / G::U_SLOTS) - 1) & 1);
+                        if (lane == 0) {
+                            const float* src =
+                                p.u_tc + ((((size_t)cb * p.num_kb + kb) * 16 + h * G::XPU) * P) * (BM * BC);
+                            mbar_arrive_expect_tx(&u_full[us], G::UNIT);
+                            bulk_load(su + us * G::UNIT, src, G::UNIT, &u_full[us]);
                         }
                     }
-                    umma_commit(&u_empty[us]);
-                    if (half == G::UNITS_PER_CB - 1) {
-                        umma_commit(&v_empty[vs]);
-                        TC_TRACE(5, cb);
+                }
+            }
+        } else if (warp == MMA_WARP) {
+            // ------------------------------ MMA issuer ----------------------------
+            constexpr uint32_t IDESC = umma_idesc_tf32(BM, BN);
+            int unit = 0, gcb = 0, it = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+                if (it > 0) mbar_wait(acc_empty, (it - 1) & 1);  // epilogue drained TMEM
+                tc_fence_after();
+                for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                    const int vs = gcb & 1;
+                    mbar_wait(&v_full[vs], (gcb >> 1) & 1);
+                    for (int half = 0; half < G::UNITS_PER_CB; ++half, ++unit) {
+                        const int us = unit % G::U_SLOTS;
+                        mbar_wait(&u_full[us], (unit / G::U_SLOTS) & 1);
+                        tc_fence_after();
+                        if (lane == 0) {
+                            const uint32_t ubase = smem_u32(su + us * G::UNIT);
+                            const uint32_t vbase = smem_u32(sv + vs * G::V_SLOT);
+#pragma unroll
+                            for (int q = 0; q < G::XPU; ++q) {
+                                const int xi = half * G::XPU + q;
+                                const uint32_t d = tmem + xi * BN;
+                                const uint32_t a0 = ubase + (q * P) * A_TILE, b0 = vbase + (xi * P) * B_TILE;
+                                const uint64_t ab = umma_desc(a0, 128, 256), bb = umma_desc(b0, 128, 256);
+                                umma_tf32(d, ab, bb, IDESC, cb > 0 ? 1u : 0u);
+                                if constexpr (P == 2) {
+                                    const uint64_t as = umma_desc(a0 + A_TILE, 128, 256);
+                                    const uint64_t bs = umma_desc(b0 + B_TILE, 128, 256);
+                                    umma_tf32(d, ab, bs, IDESC, 1u);
+                                    umma_tf32(d, as, bb, IDESC, 1u);
+                                }
+                            }
+                            umma_commit(&u_empty[us]);
+                            if (half == G::UNITS_PER_CB - 1) umma_commit(&v_empty[vs]);
+                        }
+                        __syncwarp();
                     }
                 }
+                if (lane == 0) umma_commit(acc_full);
                 __syncwarp();
             }
         }
-        if (lane == 0) umma_commit(acc_full);
-        __syncwarp();
-    } else {
+    } else if (warp >= ITF_WARP0) {
+        setmaxnreg_dec<REG_ITF>();
         // ------------------------------ ITF warps -----------------------------
         // thread -> (c, nu) with lanes over (nu%8, c%4): conflict-free K-major stores
-        const int nl = (warp & 3) * 8 + (lane >> 2);
-        const int cl = (warp >> 2) * 4 + (lane & 3);
+        const int iw = warp - ITF_WARP0;
+        const int nl = (iw & 3) * 8 + (lane >> 2);
+        const int cl = (iw >> 2) * 4 + (lane & 3);
         const uint32_t voff = (nl >> 3) * 256 + (cl >> 2) * 128 + (nl & 7) * 16 + (cl & 3) * 4;
-        for (int cb = 0; cb < NCB; ++cb) {
-            const int xs = cb % G::X_SLOTS, vs = cb & 1;
-            mbar_wait(&x_full[xs], (cb / G::X_SLOTS) & 1);
-            if (tid == 0) TC_TRACE(2, cb);
-            const float* xsrc = sx + xs * (XS_BYTES / 4) + cl * 16 * BN + nl;
-            float d[16], t[16];
+        int gcb = 0;
+        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+            for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                const int xs = gcb % G::X_SLOTS, vs = gcb & 1;
+                mbar_wait(&x_full[xs], (gcb / G::X_SLOTS) & 1);
+                const float* xsrc = sx + xs * (XS_BYTES / 4) + cl * 16 * BN + nl;
+                float d[16], t[16];
 #pragma unroll
-            for (int e = 0; e < 16; ++e) d[e] = xsrc[e * BN];
-            itf_4x4(d, t);  // consumes the loads: the x slot can be released
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&x_empty[xs]);
-            if (cb >= 2) mbar_wait(&v_empty[vs], ((cb >> 1) - 1) & 1);
-            uint8_t* vdst = sv + vs * G::V_SLOT + voff;
+                for (int e = 0; e < 16; ++e) d[e] = xsrc[e * BN];
+                itf_4x4(d, t);  // consumes the loads: the x slot can be released
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&x_empty[xs]);
+                if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
+                uint8_t* vdst = sv + vs * G::V_SLOT + voff;
 #pragma unroll
-            for (int xi = 0; xi < 16; ++xi) {
-                const float big = to_tf32(t[xi]);
-                *reinterpret_cast<float*>(vdst + (xi * P) * B_TILE) = big;
-                if constexpr (P == 2) *reinterpret_cast<float*>(vdst + (xi * P + 1) * B_TILE) = to_tf32(t[xi] - big);
+                for (int xi = 0; xi < 16; ++xi) {
+                    const float big = to_tf32(t[xi]);
+                    *reinterpret_cast<float*>(vdst + (xi * P) * B_TILE) = big;
+                    if constexpr (P == 2)
+                        *reinterpret_cast<float*>(vdst + (xi * P + 1) * B_TILE) = to_tf32(t[xi] - big);
+                }
+                fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&v_full[vs]);
             }
-            fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&v_full[vs]);
-            if (tid == 0) TC_TRACE(3, cb);
         }
-
+    } else {
+        setmaxnreg_inc<REG_EPI>();
         // ------------------------------ epilogue ------------------------------
-        mbar_wait(acc_full, 0);
-        if (tid == 0) TC_TRACE(6, 0);
-        tc_fence_after();
-        const int kl = (warp & 3) * 32 + lane;  // TMEM lane = filter within the tile
-        const int k = k0 + kl;
-        const uint32_t trow = tmem + ((uint32_t)((warp & 3) * 32) << 16);
-        const size_t HWN = (size_t)p.H * p.W * p.N;
+        // thread = TMEM lane = filter k of the tile; all 32 nu of the 16 accumulators
+        const int kl = warp * 32 + lane;
+        const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
         const size_t dW = (size_t)p.W * p.N;
-        for (int ch = 0; ch < 2; ++ch) {
-            const int nb0 = (warp >> 2) * 16 + ch * 8;  // 8 nu per chunk
-            float m[16][8];
+        int it = 0;
+        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+            const int k = (tile % p.num_kb) * BM + kl;
+            const int nu0 = (tile / p.num_kb) * BN;
+            mbar_wait(acc_full, it & 1);
+            tc_fence_after();
+            float o[BN][4];  // OTF results of this filter for the 32 nu
 #pragma unroll
-            for (int xi = 0; xi < 16; ++xi) tmem_ld8(trow + xi * BN + nb0, m[xi]);
-            tmem_ld_wait();
-            if (k >= p.K) continue;
-            float o[8][4];
+            for (int ch = 0; ch < BN / 4; ++ch) {
+                float m[16][4];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) {
-                float mm[16];
+                for (int xi = 0; xi < 16; ++xi) tmem_ld4(trow + xi * BN + ch * 4, m[xi]);
+                tmem_ld_wait();
 #pragma unroll
-                for (int xi = 0; xi < 16; ++xi) mm[xi] = m[xi][j];
-                otf_2x2(mm, o[j]);
+                for (int j = 0; j < 4; ++j) {
+                    float mm[16];
+#pragma unroll
+                    for (int xi = 0; xi < 16; ++xi) mm[xi] = m[xi][j];
+                    otf_2x2(mm, o[ch * 4 + j]);
+                }
             }
-            const int nu_first = nu0 + nb0;
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(acc_empty);  // TMEM free for the next tile's MMAs
+            if (k >= p.K) continue;
             if constexpr (XM == 2) {
-                // N % 32 == 0: the 8 nu are 8 consecutive n of one tile -> 2 x float4 per output pixel
-                const int t = nu_first / p.N, n = nu_first - t * p.N;
+                // N % 32 == 0: the 32 nu are 32 consecutive n of one image tile -> 128 B rows
+                const int t = nu0 / p.N, n = nu0 - t * p.N;
                 const int th = t / p.TW, tw = t - th * p.TW;
                 const int i0 = 2 * th, j0 = 2 * tw;
                 float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
@@ -365,13 +386,14 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                     const int a = q >> 1, b = q & 1;
                     if (i0 + a >= p.H || j0 + b >= p.W) continue;  // odd H/W (L1155)
                     float* dst = yk + a * dW + b * p.N;
-                    *reinterpret_cast<float4*>(dst) = make_float4(o[0][q], o[1][q], o[2][q], o[3][q]);
-                    *reinterpret_cast<float4*>(dst + 4) = make_float4(o[4][q], o[5][q], o[6][q], o[7][q]);
+#pragma unroll
+                    for (int j = 0; j < BN; j += 4)
+                        *reinterpret_cast<float4*>(dst + j) = make_float4(o[j][q], o[j + 1][q], o[j + 2][q], o[j + 3][q]);
                 }
             } else {
 #pragma unroll
-                for (int j = 0; j < 8; ++j) {
-                    const int nu = nu_first + j;
+                for (int j = 0; j < BN; ++j) {
+                    const int nu = nu0 + j;
                     if (nu >= p.NV) break;
                     const int t = nu / p.N, n = nu - t * p.N;
                     const int th = t / p.TW, tw = t - th * p.TW;
@@ -387,7 +409,6 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     }
     tc_fence_before();
     __syncthreads();
-    if (tid == 0) TC_TRACE(7, 0);
     if (warp == 0) tmem_dealloc(tmem, 512);
 }
 

@@ -334,7 +334,7 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->load_x = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
         plan->load_u = 3;  // bulk copy of the pre-arranged operand tiles
         plan->split_c = 1;
-        plan->ctas = ((nv + BN - 1) / BN) * ((K + BM - 1) / BM);
+        plan->ctas = ((nv + BN - 1) / BN) * ((K + BM - 1) / BM);  // tiles (persistent grid <= #SMs)
         plan->threads = NT;
         plan->smem_bytes = variant == 1 ? Cfg<1>::BYTES : Cfg<2>::BYTES;
         plan->launches = 1;
@@ -428,13 +428,15 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
     prm.NV = N * ((H + 1) / 2) * prm.TW;
     prm.num_kb = (K + BM - 1) / BM;
     prm.num_cb = (C + BC - 1) / BC;
+    prm.num_tiles = ((prm.NV + BN - 1) / BN) * prm.num_kb;
     const int xm = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
     if (xm == 2) {
         const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
         const cuuint32_t box[4] = {BN, 4, 4, BC};
         if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
     }
-    const int64_t ctas = int64_t((prm.NV + BN - 1) / BN) * prm.num_kb;
+    const int sms = sm_count(dev);
+    const int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (mode == WINO_TC_TF32) {
         if (xm == 2) return launch_tc<1, 2>(prm, ctas, dev, st);
