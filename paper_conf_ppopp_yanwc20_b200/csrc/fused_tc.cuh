@@ -46,8 +46,10 @@ __device__ unsigned long long g_trace[TRACE_EVENTS * TRACE_CB];
     } while (0)
 #endif
 
-constexpr int BM = 128;        // filters per tile (UMMA M)
-constexpr int BN = 32;         // nu per tile (UMMA N)
+constexpr int BN = 32;         // nu per UMMA (N); a tile has 128 / MM such halves
+// MM (template) = filters per tile = UMMA M: 128, or 64 with TWO accumulators per
+// xi interleaved in TMEM lanes (rows 0-15 of each 32-lane quadrant hold nu-half 0,
+// lanes 16-31 hold nu-half 1; scripts/microbench/umma_m64.cu) -> tile 64 x 64.
 constexpr int BC = 8;          // channels per block (UMMA K for tf32)
 constexpr int EPI_WARPS = 4;   // warps 0..3: epilogue (TMEM lane quadrants 0..3)
 constexpr int ITF_WARP0 = 4;   // warps 4..11: ITF
@@ -57,8 +59,9 @@ constexpr int MMA_WARP = 13;   // tcgen05.mma issuer
 constexpr int XPROD_WARP = 14; // TMA / cp.async producer of raw x
 constexpr int NT = 512;        // 16 warps (warp 15 idle; warpgroup-granular register split)
 constexpr int REG_EPI = 232, REG_ITF = 88, REG_PROD = 56;  // 128*232 + 256*88 + 128*56 = 59264
-constexpr int A_TILE = BM * BC * 4;  // one (xi, plane) A operand: 4 KB
-constexpr int B_TILE = BN * BC * 4;  // one (xi, plane) B operand: 1 KB
+template <int MM>
+constexpr int a_tile() { return MM * BC * 4; }  // one (xi, plane) A operand: 4 / 2 KB
+constexpr int B_TILE = BN * BC * 4;  // one (xi, plane, nu-half) B operand: 1 KB
 constexpr int XS_BYTES = BC * 16 * BN * 4;  // raw x box: 16 KB
 constexpr int X_PREFETCH = 6;               // channel blocks of x prefetched into L2 ahead
 // U ring unit: 64 KB = all 16 xi (TF32) or 8 xi x 2 planes (3xTF32) of one channel
@@ -70,19 +73,25 @@ template <int P>
 constexpr int xi_per_unit() { return P == 1 ? 16 : 8; }
 
 // u_tc layout (written by tc_filter_kernel, read with bulk copies):
-//   [cb = C/8][kb = K/128][xi 16][plane P][m/8 16][c/4 2][m%8 8][c%4 4]  fp32
-// i.e. per (cb, kb, xi, plane) one 4 KB K-major SWIZZLE_NONE UMMA A tile
+//   [cb = C/8][kb = K/MM][xi 16][plane P][m/8][c/4 2][m%8 8][c%4 4]  fp32
+// i.e. per (cb, kb, xi, plane) one K-major SWIZZLE_NONE UMMA A tile of MM rows
 // (LBO = 128 B between the two 16 B K-chunks, SBO = 256 B between 8-row groups).
-__host__ __device__ inline size_t u_tc_floats(int C, int K, int planes) {
-    return size_t((C + BC - 1) / BC) * ((K + BM - 1) / BM) * 16 * planes * (BM * BC);
+__host__ __device__ inline size_t u_tc_floats(int C, int K, int planes, int MM) {
+    return size_t((C + BC - 1) / BC) * ((K + MM - 1) / MM) * 16 * planes * (MM * BC);
 }
+// Tile height used for a shape: the filter transform and the conv must agree.
+#ifdef WINO_TC_MM64_ALL
+__host__ __device__ inline int tc_mm(int, int planes) { return planes == 1 ? 64 : 128; }  // A/B builds
+#else
+__host__ __device__ inline int tc_mm(int K, int planes) { return (planes == 1 && K <= 64) ? 64 : 128; }
+#endif
 
 // FTF (Eq. 5) straight into the tensor-core operand layout, rounded to TF32
 // (reading R8; 3xTF32 also stores small = rna(u - big)).  Pads K and C with zeros.
-template <int P>
+template <int P, int MM>
 __global__ void __launch_bounds__(256) tc_filter_kernel(const float* __restrict__ w, float* __restrict__ u_tc,
                                                         int C, int K) {
-    const int Kp = ((K + BM - 1) / BM) * BM, Cp = ((C + BC - 1) / BC) * BC;
+    const int Kp = ((K + MM - 1) / MM) * MM, Cp = ((C + BC - 1) / BC) * BC;
     const long idx = (long)blockIdx.x * 256 + threadIdx.x;
     if (idx >= (long)Cp * Kp) return;
     const int c = (int)(idx / Kp), k = (int)(idx - (long)c * Kp);
@@ -96,15 +105,15 @@ __global__ void __launch_bounds__(256) tc_filter_kernel(const float* __restrict_
 #pragma unroll
         for (int e = 0; e < 16; ++e) t[e] = 0.f;
     }
-    const int cb = c / BC, cl = c % BC, kb = k / BM, m = k % BM;
-    const int nkb = Kp / BM;
+    const int cb = c / BC, cl = c % BC, kb = k / MM, m = k % MM;
+    const int nkb = Kp / MM;
     const size_t inner = size_t((m >> 3) * 64 + (cl >> 2) * 32 + (m & 7) * 4 + (cl & 3));
 #pragma unroll
     for (int xi = 0; xi < 16; ++xi) {
-        const size_t base = ((((size_t)cb * nkb + kb) * 16 + xi) * P) * (BM * BC);
+        const size_t base = ((((size_t)cb * nkb + kb) * 16 + xi) * P) * (MM * BC);
         const float big = to_tf32(t[xi]);
         u_tc[base + inner] = big;
-        if (P == 2) u_tc[base + (BM * BC) + inner] = to_tf32(t[xi] - big);
+        if (P == 2) u_tc[base + (MM * BC) + inner] = to_tf32(t[xi] - big);
     }
 }
 
@@ -115,34 +124,41 @@ struct __align__(64) Params {
     float* __restrict__ y;
     int N, C, H, W, K;
     int TW, NV;
-    int num_kb;     // ceil(K/128)
+    int num_kb;     // ceil(K/MM)
     int num_cb;     // ceil(C/8)
-    int num_tiles;  // ceil(NV/32) * num_kb
+    int num_tiles;  // ceil(NV/(32*NH)) * num_kb
 };
 
-template <int P>
+template <int P, int MM, int XM>
 struct Cfg {
+    static constexpr int NH = 128 / MM;                         // nu-halves per tile (32 nu each)
     static constexpr int XPU = xi_per_unit<P>();
     static constexpr int UNITS_PER_CB = 16 / XPU;
-    static constexpr int UNIT = XPU * P * A_TILE;               // 64 KB
-    static constexpr int U_SLOTS = 2;                           // 128 KB of U in flight
+    static constexpr int A_TILE = a_tile<MM>();
+    static constexpr int UNIT = XPU * P * A_TILE;               // 64 KB (MM=128) / 32 KB (MM=64)
+    static constexpr int U_SLOTS = (MM == 64 && XM == 2) ? 3 : 2;
     static constexpr int X_SLOTS = 2;                           // raw x boxes in flight (L2-prefetched)
-    static constexpr int V_SLOT = 16 * P * B_TILE;             // 16 / 32 KB
+    static constexpr int X_SLOT = NH * XS_BYTES;
+    static constexpr int V_SLOT = 16 * NH * P * B_TILE;        // 16 / 32 KB
+    static constexpr int TAB = (XM == 2) ? 0 : 16 * BN * NH * 4;  // cp.async gather table
     static constexpr int OFF_U = 0;
     static constexpr int OFF_X = OFF_U + U_SLOTS * UNIT;
-    static constexpr int OFF_V = OFF_X + X_SLOTS * XS_BYTES;
-    static constexpr int OFF_TAB = OFF_V + 2 * V_SLOT;          // cp.async gather table (16*32 ints)
-    static constexpr int OFF_BAR = OFF_TAB + 16 * BN * 4;
+    static constexpr int OFF_V = OFF_X + X_SLOTS * X_SLOT;
+    static constexpr int OFF_TAB = OFF_V + 2 * V_SLOT;
+    static constexpr int OFF_BAR = OFF_TAB + TAB;
     // u_full/u_empty[U_SLOTS], x_full/x_empty[X_SLOTS], v_full[2], v_empty[2], acc_full, acc_empty
     static constexpr int NBAR = 2 * U_SLOTS + 2 * X_SLOTS + 6;
     static constexpr int OFF_TMEM = OFF_BAR + NBAR * 8;
     static constexpr int BYTES = OFF_TMEM + 16;
+    static_assert(BYTES <= 232448, "shared memory budget");
 };
 
 // XM: 2 = TMA x box (N % 32 == 0), 1 = cp.async 16 B gather, 0 = cp.async 4 B gather
-template <int P, int XM>
+template <int P, int XM, int MM>
 __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__ Params p) {
-    using G = Cfg<P>;
+    using G = Cfg<P, MM, XM>;
+    constexpr int NH = G::NH;
+    constexpr int TN = BN * NH;  // nu per tile
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t* const su = smem + G::OFF_U;
     float* const sx = reinterpret_cast<float*>(smem + G::OFF_X);
@@ -193,23 +209,30 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             // --------------------------- raw-x producer ---------------------------
             int gcb = 0;  // channel blocks issued so far (all tiles)
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-                const int nu0 = (tile / p.num_kb) * BN;
-                int tma_n0 = 0, tma_w0 = 0, tma_h0 = 0;
+                const int nu0 = (tile / p.num_kb) * TN;
+                int tma_n0[NH], tma_w0[NH], tma_h0[NH];
                 if constexpr (XM == 2) {
-                    const int t = nu0 / p.N;
-                    tma_n0 = nu0 - t * p.N;
-                    const int th = t / p.TW, tw = t - th * p.TW;
-                    tma_w0 = 2 * tw - 1;  // may be -1: TMA zero fill = implicit padding (Sec. 3.5)
-                    tma_h0 = 2 * th - 1;
+#pragma unroll
+                    for (int h = 0; h < NH; ++h) {  // N % 32 == 0: each half = 32 consecutive n of one image tile
+                        const int nuh = nu0 + h * BN;
+                        const int t = nuh < p.NV ? nuh / p.N : 0;
+                        tma_n0[h] = nuh < p.NV ? nuh - t * p.N : 0;
+                        const int th = t / p.TW, tw = t - th * p.TW;
+                        tma_w0[h] = nuh < p.NV ? 2 * tw - 1 : -8;  // -1: TMA zero fill = padding (Sec. 3.5);
+                        tma_h0[h] = nuh < p.NV ? 2 * th - 1 : -8;  // -8: half past NV -> all zeros
+                    }
                     // x streams from HBM (first touch): warm L2 a few blocks ahead
                     if (lane == 0)
                         for (int cb = 0; cb < X_PREFETCH && cb < NCB; ++cb)
-                            tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, cb * BC);
+#pragma unroll
+                            for (int h = 0; h < NH; ++h)
+                                tma_prefetch_l2_4d(&p.tmx, tma_n0[h], tma_w0[h], tma_h0[h], cb * BC);
                 } else {
                     // gather offsets (h*W+w)*N+n of the 4x4 window element pos of local nu (-1: padding)
                     __syncwarp();
-                    for (int e = lane; e < 16 * BN; e += 32) {
-                        const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
+                    for (int e = lane; e < 16 * TN; e += 32) {
+                        const int hh = e / (16 * BN), r = e % (16 * BN);
+                        const int pos = r / BN, nl = r % BN, nu = nu0 + hh * BN + nl;
                         int off = -1;
                         if (nu < p.NV) {
                             const int t = nu / p.N, n = nu - t * p.N;
@@ -224,23 +247,29 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                 for (int cb = 0; cb < NCB; ++cb, ++gcb) {
                     const int xs = gcb % G::X_SLOTS;
                     if (gcb >= G::X_SLOTS) mbar_wait(&x_empty[xs], ((gcb / G::X_SLOTS) - 1) & 1);
-                    float* xdst = sx + xs * (XS_BYTES / 4);
+                    float* xdst = sx + xs * (G::X_SLOT / 4);
                     if constexpr (XM == 2) {
                         if (lane == 0) {
-                            if (cb + X_PREFETCH < NCB)
-                                tma_prefetch_l2_4d(&p.tmx, tma_n0, tma_w0, tma_h0, (cb + X_PREFETCH) * BC);
-                            mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
-                            tma_load_4d(xdst, &p.tmx, &x_full[xs], tma_n0, tma_w0, tma_h0, cb * BC);
+                            mbar_arrive_expect_tx(&x_full[xs], G::X_SLOT);
+#pragma unroll
+                            for (int h = 0; h < NH; ++h) {
+                                if (cb + X_PREFETCH < NCB)
+                                    tma_prefetch_l2_4d(&p.tmx, tma_n0[h], tma_w0[h], tma_h0[h], (cb + X_PREFETCH) * BC);
+                                tma_load_4d(xdst + h * (XS_BYTES / 4), &p.tmx, &x_full[xs], tma_n0[h], tma_w0[h],
+                                            tma_h0[h], cb * BC);
+                            }
                         }
                     } else {
                         constexpr int VX = XM == 1 ? 4 : 1;
-                        for (int e = lane; e < BC * 16 * BN / VX; e += 32) {
-                            const int cl = e / (16 * BN / VX), r = (e % (16 * BN / VX)) * VX;
+                        constexpr int PER_C = 16 * BN / VX;  // vectors per (half, channel)
+                        for (int e = lane; e < NH * BC * PER_C; e += 32) {
+                            const int hh = e / (BC * PER_C), r0 = e % (BC * PER_C);
+                            const int cl = r0 / PER_C, r = (r0 % PER_C) * VX;
                             const int c = cb * BC + cl;
-                            const int off = xtab[r];
+                            const int off = xtab[hh * 16 * BN + r];
                             const bool ok = (c < p.C) && (off >= 0);
                             const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
-                            const uint32_t dst = smem_u32(xdst + cl * 16 * BN + r);
+                            const uint32_t dst = smem_u32(xdst + hh * (XS_BYTES / 4) + cl * 16 * BN + r);
                             if constexpr (VX == 4) cp_async16(dst, src, ok);
                             else cp_async4(dst, src, ok);
                         }
@@ -261,7 +290,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                         if (unit >= G::U_SLOTS) mbar_wait(&u_empty[us], ((unit / G::U_SLOTS) - 1) & 1);
                         if (lane == 0) {
                             const float* src =
-                                p.u_tc + ((((size_t)cb * p.num_kb + kb) * 16 + h * G::XPU) * P) * (BM * BC);
+                                p.u_tc + ((((size_t)cb * p.num_kb + kb) * 16 + h * G::XPU) * P) * (MM * BC);
                             mbar_arrive_expect_tx(&u_full[us], G::UNIT);
                             bulk_load(su + us * G::UNIT, src, G::UNIT, &u_full[us]);
                         }
@@ -270,7 +299,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             }
         } else if (warp == MMA_WARP) {
             // ------------------------------ MMA issuer ----------------------------
-            constexpr uint32_t IDESC = umma_idesc_tf32(BM, BN);
+            constexpr uint32_t IDESC = umma_idesc_tf32(MM, BN);
             int unit = 0, gcb = 0, it = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
                 if (it > 0) mbar_wait(acc_empty, (it - 1) & 1);  // epilogue drained TMEM
@@ -288,15 +317,21 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
 #pragma unroll
                             for (int q = 0; q < G::XPU; ++q) {
                                 const int xi = half * G::XPU + q;
-                                const uint32_t d = tmem + xi * BN;
-                                const uint32_t a0 = ubase + (q * P) * A_TILE, b0 = vbase + (xi * P) * B_TILE;
-                                const uint64_t ab = umma_desc(a0, 128, 256), bb = umma_desc(b0, 128, 256);
-                                umma_tf32(d, ab, bb, IDESC, cb > 0 ? 1u : 0u);
-                                if constexpr (P == 2) {
-                                    const uint64_t as = umma_desc(a0 + A_TILE, 128, 256);
-                                    const uint64_t bs = umma_desc(b0 + B_TILE, 128, 256);
-                                    umma_tf32(d, ab, bs, IDESC, 1u);
-                                    umma_tf32(d, as, bb, IDESC, 1u);
+                                const uint32_t a0 = ubase + (q * P) * G::A_TILE;
+                                const uint64_t ab = umma_desc(a0, 128, 256);
+#pragma unroll
+                                for (int h = 0; h < NH; ++h) {
+                                    // nu-half h accumulates in TMEM lanes 16h.. of each quadrant (MM = 64)
+                                    const uint32_t d = tmem + xi * BN + ((uint32_t)(16 * h) << 16);
+                                    const uint32_t b0 = vbase + ((xi * NH + h) * P) * B_TILE;
+                                    const uint64_t bb = umma_desc(b0, 128, 256);
+                                    umma_tf32(d, ab, bb, IDESC, cb > 0 ? 1u : 0u);
+                                    if constexpr (P == 2) {
+                                        const uint64_t as = umma_desc(a0 + G::A_TILE, 128, 256);
+                                        const uint64_t bs = umma_desc(b0 + B_TILE, 128, 256);
+                                        umma_tf32(d, ab, bs, IDESC, 1u);
+                                        umma_tf32(d, as, bb, IDESC, 1u);
+                                    }
                                 }
                             }
                             umma_commit(&u_empty[us]);
@@ -322,22 +357,28 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             for (int cb = 0; cb < NCB; ++cb, ++gcb) {
                 const int xs = gcb % G::X_SLOTS, vs = gcb & 1;
                 mbar_wait(&x_full[xs], (gcb / G::X_SLOTS) & 1);
-                const float* xsrc = sx + xs * (XS_BYTES / 4) + cl * 16 * BN + nl;
-                float d[16], t[16];
+                float t[NH][16];
 #pragma unroll
-                for (int e = 0; e < 16; ++e) d[e] = xsrc[e * BN];
-                itf_4x4(d, t);  // consumes the loads: the x slot can be released
+                for (int h = 0; h < NH; ++h) {
+                    const float* xsrc = sx + xs * (G::X_SLOT / 4) + h * (XS_BYTES / 4) + cl * 16 * BN + nl;
+                    float d[16];
+#pragma unroll
+                    for (int e = 0; e < 16; ++e) d[e] = xsrc[e * BN];
+                    itf_4x4(d, t[h]);  // consumes the loads
+                }
                 __syncwarp();
-                if (lane == 0) mbar_arrive(&x_empty[xs]);
+                if (lane == 0) mbar_arrive(&x_empty[xs]);  // the x slot can be refilled
                 if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
                 uint8_t* vdst = sv + vs * G::V_SLOT + voff;
 #pragma unroll
-                for (int xi = 0; xi < 16; ++xi) {
-                    const float big = to_tf32(t[xi]);
-                    *reinterpret_cast<float*>(vdst + (xi * P) * B_TILE) = big;
-                    if constexpr (P == 2)
-                        *reinterpret_cast<float*>(vdst + (xi * P + 1) * B_TILE) = to_tf32(t[xi] - big);
-                }
+                for (int h = 0; h < NH; ++h)
+#pragma unroll
+                    for (int xi = 0; xi < 16; ++xi) {
+                        const float big = to_tf32(t[h][xi]);
+                        *reinterpret_cast<float*>(vdst + ((xi * NH + h) * P) * B_TILE) = big;
+                        if constexpr (P == 2)
+                            *reinterpret_cast<float*>(vdst + ((xi * NH + h) * P + 1) * B_TILE) = to_tf32(t[h][xi] - big);
+                    }
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&v_full[vs]);
@@ -347,13 +388,15 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         setmaxnreg_inc<REG_EPI>();
         // ------------------------------ epilogue ------------------------------
         // thread = TMEM lane = filter k of the tile; all 32 nu of the 16 accumulators
-        const int kl = warp * 32 + lane;
+        // MM = 128: lane = filter; MM = 64: lanes 0-15 -> filters of nu-half 0, 16-31 -> nu-half 1
+        const int kl = (MM == 128) ? warp * 32 + lane : warp * 16 + (lane & 15);
+        const int hsel = (MM == 128) ? 0 : (lane >> 4);
         const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
         const size_t dW = (size_t)p.W * p.N;
         int it = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
-            const int k = (tile % p.num_kb) * BM + kl;
-            const int nu0 = (tile / p.num_kb) * BN;
+            const int k = (tile % p.num_kb) * MM + kl;
+            const int nu0 = (tile / p.num_kb) * TN + hsel * BN;
             mbar_wait(acc_full, it & 1);
             tc_fence_after();
             float o[BN][4];  // OTF results of this filter for the 32 nu
@@ -374,7 +417,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(acc_empty);  // TMEM free for the next tile's MMAs
-            if (k >= p.K) continue;
+            if (k >= p.K || nu0 >= p.NV) continue;
             if constexpr (XM == 2) {
                 // N % 32 == 0: the 32 nu are 32 consecutive n of one image tile -> 128 B rows
                 const int t = nu0 / p.N, n = nu0 - t * p.N;

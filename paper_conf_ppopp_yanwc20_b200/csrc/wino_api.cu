@@ -169,12 +169,12 @@ wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem,
 }  // namespace
 
 namespace {
-std::atomic<uint64_t> g_attr_tc[2][3];
-template <int P, int XM>
+std::atomic<uint64_t> g_attr_tc[2][3][2];
+template <int P, int XM, int MM>
 wino_status_t launch_tc(const wino::tc::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
-    auto kern = wino::tc::fused_tc_kernel<P, XM>;
-    const int smem = wino::tc::Cfg<P>::BYTES;
-    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc[P - 1][XM]);
+    auto kern = wino::tc::fused_tc_kernel<P, XM, MM>;
+    const int smem = wino::tc::Cfg<P, MM, XM>::BYTES;
+    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc[P - 1][XM][MM == 64]);
     if (s != WINO_OK) return s;
     kern<<<dim3(static_cast<unsigned>(ctas)), wino::tc::NT, smem, st>>>(prm);
     cudaError_t e = cudaGetLastError();
@@ -327,16 +327,17 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
     if (variant == 1 || variant == 2) {  // tcgen05 TF32 (1) / 3xTF32 (2)
         using namespace wino::tc;
         const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
+        const int mm = tc_mm(K, variant == 2 ? 2 : 1);
         plan->variant = variant;
-        plan->bk = BM;
-        plan->bn = BN;
+        plan->bk = mm;
+        plan->bn = BN * (128 / mm);
         plan->bc = BC;
         plan->load_x = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
         plan->load_u = 3;  // bulk copy of the pre-arranged operand tiles
         plan->split_c = 1;
-        plan->ctas = ((nv + BN - 1) / BN) * ((K + BM - 1) / BM);  // tiles (persistent grid <= #SMs)
+        plan->ctas = ((nv + plan->bn - 1) / plan->bn) * ((K + mm - 1) / mm);  // tiles (persistent grid <= #SMs)
         plan->threads = NT;
-        plan->smem_bytes = variant == 1 ? Cfg<1>::BYTES : Cfg<2>::BYTES;
+        plan->smem_bytes = variant == 1 ? (mm == 64 ? Cfg<1, 64, 2>::BYTES : Cfg<1, 128, 2>::BYTES) : Cfg<2, 128, 2>::BYTES;
         plan->launches = 1;
         return WINO_OK;
     }
@@ -373,7 +374,8 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
 
 size_t wino_filter_workspace_bytes_tc(int C, int K, wino_tc_mode_t mode) {
     if (C <= 0 || K <= 0 || (mode != WINO_TC_TF32 && mode != WINO_TC_3XTF32)) return 0;
-    return wino::tc::u_tc_floats(C, K, mode == WINO_TC_3XTF32 ? 2 : 1) * sizeof(float);
+    const int planes = mode == WINO_TC_3XTF32 ? 2 : 1;
+    return wino::tc::u_tc_floats(C, K, planes, wino::tc::tc_mm(K, planes)) * sizeof(float);
 }
 
 wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int C, int K, wino_tc_mode_t mode,
@@ -387,12 +389,15 @@ wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int 
     int dev;
     wino_status_t s = check_device(&dev);
     if (s != WINO_OK) return s;
-    const int64_t Kp = ((K + wino::tc::BM - 1) / wino::tc::BM) * wino::tc::BM;
+    const int planes = mode == WINO_TC_3XTF32 ? 2 : 1;
+    const int mm = wino::tc::tc_mm(K, planes);
+    const int64_t Kp = ((K + mm - 1) / mm) * mm;
     const int64_t Cp = ((C + wino::tc::BC - 1) / wino::tc::BC) * wino::tc::BC;
     const unsigned blocks = static_cast<unsigned>((Cp * Kp + 255) / 256);
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    if (mode == WINO_TC_TF32) wino::tc::tc_filter_kernel<1><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
-    else wino::tc::tc_filter_kernel<2><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
+    if (planes == 1 && mm == 64) wino::tc::tc_filter_kernel<1, 64><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
+    else if (planes == 1) wino::tc::tc_filter_kernel<1, 128><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
+    else wino::tc::tc_filter_kernel<2, 128><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
@@ -426,9 +431,12 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
     prm.K = K;
     prm.TW = (W + 1) / 2;
     prm.NV = N * ((H + 1) / 2) * prm.TW;
-    prm.num_kb = (K + BM - 1) / BM;
+    const int planes = mode == WINO_TC_3XTF32 ? 2 : 1;
+    const int mm = tc_mm(K, planes);
+    const int tn = BN * (128 / mm);
+    prm.num_kb = (K + mm - 1) / mm;
     prm.num_cb = (C + BC - 1) / BC;
-    prm.num_tiles = ((prm.NV + BN - 1) / BN) * prm.num_kb;
+    prm.num_tiles = ((prm.NV + tn - 1) / tn) * prm.num_kb;
     const int xm = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
     if (xm == 2) {
         const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
@@ -438,14 +446,19 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
     const int sms = sm_count(dev);
     const int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    if (mode == WINO_TC_TF32) {
-        if (xm == 2) return launch_tc<1, 2>(prm, ctas, dev, st);
-        if (xm == 1) return launch_tc<1, 1>(prm, ctas, dev, st);
-        return launch_tc<1, 0>(prm, ctas, dev, st);
+    if (mode == WINO_TC_TF32 && mm == 64) {
+        if (xm == 2) return launch_tc<1, 2, 64>(prm, ctas, dev, st);
+        if (xm == 1) return launch_tc<1, 1, 64>(prm, ctas, dev, st);
+        return launch_tc<1, 0, 64>(prm, ctas, dev, st);
     }
-    if (xm == 2) return launch_tc<2, 2>(prm, ctas, dev, st);
-    if (xm == 1) return launch_tc<2, 1>(prm, ctas, dev, st);
-    return launch_tc<2, 0>(prm, ctas, dev, st);
+    if (mode == WINO_TC_TF32) {
+        if (xm == 2) return launch_tc<1, 2, 128>(prm, ctas, dev, st);
+        if (xm == 1) return launch_tc<1, 1, 128>(prm, ctas, dev, st);
+        return launch_tc<1, 0, 128>(prm, ctas, dev, st);
+    }
+    if (xm == 2) return launch_tc<2, 2, 128>(prm, ctas, dev, st);
+    if (xm == 1) return launch_tc<2, 1, 128>(prm, ctas, dev, st);
+    return launch_tc<2, 0, 128>(prm, ctas, dev, st);
 }
 
 

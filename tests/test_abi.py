@@ -112,12 +112,16 @@ def test_tc_workspace_and_plan():
     # [ceil(C/8)][ceil(K/128)][16 xi][planes][128 x 8] floats
     for (C, K) in [(1, 1), (8, 128), (9, 129), (512, 512), (64, 64)]:
         for mode, planes in [("tf32", 1), ("3xtf32", 2)]:
-            want = -(-C // 8) * -(-K // 128) * 16 * planes * 128 * 8 * 4
+            mm = 64 if (planes == 1 and K <= 64) else 128  # tile height rule of the tc kernel
+            want = -(-C // 8) * -(-K // mm) * 16 * planes * mm * 8 * 4
             assert wino.filter_workspace_bytes_tc(C, K, mode) == want
     assert wino.lib().wino_filter_workspace_bytes_tc(8, 8, 5) == 0
     c = CONFIGS["conv3_x"]
     p = wino.plan(c.N, c.C, c.H, c.W, c.K, variant=1)
-    assert (p.bk, p.bn, p.bc, p.threads) == (128, 32, 8, 352)
+    assert (p.bk, p.bn, p.bc, p.threads) == (128, 32, 8, 512)
+    c2 = CONFIGS["conv2_x"]  # K = 64: 64-filter tiles with two nu-halves in TMEM
+    p2 = wino.plan(c2.N, c2.C, c2.H, c2.W, c2.K, variant=1)
+    assert (p2.bk, p2.bn) == (64, 64)
     assert p.ctas == -(-(c.N * c.tiles) // 32) * -(-c.K // 128)
     assert p.smem_bytes <= 232448 and wino.plan(c.N, c.C, c.H, c.W, c.K, variant=2).smem_bytes <= 232448
 
