@@ -2,11 +2,12 @@
 //
 // Same method, tiling and FFMA micro-kernel as fused_fp32.cuh (Yan, Wang & Chu,
 // Sec. 3-4, Alg. 1), re-organised for Blackwell:
-//   * warpgroups 0-1 (8 warps, 224 registers each via setmaxnreg) only run the
+//   * warpgroups 0-1 (8 warps, 208 registers each via setmaxnreg) only run the
 //     16-batched GEMM (LDS.128 fragments + FFMA, Fig. 3 arrangement, bank-aware
 //     order) and the output transform;
-//   * warpgroup 2 (56 registers): one warp issues the TMA boxes, three perform
-//     the ITF (Eq. 6) of the coming stages into a ring of V buffers;
+//   * warpgroup 2 (88 registers): one warp issues the TMA boxes, two perform
+//     the ITF (Eq. 6) of the coming stages (LDS.128 / STS.128 along nu) into a
+//     ring of V buffers;
 //   * stages are handed over with mbarriers (full / empty / V-full / V-empty),
 //     so the compute warps never wait at a CTA-wide barrier and never stall on
 //     the ITF's load-to-use latency (the paper interleaves ITF and FFMA in one
@@ -42,8 +43,8 @@ constexpr int NT = 384;             // 2 compute warpgroups + 1 producer/ITF war
 constexpr int COMPUTE_THREADS = 256;
 constexpr int S = 3;                // TMA stage ring (u 32 KB + raw x 16 KB per stage)
 constexpr int SV = 2;               // V ring (16 KB each)
-constexpr int REG_COMPUTE = 224, REG_PRODUCER = 56;  // 256*224 + 128*56 = 64512 <= 65536
-constexpr int ITF_WARPS = 3;        // warps 9..11; warp 8 only issues TMA
+constexpr int REG_COMPUTE = 208, REG_PRODUCER = 88;  // 256*208 + 128*88 = 64512 <= 65536
+constexpr int ITF_WARPS = 2;        // warps 9..10 (float4 along nu); warp 8 only issues TMA; 11 idle
 constexpr int ER_LD = BN + 4;       // padded row of the epilogue buffer
 constexpr int ER_KROWS = 16;        // filters per epilogue round
 constexpr int ER_FLOATS = 16 * ER_KROWS * ER_LD;  // [xi][16 k][36]
@@ -110,30 +111,32 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             }
             return;
         }
-        // ---------------- ITF (Sec. 4.2) on warps 9..11 ----------------
-        // 256 (c, nu) tiles per stage; lanes along nu (conflict-free LDS and STS),
-        // warp w handles channels c = (w - 9) + 3j.
-        const int cw = warp - 9;
+        // ---------------- ITF (Sec. 4.2) on warps 9..10 ----------------
+        // 256 (c, nu) tiles per stage; a thread transforms 4 consecutive nu of one
+        // channel with LDS.128 / STS.128 (a quarter-warp covers one 128 B row:
+        // conflict-free): lane -> (c = 4 (w - 9) + lane / 8, nu4 = lane % 8).
+        if (warp > 8 + ITF_WARPS) return;
+        const int c = 4 * (warp - 9) + (lane >> 3), n4 = 4 * (lane & 7);
         int G = 0;
         for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
             for (int g = 0; g < NIT; ++g, ++G) {
                 const int slot = G % S, vb = G % SV;
                 mbar_wait(&full[slot], (G / S) & 1);
                 if (G >= SV) mbar_wait(&vempty[vb], ((G / SV) - 1) & 1);
-                const float* xs = smem + slot * STAGE_FLOATS + US_FLOATS + lane;
-                float* v = vs + vb * VS_FLOATS + lane;
+                const float* xs = smem + slot * STAGE_FLOATS + US_FLOATS + c * 16 * BN + n4;
+                float* v = vs + vb * VS_FLOATS + c * BN + n4;
+                float d[4][16];
 #pragma unroll
-                for (int j = 0; j < 3; ++j) {
-                    const int c = cw + 3 * j;
-                    if (c < BC) {
-                        float d[16], t[16];
-#pragma unroll
-                        for (int e = 0; e < 16; ++e) d[e] = xs[(c * 16 + e) * BN];
-                        itf_4x4(d, t);
-#pragma unroll
-                        for (int e = 0; e < 16; ++e) v[(e * BC + c) * BN] = t[e];
-                    }
+                for (int e = 0; e < 16; ++e) {
+                    const float4 q = *reinterpret_cast<const float4*>(xs + e * BN);
+                    d[0][e] = q.x; d[1][e] = q.y; d[2][e] = q.z; d[3][e] = q.w;
                 }
+                float t[4][16];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) itf_4x4(d[j], t[j]);
+#pragma unroll
+                for (int e = 0; e < 16; ++e)
+                    *reinterpret_cast<float4*>(v + e * BC * BN) = make_float4(t[0][e], t[1][e], t[2][e], t[3][e]);
                 __syncwarp();
                 if (lane == 0) {
                     mbar_arrive(&empty[slot]);  // raw x of this slot consumed

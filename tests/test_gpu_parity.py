@@ -46,6 +46,9 @@ EDGE = [
     (1, 1, 1, 1, 1), (1, 8, 8, 8, 8), (3, 7, 5, 5, 5), (2, 9, 65, 7, 7), (33, 8, 64, 3, 3),
     (4, 20, 70, 13, 9), (5, 17, 130, 6, 10), (64, 16, 128, 2, 2), (1, 3, 3, 1, 17),
     (6, 12, 3, 14, 1), (32, 24, 96, 4, 6), (2, 64, 64, 16, 16), (7, 40, 72, 11, 12),
+    # persistent warp-specialised FP32 path (N % 32 == 0, K % 4 == 0): C tails, K tails,
+    # odd planes, more tiles than SMs
+    (32, 7, 68, 5, 9), (64, 13, 132, 3, 7), (96, 1, 4, 9, 2), (32, 16, 64, 40, 40),
 ]
 
 
