@@ -59,6 +59,13 @@ def _load():
         for name in ("oracle_ftf_tile", "oracle_itf_tile", "oracle_otf_tile"):
             getattr(lib, name).argtypes = [dp, dp]
             getattr(lib, name).restype = None
+        lib.oracle_filter_transform_f4.argtypes = [dp, dp, i, i]
+        lib.oracle_filter_transform_f4.restype = None
+        lib.oracle_winograd_f4_conv.argtypes = [dp, dp, dp, i, i, i, i, i]
+        lib.oracle_winograd_f4_conv.restype = ctypes.c_int
+        for name in ("oracle_ftf4_tile", "oracle_itf4_tile", "oracle_otf4_tile"):
+            getattr(lib, name).argtypes = [dp, dp]
+            getattr(lib, name).restype = None
         lib.oracle_num_threads.argtypes = []
         lib.oracle_num_threads.restype = ctypes.c_int
         _lib = lib
@@ -126,6 +133,38 @@ def winograd_conv(x_chwn, w_crsk, return_u: bool = False):
     if rc != 0:
         raise MemoryError("oracle_winograd_conv: allocation failed")
     return (y, u) if return_u else y
+
+
+def filter_transform_f4(w_crsk) -> np.ndarray:
+    """NEXT row N1: F(4x4,3x3) filter transform U4 (C,6,6,K) = G4 w G4^T (Lavin-Gray matrices)."""
+    w = _f64(w_crsk)
+    C, K = w.shape[0], w.shape[3]
+    u = np.empty((C, 6, 6, K), dtype=np.float64)
+    _load().oracle_filter_transform_f4(_ptr(w), _ptr(u), C, K)
+    return u
+
+
+def winograd_f4_conv(x_chwn, w_crsk) -> np.ndarray:
+    """NEXT row N1: naive F(4x4,3x3) Winograd conv in fp64 (same steps as Eq. 5-8, alpha = 6)."""
+    x, w = _f64(x_chwn), _f64(w_crsk)
+    C, H, W, N = x.shape
+    K = w.shape[3]
+    y = np.empty((K, H, W, N), dtype=np.float64)
+    if _load().oracle_winograd_f4_conv(_ptr(x), _ptr(w), _ptr(y), N, C, H, W, K) != 0:
+        raise MemoryError("oracle_winograd_f4_conv: allocation failed")
+    return y
+
+
+def ftf4_tile(g3x3) -> np.ndarray:
+    return _tile("oracle_ftf4_tile", g3x3, 36).reshape(6, 6)
+
+
+def itf4_tile(d6x6) -> np.ndarray:
+    return _tile("oracle_itf4_tile", d6x6, 36).reshape(6, 6)
+
+
+def otf4_tile(m6x6) -> np.ndarray:
+    return _tile("oracle_otf4_tile", m6x6, 16).reshape(4, 4)
 
 
 def _tile(fn, inp, n_out):

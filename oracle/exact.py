@@ -111,3 +111,34 @@ def convolve_tile_flipped(d, g):
     """2x2 valid *convolution* (flipped filter) -- used to show the orientation."""
     return [[sum((d[y + r][x + s] * g[2 - r][2 - s] for r in range(3) for s in range(3)), Fr(0))
              for x in range(2)] for y in range(2)]
+
+
+# --------------------------------------------------------------------------
+# NEXT row N1: F(4x4,3x3) (Lavin-Gray matrices, points 0, +-1, +-2, inf).
+# PAPER.md gives no F(4x4) matrices (it cites [11, 26], L117); these are pinned
+# only by the exact identity below (tests/test_oracle.py).
+# --------------------------------------------------------------------------
+AT4 = [[Fr(v) for v in row] for row in [[1, 1, 1, 1, 1, 0], [0, 1, -1, 2, -2, 0], [0, 1, 1, 4, 4, 0],
+                                         [0, 1, -1, 8, -8, 1]]]
+G4 = [[Fr(1, 4), Fr(0), Fr(0)],
+      [Fr(-1, 6), Fr(-1, 6), Fr(-1, 6)],
+      [Fr(-1, 6), Fr(1, 6), Fr(-1, 6)],
+      [Fr(1, 24), Fr(1, 12), Fr(1, 6)],
+      [Fr(1, 24), Fr(-1, 12), Fr(1, 6)],
+      [Fr(0), Fr(0), Fr(1)]]
+BT4 = [[Fr(v) for v in row] for row in [[4, 0, -5, 0, 1, 0], [0, -4, -4, 1, 1, 0], [0, 4, -4, -1, 1, 0],
+                                         [0, -2, -1, 2, 1, 0], [0, 2, -1, -2, 1, 0], [0, 4, 0, -5, 0, 1]]]
+
+
+def winograd_f4_tile(d, g):
+    """F(4x4,3x3): AT4 [(G4 g G4^T) (.) (BT4 d BT4^T)] AT4^T for a 6x6 tile d, 3x3 filter g."""
+    u = matmul(matmul(G4, g), transpose(G4))
+    v = matmul(matmul(BT4, d), transpose(BT4))
+    m = [[u[i][j] * v[i][j] for j in range(6)] for i in range(6)]
+    return matmul(matmul(AT4, m), transpose(AT4))
+
+
+def correlate_tile_f4(d, g):
+    """Brute force: 4x4 valid correlation of a 6x6 tile with a 3x3 filter."""
+    return [[sum((d[y + r][x + s] * g[r][s] for r in range(3) for s in range(3)), Fr(0))
+             for x in range(4)] for y in range(4)]

@@ -256,3 +256,135 @@ int oracle_winograd_conv(const double* x, const double* w, double* y, double* u_
     if (!u_out) free(U);
     return failed;
 }
+
+/* ========================================================================= *
+ * NEXT row N1: Winograd F(4x4,3x3).  PAPER.md only points to
+ * the matrices ("the transformation matrices for ... F(4x4,3x3) ... are also
+ * given in [11, 26]", L117; "We expect greater speedup in the future if the
+ * fused F(4x4,3x3) is well optimized", L1271).  The matrices below are the
+ * Lavin-Gray F(4x4,3x3) ones (interpolation points 0, +-1, +-2, inf); they are
+ * pinned by the exact-rational identity tests (tests/test_oracle.py), not by
+ * the paper's text.  Same steps as Eq. 5-8 with alpha = 6, 4x4 outputs per tile.
+ * ========================================================================= */
+static const double AT4[4][6] = {{1, 1, 1, 1, 1, 0},
+                                 {0, 1, -1, 2, -2, 0},
+                                 {0, 1, 1, 4, 4, 0},
+                                 {0, 1, -1, 8, -8, 1}};
+static const double G4[6][3] = {{1.0 / 4, 0, 0},
+                                {-1.0 / 6, -1.0 / 6, -1.0 / 6},
+                                {-1.0 / 6, 1.0 / 6, -1.0 / 6},
+                                {1.0 / 24, 1.0 / 12, 1.0 / 6},
+                                {1.0 / 24, -1.0 / 12, 1.0 / 6},
+                                {0, 0, 1}};
+static const double BT4[6][6] = {{4, 0, -5, 0, 1, 0},
+                                 {0, -4, -4, 1, 1, 0},
+                                 {0, 4, -4, -1, 1, 0},
+                                 {0, -2, -1, 2, 1, 0},
+                                 {0, 2, -1, -2, 1, 0},
+                                 {0, 4, 0, -5, 0, 1}};
+
+/* U = G4 g G4^T (6x6) */
+void oracle_ftf4_tile(const double* g9, double* u36) {
+    double t[6][3];
+    for (int a = 0; a < 6; ++a)
+        for (int b = 0; b < 3; ++b) {
+            double s = 0.0;
+            for (int m = 0; m < 3; ++m) s += G4[a][m] * g9[m * 3 + b];
+            t[a][b] = s;
+        }
+    for (int a = 0; a < 6; ++a)
+        for (int b = 0; b < 6; ++b) {
+            double s = 0.0;
+            for (int m = 0; m < 3; ++m) s += t[a][m] * G4[b][m];
+            u36[a * 6 + b] = s;
+        }
+}
+/* V = BT4 d BT4^T (6x6) */
+void oracle_itf4_tile(const double* d36, double* v36) {
+    double t[6][6];
+    for (int a = 0; a < 6; ++a)
+        for (int b = 0; b < 6; ++b) {
+            double s = 0.0;
+            for (int m = 0; m < 6; ++m) s += BT4[a][m] * d36[m * 6 + b];
+            t[a][b] = s;
+        }
+    for (int a = 0; a < 6; ++a)
+        for (int b = 0; b < 6; ++b) {
+            double s = 0.0;
+            for (int m = 0; m < 6; ++m) s += t[a][m] * BT4[b][m];
+            v36[a * 6 + b] = s;
+        }
+}
+/* Y = AT4 M AT4^T (4x4) */
+void oracle_otf4_tile(const double* m36, double* o16) {
+    double t[4][6];
+    for (int a = 0; a < 4; ++a)
+        for (int b = 0; b < 6; ++b) {
+            double s = 0.0;
+            for (int q = 0; q < 6; ++q) s += AT4[a][q] * m36[q * 6 + b];
+            t[a][b] = s;
+        }
+    for (int a = 0; a < 4; ++a)
+        for (int b = 0; b < 4; ++b) {
+            double s = 0.0;
+            for (int q = 0; q < 6; ++q) s += t[a][q] * AT4[b][q];
+            o16[a * 4 + b] = s;
+        }
+}
+
+/* U4 (C,6,6,K) */
+void oracle_filter_transform_f4(const double* w, double* u, int C, int K) {
+#pragma omp parallel for schedule(static)
+    for (long ck = 0; ck < (long)C * K; ++ck) {
+        int c = (int)(ck / K), k = (int)(ck % K);
+        double g[9], t[36];
+        for (int e = 0; e < 9; ++e) g[e] = w[((size_t)c * 9 + e) * K + k];
+        oracle_ftf4_tile(g, t);
+        for (int e = 0; e < 36; ++e) u[((size_t)c * 36 + e) * K + k] = t[e];
+    }
+}
+
+/* Naive F(4x4,3x3) Winograd conv, pad 1: windows start at (4th-1, 4tw-1). */
+int oracle_winograd_f4_conv(const double* x, const double* w, double* y, int N, int C, int H, int W, int K) {
+    double* U = (double*)malloc(sizeof(double) * 36 * (size_t)C * K);
+    if (!U) return 1;
+    oracle_filter_transform_f4(w, U, C, K);
+    int TH = (H + 3) / 4, TW = (W + 3) / 4;
+    int failed = 0;
+#pragma omp parallel
+    {
+        double* V = (double*)malloc(sizeof(double) * 36 * (size_t)C * N);
+        if (!V) {
+#pragma omp atomic write
+            failed = 1;
+        }
+#pragma omp for schedule(dynamic, 1)
+        for (long t = 0; t < (long)TH * TW; ++t) {
+            if (!V) continue;
+            int th = (int)(t / TW), tw = (int)(t % TW);
+            for (int c = 0; c < C; ++c)
+                for (int n = 0; n < N; ++n) {
+                    double d[36];
+                    for (int a = 0; a < 6; ++a)
+                        for (int b = 0; b < 6; ++b) d[a * 6 + b] = xhat(x, N, H, W, c, 4 * th - 1 + a, 4 * tw - 1 + b, n);
+                    oracle_itf4_tile(d, V + ((size_t)c * N + n) * 36);
+                }
+            for (int k = 0; k < K; ++k)
+                for (int n = 0; n < N; ++n) {
+                    double m[36], o[16];
+                    for (int e = 0; e < 36; ++e) m[e] = 0.0;
+                    for (int c = 0; c < C; ++c)
+                        for (int e = 0; e < 36; ++e) m[e] += U[((size_t)c * 36 + e) * K + k] * V[((size_t)c * N + n) * 36 + e];
+                    oracle_otf4_tile(m, o);
+                    for (int a = 0; a < 4; ++a)
+                        for (int b = 0; b < 4; ++b) {
+                            int i = 4 * th + a, j = 4 * tw + b;
+                            if (i < H && j < W) y[(((size_t)k * H + i) * W + j) * N + n] = o[a * 4 + b];
+                        }
+                }
+        }
+        free(V);
+    }
+    free(U);
+    return failed;
+}

@@ -279,3 +279,38 @@ def test_max_rel_err_metric():
     assert oracle.max_rel_err(ref + np.array([0, 0.004, 0]), ref) == pytest.approx(1e-3)
     assert oracle.max_rel_err(np.zeros(3), np.zeros(3)) == 0.0
     assert oracle.max_rel_err(np.ones(3), np.zeros(3)) == float("inf")
+
+
+# --------------------------------------------------------------------------
+# NEXT row N1: F(4x4,3x3) oracle pins
+# --------------------------------------------------------------------------
+def test_f4_identity_exact_rational():
+    rng = random.Random(44)
+    for _ in range(60):
+        d = [[_rand_frac(rng) for _ in range(6)] for _ in range(6)]
+        g = [[_rand_frac(rng) for _ in range(3)] for _ in range(3)]
+        assert exact.winograd_f4_tile(d, g) == exact.correlate_tile_f4(d, g)
+
+
+def test_f4_c_tiles_match_exact():
+    rng = random.Random(45)
+    as_np = lambda a: np.array([[float(v) for v in r] for r in a])
+    for _ in range(50):
+        g = [[Fr(rng.randint(-9, 9)) for _ in range(3)] for _ in range(3)]
+        d = [[Fr(rng.randint(-9, 9)) for _ in range(6)] for _ in range(6)]
+        m = [[Fr(rng.randint(-9, 9)) for _ in range(6)] for _ in range(6)]
+        u = exact.matmul(exact.matmul(exact.G4, g), exact.transpose(exact.G4))
+        v = exact.matmul(exact.matmul(exact.BT4, d), exact.transpose(exact.BT4))
+        o = exact.matmul(exact.matmul(exact.AT4, m), exact.transpose(exact.AT4))
+        assert np.allclose(oracle.ftf4_tile(as_np(g)), as_np(u), rtol=0, atol=1e-13)
+        assert np.array_equal(oracle.itf4_tile(as_np(d)), as_np(v))
+        assert np.array_equal(oracle.otf4_tile(as_np(m)), as_np(o))
+
+
+@pytest.mark.parametrize("shape", [(2, 3, 4, 7, 7), (1, 8, 5, 8, 8), (3, 5, 2, 1, 9), (2, 16, 8, 14, 13)])
+def test_f4_winograd_vs_direct(shape):
+    N, C, K, H, W = shape
+    rng = np.random.default_rng(9 + C)
+    x = rng.uniform(-1, 1, (C, H, W, N))
+    w = rng.uniform(-1, 1, (C, 3, 3, K))
+    assert oracle.max_rel_err(oracle.winograd_f4_conv(x, w), oracle.direct_conv(x, w)) <= 1e-12
