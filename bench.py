@@ -288,13 +288,23 @@ def main():
     def measure(variant, sample_clocks):
         """Warm up, capture the step in a CUDA graph, time args.steps replays (L2 flushed
         before each, outside the events), then a per-layer breakdown.  Max over ranks."""
-        tc = variant != "fp32"
-        vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[variant]
-        launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=vid).launches
-                       for d in per if d["n"] > 0)
+        f4 = variant == "f4_fp32"  # NEXT row N1: fused F(4x4,3x3), FTF4 + one fused launch per layer
+        tc = variant in ("tf32", "3xtf32")
+        if f4:
+            launches = sum(2 for d in per if d["n"] > 0)
+        else:
+            vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[variant]
+            launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K,
+                                         variant=vid).launches for d in per if d["n"] > 0)
         for d in per:
             # transformed filter: computed on rank 0, broadcast once over NVLink (NCCL)
-            if tc:
+            if f4:
+                d["u"] = torch.empty((d["cfg"].C, 6, 6, d["cfg"].K), dtype=torch.float32, device=dev)
+                if rank == 0:
+                    wino.filter_transform_f4(d["w"], out=d["u"])
+                if world > 1:
+                    dist.broadcast(d["u"], src=0)
+            elif tc:
                 d["u"] = wino.filter_transform_tc(d["w"], variant)
                 if world > 1:
                     dist.broadcast(d["u"].data, src=0)
@@ -309,12 +319,16 @@ def main():
             if d["n"] == 0:
                 return
             if ftf:
-                if tc:
+                if f4:
+                    wino.filter_transform_f4(d["w"], out=d["u"])
+                elif tc:
                     wino.filter_transform_tc(d["w"], variant, out=d["u"])
                 else:
                     wino.filter_transform(d["w"], out=d["u"])
             if conv:
-                if tc:
+                if f4:
+                    wino.conv2d_f4(d["x"], d["u"], out=d["y"])
+                elif tc:
                     wino.conv2d_tc(d["x"], d["u"], out=d["y"])
                 else:
                     wino.conv2d(d["x"], d["u"], out=d["y"])
@@ -395,7 +409,9 @@ def main():
     main_m = measure(args.variant, sample_clocks=True)
     others = {}
     if not args.no_variants:
-        for v in ("fp32", "tf32", "3xtf32"):
+        for v in ("fp32", "tf32", "3xtf32", "f4_fp32"):
+            if v == "f4_fp32" and any(d["n"] % 16 for d in per if d["n"]):
+                continue  # the F(4x4) kernel needs N % 16 == 0 per rank
             if v != args.variant:
                 others[v] = measure(v, sample_clocks=False)
     ms_step, conv_ms, ftf_ms = main_m["ms_step"], main_m["conv_ms"], main_m["ftf_ms"]
@@ -489,8 +505,8 @@ def main():
         vrep[v] = {"value": val, "ms_per_step": m["ms_step"], "pct_fp32_peak_eff": 100 * val / fp32_peak,
                    "layers_eff_tflops": {d["cfg"].name: d["cfg"].eff_flops / (m["conv_ms"][i] * 1e-3) / 1e12
                                          for i, d in enumerate(per) if d["n"]},
-                   "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4}[v]}
-        if v != "fp32":
+                   "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4}[v]}
+        if v in ("tf32", "3xtf32"):
             ach = ewmm_flops / (sum(m["conv_ms"]) * 1e-3) / 1e12
             mult = 3 if v == "3xtf32" else 1
             vrep[v]["roofline"] = {"bound": "tensor", "achieved": ach * mult, "peak": tf32_peak,

@@ -146,6 +146,22 @@ wino_status_t wino_conv2d_f2x3_fwd_host(const float* x_host, const float* w_host
                                         void* ws_dev, size_t ws_bytes, wino_stream_t stream);
 
 /*
+ * NEXT row N1: fused Winograd F(4x4,3x3), FP32 FFMA.  The paper
+ * restricts itself to F(2x2,3x3) (L117) and anticipates a well-optimised fused
+ * F(4x4,3x3) (Sec. 8.1).  Lavin-Gray matrices (6x6 windows at stride 4,
+ * 36 Winograd elements, 4x4 outputs per tile); same computation (Eq. 4).
+ *   u4 : (C,6,6,K) = G4 w G4^T, element (r',s') at [c][r'][s'][k]
+ *        (36*C*K floats, wino_filter_workspace_bytes_f4)
+ * The fused kernel needs N % 16 == 0 and K % 4 == 0 (TMA boxes); other shapes
+ * return WINO_ERR_UNSUPPORTED.  Otherwise arguments and errors as the F(2x2) calls.
+ */
+size_t wino_filter_workspace_bytes_f4(int C, int K);
+wino_status_t wino_filter_transform_f4(const float* w_dev, float* u4_dev, int C, int K, wino_stream_t stream);
+wino_status_t wino_conv2d_f4x3_fwd(const float* x_dev, const float* u4_dev, float* y_dev,
+                                   int N, int C, int H, int W, int K, int pad, int stride,
+                                   wino_stream_t stream);
+
+/*
  * Multi-layer end-to-end call on HOST buffers with copy/compute overlap: for
  * each layer the weights and input are copied in on a library-owned copy-in
  * stream, the FTF + fused FP32 convolution run on `stream`, and the output is

@@ -23,6 +23,7 @@ __all__ = [
     "conv2d_host", "host_workspace_bytes", "plan", "Plan", "TC_TF32", "TC_3XTF32",
     "TcFilter", "filter_workspace_bytes_tc", "filter_transform_tc", "conv2d_tc",
     "host_multi_workspace_bytes", "conv2d_host_multi",
+    "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -109,6 +110,12 @@ def lib() -> ctypes.CDLL:
     L.wino_host_multi_workspace_bytes.argtypes = [ctypes.POINTER(_HostLayer), i]
     L.wino_conv2d_f2x3_fwd_host_multi.restype = i
     L.wino_conv2d_f2x3_fwd_host_multi.argtypes = [ctypes.POINTER(_HostLayer), i, vp, st, vp]
+    L.wino_filter_workspace_bytes_f4.restype = st
+    L.wino_filter_workspace_bytes_f4.argtypes = [i, i]
+    L.wino_filter_transform_f4.restype = i
+    L.wino_filter_transform_f4.argtypes = [vp, vp, i, i, vp]
+    L.wino_conv2d_f4x3_fwd.restype = i
+    L.wino_conv2d_f4x3_fwd.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
     L.wino_plan.restype = i
     L.wino_plan.argtypes = [i, i, i, i, i, i, ctypes.POINTER(_Plan)]
     _lib = L
@@ -255,6 +262,50 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
         if variant != "fp32":
             raise ValueError(f"conv2d runs the FP32 kernel; use conv2d_tc for {variant!r}")
         _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
+    return out
+
+
+def filter_workspace_bytes_f4(C: int, K: int) -> int:
+    return int(lib().wino_filter_workspace_bytes_f4(C, K))
+
+
+def filter_transform_f4(w: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """NEXT row N1: F(4x4,3x3) filter transform w (C,3,3,K) -> u4 (C,6,6,K) on the GPU."""
+    _need_cuda_f32(w, "w", 4)
+    C, r, s, K = w.shape
+    if (r, s) != (3, 3):
+        raise ValueError(f"w must be (C,3,3,K), got {tuple(w.shape)}")
+    if out is None:
+        out = torch.empty((C, 6, 6, K), dtype=torch.float32, device=w.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (C, 6, 6, K):
+        raise ValueError("out must be (C,6,6,K)")
+    with torch.cuda.device(w.device):
+        _check(lib().wino_filter_transform_f4(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                              C, K, _stream_ptr(stream)), "wino_filter_transform_f4")
+    return out
+
+
+def conv2d_f4(x: torch.Tensor, u4: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """NEXT row N1: fused Winograd F(4x4,3x3) forward conv (FP32), pad 1 stride 1:
+    x (C,H,W,N), u4 (C,6,6,K) -> y (K,H,W,N).  Needs N % 16 == 0 and K % 4 == 0."""
+    _need_cuda_f32(x, "x", 4)
+    _need_cuda_f32(u4, "u4", 4)
+    C, H, W, N = x.shape
+    if u4.shape[0] != C or tuple(u4.shape[1:3]) != (6, 6):
+        raise ValueError(f"u4 must be (C,6,6,K) with C={C}, got {tuple(u4.shape)}")
+    if u4.device != x.device:
+        raise ValueError("x and u4 must be on the same device")
+    K = u4.shape[3]
+    if out is None:
+        out = torch.empty((K, H, W, N), dtype=torch.float32, device=x.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (K, H, W, N):
+        raise ValueError("out must be (K,H,W,N)")
+    with torch.cuda.device(x.device):
+        _check(lib().wino_conv2d_f4x3_fwd(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u4.data_ptr()),
+                                          ctypes.c_void_p(out.data_ptr()), N, C, H, W, K, 1, 1,
+                                          _stream_ptr(stream)), "wino_conv2d_f4x3_fwd")
     return out
 
 

@@ -17,6 +17,7 @@
 #include "fused_fp32.cuh"
 #include "fused_fp32_ws.cuh"
 #include "fused_tc.cuh"
+#include "fused_f4_fp32.cuh"
 
 namespace {
 
@@ -155,6 +156,7 @@ bool encode_map(CUtensorMap* m, const float* base, int rank, const cuuint64_t* d
 
 std::atomic<uint64_t> g_attr_fp32[3][3];
 std::atomic<uint64_t> g_attr_ws;
+std::atomic<uint64_t> g_attr_f4;
 
 template <int XM, int UM>
 wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem, int dev, cudaStream_t st) {
@@ -603,6 +605,72 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
     WINO_TRY(cudaStreamWaitEvent(st, eo, 0));  // caller's stream completes after every copy
 #undef WINO_TRY
     return WINO_OK;
+}
+
+size_t wino_filter_workspace_bytes_f4(int C, int K) {
+    if (C <= 0 || K <= 0) return 0;
+    return size_t(36) * size_t(C) * size_t(K) * sizeof(float);
+}
+
+wino_status_t wino_filter_transform_f4(const float* w_dev, float* u4_dev, int C, int K, wino_stream_t stream) {
+    if (!w_dev || !u4_dev || C <= 0 || K <= 0) return WINO_ERR_INVALID_ARG;
+    if (int64_t(36) * C * K > kMaxElems) return WINO_ERR_TOO_LARGE;
+    if (!aligned16(w_dev) || !aligned16(u4_dev)) return WINO_ERR_MISALIGNED;
+    if (overlaps(w_dev, size_t(9) * C * K * 4, u4_dev, size_t(36) * C * K * 4)) return WINO_ERR_INVALID_ARG;
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    const unsigned blocks = static_cast<unsigned>((int64_t(C) * K + 255) / 256);
+    wino::f4::ftf4_kernel<<<blocks, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(w_dev, u4_dev, C, K);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
+wino_status_t wino_conv2d_f4x3_fwd(const float* x_dev, const float* u4_dev, float* y_dev, int N, int C, int H,
+                                   int W, int K, int pad, int stride, wino_stream_t stream) {
+    if (!x_dev || !u4_dev || !y_dev) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (int64_t(36) * C * K > kMaxElems) return WINO_ERR_TOO_LARGE;
+    if (N % 16 != 0 || K % 4 != 0) return WINO_ERR_UNSUPPORTED;
+    if (!aligned16(x_dev) || !aligned16(u4_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t yb = size_t(K) * hwn * 4;
+    if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) || overlaps(y_dev, yb, u4_dev, size_t(36) * C * K * 4))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    using namespace wino::f4;
+    Params prm;
+    std::memset(&prm, 0, sizeof(prm));
+    prm.y = y_dev;
+    prm.N = N;
+    prm.C = C;
+    prm.H = H;
+    prm.W = W;
+    prm.K = K;
+    prm.TW = (W + 3) / 4;
+    prm.NV = N * ((H + 3) / 4) * prm.TW;
+    prm.num_kb = (K + BK - 1) / BK;
+    prm.num_it = (C + BC - 1) / BC;
+    prm.num_tiles = ((prm.NV + BN - 1) / BN) * prm.num_kb;
+    {
+        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
+        const cuuint32_t box[4] = {BN, 6, 6, BC};
+        if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    {
+        const cuuint64_t dims[3] = {cuuint64_t(K), 36, cuuint64_t(C)};
+        const cuuint32_t box[3] = {BK, 36, BC};
+        if (!encode_map(&prm.tmu, u4_dev, 3, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    auto kern = fused_f4_kernel;
+    if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4)) != WINO_OK) return s;
+    const int sms = sm_count(dev);
+    const int grid = prm.num_tiles < sms ? prm.num_tiles : sms;
+    kern<<<grid, NT, Smem::bytes, reinterpret_cast<cudaStream_t>(stream)>>>(prm);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 
 }  // extern "C"

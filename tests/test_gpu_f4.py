@@ -1,0 +1,100 @@
+"""GPU parity for NEXT row N1: fused F(4x4,3x3) FP32 kernel vs the fp64 oracle.
+
+The F(4x4) transforms carry the constants 1/4, 1/6, 1/12, 1/24 (G4) and 4, 5,
+2, 8 (B4, A4), so unlike F(2x2) no input class is exact in FP32: every case is
+compared with a relative tolerance (F4_TOL), against
+both the direct definition (Eq. 4) and the oracle's step-by-step F(4x4)
+Winograd (oracle.winograd_f4_conv).  The transformed filter u4 is compared
+with oracle.filter_transform_f4 element by element.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth_inputs import CONFIGS, Conv3x3Config, make_inputs, sample_points
+
+pytestmark = pytest.mark.gpu
+
+F4_TOL = 1e-4   # FP32 bar of north_star, kept for F(4x4)
+FTF4_TOL = 1e-6
+DEV = "cuda:0"
+
+
+@pytest.fixture(scope="module")
+def wino():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ppopp_yanwc20_b200 as w
+    w.lib()
+    return w
+
+
+def _run(wino, x, w):
+    u4 = wino.filter_transform_f4(w.to(DEV))
+    y = wino.conv2d_f4(x.to(DEV), u4)
+    torch.cuda.synchronize()
+    return u4.cpu(), y.cpu()
+
+
+# (N, C, K, H, W): N % 16 == 0, K % 4 == 0.  Channel tails (C % 4), filter tails
+# (K % 64), plane tails (H, W % 4), 1x1 planes, more tiles than SMs.
+F4_EDGE = [
+    (16, 1, 4, 1, 1), (16, 3, 8, 5, 5), (16, 7, 68, 9, 7), (32, 13, 132, 6, 10),
+    (16, 64, 64, 14, 14), (48, 5, 36, 4, 4), (16, 2, 4, 3, 17), (32, 16, 64, 40, 40),
+    (64, 9, 200, 7, 7),
+]
+
+
+@pytest.mark.parametrize("kind", ["uniform", "smallint"])
+@pytest.mark.parametrize("shape", F4_EDGE, ids=[str(s) for s in F4_EDGE])
+def test_f4_edge_shapes(wino, shape, kind):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("f4edge", N, C, K, H, W), kind=kind)
+    u4, y = _run(wino, x, w)
+    assert oracle.max_rel_err(u4.double().numpy(), oracle.filter_transform_f4(w)) <= FTF4_TOL
+    yd = y.double().numpy()
+    assert np.isfinite(yd).all()
+    assert oracle.max_rel_err(yd, oracle.direct_conv(x, w)) <= F4_TOL
+
+
+def test_f4_matches_oracle_f4_winograd(wino):
+    """Same result as the oracle's naive F(4x4) steps (not only the definition)."""
+    x, w = make_inputs(Conv3x3Config("f4", 32, 24, 72, 13, 11), kind="uniform")
+    _, y = _run(wino, x, w)
+    assert oracle.max_rel_err(y.double().numpy(), oracle.winograd_f4_conv(x, w)) <= F4_TOL
+
+
+@pytest.mark.parametrize("kind", ["uniform", "resnet"])
+@pytest.mark.parametrize("name", ["conv2_x", "conv3_x", "conv4_x", "conv5_x"])
+def test_f4_full_configs_sampled(wino, name, kind):
+    cfg = CONFIGS[name]
+    x, w = make_inputs(cfg, kind=kind)
+    u4, y = _run(wino, x, w)
+    assert oracle.max_rel_err(u4.double().numpy(), oracle.filter_transform_f4(w)) <= FTF4_TOL
+    idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 4000)
+    ref = oracle.direct_sample(x, w, idx)
+    ii = idx.numpy()
+    got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
+    assert np.isfinite(y.numpy()).all()
+    assert float(np.max(np.abs(got - ref))) / float(np.max(np.abs(ref))) <= F4_TOL
+
+
+def test_f4_deterministic_and_overwrites(wino):
+    x, w = make_inputs(Conv3x3Config("f4", 32, 20, 68, 9, 9), kind="uniform")
+    xd, wd = x.to(DEV), w.to(DEV)
+    u4 = wino.filter_transform_f4(wd)
+    y1 = wino.conv2d_f4(xd, u4)
+    y2 = torch.full_like(y1, float("nan"))
+    wino.conv2d_f4(xd, u4, out=y2)
+    torch.cuda.synchronize()
+    assert torch.equal(y1, y2)
+
+
+@pytest.mark.parametrize("shape", [(8, 4, 8, 5, 5), (16, 4, 6, 5, 5), (24, 3, 8, 4, 4)])
+def test_f4_unsupported_shapes_raise(wino, shape):
+    N, C, K, H, W = shape
+    x = torch.zeros((C, H, W, N), device=DEV)
+    u4 = torch.zeros((C, 6, 6, K), device=DEV)
+    with pytest.raises(wino.WinoError, match="UNSUPPORTED"):
+        wino.conv2d_f4(x, u4)
