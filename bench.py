@@ -144,6 +144,14 @@ def _init_dist(backend="nccl"):
     return rank, world, local
 
 
+def _ewmm_flops(c, variant):
+    """Algorithmic multiply-add flops of the Winograd-domain GEMMs (Eq. 7): 2 x alpha^2 x
+    K x C x N x tiles; alpha = 4 for F(2x2,3x3), 6 for F(4x4,3x3)."""
+    if variant == "f4_fp32":
+        return 2 * 36 * c.K * c.C * c.N * ((c.H + 3) // 4) * ((c.W + 3) // 4)
+    return 32 * c.K * c.C * c.N * c.tiles
+
+
 def _max_over_ranks(v: float, world: int, device) -> float:
     if world == 1:
         return v
@@ -229,7 +237,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default="resnet_3x3", choices=["resnet_3x3", *RESNET_LAYERS, "tiny"])
-    ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32"])
+    ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32", "f4_fp32"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
@@ -460,7 +468,7 @@ def main():
     for i, d in enumerate(per):
         c = d["cfg"]
         eff = c.eff_flops / (conv_ms[i] * 1e-3) / 1e12
-        ew = 32 * c.K * c.C * c.N * c.tiles
+        ew = _ewmm_flops(c, args.variant)
         ewmm_flops += ew
         conv_total_ms += conv_ms[i]
         layer_rep[c.name] = {
@@ -506,6 +514,11 @@ def main():
                    "layers_eff_tflops": {d["cfg"].name: d["cfg"].eff_flops / (m["conv_ms"][i] * 1e-3) / 1e12
                                          for i, d in enumerate(per) if d["n"]},
                    "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4}[v]}
+        if v == "f4_fp32":
+            ach = sum(_ewmm_flops(d["cfg"], v) for d in per if d["n"]) / (sum(m["conv_ms"]) * 1e-3) / 1e12
+            vrep[v]["roofline"] = {"bound": "alu", "achieved": ach, "peak": fp32_peak, "unit": "TFLOP/s",
+                                   "frac": ach / fp32_peak,
+                                   "achieved_def": "F(4x4) EWMM flops 72*K*C*N*ceil(H/4)*ceil(W/4) / conv time"}
         if v in ("tf32", "3xtf32"):
             ach = ewmm_flops / (sum(m["conv_ms"]) * 1e-3) / 1e12
             mult = 3 if v == "3xtf32" else 1
