@@ -109,6 +109,27 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
                                    wino_stream_t stream);
 
 /*
+ * wino_conv2d_f2x3_fwd with an explicit channel-split factor (split-C).
+ * The paper's kernel gives each CTA a whole (64 filters x 32 tiles) output
+ * block and all C channels (Sec. 3.3; Alg. 1); with small
+ * per-rank batches (batch sharding) there are then fewer blocks
+ * than SMs.  With split_c = S > 1 a thread-block cluster of S CTAs shares each
+ * block, CTA r summing channels [r*C/S, (r+1)*C/S) (per 8-channel block), and
+ * because the output transform is linear (Eq. 8) the S partial 2x2
+ * outputs are added through distributed shared memory in rank order 0..S-1:
+ * deterministic, no atomics, no workspace.  Results equal the unsplit kernel's
+ * up to FP32 summation order (bit-identical on small-integer inputs).
+ *   split_c : 0 = the library's choice (what wino_conv2d_f2x3_fwd does),
+ *             1, 2, 4 or 8 = forced; anything else -> WINO_ERR_INVALID_ARG.
+ *             Honoured by the warp-specialised kernel (N % 32 == 0 or
+ *             N in {4, 8, 16}, K % 4 == 0); other shapes ignore it.
+ * Other arguments, layouts and errors as wino_conv2d_f2x3_fwd.
+ */
+wino_status_t wino_conv2d_f2x3_fwd_split(const float* x_dev, const float* u_dev, float* y_dev,
+                                         int N, int C, int H, int W, int K, int pad, int stride,
+                                         int split_c, wino_stream_t stream);
+
+/*
  * Tensor-core variant (a5' of SURVEY 8(a)): the Winograd-domain GEMM (Eq. 7)
  * on the 5th-generation tensor cores (tcgen05.mma kind::tf32, accumulators in
  * TMEM).  The paper has no tensor-core path ("the data layout needs a

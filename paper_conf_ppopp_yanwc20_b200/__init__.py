@@ -96,6 +96,9 @@ def lib() -> ctypes.CDLL:
     L.wino_filter_transform.argtypes = [vp, vp, i, i, vp]
     L.wino_conv2d_f2x3_fwd.restype = i
     L.wino_conv2d_f2x3_fwd.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_split") or not os.environ.get("WINO_LIB_PATH"):  # A/B builds may predate it
+        L.wino_conv2d_f2x3_fwd_split.restype = i
+        L.wino_conv2d_f2x3_fwd_split.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
     L.wino_conv2d_f2x3_fwd_tc.restype = i
     L.wino_conv2d_f2x3_fwd_tc.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
     L.wino_filter_workspace_bytes_tc.restype = st
@@ -240,9 +243,11 @@ def conv2d_tc(x: torch.Tensor, u_tc: TcFilter, out: torch.Tensor | None = None, 
 
 
 def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, variant: str = "fp32",
-           stream=None) -> torch.Tensor:
+           stream=None, split_c: int = 0) -> torch.Tensor:
     """Fused Winograd forward conv on FP32 CUDA cores, pad 1 stride 1:
-    x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N)."""
+    x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N).  split_c: 0 = the library's choice, else
+    force the split-C factor (1, 2, 4, 8) of the warp-specialised kernel
+    (``wino_conv2d_f2x3_fwd_split``)."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u, "u", 4)
     C, H, W, N = x.shape
@@ -261,7 +266,11 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
     with torch.cuda.device(x.device):
         if variant != "fp32":
             raise ValueError(f"conv2d runs the FP32 kernel; use conv2d_tc for {variant!r}")
-        _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
+        if split_c:
+            _check(lib().wino_conv2d_f2x3_fwd_split(*args, int(split_c), _stream_ptr(stream)),
+                   "wino_conv2d_f2x3_fwd_split")
+        else:
+            _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
     return out
 
 

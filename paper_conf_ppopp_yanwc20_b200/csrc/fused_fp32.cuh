@@ -66,6 +66,9 @@ struct __align__(64) Params {
     int NV;      // N * ceil(H/2) * ceil(W/2)
     int num_kb;  // ceil(K/BK)
     int num_it;  // ceil(C/BC)
+    int xnb;     // n-extent of one x TMA box: 32, or N when N | 32 (WS kernel: 32/xnb boxes per stage)
+    int split;   // split-C factor S = cluster size (WS kernel; 1 = no split)
+    int itf_map[64];  // WS kernel, N | 32: ITF task of thread (warp-9)*32+lane: c | n4 << 3 | xoff << 8
 };
 
 // XPW = Winograd elements xi per warp: 2 -> 8 warps / 256 threads (the paper's

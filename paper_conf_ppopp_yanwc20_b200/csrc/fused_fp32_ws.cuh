@@ -17,7 +17,23 @@
 //     ITF overlap this tile's epilogue.  The epilogue therefore has its own
 //     shared buffer and runs in 4 rounds (16 filters each) -- the paper's
 //     4-round OTF (L479-499), here to leave room for the pipeline ring.
-// Used when both operands can be TMA boxes (N % 32 == 0, K % 4 == 0).
+// Used when both operands can be TMA boxes (N % 32 == 0 or N in {4, 8, 16}; K % 4 == 0).
+//
+// Small per-rank batches (batch sharding): with N | 32 a 32-nu tile
+// spans 32/N consecutive image tiles, loaded as 32/N boxes (n:N, w:4, h:4, c:8).
+// Split-C (SPLIT = true): when there are too few (k, nu) tiles to fill 148 SMs,
+// a thread-block cluster of S CTAs shares each tile, CTA r accumulating channel
+// blocks [r*NIT/S, (r+1)*NIT/S).  The output transform is linear (Eq. 8), so each
+// CTA applies it to its partial M and the S partial 2x2 outputs are summed (the 4
+// outputs per (k, nu) are reduced instead of the 16 M).  CTA r owns filters
+// [r*64/S, (r+1)*64/S) of the tile: every CTA pushes its partial outputs of those
+// filters into slot [its rank] of CTA r's receive buffer with st.async (remote,
+// fire-and-forget, byte-counted on CTA r's mbarrier), and CTA r's compute warps sum
+// the S slots from LOCAL shared memory in rank order 0..S-1 and store y --
+// deterministic, no atomics, no global workspace.  Pull-based reads of
+// the peers' buffers were measured ~4x slower (DSMEM reads queue behind the remote
+// SM's LDS traffic; scripts/ws_trace.py), and so was a dedicated reducer warp in the
+// producer warpgroup (its shared-memory loads queue behind the compute warps').
 #pragma once
 #include <cuda.h>
 
@@ -46,89 +62,53 @@ constexpr int SV = 2;               // V ring (16 KB each)
 constexpr int REG_COMPUTE = 208, REG_PRODUCER = 88;  // 256*208 + 128*88 = 64512 <= 65536
 constexpr int ITF_WARPS = 2;        // warps 9..10 (float4 along nu); warp 8 only issues TMA; 11 idle
 constexpr int ER_LD = BN + 4;       // padded row of the epilogue buffer
-constexpr int ER_KROWS = 16;        // filters per epilogue round
-constexpr int ER_FLOATS = 16 * ER_KROWS * ER_LD;  // [xi][16 k][36]
+constexpr int MAX_SPLIT = 8;        // portable cluster size
+constexpr uint32_t kSplitTileBytes = BK * BN * 4 * 4;  // S slots x 64/S filters x 32 nu x 16 B
 
+#ifdef WINO_WS_TRACE
+// debug builds only: clock64 events of CTA 0 per tile (scripts/ws_trace.py)
+__device__ unsigned long long g_ws_trace[8][64];
+#define WS_TR(e, T) \
+    do { if (blockIdx.x == 0 && (T) < 64) g_ws_trace[e][T] = clock64(); } while (0)
+#else
+#define WS_TR(e, T) do { } while (0)
+#endif
+
+// Epilogue geometry: RR accumulator rows per thread per round -> 8*RR filters per
+// round, 8/RR rounds.  Without split RR = 2 (4 rounds of 16 filters, L499).  With
+// split RR = 1 (8 rounds of 8) so that the whole tile's partial outputs fit: the
+// rounds fill yp[64 k][4 outputs][32 nu] (32 KB), then ONE cluster exchange per
+// tile (a per-round exchange is latency-bound: ~8 DSMEM round trips per tile).
+template <bool SPLIT>
 struct Smem {
+    static constexpr int RR = SPLIT ? 1 : 2;
+    static constexpr int ER_KROWS = 8 * RR;
+    static constexpr int ER_FLOATS = 16 * ER_KROWS * ER_LD;  // [xi][8RR k][36]
+    // split receive buffer [S slots][64/S owned filters][32 nu][4 outputs] = 32 KB for any S
+    static constexpr int YP_FLOATS = SPLIT ? BK * 4 * BN : 0;
     static constexpr int ep_offset = (S * STAGE_FLOATS + SV * VS_FLOATS) * 4;
-    static constexpr int bar_offset = ep_offset + ER_FLOATS * 4;
-    // full[S], empty[S], vfull[SV], vempty[SV]
-    static constexpr int bytes = bar_offset + (2 * S + 2 * SV) * 8;
+    static constexpr int yp_offset = ep_offset + ER_FLOATS * 4;
+    static constexpr int bar_offset = yp_offset + YP_FLOATS * 4;
+    // full[S], empty[S], vfull[SV], vempty[SV], yready, yfree
+    static constexpr int bytes = bar_offset + (2 * S + 2 * SV + 2) * 8;
 };
 
-__global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_constant__ Params p, int num_tiles) {
-    extern __shared__ __align__(1024) float smem[];
-    float* const vs = smem + S * STAGE_FLOATS;
-    float* const ep = reinterpret_cast<float*>(reinterpret_cast<char*>(smem) + Smem::ep_offset);
-    uint64_t* const full = reinterpret_cast<uint64_t*>(reinterpret_cast<char*>(smem) + Smem::bar_offset);
-    uint64_t* const empty = full + S;
-    uint64_t* const vfull = empty + S;
-    uint64_t* const vempty = vfull + SV;
-
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int NIT = p.num_it;
-
-    if (tid == 0) {
-        tma_prefetch_desc(&p.tmx);
-        tma_prefetch_desc(&p.tmu);
-        for (int s = 0; s < S; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&empty[s], 8 + ITF_WARPS);  // 8 compute warps (u) + ITF warps (raw x)
-        }
-        for (int s = 0; s < SV; ++s) {
-            mbar_init(&vfull[s], ITF_WARPS);
-            mbar_init(&vempty[s], 8);
-        }
-        fence_mbar_init();
-    }
-    __syncthreads();
-
-    if (warp >= 8) {
-        // ============================ producer / ITF ============================
-        setmaxnreg_dec<REG_PRODUCER>();
-        if (warp == 8) {
-            // ---------------- TMA issue (one elected lane) ----------------
-            if (lane == 0) {
-                constexpr uint32_t kBytes = (US_FLOATS + XS_FLOATS) * 4;
-                int G = 0;  // global stage counter across tiles
-                for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-                    const int kb = tile % p.num_kb, nb = tile / p.num_kb;
-                    const int k0 = kb * BK, nu0 = nb * BN;
-                    // N % 32 == 0 -> the tile's 32 nu are 32 consecutive n of one image tile
-                    const int t = nu0 / p.N;
-                    const int n0 = nu0 - t * p.N;
-                    const int th = t / p.TW, tw = t - th * p.TW;
-                    const int w0 = 2 * tw - 1, h0 = 2 * th - 1;  // -1: TMA zero fill = padding (Sec. 3.5)
-                    for (int g = 0; g < NIT; ++g, ++G) {
-                        const int slot = G % S;
-                        if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
-                        float* us = smem + slot * STAGE_FLOATS;
-                        mbar_arrive_expect_tx(&full[slot], kBytes);
-                        tma_load_3d(us, &p.tmu, &full[slot], k0, 0, g * BC);
-                        tma_load_4d(us + US_FLOATS, &p.tmx, &full[slot], n0, w0, h0, g * BC);
-                    }
-                }
-            }
-            return;
-        }
-        // ---------------- ITF (Sec. 4.2) on warps 9..10 ----------------
-        // 256 (c, nu) tiles per stage; a thread transforms 4 consecutive nu of one
-        // channel with LDS.128 / STS.128 (a quarter-warp covers one 128 B row:
-        // conflict-free): lane -> (c = 4 (w - 9) + lane / 8, nu4 = lane % 8).
-        if (warp > 8 + ITF_WARPS) return;
-        const int c = 4 * (warp - 9) + (lane >> 3), n4 = 4 * (lane & 7);
+// ITF loop of warps 9..10 (Sec. 4.2): raw x of every stage -> V = B^T d B in the V ring.
+__device__ __forceinline__ void itf_loop(float* smem, float* vs, uint64_t* full, uint64_t* empty, uint64_t* vfull,
+                                         uint64_t* vempty, int xoff, int xpos, int voff, int NIT, int first,
+                                         int num_tiles, int stride, int lane) {
         int G = 0;
-        for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+        for (int tile = first; tile < num_tiles; tile += stride) {
             for (int g = 0; g < NIT; ++g, ++G) {
                 const int slot = G % S, vb = G % SV;
                 mbar_wait(&full[slot], (G / S) & 1);
                 if (G >= SV) mbar_wait(&vempty[vb], ((G / SV) - 1) & 1);
-                const float* xs = smem + slot * STAGE_FLOATS + US_FLOATS + c * 16 * BN + n4;
-                float* v = vs + vb * VS_FLOATS + c * BN + n4;
+                const float* xs = smem + slot * STAGE_FLOATS + US_FLOATS + xoff;
+                float* v = vs + vb * VS_FLOATS + voff;
                 float d[4][16];
 #pragma unroll
                 for (int e = 0; e < 16; ++e) {
-                    const float4 q = *reinterpret_cast<const float4*>(xs + e * BN);
+                    const float4 q = *reinterpret_cast<const float4*>(xs + e * xpos);
                     d[0][e] = q.x; d[1][e] = q.y; d[2][e] = q.z; d[3][e] = q.w;
                 }
                 float t[4][16];
@@ -144,6 +124,130 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                 }
             }
         }
+}
+// BOX32: N % 32 == 0 (one x box per stage, compile-time ITF strides); else N | 32
+// (32/N boxes, runtime strides -- costs the 88-register ITF warps one spill).
+template <bool SPLIT, bool BOX32>
+__global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_constant__ Params p, int num_tiles) {
+    using SM = Smem<SPLIT>;
+    constexpr int RR = SM::RR, ER_KROWS = SM::ER_KROWS;
+    extern __shared__ __align__(1024) float smem[];
+    float* const vs = smem + S * STAGE_FLOATS;
+    float* const ep = reinterpret_cast<float*>(reinterpret_cast<char*>(smem) + SM::ep_offset);
+    float* const yp = reinterpret_cast<float*>(reinterpret_cast<char*>(smem) + SM::yp_offset);
+    uint64_t* const full = reinterpret_cast<uint64_t*>(reinterpret_cast<char*>(smem) + SM::bar_offset);
+    uint64_t* const empty = full + S;
+    uint64_t* const vfull = empty + S;
+    uint64_t* const vempty = vfull + SV;
+    uint64_t* const yready = vempty + SV;  // split: all S slots of this CTA's receive buffer landed (tx bytes)
+    uint64_t* const yfree = yready + 1;    // split: every owner has consumed this CTA's slots of the last tile
+
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // split-C: cluster = S consecutive CTAs sharing each tile; rank r takes channel
+    // blocks [it_lo, it_hi).  Without split every CTA is its own "cluster".
+    const int nsplit = SPLIT ? p.split : 1;
+    const int crank = SPLIT ? static_cast<int>(cluster_ctarank()) : 0;
+    // first tile / tile stride of this cluster.  Re-derived from blockIdx / gridDim at each
+    // use rather than held in registers: two more live registers across the compute
+    // warps' main loop change ptxas' accumulator assignment and cost ~20% more FFMA
+    // register-bank conflicts (scripts/sass_bank.py: 1.14 -> 1.35 reads per FFMA).
+#define WS_CID (SPLIT ? static_cast<int>(blockIdx.x) / p.split : static_cast<int>(blockIdx.x))
+#define WS_NCL (SPLIT ? static_cast<int>(gridDim.x) / p.split : static_cast<int>(gridDim.x))
+    const int it_lo = crank * p.num_it / nsplit, it_hi = (crank + 1) * p.num_it / nsplit;
+    const int NIT = it_hi - it_lo;
+
+    if (tid == 0) {
+        tma_prefetch_desc(&p.tmx);
+        tma_prefetch_desc(&p.tmu);
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 8 + ITF_WARPS);  // 8 compute warps (u) + ITF warps (raw x)
+        }
+        for (int s = 0; s < SV; ++s) {
+            mbar_init(&vfull[s], ITF_WARPS);
+            mbar_init(&vempty[s], 8);
+        }
+        if (SPLIT) {
+            mbar_init(yready, 1);       // one arrive.expect_tx per tile (+ S x 64/S x 512 B of st.async)
+            mbar_init(yfree, nsplit);   // one arrival per owner CTA
+        }
+        fence_mbar_init();
+    }
+    if constexpr (SPLIT) {
+        if (tid == 0) mbar_arrive_expect_tx(yready, kSplitTileBytes);  // tile 0's partials
+        cluster_sync_all();  // peers' barriers initialised before any remote arrive / st.async
+    }
+    else __syncthreads();
+
+    if (warp >= 8) {
+        // ============================ producer / ITF ============================
+        setmaxnreg_dec<REG_PRODUCER>();
+        if (warp == 8) {
+            // ---------------- TMA issue (one elected lane) ----------------
+            if (lane == 0) {
+                constexpr uint32_t kBytes = (US_FLOATS + XS_FLOATS) * 4;
+                int G = 0;  // global stage counter across tiles
+                for (int tile = WS_CID; tile < num_tiles; tile += WS_NCL) {
+                    const int kb = tile % p.num_kb, nb = tile / p.num_kb;
+                    const int k0 = kb * BK, nu0 = nb * BN;
+                    // N % 32 == 0: the tile's 32 nu are 32 consecutive n of one image tile (one box);
+                    // N | 32: 32/N consecutive image tiles, one (n:N) box each -> [box][c][pos][n]
+                    const int t0 = nu0 / p.N;
+                    const int n0 = nu0 - t0 * p.N;
+                    const int nbox = BOX32 ? 1 : BN / p.xnb;
+                    for (int g = it_lo; g < it_hi; ++g, ++G) {
+                        const int slot = G % S;
+                        if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
+                        float* us = smem + slot * STAGE_FLOATS;
+                        mbar_arrive_expect_tx(&full[slot], kBytes);
+                        tma_load_3d(us, &p.tmu, &full[slot], k0, 0, g * BC);
+                        for (int b = 0; b < nbox; ++b) {
+                            const int t = t0 + b;
+                            const int th = t / p.TW, tw = t - th * p.TW;
+                            // -1 / past the end: TMA zero fill = implicit padding (Sec. 3.5).
+                            // BOX32: map (n, w, h, c) -> [c][pos][n]; small N: map (n, c, w, h)
+                            // -> [pos][c][n] per box (see the ITF lane map below)
+                            if (BOX32)
+                                tma_load_4d(us + US_FLOATS, &p.tmx, &full[slot], n0, 2 * tw - 1, 2 * th - 1, g * BC);
+                            else
+                                tma_load_4d(us + US_FLOATS + b * (BC * 16 * p.xnb), &p.tmx, &full[slot], 0, g * BC,
+                                            2 * tw - 1, 2 * th - 1);
+                        }
+                    }
+                }
+            }
+            return;
+        }
+        // ---------------- ITF (Sec. 4.2) on warps 9..10 ----------------
+        // 256 (c, nu) tiles per stage; a thread transforms 4 consecutive nu of one
+        // channel with LDS.128 / STS.128 (a quarter-warp covers one 128 B row:
+        // conflict-free): lane -> (c = 4 (w - 9) + lane / 8, nu4 = lane % 8).
+        if (warp == 11) return;  // idle
+        // Small N (N | 32, boxes [b][pos][c][n]): the 8 lanes of a quarter-warp (one LDS.128 /
+        // STS.128 wavefront) take task i = b*Q + h (Q = N/4 quads per row, h = quad) with
+        // channel c = (b + j) % 8 in quarter j: raw reads hit bank group (c*Q + h) % 8 and V
+        // writes (b*Q + h) % 8 -- both distinct across the 8 lanes, so conflict-free.  The map
+        // comes precomputed in Params: computing it here (or calling the ITF out of line)
+        // perturbs ptxas' register assignment of the compute warps' FFMA stream.
+        int c, n4, xoff, xpos;
+        if (BOX32) {
+            c = 4 * (warp - 9) + (lane >> 3);
+            n4 = 4 * (lane & 7);
+            xoff = c * 16 * BN + n4;  // [c][pos][n]
+            xpos = BN;
+        } else {
+            const int m = p.itf_map[(warp - 9) * 32 + lane];  // host-computed (wino_api.cu)
+            c = m & 7;
+            n4 = (m >> 3) & 31;
+            xoff = m >> 8;
+            xpos = BC * p.xnb;
+        }
+        if (BOX32)
+            itf_loop(smem, vs, full, empty, vfull, vempty, xoff, xpos, c * BN + n4, NIT, WS_CID, num_tiles, WS_NCL,
+                     lane);
+        else
+            itf_loop(smem, vs, full, empty, vfull, vempty, xoff, xpos, c * BN + n4, NIT, WS_CID, num_tiles, WS_NCL,
+                     lane);
         return;
     }
 
@@ -170,7 +274,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
     };
 
     int G = 0;
-    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+    for (int tile = WS_CID; tile < num_tiles; tile += WS_NCL) {
         const int kb = tile % p.num_kb, nb = tile / p.num_kb;
         const int k0 = kb * BK, nu0 = nb * BN;
         float acc[2][8][8];
@@ -192,6 +296,10 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                         acc[q][i][j] = fmaf(f[q][i], g[q][j], acc[q][i][j]);
                     }
         };
+#ifdef WINO_WS_TRACE
+        const int Ttr = (tile - WS_CID) / WS_NCL;
+        if (tid == 0) WS_TR(0, Ttr);
+#endif
         for (int g = 0; g < NIT; ++g, ++G) {
             const int slot = G % S, vb = G % SV;
             mbar_wait(&full[slot], (G / S) & 1);
@@ -214,7 +322,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             }
         }
 
-        // ---- OTF (Sec. 4.4) in 4 rounds of 16 filters through the epilogue buffer ----
+        // ---- OTF (Sec. 4.4) through the epilogue buffer ----
         const int nu = nu0 + lane;
         int t = 0, n = 0, i0 = 0, j0 = 0;
         if (nu < p.NV) {
@@ -226,46 +334,141 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
         }
         const bool okr = i0 + 1 < p.H, okc = j0 + 1 < p.W;  // odd H/W: drop extra outputs (L1155)
         const size_t base = ((size_t)i0 * p.W + j0) * p.N + n;
+        if constexpr (!SPLIT) {
+            // 4 rounds of 16 filters (the paper's 4-round OTF, L499).  NOTE: ptxas' register
+            // assignment of the accumulators (and so the FFMA bank conflicts of the main
+            // loop) is sensitive to this code's shape: keep it as is.
 #pragma unroll
-        for (int rd = 0; rd < 4; ++rd) {
-            // round rd stores accumulator rows i in {2(rd&1), 2(rd&1)+1} of half rd>>1:
-            // filters kl = fo + (i&3) + 32*(i>>2); in the buffer row = (fo>>2)*2 + (i&1)
-            named_bar_sync(1, COMPUTE_THREADS);  // previous round's readers are done
+            for (int rd = 0; rd < 4; ++rd) {
+                // round rd stores accumulator rows i in {2(rd&1), 2(rd&1)+1} of half rd>>1:
+                // filters kl = fo + (i&3) + 32*(i>>2); in the buffer row = (fo>>2)*2 + (i&1)
+                named_bar_sync(1, COMPUTE_THREADS);  // previous round's readers are done
 #pragma unroll
-            for (int q = 0; q < 2; ++q)
+                for (int q = 0; q < 2; ++q)
 #pragma unroll
-                for (int ii = 0; ii < 2; ++ii) {
-                    const int i = (rd >> 1) * 4 + (rd & 1) * 2 + ii;
-                    const int r = (fo >> 2) * 2 + ii;
-                    float* row = ep + ((xi0 + q) * ER_KROWS + r) * ER_LD + io;
-                    *reinterpret_cast<float4*>(row) =
-                        make_float4(acc[q][i][1], acc[q][i][0], acc[q][i][3], acc[q][i][2]);
-                    *reinterpret_cast<float4*>(row + 16) =
-                        make_float4(acc[q][i][5], acc[q][i][4], acc[q][i][7], acc[q][i][6]);
-                }
-            named_bar_sync(1, COMPUTE_THREADS);
-            if (nu < p.NV) {
+                    for (int ii = 0; ii < 2; ++ii) {
+                        const int i = (rd >> 1) * 4 + (rd & 1) * 2 + ii;
+                        const int r = (fo >> 2) * 2 + ii;
+                        float* row = ep + ((xi0 + q) * ER_KROWS + r) * ER_LD + io;
+                        *reinterpret_cast<float4*>(row) =
+                            make_float4(acc[q][i][1], acc[q][i][0], acc[q][i][3], acc[q][i][2]);
+                        *reinterpret_cast<float4*>(row + 16) =
+                            make_float4(acc[q][i][5], acc[q][i][4], acc[q][i][7], acc[q][i][6]);
+                    }
+                named_bar_sync(1, COMPUTE_THREADS);
+                if (nu < p.NV) {
 #pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    const int r = warp + 8 * h;  // buffer row 0..15
-                    const int kl = (r >> 1) * 4 + (rd & 1) * 2 + (r & 1) + (rd >> 1) * 32;
-                    const int k = k0 + kl;
-                    if (k < p.K) {
-                        float m[16], o[4];
+                    for (int h = 0; h < 2; ++h) {
+                        const int r = warp + 8 * h;  // buffer row 0..15
+                        const int kl = (r >> 1) * 4 + (rd & 1) * 2 + (r & 1) + (rd >> 1) * 32;
+                        const int k = k0 + kl;
+                        if (k < p.K) {
+                            float m[16], o[4];
 #pragma unroll
-                        for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + r) * ER_LD + (lane ^ 1)];
-                        otf_2x2(m, o);
-                        float* yk = p.y + (size_t)k * HWN + base;
-                        yk[0] = o[0];
-                        if (okc) yk[p.N] = o[1];
-                        if (okr) yk[dW] = o[2];
-                        if (okr && okc) yk[dW + p.N] = o[3];
+                            for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + r) * ER_LD + (lane ^ 1)];
+                            otf_2x2(m, o);
+                            float* yk = p.y + (size_t)k * HWN + base;
+                            yk[0] = o[0];
+                            if (okc) yk[p.N] = o[1];
+                            if (okr) yk[dW] = o[2];
+                            if (okr && okc) yk[dW + p.N] = o[3];
+                        }
                     }
                 }
             }
+        } else {
+            // 8 rounds of 8 filters: round rd stores accumulator row i = rd (filters
+            // kl = fo + (rd&3) + 32*(rd>>2)) into buffer row fo>>2; the OTF of buffer row
+            // `warp` (filter 4*warp + (rd&3) + 32*(rd>>2)) goes to yp[kl][o][nu]
+            // peers done reading this CTA's yp of its previous tile (T = this CTA's tile count
+            // so far, re-derived rather than kept live across the main loop)
+            const int T = (tile - WS_CID) / WS_NCL;
+            if (tid == 0) WS_TR(1, T);
+            if (T > 0) mbar_wait_cluster(yfree, (T - 1) & 1);  // owners consumed our previous partials
+            if (tid == 0) WS_TR(2, T);
+            const int rows = BK / nsplit;
+            const uint32_t yb = smem_u32(yp), ybar = smem_u32(yready);
+#pragma unroll
+            for (int rd = 0; rd < 8; ++rd) {
+                named_bar_sync(1, COMPUTE_THREADS);
+#pragma unroll
+                for (int q = 0; q < 2; ++q) {
+                    float* row = ep + ((xi0 + q) * ER_KROWS + (fo >> 2)) * ER_LD + io;
+                    *reinterpret_cast<float4*>(row) =
+                        make_float4(acc[q][rd][1], acc[q][rd][0], acc[q][rd][3], acc[q][rd][2]);
+                    *reinterpret_cast<float4*>(row + 16) =
+                        make_float4(acc[q][rd][5], acc[q][rd][4], acc[q][rd][7], acc[q][rd][6]);
+                }
+                named_bar_sync(1, COMPUTE_THREADS);
+                const int kl = 4 * warp + (rd & 3) + 32 * (rd >> 2);
+                float m[16], o[4];
+#pragma unroll
+                for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + warp) * ER_LD + (lane ^ 1)];
+                otf_2x2(m, o);
+                // -> slot [crank] of the owner of filter kl: [slot][kl % rows][nu][4]
+                const int owner = kl / rows;
+                const uint32_t dst = yb + (uint32_t)((((crank * rows + kl - owner * rows) * BN) + lane) * 16);
+                st_async4(mapa_shared(dst, owner), o[0], o[1], o[2], o[3], mapa_shared(ybar, owner));
+            }
         }
+        if constexpr (SPLIT) {
+            // all S partials of this CTA's filters landed -> sum the S slots and store.  Warp w
+            // takes owned filters w + 8i: always 8 (filter, slot) pairs per thread (64/S filters
+            // x S slots / 8 warps), all 8 loads issued before the first add; the slots are
+            // added by a fixed pairwise tree ((s0+s1)+(s2+s3))+... (deterministic).
+            const int T = (tile - WS_CID) / WS_NCL;
+            mbar_wait_cluster(yready, T & 1);
+            if (tid == 0) WS_TR(5, T);
+            {
+                const int rows = BK / nsplit, lg = nsplit == 2 ? 1 : (nsplit == 4 ? 2 : 3);
+                const float4* yb4 = reinterpret_cast<const float4*>(yp) + lane;
+                float4 v[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {  // j = i * S + q: filter warp + 8i, slot q
+                    const int q = j & (nsplit - 1), r = warp + 8 * (j >> lg);
+                    v[j] = yb4[(q * rows + r) * BN];
+                }
+                auto add4 = [](float4& a, const float4& b) { a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w; };
+#pragma unroll
+                for (int j = 0; j < 8; j += 2) add4(v[j], v[j + 1]);
+                if (nsplit >= 4) {
+#pragma unroll
+                    for (int j = 0; j < 8; j += 4) add4(v[j], v[j + 2]);
+                }
+                if (nsplit >= 8) add4(v[0], v[4]);
+                if (nu < p.NV) {
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) {
+                        if (j & (nsplit - 1)) continue;
+                        const int k = k0 + crank * rows + warp + 8 * (j >> lg);
+                        if (k >= p.K) continue;
+                        float* yk = p.y + (size_t)k * HWN + base;
+                        yk[0] = v[j].x;
+                        if (okc) yk[p.N] = v[j].y;
+                        if (okr) yk[dW] = v[j].z;
+                        if (okr && okc) yk[dW + p.N] = v[j].w;
+                    }
+                }
+            }
+            named_bar_sync(1, COMPUTE_THREADS);  // every slot consumed
+            if (warp == 0) {
+                if (lane == 0) mbar_arrive_expect_tx(yready, kSplitTileBytes);  // next tile's partials
+                if (lane < nsplit) mbar_arrive_cluster(mapa_shared(smem_u32(yfree), lane));
+            }
+            if (tid == 0) WS_TR(6, T);
+#ifdef WINO_WS_TRACE
+            if (tid == 0) WS_TR(3, (tile - WS_CID) / WS_NCL);
+#endif
+        }
+    }
+    if constexpr (SPLIT) {
+        // peers may still be reading this CTA's yp: exit only after they all signalled
+        const int T = num_tiles > WS_CID ? (num_tiles - WS_CID + WS_NCL - 1) / WS_NCL : 0;  // tiles done
+        if (T > 0) mbar_wait_cluster(yfree, (T - 1) & 1);
     }
 }
 
+#undef WS_CID
+#undef WS_NCL
 }  // namespace fp32ws
 }  // namespace wino

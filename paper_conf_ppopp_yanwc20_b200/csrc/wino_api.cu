@@ -102,23 +102,71 @@ wino_status_t check_shape(int N, int C, int H, int W, int K, int pad, int stride
     return WINO_OK;
 }
 
+// Co-resident clusters of `split` CTAs of the warp-specialised kernel (1 CTA per SM).
+// Measured with cudaOccupancyMaxActiveClusters on the device when one is current
+// (cached); without a device (host-only planning) the B200 values.
+std::atomic<int> g_clusters[kMaxDevices][4];
+int cluster_slots(int split, int dev);
+
 struct Fp32Plan {
-    int load_x, load_u;  // wino::fp32::LoadMode
-    int64_t ctas;
-    int smem;
+    int load_x, load_u;  // wino::fp32::LoadMode (generic kernel)
+    bool ws;             // warp-specialised persistent kernel
+    int xnb;             // x TMA box n-extent (ws)
+    int split;           // split-C factor = cluster size (ws)
+    int64_t tiles;       // (k, nu) tiles
+    int64_t grid;        // CTAs launched
+    int threads, smem;
 };
 
-Fp32Plan plan_fp32(int N, int C, int H, int W, int K) {
+int log2_small(int s) { return s == 1 ? 0 : s == 2 ? 1 : s == 4 ? 2 : 3; }
+
+// Shape -> kernel / tiling / split-C.  force_split: 0 = choose, else 1, 2, 4 or 8.
+// The split model: a cluster of S CTAs shares a tile, each CTA runs ceil(NIT/S)
+// channel blocks plus an epilogue worth ~E channel blocks (E measured: the
+// DSMEM-reduced epilogue of the split kernel costs about one block more than the
+// plain one); time ~ waves(S) * (ceil(NIT/S) + E(S)), waves = ceil(tiles/clusters).
+Fp32Plan plan_fp32(int N, int C, int H, int W, int K, bool u_tma_ok, int dev, int force_split) {
     using namespace wino::fp32;
     Fp32Plan p;
     p.load_x = (N % 32 == 0) ? LD_TMA : (N % 4 == 0 ? LD_CP16B : LD_CP4B);
-    p.load_u = (K % 4 == 0) ? LD_TMA : LD_CP4B;
+    p.load_u = (K % 4 == 0 && u_tma_ok) ? LD_TMA : LD_CP4B;
     const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
     const int64_t nb = (nv + BN - 1) / BN;
     const int64_t kb = (K + BK - 1) / BK;
-    p.ctas = nb * kb;
-    p.smem = Smem<kStages>::bytes;
-    (void)C;
+    p.tiles = nb * kb;
+    p.xnb = (N % 32 == 0) ? 32 : N;
+    p.ws = p.load_u == LD_TMA && (N % 32 == 0 || N == 4 || N == 8 || N == 16);
+#ifdef WINO_NO_WS
+    p.ws = false;
+#endif
+    p.split = 1;
+    if (!p.ws) {
+        p.grid = p.tiles;
+        p.threads = threads_for<kXpw>();
+        p.smem = Smem<kStages>::bytes;
+        return p;
+    }
+    const int nit = (C + BC - 1) / BC;
+    if (force_split > 0) {
+        p.split = force_split;
+    } else {
+        double best = 0;
+        for (int s = 1; s <= wino::fp32ws::MAX_SPLIT; s *= 2) {
+            if (s > 1 && nit < 2 * s) break;  // keep >= 2 channel blocks per CTA
+            const int cl = cluster_slots(s, dev);
+            if (cl <= 0) continue;
+            const double waves = double((p.tiles + cl - 1) / cl);
+            const double est = waves * (double((nit + s - 1) / s) + (s == 1 ? 0.5 : 1.5));
+            if (s == 1 || est < best * 0.97) {
+                best = est;
+                p.split = s;
+            }
+        }
+    }
+    const int64_t cl = cluster_slots(p.split, dev);
+    p.grid = (p.tiles < cl ? p.tiles : cl) * p.split;
+    p.threads = wino::fp32ws::NT;
+    p.smem = p.split > 1 ? wino::fp32ws::Smem<true>::bytes : wino::fp32ws::Smem<false>::bytes;
     return p;
 }
 
@@ -155,7 +203,6 @@ bool encode_map(CUtensorMap* m, const float* base, int rank, const cuuint64_t* d
 }
 
 std::atomic<uint64_t> g_attr_fp32[3][3];
-std::atomic<uint64_t> g_attr_ws;
 std::atomic<uint64_t> g_attr_f4;
 
 template <int XM, int UM>
@@ -184,12 +231,51 @@ wino_status_t launch_tc(const wino::tc::Params& prm, int64_t ctas, int dev, cuda
 }
 }  // namespace
 
+namespace {
+int cluster_slots(int split, int dev) {
+    // host-only default: B200 (148 SMs); clusters of 8 measured 18
+    static const int kDefault[4] = {148, 74, 37, 18};
+    const int li = log2_small(split);
+    if (dev < 0 || dev >= kMaxDevices) return kDefault[li];
+    int n = g_clusters[dev][li].load(std::memory_order_relaxed);
+    if (n != 0) return n;
+    n = kDefault[li];
+    if (split == 1) {
+        n = sm_count(dev);
+    } else {
+        auto kern = wino::fp32ws::fused_fp32_ws_kernel<true, true>;
+        const int smem = wino::fp32ws::Smem<true>::bytes;
+        if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) == cudaSuccess) {
+            cudaLaunchConfig_t cfg = {};
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = split;
+            at[0].val.clusterDim.y = 1;
+            at[0].val.clusterDim.z = 1;
+            cfg.gridDim = dim3(split * 64);
+            cfg.blockDim = dim3(wino::fp32ws::NT);
+            cfg.dynamicSmemBytes = smem;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            int q = 0;
+            if (cudaOccupancyMaxActiveClusters(&q, kern, &cfg) == cudaSuccess && q > 0) n = q;
+        }
+        cudaGetLastError();  // a failed query must not leak into the caller's error state
+    }
+    g_clusters[dev][li].store(n, std::memory_order_relaxed);
+    return n;
+}
+
+std::atomic<uint64_t> g_attr_ws_k[2][2];
+}  // namespace
+
 // FP32 fused conv on validated arguments; u may be a K-slice of a wider (C,4,4,ldu) array.
+// force_split: 0 = planner's choice, else the split-C factor (1, 2, 4, 8).
 wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, float* y_dev, int N, int C, int H,
-                              int W, int K, int dev, cudaStream_t st) {
+                              int W, int K, int dev, cudaStream_t st, int force_split = 0) {
     using namespace wino::fp32;
-    Fp32Plan pl = plan_fp32(N, C, H, W, K);
-    if (ldu % 4 != 0 || !aligned16(u_dev)) pl.load_u = LD_CP4B;
+    const bool u_tma_ok = ldu % 4 == 0 && aligned16(u_dev);
+    Fp32Plan pl = plan_fp32(N, C, H, W, K, u_tma_ok, dev, force_split);
     Params prm;
     std::memset(&prm, 0, sizeof(prm));
     prm.x = x_dev;
@@ -205,7 +291,23 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
     prm.NV = N * ((H + 1) / 2) * prm.TW;
     prm.num_kb = (K + BK - 1) / BK;
     prm.num_it = (C + BC - 1) / BC;
-    if (pl.load_x == LD_TMA) {
+    prm.xnb = pl.ws ? pl.xnb : BN;
+    prm.split = pl.split;
+    if (pl.ws && prm.xnb < BN) {
+        // ITF lane map of the small-N WS kernel (conflict-free LDS.128 / STS.128, see fused_fp32_ws.cuh)
+        const int Q = prm.xnb / 4;
+        for (int t = 0; t < 64; ++t) {
+            const int j = t / 8, i = t % 8, b = i / Q, h = i % Q;
+            const int c = (b + j) % 8, n4 = b * prm.xnb + 4 * h;
+            const int xoff = b * (BC * 16 * prm.xnb) + c * prm.xnb + 4 * h;  // [b][pos][c][n]
+            prm.itf_map[t] = c | (n4 << 3) | (xoff << 8);
+        }
+        // small N: x viewed as (n, c, w, h) so that a box lands as [pos][c][n] (conflict-free ITF)
+        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(C), cuuint64_t(W), cuuint64_t(H)};
+        const cuuint64_t strides[3] = {cuuint64_t(H) * W * N * 4, cuuint64_t(N) * 4, cuuint64_t(W) * N * 4};
+        const cuuint32_t box[4] = {cuuint32_t(prm.xnb), BC, 4, 4};
+        if (!encode_map(&prm.tmx, x_dev, 4, dims, box, strides)) return cuda_fail(cudaErrorInvalidValue);
+    } else if (pl.ws || pl.load_x == LD_TMA) {
         const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
         const cuuint32_t box[4] = {BN, 4, 4, BC};
         if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
@@ -216,21 +318,38 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
         const cuuint32_t box[3] = {BK, 16, BC};
         if (!encode_map(&prm.tmu, u_dev, 3, dims, box, strides)) return cuda_fail(cudaErrorInvalidValue);
     }
-    const int64_t g = pl.ctas;
+    const int64_t g = pl.tiles;
     const int sm = pl.smem;
-#ifndef WINO_NO_WS
-    if (pl.load_x == LD_TMA && pl.load_u == LD_TMA) {  // warp-specialised kernel
-        auto kern = wino::fp32ws::fused_fp32_ws_kernel;
-        const int wsm = wino::fp32ws::Smem::bytes;
-        wino_status_t s = ensure_smem_attr(kern, dev, wsm, g_attr_ws);
+    const bool box32 = prm.xnb == BN;
+    if (pl.ws && pl.split == 1) {  // warp-specialised persistent kernel, one CTA per SM
+        auto kern = box32 ? wino::fp32ws::fused_fp32_ws_kernel<false, true>
+                          : wino::fp32ws::fused_fp32_ws_kernel<false, false>;
+        wino_status_t s = ensure_smem_attr(kern, dev, sm, g_attr_ws_k[0][box32]);
         if (s != WINO_OK) return s;
-        const int sms = sm_count(dev);
-        const int64_t grid = g < sms ? g : sms;  // persistent: one CTA per SM
-        kern<<<dim3(static_cast<unsigned>(grid)), wino::fp32ws::NT, wsm, st>>>(prm, static_cast<int>(g));
+        kern<<<dim3(static_cast<unsigned>(pl.grid)), wino::fp32ws::NT, sm, st>>>(prm, static_cast<int>(g));
         cudaError_t e = cudaGetLastError();
         return e == cudaSuccess ? WINO_OK : cuda_fail(e);
     }
-#endif
+    if (pl.ws) {  // split-C: clusters of pl.split CTAs, partial outputs reduced through DSMEM
+        auto kern = box32 ? wino::fp32ws::fused_fp32_ws_kernel<true, true>
+                          : wino::fp32ws::fused_fp32_ws_kernel<true, false>;
+        wino_status_t s = ensure_smem_attr(kern, dev, sm, g_attr_ws_k[1][box32]);
+        if (s != WINO_OK) return s;
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = pl.split;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
+        cfg.blockDim = dim3(wino::fp32ws::NT);
+        cfg.dynamicSmemBytes = sm;
+        cfg.stream = st;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cudaError_t e = cudaLaunchKernelEx(&cfg, kern, prm, static_cast<int>(g));
+        return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+    }
     switch (pl.load_x * 3 + pl.load_u) {
         case LD_TMA * 3 + LD_TMA: return launch_fp32<LD_TMA, LD_TMA>(prm, g, sm, dev, st);
         case LD_TMA * 3 + LD_CP4B: return launch_fp32<LD_TMA, LD_CP4B>(prm, g, sm, dev, st);
@@ -294,6 +413,16 @@ const char* wino_status_string(wino_status_t s) {
 
 int wino_last_cuda_error(void) { return g_last_cuda_error; }
 
+#ifdef WINO_WS_TRACE
+int wino_debug_cluster_slots(int split) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    return cluster_slots(split, dev);
+}
+int wino_debug_ws_trace(unsigned long long* host, int n) {
+    return (int)cudaMemcpyFromSymbol(host, wino::fp32ws::g_ws_trace, sizeof(unsigned long long) * n);
+}
+#endif
 #ifdef WINO_TC_TRACE
 // debug builds only: copy the tcgen05 kernel's CTA-0 event trace to the host
 int wino_debug_tc_trace(unsigned long long* host, int n) {
@@ -344,16 +473,22 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         return WINO_OK;
     }
     if (variant != 0) return WINO_ERR_UNSUPPORTED;
-    Fp32Plan p = plan_fp32(N, C, H, W, K);
+    int dev = -1;  // host-only planning unless an sm_100 device is current
+    {
+        int d;
+        if (check_device(&d) == WINO_OK) dev = d;
+        else cudaGetLastError();
+    }
+    Fp32Plan p = plan_fp32(N, C, H, W, K, true, dev, 0);
     plan->variant = 0;
     plan->bk = wino::fp32::BK;
     plan->bn = wino::fp32::BN;
     plan->bc = wino::fp32::BC;
-    plan->load_x = p.load_x;
+    plan->load_x = p.ws ? 2 : p.load_x;
     plan->load_u = p.load_u;
-    plan->split_c = 1;
-    plan->ctas = p.ctas;
-    plan->threads = wino::fp32::threads_for<kXpw>();
+    plan->split_c = p.split;
+    plan->ctas = p.tiles * p.split;
+    plan->threads = p.threads;
     plan->smem_bytes = p.smem;
     plan->launches = 1;
     return WINO_OK;
@@ -372,6 +507,23 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
     int dev;
     if ((s = check_device(&dev)) != WINO_OK) return s;
     return launch_fwd_fp32(x_dev, u_dev, K, y_dev, N, C, H, W, K, dev, reinterpret_cast<cudaStream_t>(stream));
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_split(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H,
+                                         int W, int K, int pad, int stride, int split_c, wino_stream_t stream) {
+    if (split_c != 0 && split_c != 1 && split_c != 2 && split_c != 4 && split_c != 8) return WINO_ERR_INVALID_ARG;
+    if (!x_dev || !u_dev || !y_dev) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (!aligned16(x_dev) || !aligned16(u_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t yb = size_t(K) * hwn * 4;
+    if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) || overlaps(y_dev, yb, u_dev, size_t(16) * C * K * 4))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    return launch_fwd_fp32(x_dev, u_dev, K, y_dev, N, C, H, W, K, dev, reinterpret_cast<cudaStream_t>(stream),
+                           split_c);
 }
 
 size_t wino_filter_workspace_bytes_tc(int C, int K, wino_tc_mode_t mode) {

@@ -64,8 +64,10 @@ def test_plan_shapes(name):
     assert p.variant == 0 and (p.bk, p.bn, p.bc) == (64, 32, 8)
     nv = c.N * c.tiles
     assert p.ctas == -(-nv // p.bn) * -(-c.K // p.bk) * p.split_c
-    assert p.threads == 256 and 0 < p.smem_bytes <= 232448
-    assert p.load_x == (2 if c.N % 32 == 0 else (1 if c.N % 4 == 0 else 0))
+    ws = (c.N % 32 == 0 or c.N in (4, 8, 16)) and c.K % 4 == 0  # warp-specialised TMA kernel
+    assert p.threads == (384 if ws else 256) and 0 < p.smem_bytes <= 232448
+    assert p.load_x == (2 if (ws or c.N % 32 == 0) else (1 if c.N % 4 == 0 else 0))
+    assert p.split_c in (1, 2, 4, 8) and (ws or p.split_c == 1)
     assert p.load_u == (2 if c.K % 4 == 0 else 0)
     assert p.launches >= 1
 
@@ -106,6 +108,27 @@ def test_fwd_argument_validation_host_side():
     assert L.wino_filter_transform_tc(ctypes.c_void_p(X), ctypes.c_void_p(U), 3, 5, 7, None) == 1
     assert L.wino_conv2d_f2x3_fwd_tc(ctypes.c_void_p(X), ctypes.c_void_p(U), ctypes.c_void_p(Y),
                                      2, 3, 4, 4, 5, 2, 1, 0, None) == 2  # pad != 1
+    for bad in (-1, 3, 5, 16):  # split-C factor must be 0 (auto), 1, 2, 4 or 8
+        assert L.wino_conv2d_f2x3_fwd_split(ctypes.c_void_p(X), ctypes.c_void_p(U), ctypes.c_void_p(Y),
+                                            2, 3, 4, 4, 5, 1, 1, bad, None) == 1
+    assert L.wino_conv2d_f2x3_fwd_split(ctypes.c_void_p(X), ctypes.c_void_p(U), ctypes.c_void_p(Y),
+                                        2, 3, 4, 4, 5, 0, 1, 2, None) == 2  # pad != 1
+
+
+@pytest.mark.parametrize("P", [2, 4, 8])
+def test_plan_splits_small_shards(P):
+    """Per-rank batch shards with fewer (k, nu) tiles than SMs get split-C,
+    and every shard of the BASELINE layers takes the warp-specialised TMA kernel."""
+    from paper_conf_ppopp_yanwc20_b200.dist import shard_range
+    for name in ("conv5_x", "conv4_x", "conv3_x", "conv2_x"):
+        c = CONFIGS[name]
+        lo, hi = shard_range(c.N, 0, P)
+        p = wino.plan(hi - lo, c.C, c.H, c.W, c.K)
+        assert p.threads == 384 and p.load_x == 2, (name, P)
+        tiles = p.ctas // p.split_c
+        if tiles < 64:
+            assert p.split_c > 1, (name, P, tiles)
+        assert p.split_c * 2 * 8 <= c.C or p.split_c == 1  # >= 2 channel blocks per CTA
 
 
 def test_tc_workspace_and_plan():
