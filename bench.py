@@ -226,7 +226,8 @@ def _config(args, layers, world):
         "variant": args.variant,
         "inputs": f"uniform[-1,1) fp32, torch seeds x={SEED_X} w={SEED_W}",
         "l2": "flushed before every timed step by a 512 MiB write + 256 MiB read (outside the events)",
-        "step": "per layer: FTF kernel + fused ITF/16xGEMM/OTF kernel; the whole step replayed from one CUDA graph",
+        "step": "per layer: FTF kernel + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
+                "its own FTF); the whole step replayed from one CUDA graph",
     }
 
 
@@ -323,16 +324,16 @@ def main():
                 if world > 1:
                     dist.broadcast(d["u"], src=0)
 
-        def run_layer(d, ftf=True, conv=True):
+        def run_layer(d, ftf=True, conv=True, ftf_stream=None):
             if d["n"] == 0:
                 return
             if ftf:
                 if f4:
-                    wino.filter_transform_f4(d["w"], out=d["u"])
+                    wino.filter_transform_f4(d["w"], out=d["u"], stream=ftf_stream)
                 elif tc:
-                    wino.filter_transform_tc(d["w"], variant, out=d["u"])
+                    wino.filter_transform_tc(d["w"], variant, out=d["u"], stream=ftf_stream)
                 else:
-                    wino.filter_transform(d["w"], out=d["u"])
+                    wino.filter_transform(d["w"], out=d["u"], stream=ftf_stream)
             if conv:
                 if f4:
                     wino.conv2d_f4(d["x"], d["u"], out=d["y"])
@@ -341,9 +342,24 @@ def main():
                 else:
                     wino.conv2d(d["x"], d["u"], out=d["y"])
 
+        side = torch.cuda.Stream(dev)
+
         def step():
+            # The layers' filter transforms (a1) do not depend on the convolutions, so they run
+            # on a side stream: FTF of layer l+1 overlaps conv l (the persistent conv grids
+            # leave SMs free at small per-rank batches).  conv l waits for its own FTF only.
+            fork = torch.cuda.Event()
+            fork.record(stream)
+            side.wait_event(fork)
+            ready = []
             for d in per:
-                run_layer(d)
+                run_layer(d, conv=False, ftf_stream=side)
+                ev = torch.cuda.Event()
+                ev.record(side)
+                ready.append(ev)
+            for d, ev in zip(per, ready):
+                stream.wait_event(ev)
+                run_layer(d, ftf=False)
 
         for _ in range(args.warmup):
             flush_l2(1.0)
