@@ -238,7 +238,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default="resnet_3x3", choices=["resnet_3x3", *RESNET_LAYERS, "tiny"])
-    ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32", "f4_fp32"])
+    ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
@@ -299,7 +299,8 @@ def main():
         before each, outside the events), then a per-layer breakdown.  Max over ranks."""
         f4 = variant == "f4_fp32"  # NEXT row N1: fused F(4x4,3x3), FTF4 + one fused launch per layer
         tc = variant in ("tf32", "3xtf32")
-        if f4:
+        nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
+        if f4 or nchw:
             launches = sum(2 for d in per if d["n"] > 0)
         else:
             vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[variant]
@@ -317,6 +318,14 @@ def main():
                 d["u"] = wino.filter_transform_tc(d["w"], variant)
                 if world > 1:
                     dist.broadcast(d["u"].data, src=0)
+            elif nchw:
+                # layout change of the synthetic inputs at setup (outside the timed region)
+                d["x_nchw"] = d["x"].permute(3, 0, 1, 2).contiguous()
+                d["w_kcrs"] = d["w"].permute(3, 0, 1, 2).contiguous()
+                d["y_nchw"] = torch.empty((max(d["n"], 1), d["cfg"].K, d["cfg"].H, d["cfg"].W),
+                                          dtype=torch.float32, device=dev)
+                d["u"] = torch.empty((d["cfg"].C, 4, 4, d["cfg"].K), dtype=torch.float32, device=dev)
+                wino.filter_transform_kcrs(d["w_kcrs"], out=d["u"])
             else:
                 d["u"] = torch.empty((d["cfg"].C, 4, 4, d["cfg"].K), dtype=torch.float32, device=dev)
                 if rank == 0:
@@ -332,6 +341,8 @@ def main():
                     wino.filter_transform_f4(d["w"], out=d["u"], stream=ftf_stream)
                 elif tc:
                     wino.filter_transform_tc(d["w"], variant, out=d["u"], stream=ftf_stream)
+                elif nchw:
+                    wino.filter_transform_kcrs(d["w_kcrs"], out=d["u"], stream=ftf_stream)
                 else:
                     wino.filter_transform(d["w"], out=d["u"], stream=ftf_stream)
             if conv:
@@ -339,6 +350,8 @@ def main():
                     wino.conv2d_f4(d["x"], d["u"], out=d["y"])
                 elif tc:
                     wino.conv2d_tc(d["x"], d["u"], out=d["y"])
+                elif nchw:
+                    wino.conv2d_nchw(d["x_nchw"], d["u"], out=d["y_nchw"])
                 else:
                     wino.conv2d(d["x"], d["u"], out=d["y"])
 
@@ -433,7 +446,7 @@ def main():
     main_m = measure(args.variant, sample_clocks=True)
     others = {}
     if not args.no_variants:
-        for v in ("fp32", "tf32", "3xtf32", "f4_fp32"):
+        for v in ("fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw"):
             if v == "f4_fp32" and any(d["n"] % 16 for d in per if d["n"]):
                 continue  # the F(4x4) kernel needs N % 16 == 0 per rank
             if v != args.variant:
@@ -529,7 +542,12 @@ def main():
         vrep[v] = {"value": val, "ms_per_step": m["ms_step"], "pct_fp32_peak_eff": 100 * val / fp32_peak,
                    "layers_eff_tflops": {d["cfg"].name: d["cfg"].eff_flops / (m["conv_ms"][i] * 1e-3) / 1e12
                                          for i, d in enumerate(per) if d["n"]},
-                   "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4}[v]}
+                   "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4, "fp32_nchw": 1e-4}[v]}
+        if v == "fp32_nchw":
+            ach = sum(_ewmm_flops(d["cfg"], "fp32") for d in per if d["n"]) / (sum(m["conv_ms"]) * 1e-3) / 1e12
+            vrep[v]["roofline"] = {"bound": "alu", "achieved": ach, "peak": fp32_peak, "unit": "TFLOP/s",
+                                   "frac": ach / fp32_peak,
+                                   "achieved_def": "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) / conv time (NCHW)"}
         if v == "f4_fp32":
             ach = sum(_ewmm_flops(d["cfg"], v) for d in per if d["n"]) / (sum(m["conv_ms"]) * 1e-3) / 1e12
             vrep[v]["roofline"] = {"bound": "alu", "achieved": ach, "peak": fp32_peak, "unit": "TFLOP/s",

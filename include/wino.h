@@ -116,9 +116,10 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
  * than SMs.  With split_c = S > 1 a thread-block cluster of S CTAs shares each
  * block, CTA r summing channels [r*C/S, (r+1)*C/S) (per 8-channel block), and
  * because the output transform is linear (Eq. 8) the S partial 2x2
- * outputs are added through distributed shared memory in rank order 0..S-1:
- * deterministic, no atomics, no workspace.  Results equal the unsplit kernel's
- * up to FP32 summation order (bit-identical on small-integer inputs).
+ * outputs are pushed through distributed shared memory to the CTA owning the
+ * filter (st.async) and summed there in a fixed order: deterministic, no
+ * atomics, no workspace.  Results equal the unsplit kernel's up to FP32
+ * summation order (bit-identical on small-integer inputs).
  *   split_c : 0 = the library's choice (what wino_conv2d_f2x3_fwd does),
  *             1, 2, 4 or 8 = forced; anything else -> WINO_ERR_INVALID_ARG.
  *             Honoured by the warp-specialised kernel (N % 32 == 0 or
@@ -128,6 +129,28 @@ wino_status_t wino_conv2d_f2x3_fwd(const float* x_dev, const float* u_dev, float
 wino_status_t wino_conv2d_f2x3_fwd_split(const float* x_dev, const float* u_dev, float* y_dev,
                                          int N, int C, int H, int W, int K, int pad, int stride,
                                          int split_c, wino_stream_t stream);
+
+/*
+ * NCHW front end (NEXT row N2; Sec. 8.4: "The implementation in this
+ * work can be ported to NCHW layout with little effort ... The offsets of global
+ * and shared memory accesses need to be recomputed, while all other
+ * optimizations can be adopted").  Same computation as wino_conv2d_f2x3_fwd
+ * (Eq. 4 via Eq. 5-8), PyTorch's default layouts:
+ *   wino_filter_transform_kcrs : w_kcrs_dev (K,C,3,3) fp32 (torch conv weight)
+ *                                -> u_dev (C,4,4,K), identical to
+ *                                wino_filter_transform of the CRSK permutation.
+ *   wino_conv2d_f2x3_fwd_nchw  : x_nchw_dev (N,C,H,W), u_dev (C,4,4,K)
+ *                                -> y_nkhw_dev (N,K,H,W), fully overwritten.
+ * The input tiles are gathered with per-CTA offset tables (4 B cp.async, zero
+ * fill = padding) and the tiles of one image are the fastest-varying part of
+ * nu; the FFMA micro-kernel and output transform are the FP32 kernel's.
+ * Arguments, alignment, aliasing and errors as wino_conv2d_f2x3_fwd.
+ */
+wino_status_t wino_filter_transform_kcrs(const float* w_kcrs_dev, float* u_dev, int C, int K,
+                                         wino_stream_t stream);
+wino_status_t wino_conv2d_f2x3_fwd_nchw(const float* x_nchw_dev, const float* u_dev, float* y_nkhw_dev,
+                                        int N, int C, int H, int W, int K, int pad, int stride,
+                                        wino_stream_t stream);
 
 /*
  * Tensor-core variant (a5' of SURVEY 8(a)): the Winograd-domain GEMM (Eq. 7)

@@ -24,6 +24,7 @@ __all__ = [
     "TcFilter", "filter_workspace_bytes_tc", "filter_transform_tc", "conv2d_tc",
     "host_multi_workspace_bytes", "conv2d_host_multi",
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
+    "filter_transform_kcrs", "conv2d_nchw",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -99,6 +100,12 @@ def lib() -> ctypes.CDLL:
     if hasattr(L, "wino_conv2d_f2x3_fwd_split") or not os.environ.get("WINO_LIB_PATH"):  # A/B builds may predate it
         L.wino_conv2d_f2x3_fwd_split.restype = i
         L.wino_conv2d_f2x3_fwd_split.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
+    for name in ("wino_filter_transform_kcrs", "wino_conv2d_f2x3_fwd_nchw"):
+        if hasattr(L, name) or not os.environ.get("WINO_LIB_PATH"):  # A/B builds may predate them
+            getattr(L, name).restype = i
+    if hasattr(L, "wino_filter_transform_kcrs") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_filter_transform_kcrs.argtypes = [vp, vp, i, i, vp]
+        L.wino_conv2d_f2x3_fwd_nchw.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
     L.wino_conv2d_f2x3_fwd_tc.restype = i
     L.wino_conv2d_f2x3_fwd_tc.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
     L.wino_filter_workspace_bytes_tc.restype = st
@@ -271,6 +278,47 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
                    "wino_conv2d_f2x3_fwd_split")
         else:
             _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
+    return out
+
+
+def filter_transform_kcrs(w_kcrs: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """NEXT row N2 (Sec. 8.4): FTF from PyTorch's conv weight layout w (K,C,3,3) -> u (C,4,4,K)."""
+    _need_cuda_f32(w_kcrs, "w_kcrs", 4)
+    K, C, r, s = w_kcrs.shape
+    if (r, s) != (3, 3):
+        raise ValueError(f"w_kcrs must be (K,C,3,3), got {tuple(w_kcrs.shape)}")
+    if out is None:
+        out = torch.empty((C, 4, 4, K), dtype=torch.float32, device=w_kcrs.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (C, 4, 4, K):
+        raise ValueError("out must be (C,4,4,K)")
+    with torch.cuda.device(w_kcrs.device):
+        _check(lib().wino_filter_transform_kcrs(ctypes.c_void_p(w_kcrs.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                                C, K, _stream_ptr(stream)), "wino_filter_transform_kcrs")
+    return out
+
+
+def conv2d_nchw(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """NEXT row N2 (Sec. 8.4): fused Winograd conv on NCHW tensors, pad 1 stride 1:
+    x (N,C,H,W), u (C,4,4,K) -> y (N,K,H,W) -- torch.nn.functional.conv2d(x, w, padding=1)
+    with u = filter_transform_kcrs(w)."""
+    _need_cuda_f32(x, "x", 4)
+    _need_cuda_f32(u, "u", 4)
+    N, C, H, W = x.shape
+    if u.shape[0] != C or tuple(u.shape[1:3]) != (4, 4):
+        raise ValueError(f"u must be (C,4,4,K) with C={C}, got {tuple(u.shape)}")
+    if u.device != x.device:
+        raise ValueError("x and u must be on the same device")
+    K = u.shape[3]
+    if out is None:
+        out = torch.empty((N, K, H, W), dtype=torch.float32, device=x.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (N, K, H, W):
+        raise ValueError("out must be (N,K,H,W)")
+    with torch.cuda.device(x.device):
+        _check(lib().wino_conv2d_f2x3_fwd_nchw(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()),
+                                               ctypes.c_void_p(out.data_ptr()), N, C, H, W, K, 1, 1,
+                                               _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_nchw")
     return out
 
 

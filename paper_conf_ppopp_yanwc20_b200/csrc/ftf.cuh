@@ -26,4 +26,22 @@ __global__ void __launch_bounds__(FTF_THREADS) ftf_kernel(const float* __restric
     for (int e = 0; e < 16; ++e) uc[(size_t)e * K] = t[e];
 }
 
+// Same transform reading PyTorch's weight layout w (K,C,3,3) ("KCRS"), writing u
+// (C,4,4,K): the NCHW front end (Sec. 8.4).  k fastest across threads, so the
+// 16 stores stay coalesced; each thread's 9 loads are one contiguous 36 B run.
+__global__ void __launch_bounds__(FTF_THREADS) ftf_kcrs_kernel(const float* __restrict__ w,
+                                                               float* __restrict__ u, int C, int K) {
+    const long idx = (long)blockIdx.x * FTF_THREADS + threadIdx.x;
+    if (idx >= (long)C * K) return;
+    const int c = (int)(idx / K), k = (int)(idx - (long)c * K);
+    const float* wk = w + ((size_t)k * C + c) * 9;
+    float g[9], t[16];
+#pragma unroll
+    for (int e = 0; e < 9; ++e) g[e] = __ldg(wk + e);
+    ftf_4x4(g, t);
+    float* uc = u + (size_t)c * 16 * K + k;
+#pragma unroll
+    for (int e = 0; e < 16; ++e) uc[(size_t)e * K] = t[e];
+}
+
 }  // namespace wino

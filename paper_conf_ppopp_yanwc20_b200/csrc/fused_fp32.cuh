@@ -69,6 +69,13 @@ struct __align__(64) Params {
     int xnb;     // n-extent of one x TMA box: 32, or N when N | 32 (WS kernel: 32/xnb boxes per stage)
     int split;   // split-C factor S = cluster size (WS kernel; 1 = no split)
     int itf_map[64];  // WS kernel, N | 32: ITF task of thread (warp-9)*32+lane: c | n4 << 3 | xoff << 8
+    // Generic kernel: element strides of x (c, n, h, w) and y (k, n, h, w), so any dense
+    // layout works (CHWN / KHWN: the paper's, Table 4; NCHW / NKHW: Sec. 8.4), and
+    // the order of nu = (tile, n): tfast = 0 -> n fastest (CHWN), 1 -> tile fastest (NCHW:
+    // neighbouring lanes read / write neighbouring pixels of one image).
+    long long xs_c, xs_n, xs_h, xs_w, ys_k, ys_n, ys_h, ys_w;
+    int tfast;
+    int T;  // ceil(H/2) * ceil(W/2)
 };
 
 // XPW = Winograd elements xi per warp: 2 -> 8 warps / 256 threads (the paper's
@@ -94,7 +101,6 @@ __global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const
     const int kb = blockIdx.x % p.num_kb;
     const int nb = blockIdx.x / p.num_kb;
     const int k0 = kb * BK, nu0 = nb * BN;
-    const size_t HWN = (size_t)p.H * p.W * p.N;
 
     if constexpr (kTma) {
         if (tid == 0) {
@@ -120,10 +126,12 @@ __global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const
             const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
             int off = -1;
             if (nu < p.NV) {
-                const int t = nu / p.N, n = nu - t * p.N;
+                int t, n;
+                if (p.tfast) n = nu / p.T, t = nu - n * p.T;
+                else t = nu / p.N, n = nu - t * p.N;
                 const int th = t / p.TW, tw = t - th * p.TW;
                 const int h = 2 * th - 1 + (pos >> 2), w = 2 * tw - 1 + (pos & 3);
-                if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
+                if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (int)(n * p.xs_n + h * p.xs_h + w * p.xs_w);
             }
             xtab[e] = off;
         }
@@ -170,7 +178,7 @@ __global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const
                 const int c = c0 + cl;
                 const int off = xtab[e];
                 const bool ok = (c < p.C) && (off >= 0);
-                const float* src = ok ? p.x + (size_t)c * HWN + off : p.x;
+                const float* src = ok ? p.x + c * p.xs_c + off : p.x;
                 const uint32_t dst = smem_u32(xs + cl * 16 * BN + e);
                 if constexpr (VX == 4) cp_async16(dst, src, ok);
                 else cp_async4(dst, src, ok);
@@ -311,12 +319,14 @@ __global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const
 
     const int nu = nu0 + lane;
     if (nu < p.NV) {
-        const int t = nu / p.N, n = nu - t * p.N;
+        int t, n;
+        if (p.tfast) n = nu / p.T, t = nu - n * p.T;
+        else t = nu / p.N, n = nu - t * p.N;
         const int th = t / p.TW, tw = t - th * p.TW;
         const int i0 = 2 * th, j0 = 2 * tw;
         const bool okr = i0 + 1 < p.H, okc = j0 + 1 < p.W;  // odd H/W: drop extra outputs (L1155)
-        const size_t base = ((size_t)i0 * p.W + j0) * p.N + n;
-        const size_t dW = (size_t)p.W * p.N;
+        const long long base = n * p.ys_n + i0 * p.ys_h + j0 * p.ys_w;
+        const long long dW = p.ys_h, dN = p.ys_w;
 #pragma unroll 2
         for (int r = 0; r < BK / NWARP; ++r) {
             const int kl = warp + NWARP * r, k = k0 + kl;
@@ -325,11 +335,11 @@ __global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const
 #pragma unroll
             for (int e = 0; e < 16; ++e) m[e] = ep[(e * BK + kl) * EP_LD + (lane ^ 1)];
             otf_2x2(m, o);
-            float* yk = p.y + (size_t)k * HWN + base;
+            float* yk = p.y + k * p.ys_k + base;
             yk[0] = o[0];
-            if (okc) yk[p.N] = o[1];
+            if (okc) yk[dN] = o[1];
             if (okr) yk[dW] = o[2];
-            if (okr && okc) yk[dW + p.N] = o[3];
+            if (okr && okc) yk[dW + dN] = o[3];
         }
     }
 }

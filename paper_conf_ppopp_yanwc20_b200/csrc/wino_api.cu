@@ -271,11 +271,20 @@ std::atomic<uint64_t> g_attr_ws_k[2][2];
 
 // FP32 fused conv on validated arguments; u may be a K-slice of a wider (C,4,4,ldu) array.
 // force_split: 0 = planner's choice, else the split-C factor (1, 2, 4, 8).
+// nchw: x (N,C,H,W) / y (N,K,H,W) instead of the paper's CHWN / KHWN (generic kernel).
 wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, float* y_dev, int N, int C, int H,
-                              int W, int K, int dev, cudaStream_t st, int force_split = 0) {
+                              int W, int K, int dev, cudaStream_t st, int force_split = 0, bool nchw = false) {
     using namespace wino::fp32;
     const bool u_tma_ok = ldu % 4 == 0 && aligned16(u_dev);
     Fp32Plan pl = plan_fp32(N, C, H, W, K, u_tma_ok, dev, force_split);
+    if (nchw) {  // strided gathers (Sec. 8.4: "offsets ... need to be recomputed")
+        pl.ws = false;
+        pl.split = 1;
+        pl.load_x = LD_CP4B;
+        pl.grid = pl.tiles;
+        pl.threads = threads_for<kXpw>();
+        pl.smem = Smem<kStages>::bytes;
+    }
     Params prm;
     std::memset(&prm, 0, sizeof(prm));
     prm.x = x_dev;
@@ -293,6 +302,17 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
     prm.num_it = (C + BC - 1) / BC;
     prm.xnb = pl.ws ? pl.xnb : BN;
     prm.split = pl.split;
+    prm.T = ((H + 1) / 2) * prm.TW;
+    const long long hw = (long long)H * W;
+    if (nchw) {
+        prm.xs_c = hw, prm.xs_n = (long long)C * hw, prm.xs_h = W, prm.xs_w = 1;
+        prm.ys_k = hw, prm.ys_n = (long long)K * hw, prm.ys_h = W, prm.ys_w = 1;
+        prm.tfast = 1;
+    } else {
+        prm.xs_c = hw * N, prm.xs_n = 1, prm.xs_h = (long long)W * N, prm.xs_w = N;
+        prm.ys_k = hw * N, prm.ys_n = 1, prm.ys_h = (long long)W * N, prm.ys_w = N;
+        prm.tfast = 0;
+    }
     if (pl.ws && prm.xnb < BN) {
         // ITF lane map of the small-N WS kernel (conflict-free LDS.128 / STS.128, see fused_fp32_ws.cuh)
         const int Q = prm.xnb / 4;
@@ -524,6 +544,39 @@ wino_status_t wino_conv2d_f2x3_fwd_split(const float* x_dev, const float* u_dev,
     if ((s = check_device(&dev)) != WINO_OK) return s;
     return launch_fwd_fp32(x_dev, u_dev, K, y_dev, N, C, H, W, K, dev, reinterpret_cast<cudaStream_t>(stream),
                            split_c);
+}
+
+wino_status_t wino_filter_transform_kcrs(const float* w_kcrs_dev, float* u_dev, int C, int K, wino_stream_t stream) {
+    if (!w_kcrs_dev || !u_dev || C <= 0 || K <= 0) return WINO_ERR_INVALID_ARG;
+    if (int64_t(16) * C * K > kMaxElems) return WINO_ERR_TOO_LARGE;
+    if (!aligned16(w_kcrs_dev) || !aligned16(u_dev)) return WINO_ERR_MISALIGNED;
+    if (overlaps(w_kcrs_dev, size_t(9) * C * K * 4, u_dev, size_t(16) * C * K * 4)) return WINO_ERR_INVALID_ARG;
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    const int64_t n = int64_t(C) * K;
+    const unsigned blocks = static_cast<unsigned>((n + wino::FTF_THREADS - 1) / wino::FTF_THREADS);
+    wino::ftf_kcrs_kernel<<<blocks, wino::FTF_THREADS, 0, reinterpret_cast<cudaStream_t>(stream)>>>(w_kcrs_dev,
+                                                                                                   u_dev, C, K);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_nchw(const float* x_nchw_dev, const float* u_dev, float* y_nkhw_dev, int N, int C,
+                                        int H, int W, int K, int pad, int stride, wino_stream_t stream) {
+    if (!x_nchw_dev || !u_dev || !y_nkhw_dev) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (!aligned16(x_nchw_dev) || !aligned16(u_dev) || !aligned16(y_nkhw_dev)) return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t yb = size_t(K) * hwn * 4;
+    if (overlaps(y_nkhw_dev, yb, x_nchw_dev, size_t(C) * hwn * 4) ||
+        overlaps(y_nkhw_dev, yb, u_dev, size_t(16) * C * K * 4))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    return launch_fwd_fp32(x_nchw_dev, u_dev, K, y_nkhw_dev, N, C, H, W, K, dev,
+                           reinterpret_cast<cudaStream_t>(stream), 1, true);
 }
 
 size_t wino_filter_workspace_bytes_tc(int C, int K, wino_tc_mode_t mode) {

@@ -1,0 +1,97 @@
+"""GPU parity of NEXT row N2 -- the NCHW front end (Sec. 8.4):
+wino_filter_transform_kcrs + wino_conv2d_f2x3_fwd_nchw against the fp64 oracle
+(Eq. 4; the oracle works in the paper's CHWN / CRSK layouts, so inputs are
+permuted on the host -- a layout change, no arithmetic).
+
+Bars as tests/test_gpu_parity.py: bit-exact on small integers, <= 1e-4 of
+max|y| on random inputs; u from the KCRS weight equals u from CRSK bit for bit.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth_inputs import CONFIGS, Conv3x3Config, make_inputs, sample_points
+
+pytestmark = pytest.mark.gpu
+
+FP32_TOL = 1e-4
+DEV = "cuda:0"
+
+
+@pytest.fixture(scope="module")
+def wino():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ppopp_yanwc20_b200 as w
+    w.lib()
+    return w
+
+
+def _nchw(x_chwn):
+    return x_chwn.permute(3, 0, 1, 2).contiguous()
+
+
+def _kcrs(w_crsk):
+    return w_crsk.permute(3, 0, 1, 2).contiguous()
+
+
+def _run(wino, x, w):
+    u = wino.filter_transform_kcrs(_kcrs(w).to(DEV))
+    y = wino.conv2d_nchw(_nchw(x).to(DEV), u)
+    torch.cuda.synchronize()
+    return u.cpu(), y.cpu().permute(1, 2, 3, 0).contiguous()  # (N,K,H,W) -> (K,H,W,N)
+
+
+SHAPES = [
+    (1, 1, 1, 1, 1), (1, 8, 8, 8, 8), (3, 7, 5, 5, 5), (2, 9, 65, 7, 7), (4, 20, 70, 13, 9),
+    (5, 17, 130, 6, 10), (32, 16, 64, 9, 9), (2, 64, 64, 16, 16), (7, 40, 72, 11, 12), (1, 3, 3, 1, 17),
+]
+
+
+@pytest.mark.parametrize("shape", SHAPES, ids=[str(s) for s in SHAPES])
+def test_nchw_small_int_bit_exact(wino, shape):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nchw", N, C, K, H, W), kind="smallint")
+    u, y = _run(wino, x, w)
+    assert np.array_equal(u.double().numpy(), oracle.filter_transform(w))
+    assert np.array_equal(y.double().numpy(), oracle.direct_conv(x, w))
+
+
+@pytest.mark.parametrize("shape", SHAPES, ids=[str(s) for s in SHAPES])
+def test_nchw_random(wino, shape):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nchw", N, C, K, H, W), kind="uniform", seed_x=31, seed_w=32)
+    u, y = _run(wino, x, w)
+    assert np.array_equal(u.numpy(), wino.filter_transform(w.to(DEV)).cpu().numpy())
+    assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= FP32_TOL
+
+
+@pytest.mark.parametrize("name", ["conv5_x", "conv4_x", "conv3_x", "conv2_x"])
+def test_nchw_full_configs_sampled(wino, name):
+    cfg = CONFIGS[name]
+    for kind in ("smallint", "uniform"):
+        x, w = make_inputs(cfg, kind=kind)
+        _, y = _run(wino, x, w)
+        idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 2000)
+        ref = oracle.direct_sample(x, w, idx)
+        ii = idx.numpy()
+        got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
+        if kind == "smallint":
+            assert np.array_equal(got, ref)
+        else:
+            den = max(float(np.max(np.abs(ref))), 1e-30)
+            assert float(np.max(np.abs(got - ref))) / den <= FP32_TOL
+
+
+def test_nchw_matches_chwn_kernel(wino):
+    """Same convolution through both layouts: the NCHW path and the CHWN path agree
+    within the FP32 bound (their per-output summation orders are the same kernel's)."""
+    cfg = Conv3x3Config("both", 16, 64, 128, 14, 14)
+    x, w = make_inputs(cfg)
+    u = wino.filter_transform(w.to(DEV))
+    y_chwn = wino.conv2d(x.to(DEV), u, split_c=1)
+    y_nchw = wino.conv2d_nchw(_nchw(x).to(DEV), u).permute(1, 2, 3, 0)
+    torch.cuda.synchronize()
+    d = (y_chwn.double() - y_nchw.double()).abs().max() / y_chwn.double().abs().max()
+    assert float(d) <= FP32_TOL
