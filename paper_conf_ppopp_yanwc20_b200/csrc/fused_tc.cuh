@@ -136,11 +136,11 @@ struct Cfg {
     static constexpr int UNITS_PER_CB = 16 / XPU;
     static constexpr int A_TILE = a_tile<MM>();
     static constexpr int UNIT = XPU * P * A_TILE;               // 64 KB (MM=128) / 32 KB (MM=64)
-    static constexpr int U_SLOTS = (MM == 64 && XM == 2) ? 3 : 2;
+    static constexpr int U_SLOTS = (MM == 64 && XM >= 2) ? 3 : 2;
     static constexpr int X_SLOTS = 2;                           // raw x boxes in flight (L2-prefetched)
     static constexpr int X_SLOT = NH * XS_BYTES;
     static constexpr int V_SLOT = 16 * NH * P * B_TILE;        // 16 / 32 KB
-    static constexpr int TAB = (XM == 2) ? 0 : 16 * BN * NH * 4;  // cp.async gather table
+    static constexpr int TAB = (XM >= 2) ? 0 : 16 * BN * NH * 4;  // cp.async gather table
     static constexpr int OFF_U = 0;
     static constexpr int OFF_X = OFF_U + U_SLOTS * UNIT;
     static constexpr int OFF_V = OFF_X + X_SLOTS * X_SLOT;
@@ -153,7 +153,8 @@ struct Cfg {
     static_assert(BYTES <= 232448, "shared memory budget");
 };
 
-// XM: 2 = TMA x box (N % 32 == 0), 1 = cp.async 16 B gather, 0 = cp.async 4 B gather
+// XM: 2 = TMA x box (N % 32 == 0), 3 = 32/N TMA boxes per nu-half (N in {4, 8, 16}: the
+// per-rank batches of batch sharding), 1 = cp.async 16 B gather, 0 = cp.async 4 B gather
 template <int P, int XM, int MM>
 __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__ Params p) {
     using G = Cfg<P, MM, XM>;
@@ -194,7 +195,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         mbar_init(acc_full, 1);
         mbar_init(acc_empty, EPI_WARPS);
         fence_mbar_init();
-        if constexpr (XM == 2) tma_prefetch_desc(&p.tmx);
+        if constexpr (XM >= 2) tma_prefetch_desc(&p.tmx);
     }
     if (warp == 0) tmem_alloc(tmem_slot, 512);
     tc_fence_before();
@@ -211,7 +212,11 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
                 const int nu0 = (tile / p.num_kb) * TN;
                 int tma_n0[NH], tma_w0[NH], tma_h0[NH];
-                if constexpr (XM == 2) {
+                if constexpr (XM == 3) {
+                    // first image tile of each half; the half's 32/N boxes are tiles t0 .. t0 + 32/N - 1
+#pragma unroll
+                    for (int h = 0; h < NH; ++h) tma_n0[h] = (nu0 + h * BN) / p.N;
+                } else if constexpr (XM == 2) {
 #pragma unroll
                     for (int h = 0; h < NH; ++h) {  // N % 32 == 0: each half = 32 consecutive n of one image tile
                         const int nuh = nu0 + h * BN;
@@ -248,7 +253,22 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                     const int xs = gcb % G::X_SLOTS;
                     if (gcb >= G::X_SLOTS) mbar_wait(&x_empty[xs], ((gcb / G::X_SLOTS) - 1) & 1);
                     float* xdst = sx + xs * (G::X_SLOT / 4);
-                    if constexpr (XM == 2) {
+                    if constexpr (XM == 3) {
+                        if (lane == 0) {
+                            mbar_arrive_expect_tx(&x_full[xs], G::X_SLOT);
+                            const int nbox = BN / p.N;
+#pragma unroll
+                            for (int h = 0; h < NH; ++h)
+                                for (int b = 0; b < nbox; ++b) {
+                                    const int t = tma_n0[h] + b;
+                                    const bool live = t * p.N < p.NV;
+                                    const int th = t / p.TW, tw = t - th * p.TW;
+                                    // -1: zero fill = padding (Sec. 3.5); -8: tile past the end -> zeros
+                                    tma_load_4d(xdst + h * (XS_BYTES / 4) + b * (BC * 16 * p.N), &p.tmx, &x_full[xs], 0,
+                                                live ? 2 * tw - 1 : -8, live ? 2 * th - 1 : -8, cb * BC);
+                                }
+                        }
+                    } else if constexpr (XM == 2) {
                         if (lane == 0) {
                             mbar_arrive_expect_tx(&x_full[xs], G::X_SLOT);
 #pragma unroll
@@ -352,6 +372,9 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         const int nl = (iw & 3) * 8 + (lane >> 2);
         const int cl = (iw >> 2) * 4 + (lane & 3);
         const uint32_t voff = (nl >> 3) * 256 + (cl >> 2) * 128 + (nl & 7) * 16 + (cl & 3) * 4;
+        // raw x of (cl, nl): [c][pos][n32] (XM != 3) or [box][c][pos][n:N] (XM == 3)
+        const int xnb = XM == 3 ? p.N : BN;
+        const int xoff = (nl / xnb) * (BC * 16 * xnb) + cl * 16 * xnb + nl % xnb;
         int gcb = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
             for (int cb = 0; cb < NCB; ++cb, ++gcb) {
@@ -360,10 +383,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                 float t[NH][16];
 #pragma unroll
                 for (int h = 0; h < NH; ++h) {
-                    const float* xsrc = sx + xs * (G::X_SLOT / 4) + h * (XS_BYTES / 4) + cl * 16 * BN + nl;
+                    const float* xsrc = sx + xs * (G::X_SLOT / 4) + h * (XS_BYTES / 4) + xoff;
                     float d[16];
 #pragma unroll
-                    for (int e = 0; e < 16; ++e) d[e] = xsrc[e * BN];
+                    for (int e = 0; e < 16; ++e) d[e] = xsrc[e * xnb];
                     itf_4x4(d, t[h]);  // consumes the loads
                 }
                 __syncwarp();
@@ -432,6 +455,24 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
 #pragma unroll
                     for (int j = 0; j < BN; j += 4)
                         *reinterpret_cast<float4*>(dst + j) = make_float4(o[j][q], o[j + 1][q], o[j + 2][q], o[j + 3][q]);
+                }
+            } else if constexpr (XM == 3) {
+                // N | 32, N % 4 == 0: every group of 4 nu is 4 consecutive n of one image tile
+#pragma unroll
+                for (int j = 0; j < BN; j += 4) {
+                    const int nu = nu0 + j;
+                    if (nu >= p.NV) break;
+                    const int t = nu / p.N, n = nu - t * p.N;
+                    const int th = t / p.TW, tw = t - th * p.TW;
+                    const int i0 = 2 * th, j0 = 2 * tw;
+                    float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const int a = q >> 1, b = q & 1;
+                        if (i0 + a >= p.H || j0 + b >= p.W) continue;  // odd H/W (L1155)
+                        *reinterpret_cast<float4*>(yk + a * dW + b * p.N) =
+                            make_float4(o[j][q], o[j + 1][q], o[j + 2][q], o[j + 3][q]);
+                    }
                 }
             } else {
 #pragma unroll

@@ -218,7 +218,7 @@ wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem,
 }  // namespace
 
 namespace {
-std::atomic<uint64_t> g_attr_tc[2][3][2];
+std::atomic<uint64_t> g_attr_tc[2][4][2];
 template <int P, int XM, int MM>
 wino_status_t launch_tc(const wino::tc::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
     auto kern = wino::tc::fused_tc_kernel<P, XM, MM>;
@@ -483,7 +483,7 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->bk = mm;
         plan->bn = BN * (128 / mm);
         plan->bc = BC;
-        plan->load_x = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
+        plan->load_x = (N % 32 == 0 || N == 4 || N == 8 || N == 16) ? 2 : (N % 4 == 0 ? 1 : 0);
         plan->load_u = 3;  // bulk copy of the pre-arranged operand tiles
         plan->split_c = 1;
         plan->ctas = ((nv + plan->bn - 1) / plan->bn) * ((K + mm - 1) / mm);  // tiles (persistent grid <= #SMs)
@@ -644,25 +644,28 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
     prm.num_kb = (K + mm - 1) / mm;
     prm.num_cb = (C + BC - 1) / BC;
     prm.num_tiles = ((prm.NV + tn - 1) / tn) * prm.num_kb;
-    const int xm = (N % 32 == 0) ? 2 : (N % 4 == 0 ? 1 : 0);
-    if (xm == 2) {
+    const int xm = (N % 32 == 0) ? 2 : ((N == 4 || N == 8 || N == 16) ? 3 : (N % 4 == 0 ? 1 : 0));
+    if (xm >= 2) {
         const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
-        const cuuint32_t box[4] = {BN, 4, 4, BC};
+        const cuuint32_t box[4] = {cuuint32_t(xm == 2 ? BN : N), 4, 4, BC};
         if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
     }
     const int sms = sm_count(dev);
     const int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (mode == WINO_TC_TF32 && mm == 64) {
+        if (xm == 3) return launch_tc<1, 3, 64>(prm, ctas, dev, st);
         if (xm == 2) return launch_tc<1, 2, 64>(prm, ctas, dev, st);
         if (xm == 1) return launch_tc<1, 1, 64>(prm, ctas, dev, st);
         return launch_tc<1, 0, 64>(prm, ctas, dev, st);
     }
     if (mode == WINO_TC_TF32) {
+        if (xm == 3) return launch_tc<1, 3, 128>(prm, ctas, dev, st);
         if (xm == 2) return launch_tc<1, 2, 128>(prm, ctas, dev, st);
         if (xm == 1) return launch_tc<1, 1, 128>(prm, ctas, dev, st);
         return launch_tc<1, 0, 128>(prm, ctas, dev, st);
     }
+    if (xm == 3) return launch_tc<2, 3, 128>(prm, ctas, dev, st);
     if (xm == 2) return launch_tc<2, 2, 128>(prm, ctas, dev, st);
     if (xm == 1) return launch_tc<2, 1, 128>(prm, ctas, dev, st);
     return launch_tc<2, 0, 128>(prm, ctas, dev, st);

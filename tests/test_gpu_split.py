@@ -108,3 +108,47 @@ def test_rank_shards_sampled(wino, name, P, kind):
             assert np.isfinite(y.cpu().numpy()).all()
             den = max(float(np.max(np.abs(ref))), 1e-30)
             assert float(np.max(np.abs(got - ref))) / den <= FP32_TOL, (name, P, r)
+
+
+# ---------------------------------------------------------------------------
+# tcgen05 variant (a5') on the same small-batch shapes: N in {4, 8, 16} load 32/N
+# TMA boxes per nu-half (XM = 3).  TF32 <= 5e-3, 3xTF32 <= 1e-4; small integers
+# are exact in TF32 (tests/test_gpu_parity.py).
+# ---------------------------------------------------------------------------
+TC_TOL = {"tf32": 5e-3, "3xtf32": 1e-4}
+
+
+@pytest.mark.parametrize("variant", ["tf32", "3xtf32"])
+@pytest.mark.parametrize("shape", SMALL_N, ids=[str(s) for s in SMALL_N])
+def test_tc_small_n(wino, shape, variant):
+    N, C, K, H, W = shape
+    cfg = Conv3x3Config("tcsplit", N, C, K, H, W)
+    for kind in ("smallint", "uniform"):
+        x, w = make_inputs(cfg, kind=kind, seed_x=41, seed_w=42)
+        u = wino.filter_transform_tc(w.to(DEV), variant)
+        y = wino.conv2d_tc(x.to(DEV), u)
+        torch.cuda.synchronize()
+        ref = oracle.direct_conv(x, w)
+        if kind == "smallint":
+            assert np.array_equal(y.cpu().double().numpy(), ref)
+        else:
+            assert oracle.max_rel_err(y.cpu().double().numpy(), ref) <= TC_TOL[variant]
+
+
+@pytest.mark.parametrize("P", [2, 4, 8])
+@pytest.mark.parametrize("name", ["conv5_x", "conv4_x", "conv3_x", "conv2_x"])
+def test_tc_rank_shards_sampled(wino, name, P):
+    cfg = CONFIGS[name]
+    x, w = make_inputs(cfg, kind="uniform")
+    for variant in ("tf32", "3xtf32"):
+        u = wino.filter_transform_tc(w.to(DEV), variant)
+        lo, hi = shard_range(cfg.N, P - 1, P)
+        xs = x[..., lo:hi].contiguous()
+        y = wino.conv2d_tc(xs.to(DEV), u)
+        torch.cuda.synchronize()
+        idx = sample_points(cfg.K, cfg.H, cfg.W, hi - lo, 1000, seed=200 + P)
+        ref = oracle.direct_sample(xs, w, idx)
+        ii = idx.numpy()
+        got = y.cpu().double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
+        den = max(float(np.max(np.abs(ref))), 1e-30)
+        assert float(np.max(np.abs(got - ref))) / den <= TC_TOL[variant], (name, P, variant)
