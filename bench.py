@@ -238,7 +238,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default="resnet_3x3", choices=["resnet_3x3", *RESNET_LAYERS, "tiny"])
-    ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw"])
+    ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw",
+                                                            "nonfused_fp32"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
@@ -300,8 +301,11 @@ def main():
         f4 = variant == "f4_fp32"  # NEXT row N1: fused F(4x4,3x3), FTF4 + one fused launch per layer
         tc = variant in ("tf32", "3xtf32")
         nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
+        nonfused = variant == "nonfused_fp32"  # NEXT row N3: ITF -> 16 cuBLAS SGEMMs -> OTF (Sec. 9)
         if f4 or nchw:
             launches = sum(2 for d in per if d["n"] > 0)
+        elif nonfused:
+            launches = sum(3 for d in per if d["n"] > 0)  # FTF, ITF, OTF (the GEMMs are cuBLAS kernels)
         else:
             vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[variant]
             launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K,
@@ -318,6 +322,15 @@ def main():
                 d["u"] = wino.filter_transform_tc(d["w"], variant)
                 if world > 1:
                     dist.broadcast(d["u"].data, src=0)
+            elif nonfused:
+                c = d["cfg"]
+                d["u"] = torch.empty((c.C, 4, 4, c.K), dtype=torch.float32, device=dev)
+                d["ws_nf"] = torch.empty(wino.nonfused_workspace_bytes(max(d["n"], 1), c.C, c.H, c.W, c.K),
+                                         dtype=torch.uint8, device=dev)
+                if rank == 0:
+                    wino.filter_transform(d["w"], out=d["u"])
+                if world > 1:
+                    dist.broadcast(d["u"], src=0)
             elif nchw:
                 # layout change of the synthetic inputs at setup (outside the timed region)
                 d["x_nchw"] = d["x"].permute(3, 0, 1, 2).contiguous()
@@ -352,6 +365,8 @@ def main():
                     wino.conv2d_tc(d["x"], d["u"], out=d["y"])
                 elif nchw:
                     wino.conv2d_nchw(d["x_nchw"], d["u"], out=d["y_nchw"])
+                elif nonfused:
+                    wino.conv2d_nonfused(d["x"], d["u"], d["ws_nf"], out=d["y"])
                 else:
                     wino.conv2d(d["x"], d["u"], out=d["y"])
 
@@ -446,7 +461,7 @@ def main():
     main_m = measure(args.variant, sample_clocks=True)
     others = {}
     if not args.no_variants:
-        for v in ("fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw"):
+        for v in ("fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw", "nonfused_fp32"):
             if v == "f4_fp32" and any(d["n"] % 16 for d in per if d["n"]):
                 continue  # the F(4x4) kernel needs N % 16 == 0 per rank
             if v != args.variant:
@@ -542,7 +557,11 @@ def main():
         vrep[v] = {"value": val, "ms_per_step": m["ms_step"], "pct_fp32_peak_eff": 100 * val / fp32_peak,
                    "layers_eff_tflops": {d["cfg"].name: d["cfg"].eff_flops / (m["conv_ms"][i] * 1e-3) / 1e12
                                          for i, d in enumerate(per) if d["n"]},
-                   "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4, "fp32_nchw": 1e-4}[v]}
+                   "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4, "fp32_nchw": 1e-4,
+                                 "nonfused_fp32": 1e-4}[v]}
+        if v == "nonfused_fp32":
+            vrep[v]["note"] = ("NEXT row N3 ablation: ITF kernel -> V workspace, 16 strided-batched cuBLAS "
+                               "SGEMMs (pedantic FP32) -> OTF kernel; FTF as in the fused step")
         if v == "fp32_nchw":
             ach = sum(_ewmm_flops(d["cfg"], "fp32") for d in per if d["n"]) / (sum(m["conv_ms"]) * 1e-3) / 1e12
             vrep[v]["roofline"] = {"bound": "alu", "achieved": ach, "peak": fp32_peak, "unit": "TFLOP/s",

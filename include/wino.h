@@ -153,6 +153,31 @@ wino_status_t wino_conv2d_f2x3_fwd_nchw(const float* x_nchw_dev, const float* u_
                                         wino_stream_t stream);
 
 /*
+ * NEXT row N3: the NON-fused F(2x2,3x3) forward convolution -- the strategy the
+ * paper's fused kernel is measured against (Sec. 9: "store intermediate
+ * results in global memory ... can utilize optimized batched matrix
+ * multiplication routines. However, it needs significant amount of global
+ * memory as workspace and data loading can be the new bottleneck"; Sec. 7.3
+ * obs. 4-6 L1159-1241; the Sec. 8.1 break-even model L1245-1269).  Three
+ * launches on `stream`:
+ *   1. ITF kernel: x (C,H,W,N) -> V[16][C][NV] in ws_dev (Eq. 6),
+ *   2. 16 batched GEMMs M[xi] = U[xi]^T V[xi] -> M[16][K][NV] in ws_dev (Eq. 7),
+ *      one cuBLAS strided-batched SGEMM in pedantic FP32 (no TF32): the
+ *      "optimized batched matrix multiplication routine" of L1291,
+ *   3. OTF kernel: M -> y (K,H,W,N) (Eq. 8).
+ * NV = N*ceil(H/2)*ceil(W/2).  ws_dev: caller-owned device workspace of at least
+ * wino_nonfused_workspace_bytes(N,C,H,W,K) = 64*NV*(C+K) bytes (+ alignment),
+ * must not overlap x, u or y.  cuBLAS (libcublas.so.12) is loaded on first use;
+ * if it cannot be loaded the call returns WINO_ERR_UNSUPPORTED.  Other
+ * arguments, layouts and errors as wino_conv2d_f2x3_fwd; ws_bytes too small ->
+ * WINO_ERR_INVALID_ARG; V or M of >= 2^31 elements -> WINO_ERR_TOO_LARGE.
+ */
+size_t wino_nonfused_workspace_bytes(int N, int C, int H, int W, int K);
+wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_dev, float* y_dev,
+                                            int N, int C, int H, int W, int K, int pad, int stride,
+                                            void* ws_dev, size_t ws_bytes, wino_stream_t stream);
+
+/*
  * Tensor-core variant (a5' of SURVEY 8(a)): the Winograd-domain GEMM (Eq. 7)
  * on the 5th-generation tensor cores (tcgen05.mma kind::tf32, accumulators in
  * TMEM).  The paper has no tensor-core path ("the data layout needs a

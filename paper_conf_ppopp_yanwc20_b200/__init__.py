@@ -24,7 +24,7 @@ __all__ = [
     "TcFilter", "filter_workspace_bytes_tc", "filter_transform_tc", "conv2d_tc",
     "host_multi_workspace_bytes", "conv2d_host_multi",
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
-    "filter_transform_kcrs", "conv2d_nchw",
+    "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -106,6 +106,11 @@ def lib() -> ctypes.CDLL:
     if hasattr(L, "wino_filter_transform_kcrs") or not os.environ.get("WINO_LIB_PATH"):
         L.wino_filter_transform_kcrs.argtypes = [vp, vp, i, i, vp]
         L.wino_conv2d_f2x3_fwd_nchw.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_nonfused") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_nonfused_workspace_bytes.restype = st
+        L.wino_nonfused_workspace_bytes.argtypes = [i, i, i, i, i]
+        L.wino_conv2d_f2x3_fwd_nonfused.restype = i
+        L.wino_conv2d_f2x3_fwd_nonfused.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp, st, vp]
     L.wino_conv2d_f2x3_fwd_tc.restype = i
     L.wino_conv2d_f2x3_fwd_tc.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
     L.wino_filter_workspace_bytes_tc.restype = st
@@ -319,6 +324,37 @@ def conv2d_nchw(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = Non
         _check(lib().wino_conv2d_f2x3_fwd_nchw(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()),
                                                ctypes.c_void_p(out.data_ptr()), N, C, H, W, K, 1, 1,
                                                _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_nchw")
+    return out
+
+
+def nonfused_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
+    """Device workspace of the non-fused path: V[16][C][NV] + M[16][K][NV] floats."""
+    return int(lib().wino_nonfused_workspace_bytes(N, C, H, W, K))
+
+
+def conv2d_nonfused(x: torch.Tensor, u: torch.Tensor, ws: torch.Tensor, out: torch.Tensor | None = None,
+                    stream=None) -> torch.Tensor:
+    """NEXT row N3 (Sec. 9): NON-fused Winograd -- ITF kernel to a global workspace,
+    16 batched GEMMs (cuBLAS SGEMM), OTF kernel.  x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N);
+    ws: CUDA byte buffer of >= nonfused_workspace_bytes(N,C,H,W,K)."""
+    _need_cuda_f32(x, "x", 4)
+    _need_cuda_f32(u, "u", 4)
+    C, H, W, N = x.shape
+    if u.shape[0] != C or tuple(u.shape[1:3]) != (4, 4):
+        raise ValueError(f"u must be (C,4,4,K) with C={C}, got {tuple(u.shape)}")
+    K = u.shape[3]
+    if not ws.is_cuda or not ws.is_contiguous():
+        raise ValueError("ws must be a contiguous CUDA tensor")
+    if out is None:
+        out = torch.empty((K, H, W, N), dtype=torch.float32, device=x.device)
+    _need_cuda_f32(out, "out", 4)
+    if tuple(out.shape) != (K, H, W, N):
+        raise ValueError("out must be (K,H,W,N)")
+    with torch.cuda.device(x.device):
+        _check(lib().wino_conv2d_f2x3_fwd_nonfused(
+            ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+            N, C, H, W, K, 1, 1, ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size(),
+            _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_nonfused")
     return out
 
 

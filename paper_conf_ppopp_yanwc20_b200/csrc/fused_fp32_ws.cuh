@@ -334,6 +334,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
         }
         const bool okr = i0 + 1 < p.H, okc = j0 + 1 < p.W;  // odd H/W: drop extra outputs (L1155)
         const size_t base = ((size_t)i0 * p.W + j0) * p.N + n;
+#ifdef WINO_WS_TRACE
+        if (!SPLIT && tid == 0) WS_TR(1, (tile - WS_CID) / WS_NCL);
+#endif
         if constexpr (!SPLIT) {
             // 4 rounds of 16 filters (the paper's 4-round OTF, L499).  NOTE: ptxas' register
             // assignment of the accumulators (and so the FFMA bank conflicts of the main
@@ -342,7 +345,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             for (int rd = 0; rd < 4; ++rd) {
                 // round rd stores accumulator rows i in {2(rd&1), 2(rd&1)+1} of half rd>>1:
                 // filters kl = fo + (i&3) + 32*(i>>2); in the buffer row = (fo>>2)*2 + (i&1)
+#ifndef WS_EXP_NOBAR
                 named_bar_sync(1, COMPUTE_THREADS);  // previous round's readers are done
+#endif
 #pragma unroll
                 for (int q = 0; q < 2; ++q)
 #pragma unroll
@@ -355,7 +360,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                         *reinterpret_cast<float4*>(row + 16) =
                             make_float4(acc[q][i][5], acc[q][i][4], acc[q][i][7], acc[q][i][6]);
                     }
+#ifndef WS_EXP_NOBAR
                 named_bar_sync(1, COMPUTE_THREADS);
+#endif
                 if (nu < p.NV) {
 #pragma unroll
                     for (int h = 0; h < 2; ++h) {
@@ -368,14 +375,21 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                             for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + r) * ER_LD + (lane ^ 1)];
                             otf_2x2(m, o);
                             float* yk = p.y + (size_t)k * HWN + base;
+#ifdef WS_EXP_NOSTG
+                            if (o[0] == 1234.5f && o[1] == o[2] && o[3] == 7.f) yk[0] = o[0];
+#else
                             yk[0] = o[0];
                             if (okc) yk[p.N] = o[1];
                             if (okr) yk[dW] = o[2];
                             if (okr && okc) yk[dW + p.N] = o[3];
+#endif
                         }
                     }
                 }
             }
+#ifdef WINO_WS_TRACE
+            if (tid == 0) WS_TR(3, (tile - WS_CID) / WS_NCL);
+#endif
         } else {
             // 8 rounds of 8 filters: round rd stores accumulator row i = rd (filters
             // kl = fo + (rd&3) + 32*(rd>>2)) into buffer row fo>>2; the OTF of buffer row

@@ -18,6 +18,9 @@
 #include "fused_fp32_ws.cuh"
 #include "fused_tc.cuh"
 #include "fused_f4_fp32.cuh"
+#include "nonfused.cuh"
+
+#include <dlfcn.h>
 
 namespace {
 
@@ -878,6 +881,109 @@ wino_status_t wino_conv2d_f4x3_fwd(const float* x_dev, const float* u4_dev, floa
     const int grid = prm.num_tiles < sms ? prm.num_tiles : sms;
     kern<<<grid, NT, Smem::bytes, reinterpret_cast<cudaStream_t>(stream)>>>(prm);
     cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------------------
+// NEXT row N3: non-fused Winograd (ITF kernel -> 16 library GEMMs -> OTF kernel)
+// ---------------------------------------------------------------------------
+namespace {
+// cuBLAS is loaded on first use (dlopen), so libwino.so itself has no link-time
+// dependency on it; without cuBLAS the non-fused entry point returns UNSUPPORTED.
+typedef int (*cublasCreate_t)(void**);
+typedef int (*cublasSetStream_t)(void*, cudaStream_t);
+typedef int (*cublasSetMathMode_t)(void*, int);
+typedef int (*cublasSgemmStridedBatched_t)(void*, int, int, int, int, int, const float*, const float*, int,
+                                           long long, const float*, int, long long, const float*, float*, int,
+                                           long long, int);
+struct Cublas {
+    cublasCreate_t create = nullptr;
+    cublasSetStream_t set_stream = nullptr;
+    cublasSetMathMode_t set_math = nullptr;
+    cublasSgemmStridedBatched_t sgemm_sb = nullptr;
+    void* handle[kMaxDevices] = {};
+    bool ok = false;
+};
+std::mutex g_cublas_mu;
+Cublas g_cublas;
+bool g_cublas_tried = false;
+
+bool cublas_load() {
+    if (g_cublas_tried) return g_cublas.ok;
+    g_cublas_tried = true;
+    void* h = dlopen("libcublas.so.12", RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
+    if (!h) h = dlopen("libcublas.so.12", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libcublas.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return false;
+    g_cublas.create = reinterpret_cast<cublasCreate_t>(dlsym(h, "cublasCreate_v2"));
+    g_cublas.set_stream = reinterpret_cast<cublasSetStream_t>(dlsym(h, "cublasSetStream_v2"));
+    g_cublas.set_math = reinterpret_cast<cublasSetMathMode_t>(dlsym(h, "cublasSetMathMode"));
+    g_cublas.sgemm_sb = reinterpret_cast<cublasSgemmStridedBatched_t>(dlsym(h, "cublasSgemmStridedBatched"));
+    g_cublas.ok = g_cublas.create && g_cublas.set_stream && g_cublas.set_math && g_cublas.sgemm_sb;
+    return g_cublas.ok;
+}
+constexpr int kCublasOpN = 0, kCublasOpT = 1;
+constexpr int kCublasPedanticMath = 2;  // CUBLAS_PEDANTIC_MATH: plain FP32, no TF32 tensor-op shortcuts
+}  // namespace
+
+extern "C" {
+
+size_t wino_nonfused_workspace_bytes(int N, int C, int H, int W, int K) {
+    if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
+    const size_t nv = size_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
+    return round_up256(size_t(16) * C * nv * 4) + round_up256(size_t(16) * K * nv * 4);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_dev, float* y_dev, int N, int C,
+                                            int H, int W, int K, int pad, int stride, void* ws_dev, size_t ws_bytes,
+                                            wino_stream_t stream) {
+    if (!x_dev || !u_dev || !y_dev || !ws_dev) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (!aligned16(x_dev) || !aligned16(u_dev) || !aligned16(y_dev) || !aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
+    const size_t need = wino_nonfused_workspace_bytes(N, C, H, W, K);
+    if (ws_bytes < need) return WINO_ERR_INVALID_ARG;
+    const long long nv = (long long)N * ((H + 1) / 2) * ((W + 1) / 2);
+    if ((long long)16 * C * nv > kMaxElems || (long long)16 * K * nv > kMaxElems) return WINO_ERR_TOO_LARGE;
+    const size_t hwn = size_t(H) * W * N, yb = size_t(K) * hwn * 4;
+    if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) || overlaps(y_dev, yb, u_dev, size_t(16) * C * K * 4) ||
+        overlaps(ws_dev, need, x_dev, size_t(C) * hwn * 4) || overlaps(ws_dev, need, u_dev, size_t(16) * C * K * 4) ||
+        overlaps(ws_dev, need, y_dev, yb))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    float* v = static_cast<float*>(ws_dev);
+    float* m = reinterpret_cast<float*>(static_cast<char*>(ws_dev) + round_up256(size_t(16) * C * nv * 4));
+    const int TW = (W + 1) / 2;
+    // 1. ITF -> V [16][C][NV]
+    wino::nf::itf_nf_kernel<<<unsigned((C * nv + wino::nf::THREADS - 1) / wino::nf::THREADS), wino::nf::THREADS, 0,
+                              st>>>(x_dev, v, N, C, H, W, TW, nv);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e);
+    // 2. M[xi] = U[xi]^T V[xi], xi = 0..15, one strided-batched SGEMM.  Row-major M[k][nu]
+    //    is column-major M^T (NV x K): M^T = V^T (NV x C, ld NV) * U (C x K from u[c][xi][k],
+    //    column-major view K x C with ld 16K -> op T).
+    {
+        std::lock_guard<std::mutex> lk(g_cublas_mu);
+        if (!cublas_load()) return WINO_ERR_UNSUPPORTED;
+        if (!g_cublas.handle[dev]) {
+            if (g_cublas.create(&g_cublas.handle[dev]) != 0) return WINO_ERR_CUDA;
+            g_cublas.set_math(g_cublas.handle[dev], kCublasPedanticMath);
+        }
+        void* hd = g_cublas.handle[dev];
+        if (g_cublas.set_stream(hd, st) != 0) return WINO_ERR_CUDA;
+        const float one = 1.f, zero = 0.f;
+        if (g_cublas.sgemm_sb(hd, kCublasOpN, kCublasOpT, (int)nv, K, C, &one, v, (int)nv, (long long)C * nv, u_dev,
+                              16 * K, (long long)K, &zero, m, (int)nv, (long long)K * nv, 16) != 0)
+            return WINO_ERR_CUDA;
+    }
+    // 3. OTF -> y
+    wino::nf::otf_nf_kernel<<<unsigned((K * nv + wino::nf::THREADS - 1) / wino::nf::THREADS), wino::nf::THREADS, 0,
+                              st>>>(m, y_dev, N, K, H, W, TW, nv);
+    e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 

@@ -115,6 +115,16 @@ def test_fwd_argument_validation_host_side():
                                         2, 3, 4, 4, 5, 0, 1, 2, None) == 2  # pad != 1
 
 
+def test_nonfused_workspace_bytes():
+    """V[16][C][NV] + M[16][K][NV] floats, each rounded up to 256 B (NEXT row N3)."""
+    for name in ("conv5_x", "conv4_x", "conv3_x", "conv2_x", "tiny"):
+        c = CONFIGS[name]
+        nv = c.N * c.tiles
+        rnd = lambda b: -(-b // 256) * 256  # noqa: E731
+        assert wino.nonfused_workspace_bytes(c.N, c.C, c.H, c.W, c.K) == rnd(64 * c.C * nv) + rnd(64 * c.K * nv)
+    assert wino.nonfused_workspace_bytes(0, 3, 5, 5, 4) == 0
+
+
 @pytest.mark.parametrize("P", [2, 4, 8])
 def test_plan_splits_small_shards(P):
     """Per-rank batch shards with fewer (k, nu) tiles than SMs get split-C,

@@ -1,0 +1,90 @@
+"""GPU parity of NEXT row N3 -- the NON-fused Winograd path (Sec. 9; Sec. 7.3
+obs. 4-6): ITF kernel -> V workspace, 16 batched GEMMs (cuBLAS SGEMM, pedantic
+FP32), OTF kernel, through wino_conv2d_f2x3_fwd_nonfused, against the fp64 oracle.
+
+Bars as tests/test_gpu_parity.py: bit-exact vs Eq. 4 on small integers (every
+intermediate is an exact dyadic rational below 2^24), <= 1e-4 of max|y| on random
+inputs.  Also checked against the oracle's naive Winograd (Eq. 5-8), whose steps the
+non-fused path mirrors one launch each.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth_inputs import CONFIGS, Conv3x3Config, make_inputs, sample_points
+
+pytestmark = pytest.mark.gpu
+
+FP32_TOL = 1e-4
+DEV = "cuda:0"
+
+
+@pytest.fixture(scope="module")
+def wino():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ppopp_yanwc20_b200 as w
+    w.lib()
+    return w
+
+
+def _run(wino, x, w):
+    C, H, W, N = x.shape
+    K = w.shape[3]
+    u = wino.filter_transform(w.to(DEV))
+    ws = torch.empty(wino.nonfused_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+    y = wino.conv2d_nonfused(x.to(DEV), u, ws)
+    torch.cuda.synchronize()
+    return y.cpu()
+
+
+SHAPES = [
+    (1, 1, 1, 1, 1), (1, 8, 8, 8, 8), (3, 7, 5, 5, 5), (2, 9, 65, 7, 7), (33, 8, 64, 3, 3),
+    (4, 20, 70, 13, 9), (5, 17, 130, 6, 10), (32, 24, 96, 4, 6), (7, 40, 72, 11, 12),
+]
+
+
+@pytest.mark.parametrize("shape", SHAPES, ids=[str(s) for s in SHAPES])
+def test_nonfused_small_int_bit_exact(wino, shape):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nf", N, C, K, H, W), kind="smallint")
+    y = _run(wino, x, w)
+    assert np.array_equal(y.double().numpy(), oracle.direct_conv(x, w))
+
+
+@pytest.mark.parametrize("shape", SHAPES, ids=[str(s) for s in SHAPES])
+def test_nonfused_random(wino, shape):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nf", N, C, K, H, W), kind="uniform", seed_x=51, seed_w=52)
+    y = _run(wino, x, w).double().numpy()
+    assert oracle.max_rel_err(y, oracle.direct_conv(x, w)) <= FP32_TOL
+    assert oracle.max_rel_err(y, oracle.winograd_conv(x, w)) <= FP32_TOL
+
+
+@pytest.mark.parametrize("name", ["conv5_x", "conv4_x", "conv3_x", "conv2_x"])
+def test_nonfused_full_configs_sampled(wino, name):
+    cfg = CONFIGS[name]
+    for kind in ("smallint", "uniform"):
+        x, w = make_inputs(cfg, kind=kind)
+        y = _run(wino, x, w)
+        idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 2000)
+        ref = oracle.direct_sample(x, w, idx)
+        ii = idx.numpy()
+        got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
+        if kind == "smallint":
+            assert np.array_equal(got, ref)
+        else:
+            den = max(float(np.max(np.abs(ref))), 1e-30)
+            assert float(np.max(np.abs(got - ref))) / den <= FP32_TOL
+
+
+def test_nonfused_workspace_checks(wino):
+    cfg = Conv3x3Config("nf", 4, 8, 8, 6, 6)
+    x, w = make_inputs(cfg)
+    u = wino.filter_transform(w.to(DEV))
+    need = wino.nonfused_workspace_bytes(4, 8, 6, 6, 8)
+    small = torch.empty(need - 256, dtype=torch.uint8, device=DEV)
+    with pytest.raises(wino.WinoError) as e:
+        wino.conv2d_nonfused(x.to(DEV), u, small)
+    assert e.value.status == 1
