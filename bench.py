@@ -55,6 +55,14 @@ def _peaks():
     return fp32_tflops, hbm, src
 
 
+def _bf16_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            return float(json.load(f).get("bf16_tflops", 1590.0))
+    return 1590.0
+
+
 def _tf32_peak():
     path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     bf16 = 1590.0
@@ -239,7 +247,7 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default="resnet_3x3", choices=["resnet_3x3", *RESNET_LAYERS, "tiny"])
     ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw",
-                                                            "nonfused_fp32"])
+                                                            "nonfused_fp32", "fp16", "bf16"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
@@ -302,7 +310,8 @@ def main():
         tc = variant in ("tf32", "3xtf32")
         nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
         nonfused = variant == "nonfused_fp32"  # NEXT row N3: ITF -> 16 cuBLAS SGEMMs -> OTF (Sec. 9)
-        if f4 or nchw:
+        half = variant in ("fp16", "bf16")  # NEXT row N4: 16-bit x, w, y on tcgen05 kind::f16 (Sec. 8.3)
+        if f4 or nchw or half:
             launches = sum(2 for d in per if d["n"] > 0)
         elif nonfused:
             launches = sum(3 for d in per if d["n"] > 0)  # FTF, ITF, OTF (the GEMMs are cuBLAS kernels)
@@ -320,6 +329,14 @@ def main():
                     dist.broadcast(d["u"], src=0)
             elif tc:
                 d["u"] = wino.filter_transform_tc(d["w"], variant)
+                if world > 1:
+                    dist.broadcast(d["u"].data, src=0)
+            elif half:
+                # the synthetic fp32 inputs stored in the 16-bit type at setup (outside the timed region)
+                dt16 = torch.float16 if variant == "fp16" else torch.bfloat16
+                d["x16"], d["w16"] = d["x"].to(dt16), d["w"].to(dt16)
+                d["y16"] = torch.empty(d["y"].shape, dtype=dt16, device=dev)
+                d["u"] = wino.filter_transform_half(d["w16"])
                 if world > 1:
                     dist.broadcast(d["u"].data, src=0)
             elif nonfused:
@@ -356,6 +373,8 @@ def main():
                     wino.filter_transform_tc(d["w"], variant, out=d["u"], stream=ftf_stream)
                 elif nchw:
                     wino.filter_transform_kcrs(d["w_kcrs"], out=d["u"], stream=ftf_stream)
+                elif half:
+                    wino.filter_transform_half(d["w16"], out=d["u"], stream=ftf_stream)
                 else:
                     wino.filter_transform(d["w"], out=d["u"], stream=ftf_stream)
             if conv:
@@ -365,6 +384,8 @@ def main():
                     wino.conv2d_tc(d["x"], d["u"], out=d["y"])
                 elif nchw:
                     wino.conv2d_nchw(d["x_nchw"], d["u"], out=d["y_nchw"])
+                elif half:
+                    wino.conv2d_half(d["x16"], d["u"], out=d["y16"])
                 elif nonfused:
                     wino.conv2d_nonfused(d["x"], d["u"], d["ws_nf"], out=d["y"])
                 else:
@@ -461,7 +482,7 @@ def main():
     main_m = measure(args.variant, sample_clocks=True)
     others = {}
     if not args.no_variants:
-        for v in ("fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw", "nonfused_fp32"):
+        for v in ("fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw", "nonfused_fp32", "fp16", "bf16"):
             if v == "f4_fp32" and any(d["n"] % 16 for d in per if d["n"]):
                 continue  # the F(4x4) kernel needs N % 16 == 0 per rank
             if v != args.variant:
@@ -558,7 +579,7 @@ def main():
                    "layers_eff_tflops": {d["cfg"].name: d["cfg"].eff_flops / (m["conv_ms"][i] * 1e-3) / 1e12
                                          for i, d in enumerate(per) if d["n"]},
                    "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4, "fp32_nchw": 1e-4,
-                                 "nonfused_fp32": 1e-4}[v]}
+                                 "nonfused_fp32": 1e-4, "fp16": 5e-3, "bf16": 3e-2}[v]}
         if v == "nonfused_fp32":
             vrep[v]["note"] = ("NEXT row N3 ablation: ITF kernel -> V workspace, 16 strided-batched cuBLAS "
                                "SGEMMs (pedantic FP32) -> OTF kernel; FTF as in the fused step")
@@ -579,6 +600,15 @@ def main():
                                    "unit": "TFLOP/s", "frac": ach * mult / tf32_peak,
                                    "achieved_def": f"{mult} x EWMM flops (tcgen05 kind::tf32 work) / conv time",
                                    "peak_def": "MEASURED_PEAKS bf16_tflops x 0.5 (nominal tf32:bf16 dense ratio)"}
+        if v in ("fp16", "bf16"):
+            ach = ewmm_flops / (sum(m["conv_ms"]) * 1e-3) / 1e12
+            vrep[v]["note"] = ("NEXT row N4: x, w, y stored in " + v + "; FP32 transforms and accumulation, "
+                               "tcgen05 kind::f16 Winograd-domain GEMM")
+            vrep[v]["roofline"] = {"bound": "tensor", "achieved": ach, "peak": _bf16_peak(), "unit": "TFLOP/s",
+                                   "frac": ach / _bf16_peak(),
+                                   "achieved_def": "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) (kind::f16 work) / "
+                                                   "conv time",
+                                   "peak_def": "MEASURED_PEAKS bf16_tflops (fp16 and bf16 share the dense rate)"}
     if vrep:
         res["variants"] = vrep
     if world == 1 and not args.no_cpu_baseline:

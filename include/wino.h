@@ -200,6 +200,34 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
                                       wino_tc_mode_t mode, wino_stream_t stream);
 
 /*
+ * NEXT row N4: 16-bit version on the tensor cores.  The paper:
+ * "The implementation can be ported to the fp16 version by increasing bn to 64.
+ * To further increase the throughput with newly introduced tensor core, the data
+ * layout needs a redesign" (Sec. 8.3).  Here x, w and y are stored in the
+ * 16-bit type `type` (IEEE fp16 or bfloat16, raw 2-byte elements, same layouts as
+ * the FP32 calls: x (C,H,W,N), w (C,3,3,K), y (K,H,W,N)); the transforms and the
+ * accumulation over C run in FP32 (tcgen05.mma kind::f16, FP32 accumulators in
+ * TMEM); U, V and y are rounded to `type` with round-to-nearest-even (DESIGN.md
+ * reading R18).  Accuracy: max|y - y_ref| / max|y_ref| <= 5e-3 (fp16) and 3e-2
+ * (bf16) against Eq. 4 of the 16-bit inputs; bit-exact (y == round(y_ref)) on
+ * small-integer inputs.
+ *   u_h : wino_filter_workspace_bytes_half(C,K) bytes, opaque layout
+ *         [ceil(C/16)][ceil(K/128)][16][128 x 16 K-major tile], zero padded.
+ * Any N, C, K, H, W >= 1; N % 32 == 0 or N in {8, 16} take TMA loads.  Errors as
+ * the FP32 calls, plus WINO_ERR_INVALID_ARG for an unknown `type`.
+ */
+typedef enum {
+    WINO_HALF_FP16 = 0, /* IEEE 754 binary16 */
+    WINO_HALF_BF16 = 1  /* bfloat16          */
+} wino_half_t;
+size_t wino_filter_workspace_bytes_half(int C, int K);
+wino_status_t wino_filter_transform_half(const void* w_dev, void* u_h_dev, int C, int K, wino_half_t type,
+                                         wino_stream_t stream);
+wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, void* y_dev,
+                                        int N, int C, int H, int W, int K, int pad, int stride,
+                                        wino_half_t type, wino_stream_t stream);
+
+/*
  * End-to-end call on HOST buffers: copies w_host and x_host to the device,
  * runs the filter transform and the fused FP32 convolution, and copies y back
  * to y_host, all enqueued on `stream` (so the call returns before the copies
@@ -258,7 +286,8 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
  * used by tests and by bench.py to count launches and report tiling.
  */
 typedef struct {
-    int variant;        /* 0 = FP32 FFMA fused kernel, 1 = tcgen05 TF32 / 3xTF32   */
+    int variant;        /* 0 = FP32 FFMA fused kernel, 1 / 2 = tcgen05 TF32 / 3xTF32, */
+                        /* 3 = tcgen05 kind::f16 (FP16 / BF16, NEXT row N4)           */
     int bk, bn, bc;     /* filters, tiles and channels per CTA step (Sec. 3.3)      */
     int load_x, load_u; /* how x / u reach shared memory: 0 = cp.async 4 B,         */
                         /* 1 = cp.async 16 B, 2 = TMA tiled box (cp.async.bulk.tensor) */

@@ -25,6 +25,8 @@ __all__ = [
     "host_multi_workspace_bytes", "conv2d_host_multi",
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
+    "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
+    "conv2d_half",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -33,6 +35,9 @@ _lib = None
 
 TC_TF32 = 0
 TC_3XTF32 = 1
+HALF_FP16 = 0
+HALF_BF16 = 1
+_HALF_DTYPES = {torch.float16: HALF_FP16, torch.bfloat16: HALF_BF16}
 _STATUS = {0: "WINO_OK", 1: "WINO_ERR_INVALID_ARG", 2: "WINO_ERR_UNSUPPORTED",
            3: "WINO_ERR_MISALIGNED", 4: "WINO_ERR_TOO_LARGE", 5: "WINO_ERR_CUDA"}
 
@@ -131,6 +136,13 @@ def lib() -> ctypes.CDLL:
     L.wino_filter_transform_f4.argtypes = [vp, vp, i, i, vp]
     L.wino_conv2d_f4x3_fwd.restype = i
     L.wino_conv2d_f4x3_fwd.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_half") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_filter_workspace_bytes_half.restype = st
+        L.wino_filter_workspace_bytes_half.argtypes = [i, i]
+        L.wino_filter_transform_half.restype = i
+        L.wino_filter_transform_half.argtypes = [vp, vp, i, i, i, vp]
+        L.wino_conv2d_f2x3_fwd_half.restype = i
+        L.wino_conv2d_f2x3_fwd_half.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
     L.wino_plan.restype = i
     L.wino_plan.argtypes = [i, i, i, i, i, i, ctypes.POINTER(_Plan)]
     _lib = L
@@ -251,6 +263,71 @@ def conv2d_tc(x: torch.Tensor, u_tc: TcFilter, out: torch.Tensor | None = None, 
         _check(lib().wino_conv2d_f2x3_fwd_tc(
             ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_tc.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
             N, C, H, W, K, 1, 1, u_tc.mode, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc")
+    return out
+
+
+def _need_cuda_half(t: torch.Tensor, name: str, ndim: int):
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{name} must be a torch.Tensor")
+    if t.dtype not in _HALF_DTYPES:
+        raise TypeError(f"{name} must be float16 or bfloat16, got {t.dtype}")
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor (no CPU fallback)")
+    if t.dim() != ndim:
+        raise ValueError(f"{name} must have {ndim} dims, got shape {tuple(t.shape)}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+
+
+@dataclass
+class HalfFilter:
+    """Transformed filter in the kind::f16 operand layout (wino_filter_transform_half)."""
+    data: torch.Tensor  # flat 16-bit CUDA tensor of the filter's dtype
+    C: int
+    K: int
+    dtype: torch.dtype
+
+
+def filter_workspace_bytes_half(C: int, K: int) -> int:
+    return int(lib().wino_filter_workspace_bytes_half(C, K))
+
+
+def filter_transform_half(w: torch.Tensor, out: HalfFilter | None = None, stream=None) -> HalfFilter:
+    """NEXT row N4: FTF (Eq. 5) of a float16 / bfloat16 w (C,3,3,K) in FP32, rounded to w's type, in the
+    tcgen05 kind::f16 operand layout (Sec. 8.3, L1283)."""
+    _need_cuda_half(w, "w", 4)
+    C, r, s_, K = w.shape
+    if (r, s_) != (3, 3):
+        raise ValueError(f"w must be (C,3,3,K), got {tuple(w.shape)}")
+    nbytes = filter_workspace_bytes_half(C, K)
+    if out is None:
+        out = HalfFilter(torch.empty(nbytes // 2, dtype=w.dtype, device=w.device), C, K, w.dtype)
+    if (out.C, out.K, out.dtype) != (C, K, w.dtype) or out.data.numel() * 2 < nbytes:
+        raise ValueError("out HalfFilter does not match w")
+    with torch.cuda.device(w.device):
+        _check(lib().wino_filter_transform_half(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data.data_ptr()),
+                                                C, K, _HALF_DTYPES[w.dtype], _stream_ptr(stream)),
+               "wino_filter_transform_half")
+    return out
+
+
+def conv2d_half(x: torch.Tensor, u_h: HalfFilter, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """NEXT row N4: fused Winograd conv on float16 / bfloat16 x (C,H,W,N) -> y (K,H,W,N) of the same type,
+    Winograd-domain GEMM on tcgen05 kind::f16 with FP32 accumulation."""
+    _need_cuda_half(x, "x", 4)
+    C, H, W, N = x.shape
+    if u_h.C != C or u_h.dtype != x.dtype:
+        raise ValueError(f"u_h was built for C={u_h.C} {u_h.dtype}, x has C={C} {x.dtype}")
+    K = u_h.K
+    if out is None:
+        out = torch.empty((K, H, W, N), dtype=x.dtype, device=x.device)
+    _need_cuda_half(out, "out", 4)
+    if tuple(out.shape) != (K, H, W, N) or out.dtype != x.dtype:
+        raise ValueError("out must be (K,H,W,N) of x's dtype")
+    with torch.cuda.device(x.device):
+        _check(lib().wino_conv2d_f2x3_fwd_half(
+            ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_h.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+            N, C, H, W, K, 1, 1, _HALF_DTYPES[x.dtype], _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_half")
     return out
 
 

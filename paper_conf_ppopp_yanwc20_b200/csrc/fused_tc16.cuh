@@ -1,0 +1,463 @@
+// fused_tc16.cuh -- NEXT row N4: fused Winograd F(2x2,3x3) with FP16 or BF16
+// operands on tcgen05 tensor cores (kind::f16, FP32 accumulators in TMEM).
+//
+// Paper: "The implementation can be ported to the fp16 version by increasing bn
+// to 64.  To further increase the throughput with newly introduced tensor core,
+// the data layout needs a redesign" (Sec. 8.3).  Same method (Eq. 5-8,
+// L191-207); x, w, y are stored in the 16-bit type, the transforms and the
+// accumulation run in FP32, the Winograd-domain operands U, V and the output y
+// are rounded to the 16-bit type (round-to-nearest-even; reading R18).
+//
+// Tile: 128 filters (UMMA M) x 32 nu (UMMA N) x all 16 xi, channel blocks of 16
+// (one UMMA K step per xi).  The 16-bit operands carry twice the channels of the
+// TF32 kernel (fused_tc.cuh) in the same shared-memory bytes, so the per-block
+// operand traffic that bounds that kernel (Sec. 7.3 of DESIGN.md) buys twice the
+// Winograd-domain work here.
+// Warp roles (persistent, one CTA per SM, 512 threads):
+//   * warps 0-3   epilogue: tcgen05.ld of the 16 accumulators, OTF (Eq. 8) in
+//                 FP32 registers, TMEM released, 16-bit stores of y;
+//   * warps 4-7 / 8-11  two ITF groups taking alternate channel blocks: each
+//                 thread transforms 2 channels x 2 nu (V = B^T d B, Eq. 6, FP32)
+//                 and stores c-pairs of V as 32-bit words of the K-major B operand;
+//   * warp 12     bulk copy of the pre-arranged 16-bit U (64 KB per block);
+//   * warp 13     one thread issues tcgen05.mma.kind::f16 per xi;
+//   * warp 14     TMA of raw x (n:32, w:4, h:4, c:16), zero fill = padding (Sec. 3.5).
+#pragma once
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+
+#include <cstdint>
+
+#include "wino_ptx.cuh"
+#include "wino_transforms.cuh"
+
+namespace wino {
+namespace tc16 {
+
+constexpr int BN = 32;    // nu per tile (UMMA N)
+constexpr int MM = 128;   // filters per tile (UMMA M)
+constexpr int BC = 16;    // channels per block (UMMA K of kind::f16)
+constexpr int EPI_WARPS = 4, ITF_WARP0 = 4, ITF_WARPS = 8, ITF_GROUP = 4;
+constexpr int PROD_WARP = 12, MMA_WARP = 13, XPROD_WARP = 14;
+constexpr int NT = 512;
+constexpr int REG_EPI = 216, REG_ITF = 112, REG_PROD = 56;  // 128*216 + 256*112 + 128*56 = 63488
+constexpr int A_TILE = MM * BC * 2;       // one xi of U: 4 KB, [m/8][c/8][m%8][c%8]
+constexpr int UNIT = 16 * A_TILE;         // one channel block of U: 64 KB
+constexpr int V_SBO = 272;                // 8-row group stride of the V operand (256 + 16: fewer bank conflicts)
+constexpr int B_TILE = (BN / 8) * V_SBO;  // one xi of V: 1088 B, [nu/8 (stride 272)][c/8 (128)][nu%8][c%8]
+constexpr int XS_BYTES = BC * 16 * BN * 2;  // raw x of one block: 16 KB, [c][pos][nu]
+// x slot = gcb % 4: each ITF group owns two slots (0, 2 / 1, 3) and consumes them in order, so
+// an mbarrier phase parity can never alias a fill that has not landed (the groups drift apart).
+constexpr int U_SLOTS = 2, X_SLOTS = 4, V_SLOTS = 2;
+constexpr int V_SLOT = 16 * B_TILE;
+constexpr int OFF_U = 0;
+constexpr int OFF_X = OFF_U + U_SLOTS * UNIT;
+constexpr int OFF_V = OFF_X + X_SLOTS * XS_BYTES;
+constexpr int OFF_BAR = OFF_V + V_SLOTS * V_SLOT;
+constexpr int NBAR = 2 * U_SLOTS + 2 * X_SLOTS + 2 * V_SLOTS + 2;
+constexpr int OFF_TMEM = OFF_BAR + NBAR * 8;
+constexpr int BYTES = OFF_TMEM + 16;
+static_assert(BYTES <= 232448, "shared memory budget");
+static_assert(V_SLOTS == 2 && X_SLOTS % 2 == 0, "two ITF groups take alternate channel blocks");
+
+// u_h layout (written by tc16_filter_kernel, read with bulk copies):
+//   [cb = ceil(C/16)][kb = ceil(K/128)][xi 16][m/8 16][c/8 2][m%8 8][c%8 8]  16-bit
+// i.e. per (cb, kb, xi) one K-major SWIZZLE_NONE UMMA A tile (LBO 128 B, SBO 256 B).
+__host__ __device__ inline size_t u_h_elems(int C, int K) {
+    return size_t((C + BC - 1) / BC) * ((K + MM - 1) / MM) * 16 * (MM * BC);
+}
+
+// 16-bit type helpers: DT 0 = IEEE fp16, 1 = bf16.
+template <int DT>
+__device__ __forceinline__ float2 unpack2(uint32_t w) {
+    if constexpr (DT == 0) {
+        __half2 h = *reinterpret_cast<__half2*>(&w);
+        return __half22float2(h);
+    } else {
+        return make_float2(__uint_as_float(w << 16), __uint_as_float(w & 0xffff0000u));
+    }
+}
+template <int DT>
+__device__ __forceinline__ uint32_t pack2(float lo, float hi) {  // round-to-nearest-even
+    if constexpr (DT == 0) {
+        __half2 h = __floats2half2_rn(lo, hi);
+        return *reinterpret_cast<uint32_t*>(&h);
+    } else {
+        __nv_bfloat162 h = __floats2bfloat162_rn(lo, hi);
+        return *reinterpret_cast<uint32_t*>(&h);
+    }
+}
+template <int DT>
+__device__ __forceinline__ float to_f(uint16_t v) {
+    if constexpr (DT == 0) return __half2float(__ushort_as_half(v));
+    else return __uint_as_float(uint32_t(v) << 16);
+}
+template <int DT>
+__device__ __forceinline__ uint16_t from_f(float v) {
+    if constexpr (DT == 0) return __half_as_ushort(__float2half_rn(v));
+    else return __bfloat16_as_ushort(__float2bfloat16_rn(v));
+}
+
+// D f32, A/B fp16 (0) or bf16 (1), both K-major.
+__host__ __device__ constexpr uint32_t umma_idesc_f16(int dt, int M, int N) {
+    return (1u << 4) | (uint32_t(dt) << 7) | (uint32_t(dt) << 10) | (uint32_t(N >> 3) << 17) |
+           (uint32_t(M >> 4) << 24);
+}
+__device__ __forceinline__ void umma_f16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d_tmem),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc)
+        : "memory");
+}
+
+// FTF (Eq. 5) from 16-bit w (C,3,3,K) in FP32, rounded to the 16-bit type, straight
+// into the operand layout above.  Pads C and K with zeros.
+template <int DT>
+__global__ void __launch_bounds__(256) tc16_filter_kernel(const uint16_t* __restrict__ w, uint16_t* __restrict__ u,
+                                                          int C, int K) {
+    const int Kp = ((K + MM - 1) / MM) * MM, Cp = ((C + BC - 1) / BC) * BC;
+    const long idx = (long)blockIdx.x * 256 + threadIdx.x;
+    if (idx >= (long)Cp * Kp) return;
+    const int c = (int)(idx / Kp), k = (int)(idx - (long)c * Kp);
+    float g[9], t[16];
+    if (c < C && k < K) {
+        const uint16_t* wc = w + (size_t)c * 9 * K + k;
+#pragma unroll
+        for (int e = 0; e < 9; ++e) g[e] = to_f<DT>(wc[(size_t)e * K]);
+        ftf_4x4(g, t);
+    } else {
+#pragma unroll
+        for (int e = 0; e < 16; ++e) t[e] = 0.f;
+    }
+    const int cb = c / BC, cl = c % BC, kb = k / MM, m = k % MM;
+    const int nkb = Kp / MM;
+    const size_t inner = size_t((m >> 3) * 128 + (cl >> 3) * 64 + (m & 7) * 8 + (cl & 7));
+#pragma unroll
+    for (int xi = 0; xi < 16; ++xi) {
+        const size_t base = (((size_t)cb * nkb + kb) * 16 + xi) * (MM * BC);
+        u[base + inner] = from_f<DT>(t[xi]);
+    }
+}
+
+struct __align__(64) Params {
+    CUtensorMap tmx;  // x (C,H,W,N) 16-bit as (N, W, H, C), box (32 or N, 4, 4, 16)   [TMA paths]
+    const uint16_t* __restrict__ x;
+    const uint16_t* __restrict__ u;
+    uint16_t* __restrict__ y;
+    int N, C, H, W, K;
+    int TW, NV;
+    int num_kb, num_cb, num_tiles;
+};
+
+// XM: 2 = one TMA box per tile (N % 32 == 0), 3 = 32/N boxes (N in {8, 16}), 0 = generic gather
+template <int DT, int XM>
+__global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant__ Params p) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t* const su = smem + OFF_U;
+    uint8_t* const sx = smem + OFF_X;
+    uint8_t* const sv = smem + OFF_V;
+    uint64_t* const bars = reinterpret_cast<uint64_t*>(smem + OFF_BAR);
+    uint64_t* const u_full = bars;
+    uint64_t* const u_empty = bars + U_SLOTS;
+    uint64_t* const x_full = bars + 2 * U_SLOTS;
+    uint64_t* const x_empty = x_full + X_SLOTS;
+    uint64_t* const v_full = x_empty + X_SLOTS;
+    uint64_t* const v_empty = v_full + V_SLOTS;
+    uint64_t* const acc_full = v_empty + V_SLOTS;
+    uint64_t* const acc_empty = acc_full + 1;
+    uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + OFF_TMEM);
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int NCB = p.num_cb;
+
+    if (tid == 0) {
+        for (int s = 0; s < U_SLOTS; ++s) {
+            mbar_init(&u_full[s], 1);
+            mbar_init(&u_empty[s], 1);
+        }
+        for (int s = 0; s < X_SLOTS; ++s) {
+            mbar_init(&x_full[s], 1);
+            mbar_init(&x_empty[s], ITF_GROUP);
+        }
+        for (int s = 0; s < V_SLOTS; ++s) {
+            mbar_init(&v_full[s], ITF_GROUP);
+            mbar_init(&v_empty[s], 1);
+        }
+        mbar_init(acc_full, 1);
+        mbar_init(acc_empty, EPI_WARPS);
+        fence_mbar_init();
+        if constexpr (XM >= 2) tma_prefetch_desc(&p.tmx);
+    }
+    if (warp == 0) tmem_alloc(tmem_slot, 512);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+    const size_t HWN = (size_t)p.H * p.W * p.N;
+
+    if (warp >= PROD_WARP) {
+        setmaxnreg_dec<REG_PROD>();
+        if (warp == XPROD_WARP) {
+            // --------------------------- raw-x producer ---------------------------
+            int gcb = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+                const int nu0 = (tile / p.num_kb) * BN;
+                int tn0 = 0, tw0 = -8, th0 = -8;
+                if constexpr (XM == 2) {
+                    // N % 32 == 0: the 32 nu are 32 consecutive n of one image tile
+                    if (nu0 < p.NV) {
+                        const int t = nu0 / p.N;
+                        tn0 = nu0 - t * p.N;
+                        const int th = t / p.TW, tw = t - th * p.TW;
+                        tw0 = 2 * tw - 1;  // -1: TMA zero fill = padding (Sec. 3.5)
+                        th0 = 2 * th - 1;
+                    }
+                    if (lane == 0)
+                        for (int cb = 0; cb < 4 && cb < NCB; ++cb) tma_prefetch_l2_4d(&p.tmx, tn0, tw0, th0, cb * BC);
+                }
+                // generic gather (XM 0): lane = local nu; its window origin and image
+                const int gnu = nu0 + lane;
+                const bool glive = gnu < p.NV;
+                const int gt = glive ? gnu / p.N : 0, gn = glive ? gnu - gt * p.N : 0;
+                const int gh0 = 2 * (gt / p.TW) - 1, gw0 = 2 * (gt % p.TW) - 1;
+                for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                    const int xs = gcb % X_SLOTS;
+                    if (gcb >= X_SLOTS) mbar_wait(&x_empty[xs], ((gcb / X_SLOTS) - 1) & 1);
+                    uint8_t* xdst = sx + xs * XS_BYTES;
+                    if constexpr (XM == 2) {
+                        if (lane == 0) {
+                            mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
+                            if (cb + 4 < NCB) tma_prefetch_l2_4d(&p.tmx, tn0, tw0, th0, (cb + 4) * BC);
+                            tma_load_4d(xdst, &p.tmx, &x_full[xs], tn0, tw0, th0, cb * BC);
+                        }
+                    } else if constexpr (XM == 3) {
+                        if (lane == 0) {
+                            mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
+                            const int nbox = BN / p.N, t0 = nu0 / p.N;
+                            for (int b = 0; b < nbox; ++b) {
+                                const int t = t0 + b;
+                                const bool live = t * p.N < p.NV;
+                                const int th = t / p.TW, tw = t - th * p.TW;
+                                // [box][c][pos][n:N]; -8: tile past the end -> zeros
+                                tma_load_4d(xdst + b * (BC * 16 * p.N * 2), &p.tmx, &x_full[xs], 0,
+                                            live ? 2 * tw - 1 : -8, live ? 2 * th - 1 : -8, cb * BC);
+                            }
+                        }
+                    } else {
+                        uint16_t* xd = reinterpret_cast<uint16_t*>(xdst) + lane;  // [c][pos][nu]
+                        for (int cl = 0; cl < BC; ++cl) {
+                            const int c = cb * BC + cl;
+                            const uint16_t* xc = p.x + (size_t)c * HWN + gn;
+#pragma unroll 1
+                            for (int pos = 0; pos < 16; ++pos) {
+                                const int h = gh0 + (pos >> 2), w = gw0 + (pos & 3);
+                                const bool ok = glive && c < p.C && h >= 0 && h < p.H && w >= 0 && w < p.W;
+                                xd[(cl * 16 + pos) * BN] = ok ? xc[((size_t)h * p.W + w) * p.N] : uint16_t(0);
+                            }
+                        }
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&x_full[xs]);
+                    }
+                }
+            }
+        } else if (warp == PROD_WARP) {
+            // ------------------------ transformed-filter producer -----------------
+            int unit = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+                const int kb = tile % p.num_kb;
+                for (int cb = 0; cb < NCB; ++cb, ++unit) {
+                    const int us = unit % U_SLOTS;
+                    if (unit >= U_SLOTS) mbar_wait(&u_empty[us], ((unit / U_SLOTS) - 1) & 1);
+                    if (lane == 0) {
+                        const uint16_t* src = p.u + (((size_t)cb * p.num_kb + kb) * 16) * (MM * BC);
+                        mbar_arrive_expect_tx(&u_full[us], UNIT);
+                        bulk_load(su + us * UNIT, src, UNIT, &u_full[us]);
+                    }
+                }
+            }
+        } else if (warp == MMA_WARP) {
+            // ------------------------------ MMA issuer ----------------------------
+            constexpr uint32_t IDESC = umma_idesc_f16(DT, MM, BN);
+            int unit = 0, gcb = 0, it = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+                if (it > 0) mbar_wait(acc_empty, (it - 1) & 1);  // epilogue drained TMEM
+                tc_fence_after();
+                for (int cb = 0; cb < NCB; ++cb, ++gcb, ++unit) {
+                    const int vs = gcb & 1, us = unit % U_SLOTS;
+                    mbar_wait(&v_full[vs], (gcb >> 1) & 1);
+                    mbar_wait(&u_full[us], (unit / U_SLOTS) & 1);
+                    tc_fence_after();
+                    if (lane == 0) {
+                        const uint32_t ubase = smem_u32(su + us * UNIT);
+                        const uint32_t vbase = smem_u32(sv + vs * V_SLOT);
+#pragma unroll
+                        for (int xi = 0; xi < 16; ++xi) {
+                            const uint64_t ad = umma_desc(ubase + xi * A_TILE, 128, 256);
+                            const uint64_t bd = umma_desc(vbase + xi * B_TILE, 128, V_SBO);
+                            umma_f16(tmem + xi * BN, ad, bd, IDESC, cb > 0 ? 1u : 0u);
+                        }
+                        umma_commit(&u_empty[us]);
+                        umma_commit(&v_empty[vs]);
+                    }
+                    __syncwarp();
+                }
+                if (lane == 0) umma_commit(acc_full);
+                __syncwarp();
+            }
+        }
+    } else if (warp >= ITF_WARP0) {
+        setmaxnreg_dec<REG_ITF>();
+        // ------------------------------ ITF warps -----------------------------
+        // group g takes channel blocks gcb % 2 == g; thread -> channels (2cp, 2cp+1) x nu (2np, 2np+1)
+        const int g = (warp - ITF_WARP0) / ITF_GROUP, gw = (warp - ITF_WARP0) % ITF_GROUP;
+        const int cp = 2 * gw + (lane >> 4), np = lane & 15;
+        // raw x word (nu pair) of channel c, window element pos:
+        //   XM 0/2: [c][pos][nu32] -> word c*256 + pos*16 + np; lanes 16-31 read pos^1 first
+        //           (pos*16 words apart -> the two half-warps hit disjoint banks)
+        //   XM 3:   [box][c][pos][n:N] -> word box*(BC*8N) + c*8N + pos*N/2 + (n/2)
+        const int par = (XM == 3) ? 0 : (lane >> 4);
+        int wbase, wc, wp;
+        if constexpr (XM == 3) {
+            const int nu = 2 * np, b = nu / p.N, n = nu - b * p.N;
+            wbase = b * (BC * 8 * p.N) + (n >> 1);
+            wc = 8 * p.N;
+            wp = p.N >> 1;
+        } else {
+            wbase = np;
+            wc = 256;
+            wp = 16;
+        }
+        // V words: row nu, K pair cp -> byte (nu/8)*V_SBO + (cp/4)*128 + (nu%8)*16 + (cp%4)*4
+        const uint32_t voff0 = ((2 * np) >> 3) * V_SBO + (cp >> 2) * 128 + ((2 * np) & 7) * 16 + (cp & 3) * 4;
+        int gcb = 0;
+        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+            for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                if ((gcb & 1) != g) continue;
+                const int xs = gcb % X_SLOTS, vs = g;
+                mbar_wait(&x_full[xs], (gcb / X_SLOTS) & 1);
+                const uint32_t* xw = reinterpret_cast<const uint32_t*>(sx + xs * XS_BYTES) + wbase;
+                uint32_t r[2][16];
+#pragma unroll
+                for (int j = 0; j < 2; ++j) {
+                    const uint32_t* xc = xw + (2 * cp + j) * wc;
+#pragma unroll
+                    for (int e = 0; e < 16; ++e) {
+                        const int pe = e ^ par;
+                        r[j][e] = xc[pe * wp];
+                    }
+                }
+                // undo the pos swap of the upper half-warp
+#pragma unroll
+                for (int j = 0; j < 2; ++j)
+#pragma unroll
+                    for (int e = 0; e < 16; e += 2) {
+                        const uint32_t a = r[j][e], b = r[j][e + 1];
+                        r[j][e] = par ? b : a;
+                        r[j][e + 1] = par ? a : b;
+                    }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&x_empty[xs]);
+                if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
+                uint8_t* vdst = sv + vs * V_SLOT + voff0;
+#pragma unroll
+                for (int i = 0; i < 2; ++i) {  // nu = 2np + i
+                    float v0[16], v1[16];
+                    {
+                        float d0[16], d1[16];
+#pragma unroll
+                        for (int e = 0; e < 16; ++e) {
+                            const float2 a = unpack2<DT>(r[0][e]), b = unpack2<DT>(r[1][e]);
+                            d0[e] = i ? a.y : a.x;
+                            d1[e] = i ? b.y : b.x;
+                        }
+                        itf_4x4(d0, v0);
+                        itf_4x4(d1, v1);
+                    }
+#pragma unroll
+                    for (int xi = 0; xi < 16; ++xi)
+                        *reinterpret_cast<uint32_t*>(vdst + xi * B_TILE + i * 16) = pack2<DT>(v0[xi], v1[xi]);
+                }
+                fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&v_full[vs]);
+            }
+        }
+    } else {
+        setmaxnreg_inc<REG_EPI>();
+        // ------------------------------ epilogue ------------------------------
+        const int kl = warp * 32 + lane;  // TMEM lane = filter of the tile
+        const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
+        const size_t dW = (size_t)p.W * p.N;
+        int it = 0;
+        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+            const int k = (tile % p.num_kb) * MM + kl;
+            const int nu0 = (tile / p.num_kb) * BN;
+            mbar_wait(acc_full, it & 1);
+            tc_fence_after();
+            float o[BN][4];
+#pragma unroll
+            for (int ch = 0; ch < BN / 4; ++ch) {
+                float m[16][4];
+#pragma unroll
+                for (int xi = 0; xi < 16; ++xi) tmem_ld4(trow + xi * BN + ch * 4, m[xi]);
+                tmem_ld_wait();
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    float mm[16];
+#pragma unroll
+                    for (int xi = 0; xi < 16; ++xi) mm[xi] = m[xi][j];
+                    otf_2x2(mm, o[ch * 4 + j]);
+                }
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(acc_empty);  // TMEM free for the next tile's MMAs
+            if (k >= p.K || nu0 >= p.NV) continue;
+            if constexpr (XM == 2 || XM == 3) {
+                // groups of 8 nu = 8 consecutive n of one image tile (N % 8 == 0) -> 16 B stores
+#pragma unroll
+                for (int j = 0; j < BN; j += 8) {
+                    const int nu = nu0 + j;
+                    if (nu >= p.NV) break;
+                    const int t = nu / p.N, n = nu - t * p.N;
+                    const int th = t / p.TW, tw = t - th * p.TW;
+                    const int i0 = 2 * th, j0 = 2 * tw;
+                    uint16_t* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const int a = q >> 1, b = q & 1;
+                        if (i0 + a >= p.H || j0 + b >= p.W) continue;  // odd H/W (L1155)
+                        uint4 v;
+                        v.x = pack2<DT>(o[j][q], o[j + 1][q]);
+                        v.y = pack2<DT>(o[j + 2][q], o[j + 3][q]);
+                        v.z = pack2<DT>(o[j + 4][q], o[j + 5][q]);
+                        v.w = pack2<DT>(o[j + 6][q], o[j + 7][q]);
+                        *reinterpret_cast<uint4*>(yk + a * dW + b * p.N) = v;
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int j = 0; j < BN; ++j) {
+                    const int nu = nu0 + j;
+                    if (nu >= p.NV) break;
+                    const int t = nu / p.N, n = nu - t * p.N;
+                    const int th = t / p.TW, tw = t - th * p.TW;
+                    const int i0 = 2 * th, j0 = 2 * tw;
+                    uint16_t* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+                    yk[0] = from_f<DT>(o[j][0]);
+                    if (j0 + 1 < p.W) yk[p.N] = from_f<DT>(o[j][1]);
+                    if (i0 + 1 < p.H) yk[dW] = from_f<DT>(o[j][2]);
+                    if (i0 + 1 < p.H && j0 + 1 < p.W) yk[dW + p.N] = from_f<DT>(o[j][3]);
+                }
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) tmem_dealloc(tmem, 512);
+}
+
+}  // namespace tc16
+}  // namespace wino

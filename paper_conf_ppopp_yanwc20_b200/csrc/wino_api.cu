@@ -17,6 +17,7 @@
 #include "fused_fp32.cuh"
 #include "fused_fp32_ws.cuh"
 #include "fused_tc.cuh"
+#include "fused_tc16.cuh"
 #include "fused_f4_fp32.cuh"
 #include "nonfused.cuh"
 
@@ -188,18 +189,19 @@ PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
 }
 
 // fp32 tensor map, dims innermost first; strides (bytes, dims 1..rank-1) default to dense.
-bool encode_map(CUtensorMap* m, const float* base, int rank, const cuuint64_t* dims, const cuuint32_t* box,
-                const cuuint64_t* strides_in = nullptr) {
+bool encode_map(CUtensorMap* m, const void* base, int rank, const cuuint64_t* dims, const cuuint32_t* box,
+                const cuuint64_t* strides_in = nullptr,
+                CUtensorMapDataType dtype = CU_TENSOR_MAP_DATA_TYPE_FLOAT32, int esize = 4) {
     auto enc = tensor_map_encoder();
     if (!enc) return false;
     cuuint64_t strides[4];
-    cuuint64_t acc = 4;
+    cuuint64_t acc = esize;
     for (int i = 0; i < rank - 1; ++i) {
         acc *= dims[i];
         strides[i] = strides_in ? strides_in[i] : acc;
     }
     cuuint32_t estr[5] = {1, 1, 1, 1, 1};
-    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, rank, const_cast<float*>(base), dims, strides, box, estr,
+    CUresult r = enc(m, dtype, rank, const_cast<void*>(base), dims, strides, box, estr,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);  // OOB elements read as zero
     return r == CUDA_SUCCESS;
@@ -495,6 +497,22 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->launches = 1;
         return WINO_OK;
     }
+    if (variant == 3) {  // tcgen05 kind::f16 (FP16 / BF16 operands, NEXT row N4)
+        using namespace wino::tc16;
+        const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
+        plan->variant = 3;
+        plan->bk = MM;
+        plan->bn = BN;
+        plan->bc = BC;
+        plan->load_x = (N % 32 == 0 || N == 8 || N == 16) ? 2 : 0;
+        plan->load_u = 3;
+        plan->split_c = 1;
+        plan->ctas = ((nv + BN - 1) / BN) * ((K + MM - 1) / MM);
+        plan->threads = NT;
+        plan->smem_bytes = BYTES;
+        plan->launches = 1;
+        return WINO_OK;
+    }
     if (variant != 0) return WINO_ERR_UNSUPPORTED;
     int dev = -1;  // host-only planning unless an sm_100 device is current
     {
@@ -674,6 +692,100 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
     return launch_tc<2, 0, 128>(prm, ctas, dev, st);
 }
 
+
+extern "C++" {
+namespace {
+std::atomic<uint64_t> g_attr_tc16[2][4];
+template <int DT, int XM>
+wino_status_t launch_tc16(const wino::tc16::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
+    auto kern = wino::tc16::fused_tc16_kernel<DT, XM>;
+    wino_status_t s = ensure_smem_attr(kern, dev, wino::tc16::BYTES, g_attr_tc16[DT][XM]);
+    if (s != WINO_OK) return s;
+    kern<<<dim3(static_cast<unsigned>(ctas)), wino::tc16::NT, wino::tc16::BYTES, st>>>(prm);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+bool half_type_ok(wino_half_t t) { return t == WINO_HALF_FP16 || t == WINO_HALF_BF16; }
+}  // namespace
+}  // extern "C++"
+
+size_t wino_filter_workspace_bytes_half(int C, int K) {
+    if (C <= 0 || K <= 0) return 0;
+    return wino::tc16::u_h_elems(C, K) * 2;
+}
+
+wino_status_t wino_filter_transform_half(const void* w_dev, void* u_h_dev, int C, int K, wino_half_t type,
+                                         wino_stream_t stream) {
+    if (!w_dev || !u_h_dev || C <= 0 || K <= 0 || !half_type_ok(type)) return WINO_ERR_INVALID_ARG;
+    const size_t ub = wino_filter_workspace_bytes_half(C, K);
+    if (ub / 2 > size_t(kMaxElems) || int64_t(9) * C * K > kMaxElems) return WINO_ERR_TOO_LARGE;
+    if (!aligned16(w_dev) || !aligned16(u_h_dev)) return WINO_ERR_MISALIGNED;
+    if (overlaps(w_dev, size_t(9) * C * K * 2, u_h_dev, ub)) return WINO_ERR_INVALID_ARG;
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    using namespace wino::tc16;
+    const int64_t Kp = ((K + MM - 1) / MM) * MM, Cp = ((C + BC - 1) / BC) * BC;
+    const unsigned blocks = static_cast<unsigned>((Cp * Kp + 255) / 256);
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const uint16_t* w = static_cast<const uint16_t*>(w_dev);
+    uint16_t* u = static_cast<uint16_t*>(u_h_dev);
+    if (type == WINO_HALF_FP16) tc16_filter_kernel<0><<<blocks, 256, 0, st>>>(w, u, C, K);
+    else tc16_filter_kernel<1><<<blocks, 256, 0, st>>>(w, u, C, K);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, void* y_dev, int N, int C, int H,
+                                        int W, int K, int pad, int stride, wino_half_t type, wino_stream_t stream) {
+    if (!x_dev || !u_h_dev || !y_dev || !half_type_ok(type)) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (wino_filter_workspace_bytes_half(C, K) / 2 > size_t(kMaxElems)) return WINO_ERR_TOO_LARGE;
+    if (!aligned16(x_dev) || !aligned16(u_h_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t yb = size_t(K) * hwn * 2;
+    if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 2) ||
+        overlaps(y_dev, yb, u_h_dev, wino_filter_workspace_bytes_half(C, K)))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    using namespace wino::tc16;
+    Params prm;
+    std::memset(&prm, 0, sizeof(prm));
+    prm.x = static_cast<const uint16_t*>(x_dev);
+    prm.u = static_cast<const uint16_t*>(u_h_dev);
+    prm.y = static_cast<uint16_t*>(y_dev);
+    prm.N = N;
+    prm.C = C;
+    prm.H = H;
+    prm.W = W;
+    prm.K = K;
+    prm.TW = (W + 1) / 2;
+    prm.NV = N * ((H + 1) / 2) * prm.TW;
+    prm.num_kb = (K + MM - 1) / MM;
+    prm.num_cb = (C + BC - 1) / BC;
+    prm.num_tiles = ((prm.NV + BN - 1) / BN) * prm.num_kb;
+    const int xm = (N % 32 == 0) ? 2 : ((N == 8 || N == 16) ? 3 : 0);
+    if (xm >= 2) {
+        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
+        const cuuint32_t box[4] = {cuuint32_t(xm == 2 ? BN : N), 4, 4, BC};
+        const CUtensorMapDataType dt =
+            type == WINO_HALF_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
+        if (!encode_map(&prm.tmx, x_dev, 4, dims, box, nullptr, dt, 2)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    const int sms = sm_count(dev);
+    const int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (type == WINO_HALF_FP16) {
+        if (xm == 2) return launch_tc16<0, 2>(prm, ctas, dev, st);
+        if (xm == 3) return launch_tc16<0, 3>(prm, ctas, dev, st);
+        return launch_tc16<0, 0>(prm, ctas, dev, st);
+    }
+    if (xm == 2) return launch_tc16<1, 2>(prm, ctas, dev, st);
+    if (xm == 3) return launch_tc16<1, 3>(prm, ctas, dev, st);
+    return launch_tc16<1, 0>(prm, ctas, dev, st);
+}
 
 size_t wino_host_workspace_bytes(int N, int C, int H, int W, int K) {
     if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
