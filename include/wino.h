@@ -212,7 +212,8 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
  * (bf16) against Eq. 4 of the 16-bit inputs; bit-exact (y == round(y_ref)) on
  * small-integer inputs.
  *   u_h : wino_filter_workspace_bytes_half(C,K) bytes, opaque layout
- *         [ceil(C/16)][ceil(K/128)][16][128 x 16 K-major tile], zero padded.
+ *         [ceil(C/16)][ceil(K/MM)][16][MM x 16 K-major tile], zero padded, with the
+ *         tile height MM = 64 when K <= 64, else 128.
  * Any N, C, K, H, W >= 1; N % 32 == 0 or N in {8, 16} take TMA loads.  Errors as
  * the FP32 calls, plus WINO_ERR_INVALID_ARG for an unknown `type`.
  */

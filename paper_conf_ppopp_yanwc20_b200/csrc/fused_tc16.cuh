@@ -35,37 +35,73 @@
 namespace wino {
 namespace tc16 {
 
-constexpr int BN = 32;    // nu per tile (UMMA N)
-constexpr int MM = 128;   // filters per tile (UMMA M)
+#ifdef WINO_TC16_TRACE
+// Debug-only event trace (CTA 0): [event][gcb] = clock64 at the event.
+constexpr int TRACE_EVENTS = 8, TRACE_CB = 256;
+__device__ unsigned long long g_trace16[TRACE_EVENTS * TRACE_CB];
+#define TC16_TRACE(ev, cb)                                                                          \
+    do {                                                                                           \
+        if (blockIdx.x == 0 && (cb) < TRACE_CB) g_trace16[(ev) * TRACE_CB + (cb)] = clock64();     \
+    } while (0)
+#else
+#define TC16_TRACE(ev, cb) \
+    do {                   \
+    } while (0)
+#endif
+
+constexpr int BN = 32;    // nu per UMMA (N); a tile has NH = 128 / MM such halves
 constexpr int BC = 16;    // channels per block (UMMA K of kind::f16)
 constexpr int EPI_WARPS = 4, ITF_WARP0 = 4, ITF_WARPS = 8, ITF_GROUP = 4;
 constexpr int PROD_WARP = 12, MMA_WARP = 13, XPROD_WARP = 14;
 constexpr int NT = 512;
 constexpr int REG_EPI = 216, REG_ITF = 112, REG_PROD = 56;  // 128*216 + 256*112 + 128*56 = 63488
-constexpr int A_TILE = MM * BC * 2;       // one xi of U: 4 KB, [m/8][c/8][m%8][c%8]
-constexpr int UNIT = 16 * A_TILE;         // one channel block of U: 64 KB
-constexpr int V_SBO = 272;                // 8-row group stride of the V operand (256 + 16: fewer bank conflicts)
-constexpr int B_TILE = (BN / 8) * V_SBO;  // one xi of V: 1088 B, [nu/8 (stride 272)][c/8 (128)][nu%8][c%8]
-constexpr int XS_BYTES = BC * 16 * BN * 2;  // raw x of one block: 16 KB, [c][pos][nu]
-// x slot = gcb % 4: each ITF group owns two slots (0, 2 / 1, 3) and consumes them in order, so
-// an mbarrier phase parity can never alias a fill that has not landed (the groups drift apart).
-constexpr int U_SLOTS = 2, X_SLOTS = 4, V_SLOTS = 2;
-constexpr int V_SLOT = 16 * B_TILE;
-constexpr int OFF_U = 0;
-constexpr int OFF_X = OFF_U + U_SLOTS * UNIT;
-constexpr int OFF_V = OFF_X + X_SLOTS * XS_BYTES;
-constexpr int OFF_BAR = OFF_V + V_SLOTS * V_SLOT;
-constexpr int NBAR = 2 * U_SLOTS + 2 * X_SLOTS + 2 * V_SLOTS + 2;
-constexpr int OFF_TMEM = OFF_BAR + NBAR * 8;
-constexpr int BYTES = OFF_TMEM + 16;
-static_assert(BYTES <= 232448, "shared memory budget");
-static_assert(V_SLOTS == 2 && X_SLOTS % 2 == 0, "two ITF groups take alternate channel blocks");
+constexpr int V_SBO = 256;                // 8-row group stride of the V operand
+constexpr int B_TILE = (BN / 8) * V_SBO;  // one (xi, nu-half) of V: 1 KB, [nu/8][c/8 (LBO 128)][nu%8][c%8]
+constexpr int XS_BYTES = BC * 16 * BN * 2;  // raw x of one block and nu-half: 16 KB, [c][pos][nu]
 
+// Per tile height MM (filters = UMMA M):
+//  * MM = 128: tile 128 k x 32 nu; the two ITF groups take alternate channel blocks; x slot =
+//    gcb % 4 (each group owns two slots and consumes them in order, so an mbarrier phase
+//    parity never aliases a fill that has not landed while the groups drift apart).
+//  * MM = 64: tile 64 k x 64 nu (two nu-halves; their M = 64 accumulators interleave in TMEM
+//    lanes 0-15 / 16-31 of each quadrant, scripts/microbench/umma_m64.cu); ITF group g
+//    transforms nu-half g of every channel block.  Half the filter bytes per (k, nu) pair.
+template <int MM>
+struct Cfg {
+    static constexpr int NH = 128 / MM;
+    static constexpr int TN = BN * NH;
+    static constexpr int A_TILE = MM * BC * 2;  // one xi of U, [m/8][c/8][m%8][c%8]
+    static constexpr int UNIT = 16 * A_TILE;    // one channel block of U: 64 / 32 KB
+    static constexpr int U_SLOTS = NH == 1 ? 2 : 3;
+    static constexpr int X_SLOTS = NH == 1 ? 4 : 2;
+    static constexpr int V_SLOTS = 2;
+    static constexpr int X_SLOT = NH * XS_BYTES;
+    static constexpr int V_SLOT = 16 * NH * B_TILE;
+    static constexpr int ITF_PER_X = NH == 1 ? ITF_GROUP : ITF_WARPS;  // warps consuming one x / V slot
+    static constexpr int OFF_U = 0;
+    static constexpr int OFF_X = OFF_U + U_SLOTS * UNIT;
+    static constexpr int OFF_V = OFF_X + X_SLOTS * X_SLOT;
+    static constexpr int OFF_BAR = OFF_V + V_SLOTS * V_SLOT;
+    static constexpr int NBAR = 2 * U_SLOTS + 2 * X_SLOTS + 2 * V_SLOTS + 2;
+    static constexpr int OFF_TMEM = OFF_BAR + NBAR * 8;
+    static constexpr int BYTES = OFF_TMEM + 16;
+    static_assert(BYTES <= 232448, "shared memory budget");
+};
+
+// Tile height of a shape (the filter transform and the conv must agree).
+__host__ __device__ inline int tc16_mm(int K) {
+#if defined(WINO_TC16_MM)
+    return WINO_TC16_MM;  // A/B builds
+#else
+    return K <= 64 ? 64 : 128;
+#endif
+}
 // u_h layout (written by tc16_filter_kernel, read with bulk copies):
-//   [cb = ceil(C/16)][kb = ceil(K/128)][xi 16][m/8 16][c/8 2][m%8 8][c%8 8]  16-bit
+//   [cb = ceil(C/16)][kb = ceil(K/MM)][xi 16][m/8][c/8 2][m%8 8][c%8 8]  16-bit
 // i.e. per (cb, kb, xi) one K-major SWIZZLE_NONE UMMA A tile (LBO 128 B, SBO 256 B).
 __host__ __device__ inline size_t u_h_elems(int C, int K) {
-    return size_t((C + BC - 1) / BC) * ((K + MM - 1) / MM) * 16 * (MM * BC);
+    const int mm = tc16_mm(K);
+    return size_t((C + BC - 1) / BC) * ((K + mm - 1) / mm) * 16 * (mm * BC);
 }
 
 // 16-bit type helpers: DT 0 = IEEE fp16, 1 = bf16.
@@ -114,7 +150,7 @@ __device__ __forceinline__ void umma_f16(uint32_t d_tmem, uint64_t a, uint64_t b
 
 // FTF (Eq. 5) from 16-bit w (C,3,3,K) in FP32, rounded to the 16-bit type, straight
 // into the operand layout above.  Pads C and K with zeros.
-template <int DT>
+template <int DT, int MM>
 __global__ void __launch_bounds__(256) tc16_filter_kernel(const uint16_t* __restrict__ w, uint16_t* __restrict__ u,
                                                           int C, int K) {
     const int Kp = ((K + MM - 1) / MM) * MM, Cp = ((C + BC - 1) / BC) * BC;
@@ -151,14 +187,18 @@ struct __align__(64) Params {
     int num_kb, num_cb, num_tiles;
 };
 
-// XM: 2 = one TMA box per tile (N % 32 == 0), 3 = 32/N boxes (N in {8, 16}), 0 = generic gather
-template <int DT, int XM>
+// XM: 2 = one TMA box per nu-half (N % 32 == 0), 3 = 32/N boxes per half (N in {8, 16}),
+// 0 = generic gather by the x-producer warp
+template <int DT, int XM, int MM>
 __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant__ Params p) {
+    using G = Cfg<MM>;
+    constexpr int NH = G::NH, TN = G::TN;
+    constexpr int U_SLOTS = G::U_SLOTS, X_SLOTS = G::X_SLOTS, V_SLOTS = G::V_SLOTS;
     extern __shared__ __align__(1024) uint8_t smem[];
-    uint8_t* const su = smem + OFF_U;
-    uint8_t* const sx = smem + OFF_X;
-    uint8_t* const sv = smem + OFF_V;
-    uint64_t* const bars = reinterpret_cast<uint64_t*>(smem + OFF_BAR);
+    uint8_t* const su = smem + G::OFF_U;
+    uint8_t* const sx = smem + G::OFF_X;
+    uint8_t* const sv = smem + G::OFF_V;
+    uint64_t* const bars = reinterpret_cast<uint64_t*>(smem + G::OFF_BAR);
     uint64_t* const u_full = bars;
     uint64_t* const u_empty = bars + U_SLOTS;
     uint64_t* const x_full = bars + 2 * U_SLOTS;
@@ -167,7 +207,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
     uint64_t* const v_empty = v_full + V_SLOTS;
     uint64_t* const acc_full = v_empty + V_SLOTS;
     uint64_t* const acc_empty = acc_full + 1;
-    uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + OFF_TMEM);
+    uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + G::OFF_TMEM);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int NCB = p.num_cb;
@@ -179,10 +219,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
         }
         for (int s = 0; s < X_SLOTS; ++s) {
             mbar_init(&x_full[s], 1);
-            mbar_init(&x_empty[s], ITF_GROUP);
+            mbar_init(&x_empty[s], G::ITF_PER_X);
         }
         for (int s = 0; s < V_SLOTS; ++s) {
-            mbar_init(&v_full[s], ITF_GROUP);
+            mbar_init(&v_full[s], G::ITF_PER_X);
             mbar_init(&v_empty[s], 1);
         }
         mbar_init(acc_full, 1);
@@ -203,39 +243,47 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
             // --------------------------- raw-x producer ---------------------------
             int gcb = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-                const int nu0 = (tile / p.num_kb) * BN;
-                int tn0 = 0, tw0 = -8, th0 = -8;
+                const int nu0 = (tile / p.num_kb) * TN;
+                int tn0[NH], tw0[NH], th0[NH];
                 if constexpr (XM == 2) {
-                    // N % 32 == 0: the 32 nu are 32 consecutive n of one image tile
-                    if (nu0 < p.NV) {
-                        const int t = nu0 / p.N;
-                        tn0 = nu0 - t * p.N;
-                        const int th = t / p.TW, tw = t - th * p.TW;
-                        tw0 = 2 * tw - 1;  // -1: TMA zero fill = padding (Sec. 3.5)
-                        th0 = 2 * th - 1;
+                    // N % 32 == 0: each nu-half = 32 consecutive n of one image tile
+#pragma unroll
+                    for (int h = 0; h < NH; ++h) {
+                        const int nuh = nu0 + h * BN;
+                        tn0[h] = 0;
+                        tw0[h] = -8;  // half past NV -> all zeros
+                        th0[h] = -8;
+                        if (nuh < p.NV) {
+                            const int t = nuh / p.N;
+                            tn0[h] = nuh - t * p.N;
+                            const int th = t / p.TW, tw = t - th * p.TW;
+                            tw0[h] = 2 * tw - 1;  // -1: TMA zero fill = padding (Sec. 3.5)
+                            th0[h] = 2 * th - 1;
+                        }
                     }
                     if (lane == 0)
-                        for (int cb = 0; cb < 4 && cb < NCB; ++cb) tma_prefetch_l2_4d(&p.tmx, tn0, tw0, th0, cb * BC);
+                        for (int cb = 0; cb < 4 && cb < NCB; ++cb)
+#pragma unroll
+                            for (int h = 0; h < NH; ++h) tma_prefetch_l2_4d(&p.tmx, tn0[h], tw0[h], th0[h], cb * BC);
                 }
-                // generic gather (XM 0): lane = local nu; its window origin and image
-                const int gnu = nu0 + lane;
-                const bool glive = gnu < p.NV;
-                const int gt = glive ? gnu / p.N : 0, gn = glive ? gnu - gt * p.N : 0;
-                const int gh0 = 2 * (gt / p.TW) - 1, gw0 = 2 * (gt % p.TW) - 1;
                 for (int cb = 0; cb < NCB; ++cb, ++gcb) {
                     const int xs = gcb % X_SLOTS;
                     if (gcb >= X_SLOTS) mbar_wait(&x_empty[xs], ((gcb / X_SLOTS) - 1) & 1);
-                    uint8_t* xdst = sx + xs * XS_BYTES;
+                    uint8_t* xdst = sx + xs * G::X_SLOT;
+                    if (lane == 0) TC16_TRACE(0, gcb);
                     if constexpr (XM == 2) {
                         if (lane == 0) {
-                            mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
-                            if (cb + 4 < NCB) tma_prefetch_l2_4d(&p.tmx, tn0, tw0, th0, (cb + 4) * BC);
-                            tma_load_4d(xdst, &p.tmx, &x_full[xs], tn0, tw0, th0, cb * BC);
+                            mbar_arrive_expect_tx(&x_full[xs], G::X_SLOT);
+#pragma unroll
+                            for (int h = 0; h < NH; ++h) {
+                                if (cb + 4 < NCB) tma_prefetch_l2_4d(&p.tmx, tn0[h], tw0[h], th0[h], (cb + 4) * BC);
+                                tma_load_4d(xdst + h * XS_BYTES, &p.tmx, &x_full[xs], tn0[h], tw0[h], th0[h], cb * BC);
+                            }
                         }
                     } else if constexpr (XM == 3) {
                         if (lane == 0) {
-                            mbar_arrive_expect_tx(&x_full[xs], XS_BYTES);
-                            const int nbox = BN / p.N, t0 = nu0 / p.N;
+                            mbar_arrive_expect_tx(&x_full[xs], G::X_SLOT);
+                            const int nbox = TN / p.N, t0 = nu0 / p.N;
                             for (int b = 0; b < nbox; ++b) {
                                 const int t = t0 + b;
                                 const bool live = t * p.N < p.NV;
@@ -246,15 +294,23 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                             }
                         }
                     } else {
-                        uint16_t* xd = reinterpret_cast<uint16_t*>(xdst) + lane;  // [c][pos][nu]
-                        for (int cl = 0; cl < BC; ++cl) {
-                            const int c = cb * BC + cl;
-                            const uint16_t* xc = p.x + (size_t)c * HWN + gn;
+                        // generic gather: lane = local nu of each half, layout [h][c][pos][nu]
 #pragma unroll 1
-                            for (int pos = 0; pos < 16; ++pos) {
-                                const int h = gh0 + (pos >> 2), w = gw0 + (pos & 3);
-                                const bool ok = glive && c < p.C && h >= 0 && h < p.H && w >= 0 && w < p.W;
-                                xd[(cl * 16 + pos) * BN] = ok ? xc[((size_t)h * p.W + w) * p.N] : uint16_t(0);
+                        for (int h = 0; h < NH; ++h) {
+                            const int gnu = nu0 + h * BN + lane;
+                            const bool glive = gnu < p.NV;
+                            const int gt = glive ? gnu / p.N : 0, gn = glive ? gnu - gt * p.N : 0;
+                            const int gh0 = 2 * (gt / p.TW) - 1, gw0 = 2 * (gt % p.TW) - 1;
+                            uint16_t* xd = reinterpret_cast<uint16_t*>(xdst + h * XS_BYTES) + lane;
+                            for (int cl = 0; cl < BC; ++cl) {
+                                const int c = cb * BC + cl;
+                                const uint16_t* xc = p.x + (size_t)c * HWN + gn;
+#pragma unroll 1
+                                for (int pos = 0; pos < 16; ++pos) {
+                                    const int hh = gh0 + (pos >> 2), ww = gw0 + (pos & 3);
+                                    const bool ok = glive && c < p.C && hh >= 0 && hh < p.H && ww >= 0 && ww < p.W;
+                                    xd[(cl * 16 + pos) * BN] = ok ? xc[((size_t)hh * p.W + ww) * p.N] : uint16_t(0);
+                                }
                             }
                         }
                         __syncwarp();
@@ -271,9 +327,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                     const int us = unit % U_SLOTS;
                     if (unit >= U_SLOTS) mbar_wait(&u_empty[us], ((unit / U_SLOTS) - 1) & 1);
                     if (lane == 0) {
+                        TC16_TRACE(1, unit);
                         const uint16_t* src = p.u + (((size_t)cb * p.num_kb + kb) * 16) * (MM * BC);
-                        mbar_arrive_expect_tx(&u_full[us], UNIT);
-                        bulk_load(su + us * UNIT, src, UNIT, &u_full[us]);
+                        mbar_arrive_expect_tx(&u_full[us], G::UNIT);
+                        bulk_load(su + us * G::UNIT, src, G::UNIT, &u_full[us]);
                     }
                 }
             }
@@ -287,16 +344,23 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                 for (int cb = 0; cb < NCB; ++cb, ++gcb, ++unit) {
                     const int vs = gcb & 1, us = unit % U_SLOTS;
                     mbar_wait(&v_full[vs], (gcb >> 1) & 1);
+                    if (lane == 0) TC16_TRACE(4, gcb);
                     mbar_wait(&u_full[us], (unit / U_SLOTS) & 1);
                     tc_fence_after();
                     if (lane == 0) {
-                        const uint32_t ubase = smem_u32(su + us * UNIT);
-                        const uint32_t vbase = smem_u32(sv + vs * V_SLOT);
+                        TC16_TRACE(5, gcb);
+                        const uint32_t ubase = smem_u32(su + us * G::UNIT);
+                        const uint32_t vbase = smem_u32(sv + vs * G::V_SLOT);
 #pragma unroll
                         for (int xi = 0; xi < 16; ++xi) {
-                            const uint64_t ad = umma_desc(ubase + xi * A_TILE, 128, 256);
-                            const uint64_t bd = umma_desc(vbase + xi * B_TILE, 128, V_SBO);
-                            umma_f16(tmem + xi * BN, ad, bd, IDESC, cb > 0 ? 1u : 0u);
+                            const uint64_t ad = umma_desc(ubase + xi * G::A_TILE, 128, 256);
+#pragma unroll
+                            for (int h = 0; h < NH; ++h) {
+                                // nu-half h accumulates in TMEM lanes 16h.. of each quadrant (MM = 64)
+                                const uint64_t bd = umma_desc(vbase + (xi * NH + h) * B_TILE, 128, V_SBO);
+                                umma_f16(tmem + xi * BN + ((uint32_t)(16 * h) << 16), ad, bd, IDESC,
+                                         cb > 0 ? 1u : 0u);
+                            }
                         }
                         umma_commit(&u_empty[us]);
                         umma_commit(&v_empty[vs]);
@@ -310,90 +374,96 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
     } else if (warp >= ITF_WARP0) {
         setmaxnreg_dec<REG_ITF>();
         // ------------------------------ ITF warps -----------------------------
-        // group g takes channel blocks gcb % 2 == g; thread -> channels (2cp, 2cp+1) x nu (2np, 2np+1)
+        // group g (warps 4-7 / 8-11): MM = 128 -> channel blocks gcb % 2 == g; MM = 64 -> nu-half g.
+        // Thread -> channels (2cp, 2cp+1) x nu (2np, 2np+1) of its half.
         const int g = (warp - ITF_WARP0) / ITF_GROUP, gw = (warp - ITF_WARP0) % ITF_GROUP;
+        const int hh = NH == 2 ? g : 0;
         const int cp = 2 * gw + (lane >> 4), np = lane & 15;
         // raw x word (nu pair) of channel c, window element pos:
-        //   XM 0/2: [c][pos][nu32] -> word c*256 + pos*16 + np; lanes 16-31 read pos^1 first
-        //           (pos*16 words apart -> the two half-warps hit disjoint banks)
+        //   XM 0/2: [h][c][pos][nu32] -> word h*4096 + c*256 + pos*16 + np; lanes 16-31 read pos^1
+        //           first (pos*16 words apart -> the two half-warps hit disjoint banks)
         //   XM 3:   [box][c][pos][n:N] -> word box*(BC*8N) + c*8N + pos*N/2 + (n/2)
         const int par = (XM == 3) ? 0 : (lane >> 4);
         int wbase, wc, wp;
         if constexpr (XM == 3) {
-            const int nu = 2 * np, b = nu / p.N, n = nu - b * p.N;
+            const int nu = hh * BN + 2 * np, b = nu / p.N, n = nu - b * p.N;
             wbase = b * (BC * 8 * p.N) + (n >> 1);
             wc = 8 * p.N;
             wp = p.N >> 1;
         } else {
-            wbase = np;
+            wbase = hh * (XS_BYTES / 4) + np;
             wc = 256;
             wp = 16;
         }
-        // V words: row nu, K pair cp -> byte (nu/8)*V_SBO + (cp/4)*128 + (nu%8)*16 + (cp%4)*4
-        const uint32_t voff0 = ((2 * np) >> 3) * V_SBO + (cp >> 2) * 128 + ((2 * np) & 7) * 16 + (cp & 3) * 4;
+        // V word (row nu, K pair cp) at byte (nu/8)*V_SBO + (cp/4)*128 + (nu%8)*16 + (cp%4)*4; lanes with
+        // (np/4) odd store their nu+1 row first (2-way instead of 4-way bank conflicts)
+        const int sw = (np >> 2) & 1;
+        const uint32_t voff0 = hh * B_TILE + ((2 * np) >> 3) * V_SBO + (cp >> 2) * 128 + ((2 * np) & 7) * 16 + (cp & 3) * 4;
         int gcb = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
             for (int cb = 0; cb < NCB; ++cb, ++gcb) {
-                if ((gcb & 1) != g) continue;
-                const int xs = gcb % X_SLOTS, vs = g;
+                if (NH == 1 && (gcb & 1) != g) continue;
+                const int xs = gcb % X_SLOTS, vs = gcb & 1;
                 mbar_wait(&x_full[xs], (gcb / X_SLOTS) & 1);
-                const uint32_t* xw = reinterpret_cast<const uint32_t*>(sx + xs * XS_BYTES) + wbase;
+                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(2, gcb);
+                const uint32_t* xw = reinterpret_cast<const uint32_t*>(sx + xs * G::X_SLOT) + wbase;
                 uint32_t r[2][16];
 #pragma unroll
                 for (int j = 0; j < 2; ++j) {
                     const uint32_t* xc = xw + (2 * cp + j) * wc;
 #pragma unroll
-                    for (int e = 0; e < 16; ++e) {
-                        const int pe = e ^ par;
-                        r[j][e] = xc[pe * wp];
-                    }
+                    for (int e = 0; e < 16; ++e) r[j][e] = xc[(e ^ par) * wp];
                 }
-                // undo the pos swap of the upper half-warp
-#pragma unroll
-                for (int j = 0; j < 2; ++j)
-#pragma unroll
-                    for (int e = 0; e < 16; e += 2) {
-                        const uint32_t a = r[j][e], b = r[j][e + 1];
-                        r[j][e] = par ? b : a;
-                        r[j][e + 1] = par ? a : b;
-                    }
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&x_empty[xs]);
-                if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
-                uint8_t* vdst = sv + vs * V_SLOT + voff0;
+                // V = B^T d B (Eq. 6) in FP32 for the 4 tiles, packed as c-pairs, BEFORE waiting
+                // for the V slot (the transform overlaps the tensor cores' use of the slot)
+                uint32_t vw[2][16];
 #pragma unroll
                 for (int i = 0; i < 2; ++i) {  // nu = 2np + i
-                    float v0[16], v1[16];
-                    {
-                        float d0[16], d1[16];
+                    float d0[16], d1[16], v0[16], v1[16];
 #pragma unroll
-                        for (int e = 0; e < 16; ++e) {
-                            const float2 a = unpack2<DT>(r[0][e]), b = unpack2<DT>(r[1][e]);
-                            d0[e] = i ? a.y : a.x;
-                            d1[e] = i ? b.y : b.x;
-                        }
-                        itf_4x4(d0, v0);
-                        itf_4x4(d1, v1);
+                    for (int e = 0; e < 16; ++e) {
+                        // the upper half-warp loaded pos e^1 into slot e
+                        const uint32_t a0 = r[0][e], a1 = r[0][e ^ 1], b0 = r[1][e], b1 = r[1][e ^ 1];
+                        const float2 a = unpack2<DT>(par ? a1 : a0), b = unpack2<DT>(par ? b1 : b0);
+                        d0[e] = i ? a.y : a.x;
+                        d1[e] = i ? b.y : b.x;
                     }
+                    itf_4x4(d0, v0);
+                    itf_4x4(d1, v1);
 #pragma unroll
-                    for (int xi = 0; xi < 16; ++xi)
-                        *reinterpret_cast<uint32_t*>(vdst + xi * B_TILE + i * 16) = pack2<DT>(v0[xi], v1[xi]);
+                    for (int xi = 0; xi < 16; ++xi) vw[i][xi] = pack2<DT>(v0[xi], v1[xi]);
                 }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&x_empty[xs]);  // the x slot can be refilled
+                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(3, gcb);
+                if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
+                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(6, gcb);
+                uint8_t* vdst = sv + vs * G::V_SLOT + voff0;
+#pragma unroll
+                for (int s = 0; s < 2; ++s)
+#pragma unroll
+                    for (int xi = 0; xi < 16; ++xi) {
+                        const uint32_t val = sw ? vw[s ^ 1][xi] : vw[s][xi];
+                        *reinterpret_cast<uint32_t*>(vdst + xi * NH * B_TILE + (s ^ sw) * 16) = val;
+                    }
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&v_full[vs]);
+                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(7, gcb);
             }
         }
     } else {
         setmaxnreg_inc<REG_EPI>();
         // ------------------------------ epilogue ------------------------------
-        const int kl = warp * 32 + lane;  // TMEM lane = filter of the tile
+        // MM = 128: TMEM lane = filter; MM = 64: lanes 0-15 -> filters of nu-half 0, 16-31 -> nu-half 1
+        const int kl = (MM == 128) ? warp * 32 + lane : warp * 16 + (lane & 15);
+        const int hsel = (MM == 128) ? 0 : (lane >> 4);
         const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
         const size_t dW = (size_t)p.W * p.N;
         int it = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
             const int k = (tile % p.num_kb) * MM + kl;
-            const int nu0 = (tile / p.num_kb) * BN;
+            const int nu0 = (tile / p.num_kb) * TN + hsel * BN;
             mbar_wait(acc_full, it & 1);
             tc_fence_after();
             float o[BN][4];

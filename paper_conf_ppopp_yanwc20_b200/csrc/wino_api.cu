@@ -448,6 +448,11 @@ int wino_debug_ws_trace(unsigned long long* host, int n) {
     return (int)cudaMemcpyFromSymbol(host, wino::fp32ws::g_ws_trace, sizeof(unsigned long long) * n);
 }
 #endif
+#ifdef WINO_TC16_TRACE
+int wino_debug_tc16_trace(unsigned long long* host, int n) {
+    return (int)cudaMemcpyFromSymbol(host, wino::tc16::g_trace16, sizeof(unsigned long long) * n);
+}
+#endif
 #ifdef WINO_TC_TRACE
 // debug builds only: copy the tcgen05 kernel's CTA-0 event trace to the host
 int wino_debug_tc_trace(unsigned long long* host, int n) {
@@ -500,16 +505,17 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
     if (variant == 3) {  // tcgen05 kind::f16 (FP16 / BF16 operands, NEXT row N4)
         using namespace wino::tc16;
         const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
+        const int mm = tc16_mm(K), tn = BN * (128 / mm);
         plan->variant = 3;
-        plan->bk = MM;
-        plan->bn = BN;
+        plan->bk = mm;
+        plan->bn = tn;
         plan->bc = BC;
         plan->load_x = (N % 32 == 0 || N == 8 || N == 16) ? 2 : 0;
         plan->load_u = 3;
         plan->split_c = 1;
-        plan->ctas = ((nv + BN - 1) / BN) * ((K + MM - 1) / MM);
+        plan->ctas = ((nv + tn - 1) / tn) * ((K + mm - 1) / mm);
         plan->threads = NT;
-        plan->smem_bytes = BYTES;
+        plan->smem_bytes = mm == 64 ? Cfg<64>::BYTES : Cfg<128>::BYTES;
         plan->launches = 1;
         return WINO_OK;
     }
@@ -695,17 +701,24 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
 
 extern "C++" {
 namespace {
-std::atomic<uint64_t> g_attr_tc16[2][4];
-template <int DT, int XM>
+std::atomic<uint64_t> g_attr_tc16[2][4][2];
+template <int DT, int XM, int MM>
 wino_status_t launch_tc16(const wino::tc16::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
-    auto kern = wino::tc16::fused_tc16_kernel<DT, XM>;
-    wino_status_t s = ensure_smem_attr(kern, dev, wino::tc16::BYTES, g_attr_tc16[DT][XM]);
+    auto kern = wino::tc16::fused_tc16_kernel<DT, XM, MM>;
+    constexpr int smem = wino::tc16::Cfg<MM>::BYTES;
+    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc16[DT][XM][MM == 64]);
     if (s != WINO_OK) return s;
-    kern<<<dim3(static_cast<unsigned>(ctas)), wino::tc16::NT, wino::tc16::BYTES, st>>>(prm);
+    kern<<<dim3(static_cast<unsigned>(ctas)), wino::tc16::NT, smem, st>>>(prm);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 bool half_type_ok(wino_half_t t) { return t == WINO_HALF_FP16 || t == WINO_HALF_BF16; }
+template <int DT, int MM>
+wino_status_t launch_tc16_xm(const wino::tc16::Params& prm, int xm, int64_t ctas, int dev, cudaStream_t st) {
+    if (xm == 2) return launch_tc16<DT, 2, MM>(prm, ctas, dev, st);
+    if (xm == 3) return launch_tc16<DT, 3, MM>(prm, ctas, dev, st);
+    return launch_tc16<DT, 0, MM>(prm, ctas, dev, st);
+}
 }  // namespace
 }  // extern "C++"
 
@@ -725,13 +738,19 @@ wino_status_t wino_filter_transform_half(const void* w_dev, void* u_h_dev, int C
     wino_status_t s = check_device(&dev);
     if (s != WINO_OK) return s;
     using namespace wino::tc16;
-    const int64_t Kp = ((K + MM - 1) / MM) * MM, Cp = ((C + BC - 1) / BC) * BC;
+    const int mm = tc16_mm(K);
+    const int64_t Kp = ((K + mm - 1) / mm) * mm, Cp = ((C + BC - 1) / BC) * BC;
     const unsigned blocks = static_cast<unsigned>((Cp * Kp + 255) / 256);
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     const uint16_t* w = static_cast<const uint16_t*>(w_dev);
     uint16_t* u = static_cast<uint16_t*>(u_h_dev);
-    if (type == WINO_HALF_FP16) tc16_filter_kernel<0><<<blocks, 256, 0, st>>>(w, u, C, K);
-    else tc16_filter_kernel<1><<<blocks, 256, 0, st>>>(w, u, C, K);
+    if (type == WINO_HALF_FP16) {
+        if (mm == 64) tc16_filter_kernel<0, 64><<<blocks, 256, 0, st>>>(w, u, C, K);
+        else tc16_filter_kernel<0, 128><<<blocks, 256, 0, st>>>(w, u, C, K);
+    } else {
+        if (mm == 64) tc16_filter_kernel<1, 64><<<blocks, 256, 0, st>>>(w, u, C, K);
+        else tc16_filter_kernel<1, 128><<<blocks, 256, 0, st>>>(w, u, C, K);
+    }
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
@@ -763,9 +782,10 @@ wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, 
     prm.K = K;
     prm.TW = (W + 1) / 2;
     prm.NV = N * ((H + 1) / 2) * prm.TW;
-    prm.num_kb = (K + MM - 1) / MM;
+    const int mm = tc16_mm(K), tn = BN * (128 / mm);
+    prm.num_kb = (K + mm - 1) / mm;
     prm.num_cb = (C + BC - 1) / BC;
-    prm.num_tiles = ((prm.NV + BN - 1) / BN) * prm.num_kb;
+    prm.num_tiles = ((prm.NV + tn - 1) / tn) * prm.num_kb;
     const int xm = (N % 32 == 0) ? 2 : ((N == 8 || N == 16) ? 3 : 0);
     if (xm >= 2) {
         const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
@@ -777,14 +797,9 @@ wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, 
     const int sms = sm_count(dev);
     const int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    if (type == WINO_HALF_FP16) {
-        if (xm == 2) return launch_tc16<0, 2>(prm, ctas, dev, st);
-        if (xm == 3) return launch_tc16<0, 3>(prm, ctas, dev, st);
-        return launch_tc16<0, 0>(prm, ctas, dev, st);
-    }
-    if (xm == 2) return launch_tc16<1, 2>(prm, ctas, dev, st);
-    if (xm == 3) return launch_tc16<1, 3>(prm, ctas, dev, st);
-    return launch_tc16<1, 0>(prm, ctas, dev, st);
+    if (type == WINO_HALF_FP16)
+        return mm == 64 ? launch_tc16_xm<0, 64>(prm, xm, ctas, dev, st) : launch_tc16_xm<0, 128>(prm, xm, ctas, dev, st);
+    return mm == 64 ? launch_tc16_xm<1, 64>(prm, xm, ctas, dev, st) : launch_tc16_xm<1, 128>(prm, xm, ctas, dev, st);
 }
 
 size_t wino_host_workspace_bytes(int N, int C, int H, int W, int K) {

@@ -51,12 +51,14 @@ def _run(wino, xh, wh):
 
 
 def _unpack_u(uh):
-    """(C,4,4,K) from the documented operand layout [cb][kb][xi][m/8][c/8][m%8][c%8]."""
+    """(C,4,4,K) from the documented operand layout [cb][kb][xi][m/8][c/8][m%8][c%8], MM = 64 rows
+    per kb when K <= 64, else 128 (include/wino.h)."""
     C, K = uh.C, uh.K
-    ncb, nkb = (C + 15) // 16, (K + 127) // 128
-    a = uh.data.cpu().float().reshape(ncb, nkb, 16, 16, 2, 8, 8)
+    mm = 64 if K <= 64 else 128
+    ncb, nkb = (C + 15) // 16, (K + mm - 1) // mm
+    a = uh.data.cpu().float().reshape(ncb, nkb, 16, mm // 8, 2, 8, 8)
     # -> [cb][c/8][c%8][xi][kb][m/8][m%8]
-    a = a.permute(0, 4, 6, 2, 1, 3, 5).reshape(ncb * 16, 16, nkb * 128)
+    a = a.permute(0, 4, 6, 2, 1, 3, 5).reshape(ncb * 16, 16, nkb * mm)
     return a[:C, :, :K].reshape(C, 4, 4, K)
 
 
