@@ -149,31 +149,44 @@ __device__ __forceinline__ void umma_f16(uint32_t d_tmem, uint64_t a, uint64_t b
 }
 
 // FTF (Eq. 5) from 16-bit w (C,3,3,K) in FP32, rounded to the 16-bit type, straight
-// into the operand layout above.  Pads C and K with zeros.
+// into the operand layout above.  One thread per (8 consecutive channels, filter k):
+// the 8 channels of a core-matrix row are one 16 B store per xi, and consecutive k
+// (threads) are consecutive rows -> coalesced.  Pads C and K with zeros.
 template <int DT, int MM>
 __global__ void __launch_bounds__(256) tc16_filter_kernel(const uint16_t* __restrict__ w, uint16_t* __restrict__ u,
                                                           int C, int K) {
-    const int Kp = ((K + MM - 1) / MM) * MM, Cp = ((C + BC - 1) / BC) * BC;
+    const int Kp = ((K + MM - 1) / MM) * MM, C8 = (C + BC - 1) / BC * (BC / 8);
     const long idx = (long)blockIdx.x * 256 + threadIdx.x;
-    if (idx >= (long)Cp * Kp) return;
-    const int c = (int)(idx / Kp), k = (int)(idx - (long)c * Kp);
-    float g[9], t[16];
-    if (c < C && k < K) {
-        const uint16_t* wc = w + (size_t)c * 9 * K + k;
+    if (idx >= (long)C8 * Kp) return;
+    const int c8 = (int)(idx / Kp), k = (int)(idx - (long)c8 * Kp);
+    uint32_t pk[16][4];
 #pragma unroll
-        for (int e = 0; e < 9; ++e) g[e] = to_f<DT>(wc[(size_t)e * K]);
-        ftf_4x4(g, t);
-    } else {
+    for (int cc = 0; cc < 8; cc += 2) {
+        float t[2][16];
 #pragma unroll
-        for (int e = 0; e < 16; ++e) t[e] = 0.f;
+        for (int h = 0; h < 2; ++h) {
+            const int c = c8 * 8 + cc + h;
+            if (c < C && k < K) {
+                float g[9];
+                const uint16_t* wc = w + (size_t)c * 9 * K + k;
+#pragma unroll
+                for (int e = 0; e < 9; ++e) g[e] = to_f<DT>(wc[(size_t)e * K]);
+                ftf_4x4(g, t[h]);
+            } else {
+#pragma unroll
+                for (int e = 0; e < 16; ++e) t[h][e] = 0.f;
+            }
+        }
+#pragma unroll
+        for (int xi = 0; xi < 16; ++xi) pk[xi][cc >> 1] = pack2<DT>(t[0][xi], t[1][xi]);
     }
-    const int cb = c / BC, cl = c % BC, kb = k / MM, m = k % MM;
+    const int cb = c8 / (BC / 8), ch = c8 % (BC / 8), kb = k / MM, m = k % MM;
     const int nkb = Kp / MM;
-    const size_t inner = size_t((m >> 3) * 128 + (cl >> 3) * 64 + (m & 7) * 8 + (cl & 7));
+    const size_t inner = size_t((m >> 3) * 128 + ch * 64 + (m & 7) * 8);
 #pragma unroll
     for (int xi = 0; xi < 16; ++xi) {
         const size_t base = (((size_t)cb * nkb + kb) * 16 + xi) * (MM * BC);
-        u[base + inner] = from_f<DT>(t[xi]);
+        *reinterpret_cast<uint4*>(u + base + inner) = make_uint4(pk[xi][0], pk[xi][1], pk[xi][2], pk[xi][3]);
     }
 }
 

@@ -626,8 +626,8 @@ wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int 
     const int planes = mode == WINO_TC_3XTF32 ? 2 : 1;
     const int mm = wino::tc::tc_mm(K, planes);
     const int64_t Kp = ((K + mm - 1) / mm) * mm;
-    const int64_t Cp = ((C + wino::tc::BC - 1) / wino::tc::BC) * wino::tc::BC;
-    const unsigned blocks = static_cast<unsigned>((Cp * Kp + 255) / 256);
+    const int64_t C4 = ((C + wino::tc::BC - 1) / wino::tc::BC) * (wino::tc::BC / 4);
+    const unsigned blocks = static_cast<unsigned>((C4 * Kp + 255) / 256);
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (planes == 1 && mm == 64) wino::tc::tc_filter_kernel<1, 64><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
     else if (planes == 1) wino::tc::tc_filter_kernel<1, 128><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
@@ -739,8 +739,8 @@ wino_status_t wino_filter_transform_half(const void* w_dev, void* u_h_dev, int C
     if (s != WINO_OK) return s;
     using namespace wino::tc16;
     const int mm = tc16_mm(K);
-    const int64_t Kp = ((K + mm - 1) / mm) * mm, Cp = ((C + BC - 1) / BC) * BC;
-    const unsigned blocks = static_cast<unsigned>((Cp * Kp + 255) / 256);
+    const int64_t Kp = ((K + mm - 1) / mm) * mm, C8 = ((C + BC - 1) / BC) * (BC / 8);
+    const unsigned blocks = static_cast<unsigned>((C8 * Kp + 255) / 256);
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     const uint16_t* w = static_cast<const uint16_t*>(w_dev);
     uint16_t* u = static_cast<uint16_t*>(u_h_dev);

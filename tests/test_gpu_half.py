@@ -74,6 +74,8 @@ EDGE = [
     (1, 1, 1, 1, 1), (1, 8, 8, 8, 8), (3, 7, 5, 5, 5), (2, 17, 130, 6, 10), (4, 20, 70, 13, 9),
     (40, 16, 16, 6, 6), (32, 16, 128, 4, 4), (32, 7, 68, 5, 9), (64, 33, 132, 3, 7), (96, 1, 4, 9, 2),
     (32, 16, 64, 40, 40), (8, 24, 136, 7, 7), (16, 40, 72, 11, 12), (16, 3, 8, 1, 17),
+    # 64-filter tiles (K <= 64) on every load path: TMA, per-tile boxes (N = 8), gather
+    (64, 20, 64, 10, 10), (8, 5, 40, 9, 6), (4, 16, 64, 6, 6), (96, 33, 17, 3, 5),
 ]
 
 
