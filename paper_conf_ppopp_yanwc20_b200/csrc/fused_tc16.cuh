@@ -418,7 +418,6 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                 if (NH == 1 && (gcb & 1) != g) continue;
                 const int xs = gcb % X_SLOTS, vs = gcb & 1;
                 mbar_wait(&x_full[xs], (gcb / X_SLOTS) & 1);
-                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(2, gcb);
                 const uint32_t* xw = reinterpret_cast<const uint32_t*>(sx + xs * G::X_SLOT) + wbase;
                 uint32_t r[2][16];
 #pragma unroll
@@ -448,9 +447,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                 }
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&x_empty[xs]);  // the x slot can be refilled
-                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(3, gcb);
                 if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
-                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(6, gcb);
                 uint8_t* vdst = sv + vs * G::V_SLOT + voff0;
 #pragma unroll
                 for (int s = 0; s < 2; ++s)
@@ -462,7 +459,9 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&v_full[vs]);
-                if (tid == ITF_WARP0 * 32 + g * ITF_GROUP * 32) TC16_TRACE(7, gcb);
+#ifdef WINO_TC16_TRACE
+                if (lane == 0) TC16_TRACE(gw == 0 ? 2 : gw == 1 ? 3 : gw == 2 ? 6 : 7, gcb);  // v_full arrival per warp
+#endif
             }
         }
     } else {

@@ -21,7 +21,7 @@ L.wino_debug_tc16_trace.argtypes = [ctypes.c_void_p, ctypes.c_int]
 L.wino_debug_tc16_trace(ctypes.cast(buf, ctypes.c_void_p), NE * NC)
 ev = [[buf[e * NC + c] for c in range(NC)] for e in range(NE)]
 t0 = min(v for v in ev[0] if v)
-names = ["x_issue", "u_issue", "itf_xfull", "itf_comp", "mma_vfull", "mma_issue", "itf_vempty", "itf_vfull"]
+names = ["x_issue", "u_issue", "vfull_w0", "vfull_w1", "mma_vfull", "mma_issue", "vfull_w2", "vfull_w3"]
 print("gcb " + " ".join(f"{n:>10s}" for n in names))
 for c in range(min(NC, 64)):
     if not any(ev[e][c] for e in range(NE)):
