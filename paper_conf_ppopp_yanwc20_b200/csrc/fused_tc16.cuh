@@ -231,7 +231,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
             mbar_init(&u_empty[s], 1);
         }
         for (int s = 0; s < X_SLOTS; ++s) {
-            mbar_init(&x_full[s], 1);
+            mbar_init(&x_full[s], XM == 0 ? 32 : 1);  // gather: every lane releases its own stores
             mbar_init(&x_empty[s], G::ITF_PER_X);
         }
         for (int s = 0; s < V_SLOTS; ++s) {
@@ -326,8 +326,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                                 }
                             }
                         }
-                        __syncwarp();
-                        if (lane == 0) mbar_arrive(&x_full[xs]);
+                        mbar_arrive(&x_full[xs]);
                     }
                 }
             }
