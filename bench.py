@@ -235,7 +235,8 @@ def _config(args, layers, world):
         "inputs": f"uniform[-1,1) fp32, torch seeds x={SEED_X} w={SEED_W}",
         "l2": "flushed before every timed step by a 512 MiB write + 256 MiB read (outside the events)",
         "step": "per layer: FTF kernel + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
-                "its own FTF); the whole step replayed from one CUDA graph",
+                "its own FTF; fp32: wino_conv2d_f2x3_fwd_ws with a stream-K workspace, the planner picks regular / "
+                "split-C / stream-K + fixup per layer); the whole step replayed from one CUDA graph",
     }
 
 
@@ -316,7 +317,8 @@ def main():
         elif nonfused:
             launches = sum(3 for d in per if d["n"] > 0)  # FTF, ITF, OTF (the GEMMs are cuBLAS kernels)
         else:
-            vid = {"fp32": 0, "tf32": 1, "3xtf32": 2}[variant]
+            # fp32: with the stream-K workspace (variant 4 plans it), which may add a fixup launch
+            vid = {"fp32": 4, "tf32": 1, "3xtf32": 2}[variant]
             launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K,
                                          variant=vid).launches for d in per if d["n"] > 0)
         for d in per:
@@ -358,6 +360,10 @@ def main():
                 wino.filter_transform_kcrs(d["w_kcrs"], out=d["u"])
             else:
                 d["u"] = torch.empty((d["cfg"].C, 4, 4, d["cfg"].K), dtype=torch.float32, device=dev)
+                c = d["cfg"]
+                # device workspace of the stream-K plan (wino_conv2d_f2x3_fwd_ws; the planner decides)
+                d["ws_sk"] = torch.empty(max(wino.conv_workspace_bytes(max(d["n"], 1), c.C, c.H, c.W, c.K), 16),
+                                         dtype=torch.uint8, device=dev)
                 if rank == 0:
                     wino.filter_transform(d["w"], out=d["u"])
                 if world > 1:
@@ -389,7 +395,7 @@ def main():
                 elif nonfused:
                     wino.conv2d_nonfused(d["x"], d["u"], d["ws_nf"], out=d["y"])
                 else:
-                    wino.conv2d(d["x"], d["u"], out=d["y"])
+                    wino.conv2d(d["x"], d["u"], out=d["y"], ws=d["ws_sk"])
 
         side = torch.cuda.Stream(dev)
 

@@ -178,6 +178,31 @@ wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_d
                                             void* ws_dev, size_t ws_bytes, wino_stream_t stream);
 
 /*
+ * The fused FP32 convolution with a caller-provided device workspace, which lets the
+ * library run the warp-specialised kernel in stream-K mode: the tiles x channel-block
+ * iteration space is cut into one equal contiguous range per SM (Alg. 1's loop over C,
+ * L351-355, split across CTAs at range boundaries), partial tiles are written to the
+ * workspace and a second small kernel adds each cut tile's partial outputs (Eq. 8 is
+ * linear) in a fixed order -- deterministic, no atomics.  It removes the wave
+ * quantisation of tiles over SMs (e.g. 392 tiles on 148 SMs) and keeps small per-rank
+ * batches (batch sharding) on every SM.
+ *   ws_dev / ws_bytes : >= wino_conv_workspace_bytes(N,C,H,W,K) bytes (SM count x 64 KiB;
+ *                       the current device's SM count, 148 when no device is current),
+ *                       16-byte aligned, not overlapping x, u or y; may be NULL / 0 when
+ *                       sk = 1.  Contents need no initialisation and are clobbered.
+ *   sk                : 0 = the planner's choice (stream-K where its estimate beats the
+ *                       regular / split-C plans and the workspace suffices), 1 = never,
+ *                       2 = always when the warp-specialised kernel applies
+ *                       (N % 32 == 0 or N in {4, 8, 16}, K % 4 == 0; else the regular
+ *                       plan).  sk = 2 with a short workspace -> WINO_ERR_INVALID_ARG.
+ * Arguments and errors otherwise as wino_conv2d_f2x3_fwd.
+ */
+size_t wino_conv_workspace_bytes(int N, int C, int H, int W, int K);
+wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, float* y_dev,
+                                      int N, int C, int H, int W, int K, int pad, int stride,
+                                      int sk, void* ws_dev, size_t ws_bytes, wino_stream_t stream);
+
+/*
  * Tensor-core variant (a5' of SURVEY 8(a)): the Winograd-domain GEMM (Eq. 7)
  * on the 5th-generation tensor cores (tcgen05.mma kind::tf32, accumulators in
  * TMEM).  The paper has no tensor-core path ("the data layout needs a
@@ -288,7 +313,8 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
  */
 typedef struct {
     int variant;        /* 0 = FP32 FFMA fused kernel, 1 / 2 = tcgen05 TF32 / 3xTF32, */
-                        /* 3 = tcgen05 kind::f16 (FP16 / BF16, NEXT row N4)           */
+                        /* 3 = tcgen05 kind::f16 (FP16 / BF16, NEXT row N4),          */
+                        /* 4 = FP32 with a stream-K workspace (wino_conv2d_f2x3_fwd_ws, sk = 0) */
     int bk, bn, bc;     /* filters, tiles and channels per CTA step (Sec. 3.3)      */
     int load_x, load_u; /* how x / u reach shared memory: 0 = cp.async 4 B,         */
                         /* 1 = cp.async 16 B, 2 = TMA tiled box (cp.async.bulk.tensor) */
@@ -297,6 +323,7 @@ typedef struct {
     int threads;        /* threads per CTA                                          */
     int smem_bytes;     /* dynamic shared memory per CTA                            */
     int launches;       /* kernels launched by one wino_conv2d_f2x3_fwd* call       */
+    int stream_k;       /* 1: stream-K plan (variant 4 only)                        */
 } wino_plan_t;
 
 wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_plan_t* plan);

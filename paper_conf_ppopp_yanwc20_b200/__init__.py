@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half",
+    "conv2d_half", "conv_workspace_bytes",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -56,7 +56,7 @@ class _Plan(ctypes.Structure):
     _fields_ = [("variant", ctypes.c_int), ("bk", ctypes.c_int), ("bn", ctypes.c_int),
                 ("bc", ctypes.c_int), ("load_x", ctypes.c_int), ("load_u", ctypes.c_int),
                 ("split_c", ctypes.c_int), ("ctas", ctypes.c_int64), ("threads", ctypes.c_int),
-                ("smem_bytes", ctypes.c_int), ("launches", ctypes.c_int)]
+                ("smem_bytes", ctypes.c_int), ("launches", ctypes.c_int), ("stream_k", ctypes.c_int)]
 
 
 class _HostLayer(ctypes.Structure):
@@ -78,6 +78,7 @@ class Plan:
     threads: int
     smem_bytes: int
     launches: int
+    stream_k: int = 0
 
 
 def lib() -> ctypes.CDLL:
@@ -143,6 +144,11 @@ def lib() -> ctypes.CDLL:
         L.wino_filter_transform_half.argtypes = [vp, vp, i, i, i, vp]
         L.wino_conv2d_f2x3_fwd_half.restype = i
         L.wino_conv2d_f2x3_fwd_half.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_ws") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_conv_workspace_bytes.restype = st
+        L.wino_conv_workspace_bytes.argtypes = [i, i, i, i, i]
+        L.wino_conv2d_f2x3_fwd_ws.restype = i
+        L.wino_conv2d_f2x3_fwd_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp, st, vp]
     L.wino_plan.restype = i
     L.wino_plan.argtypes = [i, i, i, i, i, i, ctypes.POINTER(_Plan)]
     _lib = L
@@ -331,12 +337,19 @@ def conv2d_half(x: torch.Tensor, u_h: HalfFilter, out: torch.Tensor | None = Non
     return out
 
 
+def conv_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
+    """Device workspace that lets ``conv2d`` use the stream-K plan (wino_conv_workspace_bytes)."""
+    return int(lib().wino_conv_workspace_bytes(N, C, H, W, K))
+
+
 def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, variant: str = "fp32",
-           stream=None, split_c: int = 0) -> torch.Tensor:
+           stream=None, split_c: int = 0, ws: torch.Tensor | None = None, stream_k: str = "auto") -> torch.Tensor:
     """Fused Winograd forward conv on FP32 CUDA cores, pad 1 stride 1:
     x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N).  split_c: 0 = the library's choice, else
     force the split-C factor (1, 2, 4, 8) of the warp-specialised kernel
-    (``wino_conv2d_f2x3_fwd_split``)."""
+    (``wino_conv2d_f2x3_fwd_split``).  ws: a device workspace of >= conv_workspace_bytes
+    bytes enables the stream-K plan (``wino_conv2d_f2x3_fwd_ws``); stream_k = "auto"
+    (planner's choice), "off" or "on"."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u, "u", 4)
     C, H, W, N = x.shape
@@ -355,7 +368,15 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
     with torch.cuda.device(x.device):
         if variant != "fp32":
             raise ValueError(f"conv2d runs the FP32 kernel; use conv2d_tc for {variant!r}")
-        if split_c:
+        if ws is not None or stream_k == "on":
+            if split_c:
+                raise ValueError("split_c and a stream-K workspace are exclusive")
+            mode = {"auto": 0, "off": 1, "on": 2}[stream_k]
+            wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
+            if ws is not None and not ws.is_cuda:
+                raise ValueError("ws must be a CUDA tensor")
+            _check(lib().wino_conv2d_f2x3_fwd_ws(*args, mode, wp, wb, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_ws")
+        elif split_c:
             _check(lib().wino_conv2d_f2x3_fwd_split(*args, int(split_c), _stream_ptr(stream)),
                    "wino_conv2d_f2x3_fwd_split")
         else:

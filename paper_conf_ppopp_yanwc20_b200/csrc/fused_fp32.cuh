@@ -76,6 +76,12 @@ struct __align__(64) Params {
     long long xs_c, xs_n, xs_h, xs_w, ys_k, ys_n, ys_h, ys_w;
     int tfast;
     int T;  // ceil(H/2) * ceil(W/2)
+    // WS kernel, stream-K mode: the (tile, channel block) iteration space of sk_total units is
+    // cut into gridDim.x equal contiguous ranges; partial tiles go to sk_ws (2 slots of
+    // 64 k x 4 outputs x 32 nu per CTA) and are summed by sk_fixup_kernel.
+    float* __restrict__ sk_ws;
+    long long sk_total;  // tiles * num_it  (< 2^31)
+    int sk_q, sk_r;      // sk_total = gridDim * sk_q + sk_r: CTA b's range starts at b*q + min(b, r)
 };
 
 // XPW = Winograd elements xi per warp: 2 -> 8 warps / 256 threads (the paper's

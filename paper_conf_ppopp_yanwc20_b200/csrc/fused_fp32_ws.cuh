@@ -125,9 +125,16 @@ __device__ __forceinline__ void itf_loop(float* smem, float* vs, uint64_t* full,
             }
         }
 }
+// Stream-K (SK = true): CTA b of G takes units [b*total/G, (b+1)*total/G) of the flattened
+// (tile, channel block) space, unit = tile * NIT + g.  A tile is cut into segments at CTA
+// boundaries; a segment covering the whole tile stores y, a partial one stores its partial OTF
+// outputs (Eq. 8 is linear) in slot 2b (the CTA's first segment) or 2b+1 (its last) of sk_ws,
+// and sk_fixup_kernel adds the segments of each cut tile in CTA order (deterministic).
+// (the first total % G CTAs get one unit more; no division on the device)
+__host__ __device__ __forceinline__ int sk_start(const Params& p, int b) { return b * p.sk_q + min(b, p.sk_r); }
 // BOX32: N % 32 == 0 (one x box per stage, compile-time ITF strides); else N | 32
 // (32/N boxes, runtime strides -- costs the 88-register ITF warps one spill).
-template <bool SPLIT, bool BOX32>
+template <bool SPLIT, bool BOX32, bool SK = false>
 __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_constant__ Params p, int num_tiles) {
     using SM = Smem<SPLIT>;
     constexpr int RR = SM::RR, ER_KROWS = SM::ER_KROWS;
@@ -187,7 +194,19 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             if (lane == 0) {
                 constexpr uint32_t kBytes = (US_FLOATS + XS_FLOATS) * 4;
                 int G = 0;  // global stage counter across tiles
-                for (int tile = WS_CID; tile < num_tiles; tile += WS_NCL) {
+                int su = SK ? sk_start(p, blockIdx.x) : 0;
+                const int su_end = SK ? sk_start(p, blockIdx.x + 1) : 0;
+                for (int tile = SK ? 0 : WS_CID;;) {
+                    int g_lo = it_lo, g_hi = it_hi;
+                    if constexpr (SK) {
+                        if (su >= su_end) break;
+                        tile = su / p.num_it;
+                        g_lo = su - tile * p.num_it;
+                        g_hi = min(p.num_it, g_lo + (su_end - su));
+                        su += g_hi - g_lo;
+                    } else if (tile >= num_tiles) {
+                        break;
+                    }
                     const int kb = tile % p.num_kb, nb = tile / p.num_kb;
                     const int k0 = kb * BK, nu0 = nb * BN;
                     // N % 32 == 0: the tile's 32 nu are 32 consecutive n of one image tile (one box);
@@ -195,7 +214,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                     const int t0 = nu0 / p.N;
                     const int n0 = nu0 - t0 * p.N;
                     const int nbox = BOX32 ? 1 : BN / p.xnb;
-                    for (int g = it_lo; g < it_hi; ++g, ++G) {
+                    for (int g = g_lo; g < g_hi; ++g, ++G) {
                         const int slot = G % S;
                         if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
                         float* us = smem + slot * STAGE_FLOATS;
@@ -214,6 +233,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                                             2 * tw - 1, 2 * th - 1);
                         }
                     }
+                    if constexpr (!SK) tile += WS_NCL;
                 }
             }
             return;
@@ -242,7 +262,11 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             xoff = m >> 8;
             xpos = BC * p.xnb;
         }
-        if (BOX32)
+        if (SK)  // one run of this CTA's stages (the ITF does not depend on the tile)
+            itf_loop(smem, vs, full, empty, vfull, vempty, xoff, xpos, c * BN + n4,
+                     sk_start(p, blockIdx.x + 1) - sk_start(p, blockIdx.x),
+                     0, 1, 1, lane);
+        else if (BOX32)
             itf_loop(smem, vs, full, empty, vfull, vempty, xoff, xpos, c * BN + n4, NIT, WS_CID, num_tiles, WS_NCL,
                      lane);
         else
@@ -274,7 +298,26 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
     };
 
     int G = 0;
-    for (int tile = WS_CID; tile < num_tiles; tile += WS_NCL) {
+    int su = SK ? sk_start(p, blockIdx.x) : 0;
+    for (int tile = SK ? 0 : WS_CID;; tile += SK ? 0 : WS_NCL) {
+        int nst = NIT;     // channel blocks of this tile handled here
+        int sk_slot = -1;  // stream-K partial tile -> workspace slot 2b (the CTA's first segment) or
+                           // 2b + 1 (its last); whole tile -> y (-1)
+        if constexpr (SK) {
+            // (su is kept live across the main loop on purpose: re-deriving it from G changes
+            // ptxas' accumulator assignment, 1.20 -> 1.55 register reads per FFMA, sass_bank.py)
+            const int su_end = sk_start(p, blockIdx.x + 1);
+            if (su >= su_end) break;
+            tile = su / p.num_it;
+            const int g_lo = su - tile * p.num_it;
+            nst = min(p.num_it - g_lo, su_end - su);
+            if (nst != p.num_it)
+                sk_slot = 2 * static_cast<int>(blockIdx.x) +
+                          (su == sk_start(p, blockIdx.x) ? 0 : 1);
+            su += nst;
+        } else if (tile >= num_tiles) {
+            break;
+        }
         const int kb = tile % p.num_kb, nb = tile / p.num_kb;
         const int k0 = kb * BK, nu0 = nb * BN;
         float acc[2][8][8];
@@ -300,7 +343,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
         const int Ttr = (tile - WS_CID) / WS_NCL;
         if (tid == 0) WS_TR(0, Ttr);
 #endif
-        for (int g = 0; g < NIT; ++g, ++G) {
+        for (int g = 0; g < nst; ++g, ++G) {
             const int slot = G % S, vb = G % SV;
             mbar_wait(&full[slot], (G / S) & 1);
             mbar_wait(&vfull[vb], (G / SV) & 1);
@@ -374,6 +417,14 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
 #pragma unroll
                             for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + r) * ER_LD + (lane ^ 1)];
                             otf_2x2(m, o);
+                            if (SK && sk_slot >= 0) {
+                                // partial tile: [slot][kl][output][nu] for sk_fixup_kernel
+                                float* wk = p.sk_ws + ((size_t)sk_slot * BK + kl) * (4 * BN) + lane;
+                                wk[0] = o[0];
+                                wk[BN] = o[1];
+                                wk[2 * BN] = o[2];
+                                wk[3 * BN] = o[3];
+                            } else {
                             float* yk = p.y + (size_t)k * HWN + base;
 #ifdef WS_EXP_NOSTG
                             if (o[0] == 1234.5f && o[1] == o[2] && o[3] == 7.f) yk[0] = o[0];
@@ -383,6 +434,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                             if (okr) yk[dW] = o[2];
                             if (okr && okc) yk[dW + p.N] = o[3];
 #endif
+                            }
                         }
                     }
                 }
@@ -484,5 +536,68 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
 
 #undef WS_CID
 #undef WS_NCL
+
+// Stream-K fixup: blocks 8i .. 8i+7 handle the tile cut by the range boundary of CTA b = i + 1
+// (when it is the first boundary inside that tile), 8 filters each: y = sum of the tile's
+// segments' partial outputs, added in CTA order (deterministic).  256 threads = 8 filters x
+// 32 nu; each thread issues the loads of 8 segments before adding them (latency-bound otherwise).
+__global__ void __launch_bounds__(256) sk_fixup_kernel(const __grid_constant__ Params p, int G) {
+    __shared__ int slots[256];  // workspace slots of the tile's segments, CTA order (G <= 256)
+    __shared__ int nseg;
+    const int b = blockIdx.x / 8 + 1, kr = blockIdx.x % 8;
+    const int ub = sk_start(p, b);
+    const int tile = ub / p.num_it;
+    const int t0 = tile * p.num_it, t1 = t0 + p.num_it;
+    if (ub == t0 || sk_start(p, b - 1) > t0) return;  // no cut, or an earlier boundary owns it
+    if (threadIdx.x == 0) {
+        int b0 = b - 1;  // the CTA whose range holds unit t0
+        while (b0 > 0 && sk_start(p, b0) > t0) --b0;
+        int ns = 0;
+        int c0 = sk_start(p, b0);
+        for (int c = b0; c < G && c0 < t1 && ns < 256; ++c) {
+            const int c1 = sk_start(p, c + 1);
+            if (c1 > c0) slots[ns++] = 2 * c + (c0 < t0 ? 1 : 0);  // first segment of CTA c -> 2c, else its last
+            c0 = c1;
+        }
+        nseg = ns;
+    }
+    __syncthreads();
+    const int kb = tile % p.num_kb, nb = tile / p.num_kb;
+    const int lane = threadIdx.x & 31;
+    const int kl = kr * 8 + (threadIdx.x >> 5), k = kb * BK + kl;
+    const int nu = nb * BN + lane;
+    if (nu >= p.NV || k >= p.K) return;
+    const int t = nu / p.N, n = nu - t * p.N;
+    const int th = t / p.TW, tw = t - th * p.TW;
+    const int i0 = 2 * th, j0 = 2 * tw;
+    const bool okr = i0 + 1 < p.H, okc = j0 + 1 < p.W;
+    const size_t HWN = (size_t)p.H * p.W * p.N, dW = (size_t)p.W * p.N;
+    const float* wbase = p.sk_ws + (size_t)kl * (4 * BN) + lane;
+    constexpr size_t SLOT = (size_t)BK * 4 * BN;
+    const int ns = nseg;
+    float o[4] = {0.f, 0.f, 0.f, 0.f};
+    for (int i0s = 0; i0s < ns; i0s += 8) {
+        float v[8][4];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            if (i0s + i < ns) {
+                const float* wk = wbase + (size_t)slots[i0s + i] * SLOT;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) v[i][q] = wk[q * BN];
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+            if (i0s + i < ns) {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) o[q] += v[i][q];
+            }
+    }
+    float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+    yk[0] = o[0];
+    if (okc) yk[p.N] = o[1];
+    if (okr) yk[dW] = o[2];
+    if (okr && okc) yk[dW + p.N] = o[3];
+}
 }  // namespace fp32ws
 }  // namespace wino

@@ -8,6 +8,7 @@
 #include <cudaTypedefs.h>
 
 #include <atomic>
+#include <cmath>
 #include <cstdint>
 #include <cstring>
 #include <mutex>
@@ -120,16 +121,23 @@ struct Fp32Plan {
     int64_t tiles;       // (k, nu) tiles
     int64_t grid;        // CTAs launched
     int threads, smem;
+    bool sk = false;     // stream-K WS kernel (+ fixup kernel); needs the workspace
 };
 
+// Stream-K workspace: 2 partial-tile slots (64 k x 4 outputs x 32 nu fp32) per CTA.
+size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * wino::fp32::BK * 4 * wino::fp32::BN * sizeof(float); }
+
 int log2_small(int s) { return s == 1 ? 0 : s == 2 ? 1 : s == 4 ? 2 : 3; }
+// planner cost of the stream-K fixup launch, in channel-block times (~1 us each)
+constexpr double kSkFixupBlocks = 2.0;
 
 // Shape -> kernel / tiling / split-C.  force_split: 0 = choose, else 1, 2, 4 or 8.
 // The split model: a cluster of S CTAs shares a tile, each CTA runs ceil(NIT/S)
 // channel blocks plus an epilogue worth ~E channel blocks (E measured: the
 // DSMEM-reduced epilogue of the split kernel costs about one block more than the
 // plain one); time ~ waves(S) * (ceil(NIT/S) + E(S)), waves = ceil(tiles/clusters).
-Fp32Plan plan_fp32(int N, int C, int H, int W, int K, bool u_tma_ok, int dev, int force_split) {
+// sk_mode: 0 = no stream-K (no workspace), 1 = planner's choice, 2 = force stream-K.
+Fp32Plan plan_fp32(int N, int C, int H, int W, int K, bool u_tma_ok, int dev, int force_split, int sk_mode = 0) {
     using namespace wino::fp32;
     Fp32Plan p;
     p.load_x = (N % 32 == 0) ? LD_TMA : (N % 4 == 0 ? LD_CP16B : LD_CP4B);
@@ -151,7 +159,11 @@ Fp32Plan plan_fp32(int N, int C, int H, int W, int K, bool u_tma_ok, int dev, in
         return p;
     }
     const int nit = (C + BC - 1) / BC;
-    if (force_split > 0) {
+    const int sms = cluster_slots(1, dev);
+    if (double(p.tiles) * nit >= 2147483647.0) sk_mode = 0;  // stream-K unit indices are 32-bit
+    if (sk_mode == 2 && force_split <= 1) {
+        p.sk = true;
+    } else if (force_split > 0) {
         p.split = force_split;
     } else {
         double best = 0;
@@ -166,6 +178,23 @@ Fp32Plan plan_fp32(int N, int C, int H, int W, int K, bool u_tma_ok, int dev, in
                 p.split = s;
             }
         }
+        if (sk_mode == 1) {
+            // stream-K: equal shares of the tiles x channel blocks units on every SM, a tile
+            // epilogue per tile plus up to two partial ones per CTA, and the fixup launch
+            const double units = double(p.tiles) * nit;
+            const double est = std::ceil(units / sms) + (double(p.tiles) / sms + 1.0) * 0.5 + kSkFixupBlocks;
+            if (est < best * 0.97 && units >= 2.0 * sms) {
+                p.sk = true;
+                p.split = 1;
+            }
+        }
+    }
+    if (p.sk) {
+        p.split = 1;
+        p.grid = sms < 256 ? sms : 256;  // sk_fixup_kernel lists <= 256 segments per tile
+        p.threads = wino::fp32ws::NT;
+        p.smem = wino::fp32ws::Smem<false>::bytes;
+        return p;
     }
     const int64_t cl = cluster_slots(p.split, dev);
     p.grid = (p.tiles < cl ? p.tiles : cl) * p.split;
@@ -272,16 +301,21 @@ int cluster_slots(int split, int dev) {
 }
 
 std::atomic<uint64_t> g_attr_ws_k[2][2];
+std::atomic<uint64_t> g_attr_ws_sk[2];
 }  // namespace
 
 // FP32 fused conv on validated arguments; u may be a K-slice of a wider (C,4,4,ldu) array.
 // force_split: 0 = planner's choice, else the split-C factor (1, 2, 4, 8).
 // nchw: x (N,C,H,W) / y (N,K,H,W) instead of the paper's CHWN / KHWN (generic kernel).
+// sk_mode / ws: stream-K (0 = off, 1 = planner's choice, 2 = forced) when ws holds
+// sk_workspace_bytes(SM count) bytes.
 wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, float* y_dev, int N, int C, int H,
-                              int W, int K, int dev, cudaStream_t st, int force_split = 0, bool nchw = false) {
+                              int W, int K, int dev, cudaStream_t st, int force_split = 0, bool nchw = false,
+                              int sk_mode = 0, void* ws = nullptr, size_t ws_bytes = 0) {
     using namespace wino::fp32;
     const bool u_tma_ok = ldu % 4 == 0 && aligned16(u_dev);
-    Fp32Plan pl = plan_fp32(N, C, H, W, K, u_tma_ok, dev, force_split);
+    const bool ws_ok = ws != nullptr && aligned16(ws) && ws_bytes >= sk_workspace_bytes(sm_count(dev));
+    Fp32Plan pl = plan_fp32(N, C, H, W, K, u_tma_ok, dev, force_split, ws_ok && !nchw ? sk_mode : 0);
     if (nchw) {  // strided gathers (Sec. 8.4: "offsets ... need to be recomputed")
         pl.ws = false;
         pl.split = 1;
@@ -346,6 +380,23 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
     const int64_t g = pl.tiles;
     const int sm = pl.smem;
     const bool box32 = prm.xnb == BN;
+    if (pl.ws && pl.sk) {  // stream-K: equal unit ranges on every SM + fixup of the cut tiles
+        prm.sk_ws = static_cast<float*>(ws);
+        prm.sk_total = pl.tiles * prm.num_it;  // < 2^31 (planner)
+        prm.sk_q = static_cast<int>(prm.sk_total / pl.grid);
+        prm.sk_r = static_cast<int>(prm.sk_total % pl.grid);
+        auto kern = box32 ? wino::fp32ws::fused_fp32_ws_kernel<false, true, true>
+                          : wino::fp32ws::fused_fp32_ws_kernel<false, false, true>;
+        wino_status_t s = ensure_smem_attr(kern, dev, sm, g_attr_ws_sk[box32]);
+        if (s != WINO_OK) return s;
+        kern<<<dim3(static_cast<unsigned>(pl.grid)), wino::fp32ws::NT, sm, st>>>(prm, static_cast<int>(g));
+        cudaError_t e = cudaGetLastError();
+        if (e == cudaSuccess && pl.grid > 1)
+            wino::fp32ws::sk_fixup_kernel<<<dim3(static_cast<unsigned>(8 * (pl.grid - 1))), 256, 0, st>>>(
+                prm, static_cast<int>(pl.grid));
+        if (e == cudaSuccess) e = cudaGetLastError();
+        return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+    }
     if (pl.ws && pl.split == 1) {  // warp-specialised persistent kernel, one CTA per SM
         auto kern = box32 ? wino::fp32ws::fused_fp32_ws_kernel<false, true>
                           : wino::fp32ws::fused_fp32_ws_kernel<false, false>;
@@ -519,25 +570,26 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->launches = 1;
         return WINO_OK;
     }
-    if (variant != 0) return WINO_ERR_UNSUPPORTED;
+    if (variant != 0 && variant != 4) return WINO_ERR_UNSUPPORTED;
     int dev = -1;  // host-only planning unless an sm_100 device is current
     {
         int d;
         if (check_device(&d) == WINO_OK) dev = d;
         else cudaGetLastError();
     }
-    Fp32Plan p = plan_fp32(N, C, H, W, K, true, dev, 0);
-    plan->variant = 0;
+    Fp32Plan p = plan_fp32(N, C, H, W, K, true, dev, 0, variant == 4 ? 1 : 0);
+    plan->variant = variant;
     plan->bk = wino::fp32::BK;
     plan->bn = wino::fp32::BN;
     plan->bc = wino::fp32::BC;
     plan->load_x = p.ws ? 2 : p.load_x;
     plan->load_u = p.load_u;
     plan->split_c = p.split;
-    plan->ctas = p.tiles * p.split;
+    plan->ctas = p.sk ? p.grid : p.tiles * p.split;
     plan->threads = p.threads;
     plan->smem_bytes = p.smem;
-    plan->launches = 1;
+    plan->launches = p.sk ? 2 : 1;
+    plan->stream_k = p.sk ? 1 : 0;
     return WINO_OK;
 }
 
@@ -571,6 +623,37 @@ wino_status_t wino_conv2d_f2x3_fwd_split(const float* x_dev, const float* u_dev,
     if ((s = check_device(&dev)) != WINO_OK) return s;
     return launch_fwd_fp32(x_dev, u_dev, K, y_dev, N, C, H, W, K, dev, reinterpret_cast<cudaStream_t>(stream),
                            split_c);
+}
+
+size_t wino_conv_workspace_bytes(int N, int C, int H, int W, int K) {
+    if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
+    int dev = -1, sms = 148;  // host-only query: B200
+    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+    else cudaGetLastError();
+    return sk_workspace_bytes(sms);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H,
+                                      int W, int K, int pad, int stride, int sk, void* ws_dev, size_t ws_bytes,
+                                      wino_stream_t stream) {
+    if (sk < 0 || sk > 2) return WINO_ERR_INVALID_ARG;
+    if (!x_dev || !u_dev || !y_dev || (ws_bytes > 0 && !ws_dev)) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (!aligned16(x_dev) || !aligned16(u_dev) || !aligned16(y_dev) || (ws_dev && !aligned16(ws_dev)))
+        return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t yb = size_t(K) * hwn * 4, xb = size_t(C) * hwn * 4, ub = size_t(16) * C * K * 4;
+    if (overlaps(y_dev, yb, x_dev, xb) || overlaps(y_dev, yb, u_dev, ub)) return WINO_ERR_INVALID_ARG;
+    if (ws_dev && (overlaps(ws_dev, ws_bytes, x_dev, xb) || overlaps(ws_dev, ws_bytes, u_dev, ub) ||
+                   overlaps(ws_dev, ws_bytes, y_dev, yb)))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    if (sk == 2 && ws_bytes < sk_workspace_bytes(sm_count(dev))) return WINO_ERR_INVALID_ARG;
+    const int mode = sk == 0 ? 1 : (sk == 1 ? 0 : 2);  // API 0 auto / 1 off / 2 force -> planner 1 / 0 / 2
+    return launch_fwd_fp32(x_dev, u_dev, K, y_dev, N, C, H, W, K, dev, reinterpret_cast<cudaStream_t>(stream), 0,
+                           false, mode, ws_dev, ws_bytes);
 }
 
 wino_status_t wino_filter_transform_kcrs(const float* w_kcrs_dev, float* u_dev, int C, int K, wino_stream_t stream) {

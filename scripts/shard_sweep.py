@@ -43,7 +43,8 @@ def time_graph(fn, reps, flush):
         if i >= 2:
             ts.append(a.elapsed_time(b))
     ts.sort()
-    return ts[len(ts) // 2]
+    ts = ts[: max(1, len(ts) - len(ts) // 5)]  # drop the slowest fifth, average the rest
+    return sum(ts) / len(ts)  # (event timestamps are ~2 us granular: a mean resolves more)
 
 
 def main():
@@ -53,6 +54,8 @@ def main():
     ap.add_argument("--layers", default="conv5_x,conv4_x,conv3_x,conv2_x")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--split", type=int, default=0, help="force split_c (fp32 only; 0 = planner)")
+    ap.add_argument("--sk", default="none", choices=["none", "auto", "on", "off"],
+                    help="fp32: pass a stream-K workspace (wino_conv2d_f2x3_fwd_ws) with this mode")
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     dev = torch.device("cuda:0")
@@ -71,7 +74,11 @@ def main():
                 y = torch.empty((cfg.K, cfg.H, cfg.W, hi - lo), device=dev)
                 if var == "fp32":
                     u = wino.filter_transform(wd)
-                    if a.split:
+                    if a.sk != "none":
+                        wsb = torch.empty(wino.conv_workspace_bytes(hi - lo, cfg.C, cfg.H, cfg.W, cfg.K),
+                                          dtype=torch.uint8, device=dev)
+                        conv = lambda: wino.conv2d(xs, u, out=y, ws=wsb, stream_k=a.sk)  # noqa: E731
+                    elif a.split:
                         conv = lambda: wino.conv2d(xs, u, out=y, split_c=a.split)  # noqa: E731
                     else:
                         conv = lambda: wino.conv2d(xs, u, out=y)  # noqa: E731

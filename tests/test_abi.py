@@ -179,3 +179,15 @@ def test_product_package_never_imports_oracle():
                 src = open(os.path.join(dirpath, f), errors="ignore").read()
                 assert not re.search(r"^\s*(import|from)\s+oracle\b", src, re.M), f
                 assert "wino_oracle" not in src and "liboracle" not in src, f
+
+
+def test_stream_k_plan_and_workspace():
+    """Host-only planning (no device): the stream-K plan replaces the 2.65-wave conv4_x schedule
+    (392 tiles on 148 SMs) and is not taken for conv2_x (42.4 waves: nothing to gain)."""
+    c4, c2 = CONFIGS["conv4_x"], CONFIGS["conv2_x"]
+    p = wino.plan(c4.N, c4.C, c4.H, c4.W, c4.K, variant=4)
+    assert p.stream_k == 1 and p.launches == 2 and p.ctas == 148 and p.split_c == 1
+    assert wino.plan(c4.N, c4.C, c4.H, c4.W, c4.K).stream_k == 0  # no workspace -> regular plan
+    assert wino.plan(c2.N, c2.C, c2.H, c2.W, c2.K, variant=4).stream_k == 0
+    assert wino.conv_workspace_bytes(c4.N, c4.C, c4.H, c4.W, c4.K) == 148 * 2 * 64 * 4 * 32 * 4
+    assert wino.conv_workspace_bytes(0, 1, 1, 1, 1) == 0
