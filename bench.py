@@ -312,8 +312,11 @@ def main():
         nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
         nonfused = variant == "nonfused_fp32"  # NEXT row N3: ITF -> 16 cuBLAS SGEMMs -> OTF (Sec. 9)
         half = variant in ("fp16", "bf16")  # NEXT row N4: 16-bit x, w, y on tcgen05 kind::f16 (Sec. 8.3)
-        if f4 or nchw or half:
+        if f4 or half:
             launches = sum(2 for d in per if d["n"] > 0)
+        elif nchw:  # FTF, transpose, conv (+ stream-K fixup), transpose
+            launches = sum(3 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=4).launches
+                           for d in per if d["n"] > 0)
         elif nonfused:
             launches = sum(3 for d in per if d["n"] > 0)  # FTF, ITF, OTF (the GEMMs are cuBLAS kernels)
         else:
@@ -357,6 +360,10 @@ def main():
                 d["y_nchw"] = torch.empty((max(d["n"], 1), d["cfg"].K, d["cfg"].H, d["cfg"].W),
                                           dtype=torch.float32, device=dev)
                 d["u"] = torch.empty((d["cfg"].C, 4, 4, d["cfg"].K), dtype=torch.float32, device=dev)
+                c = d["cfg"]
+                # workspace of the transpose -> CHWN fused kernel -> transpose path (DESIGN 7.8)
+                d["ws_nchw"] = torch.empty(wino.nchw_workspace_bytes(max(d["n"], 1), c.C, c.H, c.W, c.K),
+                                           dtype=torch.uint8, device=dev)
                 wino.filter_transform_kcrs(d["w_kcrs"], out=d["u"])
             else:
                 d["u"] = torch.empty((d["cfg"].C, 4, 4, d["cfg"].K), dtype=torch.float32, device=dev)
@@ -389,7 +396,7 @@ def main():
                 elif tc:
                     wino.conv2d_tc(d["x"], d["u"], out=d["y"])
                 elif nchw:
-                    wino.conv2d_nchw(d["x_nchw"], d["u"], out=d["y_nchw"])
+                    wino.conv2d_nchw(d["x_nchw"], d["u"], out=d["y_nchw"], ws=d["ws_nchw"])
                 elif half:
                     wino.conv2d_half(d["x16"], d["u"], out=d["y16"])
                 elif nonfused:

@@ -172,6 +172,22 @@ wino_status_t wino_conv2d_f2x3_fwd_nchw(const float* x_nchw_dev, const float* u_
  * arguments, layouts and errors as wino_conv2d_f2x3_fwd; ws_bytes too small ->
  * WINO_ERR_INVALID_ARG; V or M of >= 2^31 elements -> WINO_ERR_TOO_LARGE.
  */
+/*
+ * NCHW with a device workspace: x is transposed to the paper's CHWN layout in the
+ * workspace, the fused FP32 convolution runs on it (warp-specialised / stream-K plans,
+ * as wino_conv2d_f2x3_fwd_ws), and y is transposed from KHWN to NKHW.  Two HBM-bound
+ * transposes (8 B per element each) buy the CHWN kernel's TMA path; faster than the
+ * strided gather of wino_conv2d_f2x3_fwd_nchw on every BASELINE layer.
+ *   ws_dev / ws_bytes : >= wino_nchw_workspace_bytes(N,C,H,W,K) bytes = |x| + |y| (fp32,
+ *                       each rounded up to 256 B) + wino_conv_workspace_bytes; 16-byte
+ *                       aligned, not overlapping x, u or y; clobbered.
+ * Arguments and errors as wino_conv2d_f2x3_fwd_nchw, plus WINO_ERR_INVALID_ARG for a
+ * NULL or short workspace.
+ */
+size_t wino_nchw_workspace_bytes(int N, int C, int H, int W, int K);
+wino_status_t wino_conv2d_f2x3_fwd_nchw_ws(const float* x_nchw_dev, const float* u_dev, float* y_nkhw_dev,
+                                           int N, int C, int H, int W, int K, int pad, int stride,
+                                           void* ws_dev, size_t ws_bytes, wino_stream_t stream);
 size_t wino_nonfused_workspace_bytes(int N, int C, int H, int W, int K);
 wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_dev, float* y_dev,
                                             int N, int C, int H, int W, int K, int pad, int stride,

@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half", "conv_workspace_bytes",
+    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -149,6 +149,11 @@ def lib() -> ctypes.CDLL:
         L.wino_conv_workspace_bytes.argtypes = [i, i, i, i, i]
         L.wino_conv2d_f2x3_fwd_ws.restype = i
         L.wino_conv2d_f2x3_fwd_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp, st, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_nchw_ws") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_nchw_workspace_bytes.restype = st
+        L.wino_nchw_workspace_bytes.argtypes = [i, i, i, i, i]
+        L.wino_conv2d_f2x3_fwd_nchw_ws.restype = i
+        L.wino_conv2d_f2x3_fwd_nchw_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp, st, vp]
     L.wino_plan.restype = i
     L.wino_plan.argtypes = [i, i, i, i, i, i, ctypes.POINTER(_Plan)]
     _lib = L
@@ -401,10 +406,17 @@ def filter_transform_kcrs(w_kcrs: torch.Tensor, out: torch.Tensor | None = None,
     return out
 
 
-def conv2d_nchw(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+def nchw_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
+    """Device workspace of the transpose + CHWN-kernel NCHW path (wino_nchw_workspace_bytes)."""
+    return int(lib().wino_nchw_workspace_bytes(N, C, H, W, K))
+
+
+def conv2d_nchw(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, stream=None,
+                ws: torch.Tensor | None = None) -> torch.Tensor:
     """NEXT row N2 (Sec. 8.4): fused Winograd conv on NCHW tensors, pad 1 stride 1:
     x (N,C,H,W), u (C,4,4,K) -> y (N,K,H,W) -- torch.nn.functional.conv2d(x, w, padding=1)
-    with u = filter_transform_kcrs(w)."""
+    with u = filter_transform_kcrs(w).  ws (>= nchw_workspace_bytes): transpose to CHWN, the
+    CHWN fused kernel, transpose back (wino_conv2d_f2x3_fwd_nchw_ws); else the strided kernel."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u, "u", 4)
     N, C, H, W = x.shape
@@ -419,9 +431,17 @@ def conv2d_nchw(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = Non
     if tuple(out.shape) != (N, K, H, W):
         raise ValueError("out must be (N,K,H,W)")
     with torch.cuda.device(x.device):
-        _check(lib().wino_conv2d_f2x3_fwd_nchw(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()),
-                                               ctypes.c_void_p(out.data_ptr()), N, C, H, W, K, 1, 1,
-                                               _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_nchw")
+        if ws is not None:
+            if not ws.is_cuda:
+                raise ValueError("ws must be a CUDA tensor")
+            _check(lib().wino_conv2d_f2x3_fwd_nchw_ws(
+                ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                N, C, H, W, K, 1, 1, ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size(),
+                _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_nchw_ws")
+        else:
+            _check(lib().wino_conv2d_f2x3_fwd_nchw(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()),
+                                                   ctypes.c_void_p(out.data_ptr()), N, C, H, W, K, 1, 1,
+                                                   _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_nchw")
     return out
 
 

@@ -21,6 +21,7 @@
 #include "fused_tc16.cuh"
 #include "fused_f4_fp32.cuh"
 #include "nonfused.cuh"
+#include "layout.cuh"
 
 #include <dlfcn.h>
 
@@ -687,6 +688,55 @@ wino_status_t wino_conv2d_f2x3_fwd_nchw(const float* x_nchw_dev, const float* u_
     if ((s = check_device(&dev)) != WINO_OK) return s;
     return launch_fwd_fp32(x_nchw_dev, u_dev, K, y_nkhw_dev, N, C, H, W, K, dev,
                            reinterpret_cast<cudaStream_t>(stream), 1, true);
+}
+
+extern "C++" {
+namespace {
+size_t round256(size_t b) { return (b + 255) & ~size_t(255); }
+cudaError_t transpose2d(const float* in, float* out, int R, long long S, cudaStream_t st) {
+    const dim3 grid(static_cast<unsigned>((S + wino::TR_TILE - 1) / wino::TR_TILE),
+                    static_cast<unsigned>((R + wino::TR_TILE - 1) / wino::TR_TILE));
+    wino::transpose2d_kernel<<<grid, dim3(wino::TR_TILE, wino::TR_ROWS), 0, st>>>(in, out, R, S);
+    return cudaGetLastError();
+}
+}  // namespace
+}  // extern "C++"
+
+size_t wino_nchw_workspace_bytes(int N, int C, int H, int W, int K) {
+    if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
+    const size_t hwn = size_t(H) * W * N;
+    return round256(size_t(C) * hwn * 4) + round256(size_t(K) * hwn * 4) + wino_conv_workspace_bytes(N, C, H, W, K);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_nchw_ws(const float* x_nchw_dev, const float* u_dev, float* y_nkhw_dev, int N,
+                                           int C, int H, int W, int K, int pad, int stride, void* ws_dev,
+                                           size_t ws_bytes, wino_stream_t stream) {
+    if (!x_nchw_dev || !u_dev || !y_nkhw_dev || !ws_dev) return WINO_ERR_INVALID_ARG;
+    wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
+    if (s != WINO_OK) return s;
+    if (!aligned16(x_nchw_dev) || !aligned16(u_dev) || !aligned16(y_nkhw_dev) || !aligned16(ws_dev))
+        return WINO_ERR_MISALIGNED;
+    const size_t hwn = size_t(H) * W * N;
+    const size_t xb = size_t(C) * hwn * 4, yb = size_t(K) * hwn * 4, ub = size_t(16) * C * K * 4;
+    if (overlaps(y_nkhw_dev, yb, x_nchw_dev, xb) || overlaps(y_nkhw_dev, yb, u_dev, ub)) return WINO_ERR_INVALID_ARG;
+    const size_t need = wino_nchw_workspace_bytes(N, C, H, W, K);
+    if (ws_bytes < need) return WINO_ERR_INVALID_ARG;
+    if (overlaps(ws_dev, ws_bytes, x_nchw_dev, xb) || overlaps(ws_dev, ws_bytes, u_dev, ub) ||
+        overlaps(ws_dev, ws_bytes, y_nkhw_dev, yb))
+        return WINO_ERR_INVALID_ARG;
+    int dev;
+    if ((s = check_device(&dev)) != WINO_OK) return s;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    float* xc = static_cast<float*>(ws_dev);                                          // (C,H,W,N)
+    float* yc = reinterpret_cast<float*>(static_cast<char*>(ws_dev) + round256(xb));  // (K,H,W,N)
+    void* wsk = static_cast<char*>(ws_dev) + round256(xb) + round256(yb);
+    const size_t wsk_bytes = ws_bytes - round256(xb) - round256(yb);
+    cudaError_t e = transpose2d(x_nchw_dev, xc, N, (long long)C * H * W, st);  // (N, CHW) -> (CHW, N)
+    if (e != cudaSuccess) return cuda_fail(e);
+    s = launch_fwd_fp32(xc, u_dev, K, yc, N, C, H, W, K, dev, st, 0, false, 1, wsk, wsk_bytes);
+    if (s != WINO_OK) return s;
+    e = transpose2d(yc, y_nkhw_dev, K * H * W, N, st);  // (KHW, N) -> (N, KHW)
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 
 size_t wino_filter_workspace_bytes_tc(int C, int K, wino_tc_mode_t mode) {

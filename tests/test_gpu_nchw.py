@@ -95,3 +95,50 @@ def test_nchw_matches_chwn_kernel(wino):
     torch.cuda.synchronize()
     d = (y_chwn.double() - y_nchw.double()).abs().max() / y_chwn.double().abs().max()
     assert float(d) <= FP32_TOL
+
+
+def _run_ws(wino, x, w):
+    u = wino.filter_transform_kcrs(_kcrs(w).to(DEV))
+    N, C, H, W = x.shape[3], x.shape[0], x.shape[1], x.shape[2]
+    ws = torch.empty(wino.nchw_workspace_bytes(N, C, H, W, w.shape[3]), dtype=torch.uint8, device=DEV)
+    y = wino.conv2d_nchw(_nchw(x).to(DEV), u, ws=ws)
+    torch.cuda.synchronize()
+    return y.cpu().permute(1, 2, 3, 0).contiguous()
+
+
+WS_SHAPES = SHAPES + [(64, 24, 40, 10, 9), (4, 40, 72, 7, 7), (16, 13, 68, 12, 5)]
+
+
+@pytest.mark.parametrize("shape", WS_SHAPES, ids=[str(s) for s in WS_SHAPES])
+def test_nchw_ws_small_int_bit_exact(wino, shape):
+    """Transpose -> CHWN fused kernel -> transpose (wino_conv2d_f2x3_fwd_nchw_ws)."""
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nchw", N, C, K, H, W), kind="smallint")
+    assert np.array_equal(_run_ws(wino, x, w).double().numpy(), oracle.direct_conv(x, w))
+
+
+@pytest.mark.parametrize("shape", WS_SHAPES, ids=[str(s) for s in WS_SHAPES])
+def test_nchw_ws_random(wino, shape):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nchw", N, C, K, H, W), kind="uniform", seed_x=41, seed_w=42)
+    y = _run_ws(wino, x, w)
+    assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= FP32_TOL
+
+
+@pytest.mark.parametrize("name", ["conv5_x", "conv4_x", "conv3_x", "conv2_x"])
+def test_nchw_ws_full_configs_sampled(wino, name):
+    cfg = CONFIGS[name]
+    x, w = make_inputs(cfg, kind="uniform")
+    y = _run_ws(wino, x, w)
+    idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 3000)
+    ref = oracle.direct_sample(x, w, idx)
+    ii = idx.numpy()
+    got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
+    assert float(np.max(np.abs(got - ref))) / float(np.max(np.abs(ref))) <= FP32_TOL
+
+
+def test_nchw_ws_short_workspace_rejected(wino):
+    x = torch.zeros((32, 8, 4, 4), device=DEV)
+    u = torch.zeros((8, 4, 4, 16), device=DEV)
+    with pytest.raises(wino.WinoError, match="INVALID_ARG"):
+        wino.conv2d_nchw(x, u, ws=torch.empty(1024, dtype=torch.uint8, device=DEV))
