@@ -257,6 +257,9 @@ def main():
     ap.add_argument("--cpu-baseline-s", type=float, default=3.0, help="oracle seconds per layer")
     ap.add_argument("--ref-step-s", type=float, default=4.0, help="oracle seconds per reference step")
     ap.add_argument("--out", default=None)
+    ap.add_argument("--shard-of", type=int, default=0,
+                    help="diagnostic: on one process / GPU, run rank 0's batch shard of a P-rank job (the per-rank "
+                         "step of --gpus P); not a bench line (the JSON is marked 'diagnostic')")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
@@ -283,7 +286,7 @@ def main():
     # ---- setup: inputs (host, full N, seeded) -> this rank's shard on device ----
     per = []
     for cfg in layers:
-        lo, hi = shard_range(cfg.N, rank, world)
+        lo, hi = shard_range(cfg.N, rank, world) if not args.shard_of else shard_range(cfg.N, 0, args.shard_of)
         x, w = make_inputs(cfg)
         xs = x[..., lo:hi].contiguous()
         n_loc = hi - lo
@@ -629,6 +632,11 @@ def main():
         fl, sec, sample = _oracle_sample(layers, args.cpu_baseline_s)
         res["cpu_baseline"] = {"value": fl / sec / 1e12, "unit": "TFLOPS", "cores": oracle.num_threads(),
                                "kind": "oracle", "sample": f"direct fp64 conv (Eq. 4) on {sample}; {sec:.1f} s"}
+    if args.shard_of:
+        res = {"diagnostic": f"rank 0 shard of a {args.shard_of}-rank job timed alone on one GPU", "ms_per_step": ms_step,
+               "projected_value_if_all_ranks_equal": total_eff / (ms_step * 1e-3) / 1e12,
+               "layers_us": {k: {"conv_us": v["conv_us"], "ftf_us": v["ftf_us"]} for k, v in layer_rep.items()},
+               "variants_ms_per_step": {k: v["ms_per_step"] for k, v in vrep.items()}}
     line = json.dumps(res)
     print(line, flush=True)
     if args.out:

@@ -201,7 +201,7 @@ struct __align__(64) Params {
 };
 
 // XM: 2 = one TMA box per nu-half (N % 32 == 0), 3 = 32/N boxes per half (N in {8, 16}),
-// 0 = generic gather by the x-producer warp
+// 0 = generic gather by the x-producer warp (a 16-bit box needs >= 8 images: 16 B rows)
 template <int DT, int XM, int MM>
 __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant__ Params p) {
     using G = Cfg<MM>;
@@ -307,23 +307,32 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                             }
                         }
                     } else {
-                        // generic gather: lane = local nu of each half, layout [h][c][pos][nu]
+                        // generic gather: lane = local nu of each half, layout [h][c][pos][nu]; the 16
+                        // window offsets are computed once per half, then 16 independent loads per channel
 #pragma unroll 1
                         for (int h = 0; h < NH; ++h) {
                             const int gnu = nu0 + h * BN + lane;
                             const bool glive = gnu < p.NV;
                             const int gt = glive ? gnu / p.N : 0, gn = glive ? gnu - gt * p.N : 0;
                             const int gh0 = 2 * (gt / p.TW) - 1, gw0 = 2 * (gt % p.TW) - 1;
+                            int off[16];
+#pragma unroll
+                            for (int pos = 0; pos < 16; ++pos) {
+                                const int hh = gh0 + (pos >> 2), ww = gw0 + (pos & 3);
+                                off[pos] = (glive && hh >= 0 && hh < p.H && ww >= 0 && ww < p.W)
+                                               ? (hh * p.W + ww) * p.N + gn
+                                               : -1;
+                            }
                             uint16_t* xd = reinterpret_cast<uint16_t*>(xdst + h * XS_BYTES) + lane;
+#pragma unroll 1
                             for (int cl = 0; cl < BC; ++cl) {
                                 const int c = cb * BC + cl;
-                                const uint16_t* xc = p.x + (size_t)c * HWN + gn;
-#pragma unroll 1
-                                for (int pos = 0; pos < 16; ++pos) {
-                                    const int hh = gh0 + (pos >> 2), ww = gw0 + (pos & 3);
-                                    const bool ok = glive && c < p.C && hh >= 0 && hh < p.H && ww >= 0 && ww < p.W;
-                                    xd[(cl * 16 + pos) * BN] = ok ? xc[((size_t)hh * p.W + ww) * p.N] : uint16_t(0);
-                                }
+                                const uint16_t* xc = p.x + (size_t)(c < p.C ? c : 0) * HWN;
+                                uint16_t v[16];
+#pragma unroll
+                                for (int pos = 0; pos < 16; ++pos) v[pos] = (c < p.C && off[pos] >= 0) ? xc[off[pos]] : 0;
+#pragma unroll
+                                for (int pos = 0; pos < 16; ++pos) xd[(cl * 16 + pos) * BN] = v[pos];
                             }
                         }
                         mbar_arrive(&x_full[xs]);

@@ -834,7 +834,7 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
 
 extern "C++" {
 namespace {
-std::atomic<uint64_t> g_attr_tc16[2][4][2];
+std::atomic<uint64_t> g_attr_tc16[2][4][2];  // [DT][XM 0..3][MM == 64]
 template <int DT, int XM, int MM>
 wino_status_t launch_tc16(const wino::tc16::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
     auto kern = wino::tc16::fused_tc16_kernel<DT, XM, MM>;
@@ -920,11 +920,11 @@ wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, 
     prm.num_cb = (C + BC - 1) / BC;
     prm.num_tiles = ((prm.NV + tn - 1) / tn) * prm.num_kb;
     const int xm = (N % 32 == 0) ? 2 : ((N == 8 || N == 16) ? 3 : 0);
+    const CUtensorMapDataType dt =
+        type == WINO_HALF_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
     if (xm >= 2) {
         const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
         const cuuint32_t box[4] = {cuuint32_t(xm == 2 ? BN : N), 4, 4, BC};
-        const CUtensorMapDataType dt =
-            type == WINO_HALF_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
         if (!encode_map(&prm.tmx, x_dev, 4, dims, box, nullptr, dt, 2)) return cuda_fail(cudaErrorInvalidValue);
     }
     const int sms = sm_count(dev);

@@ -76,6 +76,8 @@ EDGE = [
     (32, 16, 64, 40, 40), (8, 24, 136, 7, 7), (16, 40, 72, 11, 12), (16, 3, 8, 1, 17),
     # 64-filter tiles (K <= 64) on every load path: TMA, per-tile boxes (N = 8), gather
     (64, 20, 64, 10, 10), (8, 5, 40, 9, 6), (4, 16, 64, 6, 6), (96, 33, 17, 3, 5),
+    # N = 4 (batch shards): generic gather, odd and even W
+    (4, 24, 136, 7, 10), (4, 9, 40, 5, 2),
 ]
 
 
