@@ -315,8 +315,11 @@ def main():
         nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
         nonfused = variant == "nonfused_fp32"  # NEXT row N3: ITF -> 16 cuBLAS SGEMMs -> OTF (Sec. 9)
         half = variant in ("fp16", "bf16")  # NEXT row N4: 16-bit x, w, y on tcgen05 kind::f16 (Sec. 8.3)
-        if f4 or half:
+        if f4:
             launches = sum(2 for d in per if d["n"] > 0)
+        elif half:  # FTF + conv (+ stream-K fixup with the workspace, variant 5 plans it)
+            launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=5).launches
+                           for d in per if d["n"] > 0)
         elif nchw:  # FTF, transpose, conv (+ stream-K fixup), transpose
             launches = sum(3 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=4).launches
                            for d in per if d["n"] > 0)
@@ -345,6 +348,9 @@ def main():
                 d["x16"], d["w16"] = d["x"].to(dt16), d["w"].to(dt16)
                 d["y16"] = torch.empty(d["y"].shape, dtype=dt16, device=dev)
                 d["u"] = wino.filter_transform_half(d["w16"])
+                c = d["cfg"]
+                d["ws16"] = torch.empty(max(wino.half_workspace_bytes(max(d["n"], 1), c.C, c.H, c.W, c.K), 16),
+                                        dtype=torch.uint8, device=dev)
                 if world > 1:
                     dist.broadcast(d["u"].data, src=0)
             elif nonfused:
@@ -401,7 +407,7 @@ def main():
                 elif nchw:
                     wino.conv2d_nchw(d["x_nchw"], d["u"], out=d["y_nchw"], ws=d["ws_nchw"])
                 elif half:
-                    wino.conv2d_half(d["x16"], d["u"], out=d["y16"])
+                    wino.conv2d_half(d["x16"], d["u"], out=d["y16"], ws=d["ws16"])
                 elif nonfused:
                     wino.conv2d_nonfused(d["x"], d["u"], d["ws_nf"], out=d["y"])
                 else:

@@ -268,6 +268,18 @@ wino_status_t wino_filter_transform_half(const void* w_dev, void* u_h_dev, int C
 wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, void* y_dev,
                                         int N, int C, int H, int W, int K, int pad, int stride,
                                         wino_half_t type, wino_stream_t stream);
+/* The same with a caller workspace that enables a stream-K plan (as wino_conv2d_f2x3_fwd_ws:
+ * equal (tile, channel block) ranges on every SM; pieces of cut tiles leave FP32 partial
+ * outputs in the workspace, a fixup kernel adds them in CTA order and rounds once):
+ *   ws_dev / ws_bytes : >= wino_half_workspace_bytes(N,C,H,W,K) (SMs x 64 KiB), 16-byte
+ *                       aligned, not overlapping x, u or y; may be NULL / 0 when sk = 1.
+ *   sk                : 0 = planner's choice, 1 = never, 2 = always (a short workspace ->
+ *                       WINO_ERR_INVALID_ARG). */
+size_t wino_half_workspace_bytes(int N, int C, int H, int W, int K);
+wino_status_t wino_conv2d_f2x3_fwd_half_ws(const void* x_dev, const void* u_h_dev, void* y_dev,
+                                           int N, int C, int H, int W, int K, int pad, int stride,
+                                           wino_half_t type, int sk, void* ws_dev, size_t ws_bytes,
+                                           wino_stream_t stream);
 
 /*
  * End-to-end call on HOST buffers: copies w_host and x_host to the device,
@@ -331,6 +343,7 @@ typedef struct {
     int variant;        /* 0 = FP32 FFMA fused kernel, 1 / 2 = tcgen05 TF32 / 3xTF32, */
                         /* 3 = tcgen05 kind::f16 (FP16 / BF16, NEXT row N4),          */
                         /* 4 = FP32 with a stream-K workspace (wino_conv2d_f2x3_fwd_ws, sk = 0) */
+                        /* 5 = FP16 / BF16 with a stream-K workspace (..._half_ws, sk = 0)     */
     int bk, bn, bc;     /* filters, tiles and channels per CTA step (Sec. 3.3)      */
     int load_x, load_u; /* how x / u reach shared memory: 0 = cp.async 4 B,         */
                         /* 1 = cp.async 16 B, 2 = TMA tiled box (cp.async.bulk.tensor) */
@@ -339,7 +352,7 @@ typedef struct {
     int threads;        /* threads per CTA                                          */
     int smem_bytes;     /* dynamic shared memory per CTA                            */
     int launches;       /* kernels launched by one wino_conv2d_f2x3_fwd* call       */
-    int stream_k;       /* 1: stream-K plan (variant 4 only)                        */
+    int stream_k;       /* 1: stream-K plan (variants 4 and 5)                      */
 } wino_plan_t;
 
 wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_plan_t* plan);

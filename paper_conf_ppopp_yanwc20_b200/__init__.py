@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes",
+    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -144,6 +144,11 @@ def lib() -> ctypes.CDLL:
         L.wino_filter_transform_half.argtypes = [vp, vp, i, i, i, vp]
         L.wino_conv2d_f2x3_fwd_half.restype = i
         L.wino_conv2d_f2x3_fwd_half.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_half_ws") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_half_workspace_bytes.restype = st
+        L.wino_half_workspace_bytes.argtypes = [i, i, i, i, i]
+        L.wino_conv2d_f2x3_fwd_half_ws.restype = i
+        L.wino_conv2d_f2x3_fwd_half_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, i, vp, st, vp]
     if hasattr(L, "wino_conv2d_f2x3_fwd_ws") or not os.environ.get("WINO_LIB_PATH"):
         L.wino_conv_workspace_bytes.restype = st
         L.wino_conv_workspace_bytes.argtypes = [i, i, i, i, i]
@@ -322,9 +327,16 @@ def filter_transform_half(w: torch.Tensor, out: HalfFilter | None = None, stream
     return out
 
 
-def conv2d_half(x: torch.Tensor, u_h: HalfFilter, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+def half_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
+    """Device workspace that lets ``conv2d_half`` use the stream-K plan (wino_half_workspace_bytes)."""
+    return int(lib().wino_half_workspace_bytes(N, C, H, W, K))
+
+
+def conv2d_half(x: torch.Tensor, u_h: HalfFilter, out: torch.Tensor | None = None, stream=None,
+                ws: torch.Tensor | None = None, stream_k: str = "auto") -> torch.Tensor:
     """NEXT row N4: fused Winograd conv on float16 / bfloat16 x (C,H,W,N) -> y (K,H,W,N) of the same type,
-    Winograd-domain GEMM on tcgen05 kind::f16 with FP32 accumulation."""
+    Winograd-domain GEMM on tcgen05 kind::f16 with FP32 accumulation.  ws (>= half_workspace_bytes)
+    enables the stream-K plan (wino_conv2d_f2x3_fwd_half_ws): stream_k "auto" / "off" / "on"."""
     _need_cuda_half(x, "x", 4)
     C, H, W, N = x.shape
     if u_h.C != C or u_h.dtype != x.dtype:
@@ -335,10 +347,17 @@ def conv2d_half(x: torch.Tensor, u_h: HalfFilter, out: torch.Tensor | None = Non
     _need_cuda_half(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N) or out.dtype != x.dtype:
         raise ValueError("out must be (K,H,W,N) of x's dtype")
+    args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_h.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+            N, C, H, W, K, 1, 1, _HALF_DTYPES[x.dtype])
     with torch.cuda.device(x.device):
-        _check(lib().wino_conv2d_f2x3_fwd_half(
-            ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_h.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
-            N, C, H, W, K, 1, 1, _HALF_DTYPES[x.dtype], _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_half")
+        if ws is not None or stream_k == "on":
+            if ws is not None and not ws.is_cuda:
+                raise ValueError("ws must be a CUDA tensor")
+            wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
+            _check(lib().wino_conv2d_f2x3_fwd_half_ws(*args, {"auto": 0, "off": 1, "on": 2}[stream_k], wp, wb,
+                                                      _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_half_ws")
+        else:
+            _check(lib().wino_conv2d_f2x3_fwd_half(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_half")
     return out
 
 

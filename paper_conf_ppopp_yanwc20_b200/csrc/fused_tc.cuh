@@ -86,47 +86,46 @@ __host__ __device__ inline int tc_mm(int, int planes) { return planes == 1 ? 64 
 __host__ __device__ inline int tc_mm(int K, int planes) { return (planes == 1 && K <= 64) ? 64 : 128; }
 #endif
 
-// FTF (Eq. 5) straight into the tensor-core operand layout, rounded to TF32
-// (reading R8; 3xTF32 also stores small = rna(u - big)).  One thread per (4
-// consecutive channels, filter k): the 4 channels of a core-matrix row are one 16 B
-// store per (xi, plane), consecutive k (threads) are consecutive rows -> coalesced.
-// Pads K and C with zeros.
+// FTF (Eq. 5) straight into the tensor-core operand layout, rounded to TF32 (reading R8;
+// 3xTF32 also stores small = rna(u - big)).  Block = 8 channels x 32 filters, one (c, k) per
+// thread (9 coalesced loads along k); results staged in shared memory so that every store is
+// a 16 B core-matrix row (4 channels of one filter).  Grid (Kp/32, ceil(C/8)).  Pads K and C
+// with zeros.
 template <int P, int MM>
 __global__ void __launch_bounds__(256) tc_filter_kernel(const float* __restrict__ w, float* __restrict__ u_tc,
                                                         int C, int K) {
-    const int Kp = ((K + MM - 1) / MM) * MM, C4 = ((C + BC - 1) / BC) * (BC / 4);
-    const long idx = (long)blockIdx.x * 256 + threadIdx.x;
-    if (idx >= (long)C4 * Kp) return;
-    const int c4 = (int)(idx / Kp), k = (int)(idx - (long)c4 * Kp);
-    float t[4][16];
+    __shared__ __align__(16) float st[16][P][32][BC];  // [xi][plane][k][c]
+    const int kl = threadIdx.x & 31, cl = threadIdx.x >> 5;
+    const int k = blockIdx.x * 32 + kl, cb = blockIdx.y, c = cb * BC + cl;
+    float t[16];
+    if (c < C && k < K) {
+        float g[9];
+        const float* wc = w + (size_t)c * 9 * K + k;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const int c = c4 * 4 + j;
-        if (c < C && k < K) {
-            float g[9];
-            const float* wc = w + (size_t)c * 9 * K + k;
+        for (int e = 0; e < 9; ++e) g[e] = __ldg(wc + (size_t)e * K);
+        ftf_4x4(g, t);
+    } else {
 #pragma unroll
-            for (int e = 0; e < 9; ++e) g[e] = __ldg(wc + (size_t)e * K);
-            ftf_4x4(g, t[j]);
-        } else {
-#pragma unroll
-            for (int e = 0; e < 16; ++e) t[j][e] = 0.f;
-        }
+        for (int e = 0; e < 16; ++e) t[e] = 0.f;
     }
-    const int cb = c4 / (BC / 4), ch = c4 % (BC / 4), kb = k / MM, m = k % MM;
-    const int nkb = Kp / MM;
-    const size_t inner = size_t((m >> 3) * 64 + ch * 32 + (m & 7) * 4);
 #pragma unroll
     for (int xi = 0; xi < 16; ++xi) {
-        const size_t base = ((((size_t)cb * nkb + kb) * 16 + xi) * P) * (MM * BC);
-        float4 big, small;
-        big.x = to_tf32(t[0][xi]), big.y = to_tf32(t[1][xi]), big.z = to_tf32(t[2][xi]), big.w = to_tf32(t[3][xi]);
-        *reinterpret_cast<float4*>(u_tc + base + inner) = big;
-        if (P == 2) {
-            small.x = to_tf32(t[0][xi] - big.x), small.y = to_tf32(t[1][xi] - big.y);
-            small.z = to_tf32(t[2][xi] - big.z), small.w = to_tf32(t[3][xi] - big.w);
-            *reinterpret_cast<float4*>(u_tc + base + (MM * BC) + inner) = small;
-        }
+        const float big = to_tf32(t[xi]);
+        st[xi][0][kl][cl] = big;
+        if (P == 2) st[xi][P - 1][kl][cl] = to_tf32(t[xi] - big);
+    }
+    __syncthreads();
+    const int Kp = ((K + MM - 1) / MM) * MM, nkb = Kp / MM;
+#pragma unroll
+    for (int r = 0; r < 4 * P; ++r) {  // 16 xi x P planes x 32 filters x 2 chunks of 4 channels
+        const int row = r * 256 + threadIdx.x;
+        const int ch = row & 1, rk = (row >> 1) & 31, pl = (row >> 6) % P, xi = (row >> 6) / P;
+        const int kk = blockIdx.x * 32 + rk;
+        if (kk >= Kp) continue;
+        const int kb = kk / MM, m = kk % MM;
+        const size_t base = ((((size_t)cb * nkb + kb) * 16 + xi) * P + pl) * (MM * BC);
+        *reinterpret_cast<float4*>(u_tc + base + (m >> 3) * 64 + ch * 32 + (m & 7) * 4) =
+            *reinterpret_cast<const float4*>(&st[xi][pl][rk][ch * 4]);
     }
 }
 

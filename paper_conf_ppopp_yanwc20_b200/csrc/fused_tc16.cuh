@@ -148,45 +148,42 @@ __device__ __forceinline__ void umma_f16(uint32_t d_tmem, uint64_t a, uint64_t b
         : "memory");
 }
 
-// FTF (Eq. 5) from 16-bit w (C,3,3,K) in FP32, rounded to the 16-bit type, straight
-// into the operand layout above.  One thread per (8 consecutive channels, filter k):
-// the 8 channels of a core-matrix row are one 16 B store per xi, and consecutive k
-// (threads) are consecutive rows -> coalesced.  Pads C and K with zeros.
+// FTF (Eq. 5) from 16-bit w (C,3,3,K) in FP32, rounded to the 16-bit type, straight into the
+// operand layout above.  Block = 8 channels x 32 filters, one (c, k) per thread (9 coalesced
+// loads along k); the 16 results go through shared memory so that every store is a 16 B
+// core-matrix row (8 channels of one filter), consecutive filters consecutive rows.
+// Grid (ceil(Kp/32), ceil(C/16)*2).  Pads C and K with zeros.
 template <int DT, int MM>
 __global__ void __launch_bounds__(256) tc16_filter_kernel(const uint16_t* __restrict__ w, uint16_t* __restrict__ u,
                                                           int C, int K) {
-    const int Kp = ((K + MM - 1) / MM) * MM, C8 = (C + BC - 1) / BC * (BC / 8);
-    const long idx = (long)blockIdx.x * 256 + threadIdx.x;
-    if (idx >= (long)C8 * Kp) return;
-    const int c8 = (int)(idx / Kp), k = (int)(idx - (long)c8 * Kp);
-    uint32_t pk[16][4];
+    __shared__ __align__(16) uint16_t st[16][32][8];  // [xi][k][c]
+    const int kl = threadIdx.x & 31, cl = threadIdx.x >> 5;
+    const int k = blockIdx.x * 32 + kl, c8 = blockIdx.y, c = c8 * 8 + cl;
+    float t[16];
+    if (c < C && k < K) {
+        float g[9];
+        const uint16_t* wc = w + (size_t)c * 9 * K + k;
 #pragma unroll
-    for (int cc = 0; cc < 8; cc += 2) {
-        float t[2][16];
+        for (int e = 0; e < 9; ++e) g[e] = to_f<DT>(wc[(size_t)e * K]);
+        ftf_4x4(g, t);
+    } else {
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            const int c = c8 * 8 + cc + h;
-            if (c < C && k < K) {
-                float g[9];
-                const uint16_t* wc = w + (size_t)c * 9 * K + k;
-#pragma unroll
-                for (int e = 0; e < 9; ++e) g[e] = to_f<DT>(wc[(size_t)e * K]);
-                ftf_4x4(g, t[h]);
-            } else {
-#pragma unroll
-                for (int e = 0; e < 16; ++e) t[h][e] = 0.f;
-            }
-        }
-#pragma unroll
-        for (int xi = 0; xi < 16; ++xi) pk[xi][cc >> 1] = pack2<DT>(t[0][xi], t[1][xi]);
+        for (int e = 0; e < 16; ++e) t[e] = 0.f;
     }
-    const int cb = c8 / (BC / 8), ch = c8 % (BC / 8), kb = k / MM, m = k % MM;
-    const int nkb = Kp / MM;
-    const size_t inner = size_t((m >> 3) * 128 + ch * 64 + (m & 7) * 8);
 #pragma unroll
-    for (int xi = 0; xi < 16; ++xi) {
+    for (int xi = 0; xi < 16; ++xi) st[xi][kl][cl] = from_f<DT>(t[xi]);
+    __syncthreads();
+    const int Kp = ((K + MM - 1) / MM) * MM, nkb = Kp / MM;
+    const int cb = c8 / (BC / 8), ch = c8 % (BC / 8);
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {  // 16 xi x 32 rows = 512 rows of 16 B, 2 per thread
+        const int row = r * 256 + threadIdx.x, xi = row >> 5, rk = row & 31;
+        const int kk = blockIdx.x * 32 + rk;
+        if (kk >= Kp) continue;
+        const int kb = kk / MM, m = kk % MM;
         const size_t base = (((size_t)cb * nkb + kb) * 16 + xi) * (MM * BC);
-        *reinterpret_cast<uint4*>(u + base + inner) = make_uint4(pk[xi][0], pk[xi][1], pk[xi][2], pk[xi][3]);
+        *reinterpret_cast<uint4*>(u + base + (m >> 3) * 128 + ch * 64 + (m & 7) * 8) =
+            *reinterpret_cast<const uint4*>(&st[xi][rk][0]);
     }
 }
 
@@ -198,11 +195,50 @@ struct __align__(64) Params {
     int N, C, H, W, K;
     int TW, NV;
     int num_kb, num_cb, num_tiles;
+    // stream-K (SK = true): units = tile * num_cb + cb; CTA b takes [b*q + min(b, r), ...); pieces
+    // of cut tiles leave FP32 partial outputs in sk_ws (2 slots of MM x 4 x TN floats per CTA)
+    float* __restrict__ sk_ws;
+    int sk_q, sk_r;
+};
+
+__host__ __device__ __forceinline__ int sk_start(const Params& p, int b) { return b * p.sk_q + min(b, p.sk_r); }
+
+// The (tile, channel-block range) pieces a CTA processes, identical in every warp role:
+// persistent tiles blockIdx.x, +gridDim.x, ... (whole tiles), or the CTA's stream-K range.
+template <bool SK>
+struct Segs {
+    int a, b, n = 0;  // cursor, end (SK) / stride; pieces handed out so far
+    __device__ __forceinline__ explicit Segs(const Params& p) {
+        if constexpr (SK) {
+            a = sk_start(p, blockIdx.x);
+            b = sk_start(p, blockIdx.x + 1);
+        } else {
+            a = blockIdx.x;
+            b = gridDim.x;
+        }
+    }
+    __device__ __forceinline__ bool next(const Params& p, int& tile, int& lo, int& hi) {
+        if constexpr (SK) {
+            if (a >= b) return false;
+            tile = a / p.num_cb;
+            lo = a - tile * p.num_cb;
+            hi = min(p.num_cb, lo + (b - a));
+            a += hi - lo;
+        } else {
+            if (a >= p.num_tiles) return false;
+            tile = a;
+            lo = 0;
+            hi = p.num_cb;
+            a += b;
+        }
+        ++n;
+        return true;
+    }
 };
 
 // XM: 2 = one TMA box per nu-half (N % 32 == 0), 3 = 32/N boxes per half (N in {8, 16}),
 // 0 = generic gather by the x-producer warp (a 16-bit box needs >= 8 images: 16 B rows)
-template <int DT, int XM, int MM>
+template <int DT, int XM, int MM, bool SK = false>
 __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant__ Params p) {
     using G = Cfg<MM>;
     constexpr int NH = G::NH, TN = G::TN;
@@ -223,7 +259,6 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
     uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + G::OFF_TMEM);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int NCB = p.num_cb;
 
     if (tid == 0) {
         for (int s = 0; s < U_SLOTS; ++s) {
@@ -255,7 +290,9 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
         if (warp == XPROD_WARP) {
             // --------------------------- raw-x producer ---------------------------
             int gcb = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+            Segs<SK> segs(p);
+            int tile, lo, hi;
+            while (segs.next(p, tile, lo, hi)) {
                 const int nu0 = (tile / p.num_kb) * TN;
                 int tn0[NH], tw0[NH], th0[NH];
                 if constexpr (XM == 2) {
@@ -275,11 +312,11 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                         }
                     }
                     if (lane == 0)
-                        for (int cb = 0; cb < 4 && cb < NCB; ++cb)
+                        for (int cb = lo; cb < lo + 4 && cb < hi; ++cb)
 #pragma unroll
                             for (int h = 0; h < NH; ++h) tma_prefetch_l2_4d(&p.tmx, tn0[h], tw0[h], th0[h], cb * BC);
                 }
-                for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                for (int cb = lo; cb < hi; ++cb, ++gcb) {
                     const int xs = gcb % X_SLOTS;
                     if (gcb >= X_SLOTS) mbar_wait(&x_empty[xs], ((gcb / X_SLOTS) - 1) & 1);
                     uint8_t* xdst = sx + xs * G::X_SLOT;
@@ -289,7 +326,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                             mbar_arrive_expect_tx(&x_full[xs], G::X_SLOT);
 #pragma unroll
                             for (int h = 0; h < NH; ++h) {
-                                if (cb + 4 < NCB) tma_prefetch_l2_4d(&p.tmx, tn0[h], tw0[h], th0[h], (cb + 4) * BC);
+                                if (cb + 4 < hi) tma_prefetch_l2_4d(&p.tmx, tn0[h], tw0[h], th0[h], (cb + 4) * BC);
                                 tma_load_4d(xdst + h * XS_BYTES, &p.tmx, &x_full[xs], tn0[h], tw0[h], th0[h], cb * BC);
                             }
                         }
@@ -342,9 +379,11 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
         } else if (warp == PROD_WARP) {
             // ------------------------ transformed-filter producer -----------------
             int unit = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+            Segs<SK> segs(p);
+            int tile, lo, hi;
+            while (segs.next(p, tile, lo, hi)) {
                 const int kb = tile % p.num_kb;
-                for (int cb = 0; cb < NCB; ++cb, ++unit) {
+                for (int cb = lo; cb < hi; ++cb, ++unit) {
                     const int us = unit % U_SLOTS;
                     if (unit >= U_SLOTS) mbar_wait(&u_empty[us], ((unit / U_SLOTS) - 1) & 1);
                     if (lane == 0) {
@@ -359,10 +398,12 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
             // ------------------------------ MMA issuer ----------------------------
             constexpr uint32_t IDESC = umma_idesc_f16(DT, MM, BN);
             int unit = 0, gcb = 0, it = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+            Segs<SK> segs(p);
+            int tile, lo, hi;
+            for (; segs.next(p, tile, lo, hi); ++it) {
                 if (it > 0) mbar_wait(acc_empty, (it - 1) & 1);  // epilogue drained TMEM
                 tc_fence_after();
-                for (int cb = 0; cb < NCB; ++cb, ++gcb, ++unit) {
+                for (int cb = lo; cb < hi; ++cb, ++gcb, ++unit) {
                     const int vs = gcb & 1, us = unit % U_SLOTS;
                     mbar_wait(&v_full[vs], (gcb >> 1) & 1);
                     if (lane == 0) TC16_TRACE(4, gcb);
@@ -380,7 +421,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
                                 // nu-half h accumulates in TMEM lanes 16h.. of each quadrant (MM = 64)
                                 const uint64_t bd = umma_desc(vbase + (xi * NH + h) * B_TILE, 128, V_SBO);
                                 umma_f16(tmem + xi * BN + ((uint32_t)(16 * h) << 16), ad, bd, IDESC,
-                                         cb > 0 ? 1u : 0u);
+                                         cb > lo ? 1u : 0u);
                             }
                         }
                         umma_commit(&u_empty[us]);
@@ -421,8 +462,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
         const int sw = (np >> 2) & 1;
         const uint32_t voff0 = hh * B_TILE + ((2 * np) >> 3) * V_SBO + (cp >> 2) * 128 + ((2 * np) & 7) * 16 + (cp & 3) * 4;
         int gcb = 0;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-            for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+        Segs<SK> segs(p);
+        int tile, lo, hi;
+        while (segs.next(p, tile, lo, hi)) {
+            for (int cb = lo; cb < hi; ++cb, ++gcb) {
                 if (NH == 1 && (gcb & 1) != g) continue;
                 const int xs = gcb % X_SLOTS, vs = gcb & 1;
                 mbar_wait(&x_full[xs], (gcb / X_SLOTS) & 1);
@@ -481,7 +524,9 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
         const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
         const size_t dW = (size_t)p.W * p.N;
         int it = 0;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+        Segs<SK> segs(p);
+        int tile, lo, hi;
+        for (; segs.next(p, tile, lo, hi); ++it) {
             const int k = (tile % p.num_kb) * MM + kl;
             const int nu0 = (tile / p.num_kb) * TN + hsel * BN;
             mbar_wait(acc_full, it & 1);
@@ -504,6 +549,18 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(acc_empty);  // TMEM free for the next tile's MMAs
+            if (SK && hi - lo != p.num_cb) {
+                // piece of a cut tile: FP32 partial outputs -> slot 2b (the CTA's first piece) or
+                // 2b + 1 (its last), [kl][output][nu of the tile]; tc16_fixup_kernel adds and rounds
+                float* wk = p.sk_ws + ((size_t)(2 * blockIdx.x + (segs.n > 1 ? 1 : 0)) * MM + kl) * (4 * TN) + hsel * BN;
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+#pragma unroll
+                    for (int j = 0; j < BN; j += 4)
+                        *reinterpret_cast<float4*>(wk + q * TN + j) =
+                            make_float4(o[j][q], o[j + 1][q], o[j + 2][q], o[j + 3][q]);
+                continue;
+            }
             if (k >= p.K || nu0 >= p.NV) continue;
             if constexpr (XM == 2 || XM == 3) {
                 // groups of 8 nu = 8 consecutive n of one image tile (N % 8 == 0) -> 16 B stores
@@ -547,6 +604,73 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
     tc_fence_before();
     __syncthreads();
     if (warp == 0) tmem_dealloc(tmem, 512);
+}
+
+// Stream-K fixup: blocks 16i .. 16i+15 handle the tile cut by the range boundary of CTA b = i + 1
+// (when it is the first boundary inside that tile), 1/16 of its MM x TN outputs each:
+// y = RNE(sum of the pieces' FP32 partials in CTA order).  Each thread owns 4 (filter, nu)
+// outputs and issues all their loads before adding (latency-bound otherwise).
+constexpr int FIX_PARTS = 16;
+template <int DT, int MM>
+__global__ void __launch_bounds__(256) tc16_fixup_kernel(const __grid_constant__ Params p, int G) {
+    constexpr int TN = Cfg<MM>::TN;
+    constexpr int PER = MM * TN / FIX_PARTS / 256;  // outputs per thread (4)
+    __shared__ int slots[256];
+    __shared__ int nseg;
+    const int b = blockIdx.x / FIX_PARTS + 1, part = blockIdx.x % FIX_PARTS;
+    const int ub = sk_start(p, b);
+    const int tile = ub / p.num_cb;
+    const int t0 = tile * p.num_cb, t1 = t0 + p.num_cb;
+    if (ub == t0 || sk_start(p, b - 1) > t0) return;  // no cut, or an earlier boundary owns it
+    if (threadIdx.x == 0) {
+        int b0 = b - 1;
+        while (b0 > 0 && sk_start(p, b0) > t0) --b0;
+        int ns = 0, c0 = sk_start(p, b0);
+        for (int c = b0; c < G && c0 < t1 && ns < 256; ++c) {
+            const int c1 = sk_start(p, c + 1);
+            if (c1 > c0) slots[ns++] = 2 * c + (c0 < t0 ? 1 : 0);
+            c0 = c1;
+        }
+        nseg = ns;
+    }
+    __syncthreads();
+    const int ns = nseg;
+    const int kb = tile % p.num_kb, nb = tile / p.num_kb;
+    const size_t HWN = (size_t)p.H * p.W * p.N, dW = (size_t)p.W * p.N;
+    constexpr size_t SLOT = (size_t)MM * 4 * TN;
+    float o[PER][4];
+#pragma unroll
+    for (int i = 0; i < PER; ++i)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) o[i][q] = 0.f;
+    for (int sidx = 0; sidx < ns; ++sidx) {  // CTA order
+        const float* wk = p.sk_ws + slots[sidx] * SLOT;
+        float v[PER][4];
+#pragma unroll
+        for (int i = 0; i < PER; ++i) {
+            const int e = (part * PER + i) * 256 + threadIdx.x, kl = e / TN, j = e - kl * TN;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) v[i][q] = wk[((size_t)kl * 4 + q) * TN + j];
+        }
+#pragma unroll
+        for (int i = 0; i < PER; ++i)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) o[i][q] += v[i][q];
+    }
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+        const int e = (part * PER + i) * 256 + threadIdx.x, kl = e / TN, j = e - kl * TN;
+        const int k = kb * MM + kl, nu = nb * TN + j;
+        if (k >= p.K || nu >= p.NV) continue;
+        const int t = nu / p.N, n = nu - t * p.N;
+        const int th = t / p.TW, tw = t - th * p.TW;
+        const int i0 = 2 * th, j0 = 2 * tw;
+        uint16_t* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+        yk[0] = from_f<DT>(o[i][0]);
+        if (j0 + 1 < p.W) yk[p.N] = from_f<DT>(o[i][1]);
+        if (i0 + 1 < p.H) yk[dW] = from_f<DT>(o[i][2]);
+        if (i0 + 1 < p.H && j0 + 1 < p.W) yk[dW + p.N] = from_f<DT>(o[i][3]);
+    }
 }
 
 }  // namespace tc16

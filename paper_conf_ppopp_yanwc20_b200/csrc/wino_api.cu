@@ -95,6 +95,16 @@ bool overlaps(const void* a, size_t na, const void* b, size_t nb) {
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
+// stream-K workspace of the 16-bit kernel: 2 slots of MM x 4 x TN FP32 partials per CTA (64 KiB)
+size_t tc16_sk_bytes(int ctas) { return size_t(ctas) * 2 * 128 * 4 * 32 * sizeof(float); }
+// stream-K pays for the 16-bit kernel only when whole tiles would leave most SMs idle: its pieces
+// run ~1.5x slower per channel block than the persistent schedule (measured: conv5 at P = 1
+// 38.9 -> 52 us, conv2 175 -> 204 us; at P = 8 conv5 with 8 tiles 325 -> 42 us)
+bool tc16_sk_pays(int64_t tiles, int ncb, int sms) {
+    const double units = double(tiles) * ncb, reg = std::ceil(double(tiles) / sms) * ncb;
+    return 2 * tiles <= sms && 1.5 * std::ceil(units / sms) + 3.0 < 0.9 * reg;
+}
+
 constexpr int64_t kMaxElems = (int64_t(1) << 31) - 1;
 
 // Shape checks common to every conv entry point.
@@ -554,7 +564,7 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->launches = 1;
         return WINO_OK;
     }
-    if (variant == 3) {  // tcgen05 kind::f16 (FP16 / BF16 operands, NEXT row N4)
+    if (variant == 3 || variant == 5) {  // tcgen05 kind::f16 (FP16 / BF16, NEXT row N4); 5: with workspace
         using namespace wino::tc16;
         const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
         const int mm = tc16_mm(K), tn = BN * (128 / mm);
@@ -569,6 +579,16 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->threads = NT;
         plan->smem_bytes = mm == 64 ? Cfg<64>::BYTES : Cfg<128>::BYTES;
         plan->launches = 1;
+        int dev = -1, sms = 148;  // host-only planning unless an sm_100 device is current
+        if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+        else cudaGetLastError();
+        sms = sms < 256 ? sms : 256;
+        if (variant == 5 && tc16_sk_pays(plan->ctas, (C + BC - 1) / BC, sms)) {
+            plan->stream_k = 1;
+            plan->launches = 2;
+            plan->ctas = sms;
+        }
+        plan->variant = variant;
         return WINO_OK;
     }
     if (variant != 0 && variant != 4) return WINO_ERR_UNSUPPORTED;
@@ -759,8 +779,7 @@ wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int 
     const int planes = mode == WINO_TC_3XTF32 ? 2 : 1;
     const int mm = wino::tc::tc_mm(K, planes);
     const int64_t Kp = ((K + mm - 1) / mm) * mm;
-    const int64_t C4 = ((C + wino::tc::BC - 1) / wino::tc::BC) * (wino::tc::BC / 4);
-    const unsigned blocks = static_cast<unsigned>((C4 * Kp + 255) / 256);
+    const dim3 blocks(static_cast<unsigned>(Kp / 32), static_cast<unsigned>((C + wino::tc::BC - 1) / wino::tc::BC));
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (planes == 1 && mm == 64) wino::tc::tc_filter_kernel<1, 64><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
     else if (planes == 1) wino::tc::tc_filter_kernel<1, 128><<<blocks, 256, 0, st>>>(w_dev, u_tc_dev, C, K);
@@ -834,24 +853,37 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
 
 extern "C++" {
 namespace {
-std::atomic<uint64_t> g_attr_tc16[2][4][2];  // [DT][XM 0..3][MM == 64]
-template <int DT, int XM, int MM>
+std::atomic<uint64_t> g_attr_tc16[2][4][2][2];  // [DT][XM 0..3][MM == 64][SK]
+template <int DT, int XM, int MM, bool SK>
 wino_status_t launch_tc16(const wino::tc16::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
-    auto kern = wino::tc16::fused_tc16_kernel<DT, XM, MM>;
+    auto kern = wino::tc16::fused_tc16_kernel<DT, XM, MM, SK>;
     constexpr int smem = wino::tc16::Cfg<MM>::BYTES;
-    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc16[DT][XM][MM == 64]);
+    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc16[DT][XM][MM == 64][SK]);
     if (s != WINO_OK) return s;
     kern<<<dim3(static_cast<unsigned>(ctas)), wino::tc16::NT, smem, st>>>(prm);
     cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess && SK && ctas > 1) {
+        wino::tc16::tc16_fixup_kernel<DT, MM><<<dim3(static_cast<unsigned>(wino::tc16::FIX_PARTS * (ctas - 1))), 256, 0,
+                                                st>>>(
+            prm, static_cast<int>(ctas));
+        e = cudaGetLastError();
+    }
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 bool half_type_ok(wino_half_t t) { return t == WINO_HALF_FP16 || t == WINO_HALF_BF16; }
 template <int DT, int MM>
-wino_status_t launch_tc16_xm(const wino::tc16::Params& prm, int xm, int64_t ctas, int dev, cudaStream_t st) {
-    if (xm == 2) return launch_tc16<DT, 2, MM>(prm, ctas, dev, st);
-    if (xm == 3) return launch_tc16<DT, 3, MM>(prm, ctas, dev, st);
-    return launch_tc16<DT, 0, MM>(prm, ctas, dev, st);
+wino_status_t launch_tc16_xm(const wino::tc16::Params& prm, int xm, bool sk, int64_t ctas, int dev,
+                             cudaStream_t st) {
+    if (sk) {
+        if (xm == 2) return launch_tc16<DT, 2, MM, true>(prm, ctas, dev, st);
+        if (xm == 3) return launch_tc16<DT, 3, MM, true>(prm, ctas, dev, st);
+        return launch_tc16<DT, 0, MM, true>(prm, ctas, dev, st);
+    }
+    if (xm == 2) return launch_tc16<DT, 2, MM, false>(prm, ctas, dev, st);
+    if (xm == 3) return launch_tc16<DT, 3, MM, false>(prm, ctas, dev, st);
+    return launch_tc16<DT, 0, MM, false>(prm, ctas, dev, st);
 }
+
 }  // namespace
 }  // extern "C++"
 
@@ -873,7 +905,7 @@ wino_status_t wino_filter_transform_half(const void* w_dev, void* u_h_dev, int C
     using namespace wino::tc16;
     const int mm = tc16_mm(K);
     const int64_t Kp = ((K + mm - 1) / mm) * mm, C8 = ((C + BC - 1) / BC) * (BC / 8);
-    const unsigned blocks = static_cast<unsigned>((C8 * Kp + 255) / 256);
+    const dim3 blocks(static_cast<unsigned>(Kp / 32), static_cast<unsigned>(C8));
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     const uint16_t* w = static_cast<const uint16_t*>(w_dev);
     uint16_t* u = static_cast<uint16_t*>(u_h_dev);
@@ -888,17 +920,23 @@ wino_status_t wino_filter_transform_half(const void* w_dev, void* u_h_dev, int C
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 
-wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, void* y_dev, int N, int C, int H,
-                                        int W, int K, int pad, int stride, wino_half_t type, wino_stream_t stream) {
+extern "C++" {
+namespace {
+// sk: 0 = never, 1 = planner's choice, 2 = always (stream-K needs ws >= tc16_sk_bytes(SMs))
+wino_status_t conv_half(const void* x_dev, const void* u_h_dev, void* y_dev, int N, int C, int H, int W, int K,
+                        int pad, int stride, wino_half_t type, int sk, void* ws_dev, size_t ws_bytes,
+                        wino_stream_t stream) {
     if (!x_dev || !u_h_dev || !y_dev || !half_type_ok(type)) return WINO_ERR_INVALID_ARG;
     wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
     if (s != WINO_OK) return s;
     if (wino_filter_workspace_bytes_half(C, K) / 2 > size_t(kMaxElems)) return WINO_ERR_TOO_LARGE;
-    if (!aligned16(x_dev) || !aligned16(u_h_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    if (!aligned16(x_dev) || !aligned16(u_h_dev) || !aligned16(y_dev) || (ws_dev && !aligned16(ws_dev)))
+        return WINO_ERR_MISALIGNED;
     const size_t hwn = size_t(H) * W * N;
-    const size_t yb = size_t(K) * hwn * 2;
-    if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 2) ||
-        overlaps(y_dev, yb, u_h_dev, wino_filter_workspace_bytes_half(C, K)))
+    const size_t yb = size_t(K) * hwn * 2, xb = size_t(C) * hwn * 2, ub = wino_filter_workspace_bytes_half(C, K);
+    if (overlaps(y_dev, yb, x_dev, xb) || overlaps(y_dev, yb, u_h_dev, ub)) return WINO_ERR_INVALID_ARG;
+    if (ws_dev && (overlaps(ws_dev, ws_bytes, x_dev, xb) || overlaps(ws_dev, ws_bytes, u_h_dev, ub) ||
+                   overlaps(ws_dev, ws_bytes, y_dev, yb)))
         return WINO_ERR_INVALID_ARG;
     int dev;
     if ((s = check_device(&dev)) != WINO_OK) return s;
@@ -927,12 +965,49 @@ wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, 
         const cuuint32_t box[4] = {cuuint32_t(xm == 2 ? BN : N), 4, 4, BC};
         if (!encode_map(&prm.tmx, x_dev, 4, dims, box, nullptr, dt, 2)) return cuda_fail(cudaErrorInvalidValue);
     }
-    const int sms = sm_count(dev);
-    const int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
+    const int sms = sm_count(dev) < 256 ? sm_count(dev) : 256;
+    int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
+    // stream-K: equal (tile, channel block) ranges on every SM when the tiles leave SMs idle or
+    // end in a partial wave (estimate in channel-block times: waves x blocks vs units / SMs + 3)
+    const double units = double(prm.num_tiles) * prm.num_cb;
+    const bool sk_ok = ws_dev && ws_bytes >= tc16_sk_bytes(sms) && units < 2147483647.0;
+    if (sk == 2 && !sk_ok) return WINO_ERR_INVALID_ARG;
+    const bool use_sk = sk == 2 || (sk == 1 && sk_ok && tc16_sk_pays(prm.num_tiles, prm.num_cb, sms));
+    if (use_sk) {
+        ctas = sms;
+        prm.sk_ws = static_cast<float*>(ws_dev);
+        prm.sk_q = static_cast<int>(int64_t(units) / sms);
+        prm.sk_r = static_cast<int>(int64_t(units) % sms);
+    }
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (type == WINO_HALF_FP16)
-        return mm == 64 ? launch_tc16_xm<0, 64>(prm, xm, ctas, dev, st) : launch_tc16_xm<0, 128>(prm, xm, ctas, dev, st);
-    return mm == 64 ? launch_tc16_xm<1, 64>(prm, xm, ctas, dev, st) : launch_tc16_xm<1, 128>(prm, xm, ctas, dev, st);
+        return mm == 64 ? launch_tc16_xm<0, 64>(prm, xm, use_sk, ctas, dev, st)
+                        : launch_tc16_xm<0, 128>(prm, xm, use_sk, ctas, dev, st);
+    return mm == 64 ? launch_tc16_xm<1, 64>(prm, xm, use_sk, ctas, dev, st)
+                    : launch_tc16_xm<1, 128>(prm, xm, use_sk, ctas, dev, st);
+}
+}  // namespace
+}  // extern "C++"
+
+wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, void* y_dev, int N, int C, int H,
+                                        int W, int K, int pad, int stride, wino_half_t type, wino_stream_t stream) {
+    return conv_half(x_dev, u_h_dev, y_dev, N, C, H, W, K, pad, stride, type, 0, nullptr, 0, stream);
+}
+
+size_t wino_half_workspace_bytes(int N, int C, int H, int W, int K) {
+    if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
+    int dev = -1, sms = 148;
+    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+    else cudaGetLastError();
+    return tc16_sk_bytes(sms < 256 ? sms : 256);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_half_ws(const void* x_dev, const void* u_h_dev, void* y_dev, int N, int C, int H,
+                                           int W, int K, int pad, int stride, wino_half_t type, int sk,
+                                           void* ws_dev, size_t ws_bytes, wino_stream_t stream) {
+    if (sk < 0 || sk > 2 || (ws_bytes > 0 && !ws_dev)) return WINO_ERR_INVALID_ARG;
+    const int mode = sk == 0 ? 1 : (sk == 1 ? 0 : 2);  // API 0 auto / 1 off / 2 force
+    return conv_half(x_dev, u_h_dev, y_dev, N, C, H, W, K, pad, stride, type, mode, ws_dev, ws_bytes, stream);
 }
 
 size_t wino_host_workspace_bytes(int N, int C, int H, int W, int K) {

@@ -177,3 +177,57 @@ def test_half_argument_errors(wino):
     st = L.wino_conv2d_f2x3_fwd_half(p(x.data_ptr()), p(uh.data.data_ptr()), p(y.data_ptr()), 32, 16, 4, 4, 64,
                                      0, 1, 0, None)
     assert st == 2  # pad != 1 -> UNSUPPORTED
+
+
+def _run_ws(wino, xh, wh, mode):
+    C, H, W, N = xh.shape
+    K = wh.shape[3]
+    uh = wino.filter_transform_half(wh.to(DEV))
+    ws = torch.empty(wino.half_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+    y = wino.conv2d_half(xh.to(DEV), uh, ws=ws, stream_k=mode)
+    torch.cuda.synchronize()
+    return y.cpu()
+
+
+# stream-K: ranges shorter than a tile (large C, few tiles), spanning several tiles, every load path
+SK_EDGE = [(32, 512, 256, 5, 5), (4, 512, 512, 7, 7), (8, 256, 256, 14, 14), (16, 128, 128, 12, 10),
+           (32, 64, 64, 30, 30), (64, 33, 132, 9, 7), (96, 40, 17, 11, 3)]
+
+
+@pytest.mark.parametrize("dt", DTYPES, ids=IDS)
+@pytest.mark.parametrize("shape", SK_EDGE, ids=[str(s) for s in SK_EDGE])
+def test_half_stream_k_small_int_bit_exact(wino, shape, dt):
+    N, C, K, H, W = shape
+    xh, wh = _inputs(Conv3x3Config("h", N, C, K, H, W), "smallint", dt)
+    y = _run_ws(wino, xh, wh, "on")
+    assert np.array_equal(y.float().numpy(), _round(oracle.direct_conv(xh.float(), wh.float()), dt))
+
+
+@pytest.mark.parametrize("dt", DTYPES, ids=IDS)
+@pytest.mark.parametrize("shape", SK_EDGE[:4], ids=[str(s) for s in SK_EDGE[:4]])
+def test_half_stream_k_random(wino, shape, dt):
+    N, C, K, H, W = shape
+    xh, wh = _inputs(Conv3x3Config("h", N, C, K, H, W), "uniform", dt, seed_x=51, seed_w=52)
+    y = _run_ws(wino, xh, wh, "on")
+    assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(xh.float(), wh.float())) <= TOL[dt]
+
+
+@pytest.mark.parametrize("P", [1, 2, 4, 8])
+def test_half_stream_k_configs_and_shards(wino, P):
+    """BASELINE layers and their P-rank batch shards with the workspace (planner's choice)."""
+    for name in ("conv5_x", "conv4_x", "conv3_x", "conv2_x"):
+        cfg = CONFIGS[name].with_batch(CONFIGS[name].N // P)
+        xh, wh = _inputs(cfg, "smallint", torch.float16)
+        y = _run_ws(wino, xh, wh, "auto")
+        idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 1500)
+        ii = idx.numpy()
+        got = y.float().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]].astype(np.float64)
+        ref = _round(oracle.direct_sample(xh.float(), wh.float(), idx), torch.float16).astype(np.float64)
+        assert np.array_equal(got, ref), (name, cfg.N)
+
+
+def test_half_stream_k_deterministic(wino):
+    xh, wh = _inputs(CONFIGS["conv4_x"].with_batch(16), "uniform", torch.bfloat16)
+    y1 = _run_ws(wino, xh, wh, "on")
+    y2 = _run_ws(wino, xh, wh, "on")
+    assert torch.equal(y1, y2)
