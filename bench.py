@@ -327,7 +327,7 @@ def main():
             launches = sum(3 for d in per if d["n"] > 0)  # FTF, ITF, OTF (the GEMMs are cuBLAS kernels)
         else:
             # fp32: with the stream-K workspace (variant 4 plans it), which may add a fixup launch
-            vid = {"fp32": 4, "tf32": 1, "3xtf32": 2}[variant]
+            vid = {"fp32": 4, "tf32": 6, "3xtf32": 7}[variant]  # plans with the stream-K workspaces
             launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K,
                                          variant=vid).launches for d in per if d["n"] > 0)
         for d in per:
@@ -340,6 +340,9 @@ def main():
                     dist.broadcast(d["u"], src=0)
             elif tc:
                 d["u"] = wino.filter_transform_tc(d["w"], variant)
+                c = d["cfg"]
+                d["ws_tc"] = torch.empty(max(wino.tc_workspace_bytes(max(d["n"], 1), c.C, c.H, c.W, c.K), 16),
+                                         dtype=torch.uint8, device=dev)
                 if world > 1:
                     dist.broadcast(d["u"].data, src=0)
             elif half:
@@ -403,7 +406,7 @@ def main():
                 if f4:
                     wino.conv2d_f4(d["x"], d["u"], out=d["y"])
                 elif tc:
-                    wino.conv2d_tc(d["x"], d["u"], out=d["y"])
+                    wino.conv2d_tc(d["x"], d["u"], out=d["y"], ws=d["ws_tc"])
                 elif nchw:
                     wino.conv2d_nchw(d["x_nchw"], d["u"], out=d["y_nchw"], ws=d["ws_nchw"])
                 elif half:

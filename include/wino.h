@@ -239,6 +239,18 @@ wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int 
 wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev, float* y_dev,
                                       int N, int C, int H, int W, int K, int pad, int stride,
                                       wino_tc_mode_t mode, wino_stream_t stream);
+/* The same with a caller workspace that enables a stream-K plan for tile-starved shapes (as
+ * wino_conv2d_f2x3_fwd_half_ws; only the TMA x paths, N % 32 == 0 or N in {4, 8, 16}):
+ *   ws_dev / ws_bytes : >= wino_tc_workspace_bytes(N,C,H,W,K) (SMs x 64 KiB), 16-byte aligned,
+ *                       not overlapping x, u_tc or y; may be NULL / 0 when sk = 1.
+ *   sk                : 0 = planner's choice, 1 = never, 2 = always (short workspace or a
+ *                       gather-path N -> WINO_ERR_INVALID_ARG; TF32 with K <= 64, i.e.
+ *                       64-filter tiles -> WINO_ERR_UNSUPPORTED). */
+size_t wino_tc_workspace_bytes(int N, int C, int H, int W, int K);
+wino_status_t wino_conv2d_f2x3_fwd_tc_ws(const float* x_dev, const float* u_tc_dev, float* y_dev,
+                                         int N, int C, int H, int W, int K, int pad, int stride,
+                                         wino_tc_mode_t mode, int sk, void* ws_dev, size_t ws_bytes,
+                                         wino_stream_t stream);
 
 /*
  * NEXT row N4: 16-bit version on the tensor cores.  The paper:
@@ -344,6 +356,7 @@ typedef struct {
                         /* 3 = tcgen05 kind::f16 (FP16 / BF16, NEXT row N4),          */
                         /* 4 = FP32 with a stream-K workspace (wino_conv2d_f2x3_fwd_ws, sk = 0) */
                         /* 5 = FP16 / BF16 with a stream-K workspace (..._half_ws, sk = 0)     */
+                        /* 6 / 7 = TF32 / 3xTF32 with a stream-K workspace (..._tc_ws, sk = 0) */
     int bk, bn, bc;     /* filters, tiles and channels per CTA step (Sec. 3.3)      */
     int load_x, load_u; /* how x / u reach shared memory: 0 = cp.async 4 B,         */
                         /* 1 = cp.async 16 B, 2 = TMA tiled box (cp.async.bulk.tensor) */
@@ -352,7 +365,7 @@ typedef struct {
     int threads;        /* threads per CTA                                          */
     int smem_bytes;     /* dynamic shared memory per CTA                            */
     int launches;       /* kernels launched by one wino_conv2d_f2x3_fwd* call       */
-    int stream_k;       /* 1: stream-K plan (variants 4 and 5)                      */
+    int stream_k;       /* 1: stream-K plan (variants 4 - 7)                        */
 } wino_plan_t;
 
 wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_plan_t* plan);

@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes",
+    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -144,6 +144,11 @@ def lib() -> ctypes.CDLL:
         L.wino_filter_transform_half.argtypes = [vp, vp, i, i, i, vp]
         L.wino_conv2d_f2x3_fwd_half.restype = i
         L.wino_conv2d_f2x3_fwd_half.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_tc_ws") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_tc_workspace_bytes.restype = st
+        L.wino_tc_workspace_bytes.argtypes = [i, i, i, i, i]
+        L.wino_conv2d_f2x3_fwd_tc_ws.restype = i
+        L.wino_conv2d_f2x3_fwd_tc_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, i, vp, st, vp]
     if hasattr(L, "wino_conv2d_f2x3_fwd_half_ws") or not os.environ.get("WINO_LIB_PATH"):
         L.wino_half_workspace_bytes.restype = st
         L.wino_half_workspace_bytes.argtypes = [i, i, i, i, i]
@@ -263,8 +268,15 @@ def filter_transform_tc(w: torch.Tensor, variant="tf32", out: TcFilter | None = 
     return out
 
 
-def conv2d_tc(x: torch.Tensor, u_tc: TcFilter, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
-    """Fused Winograd conv with the Winograd-domain GEMM on tcgen05 (TF32 / 3xTF32)."""
+def tc_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
+    """Device workspace that lets ``conv2d_tc`` use the stream-K plan (wino_tc_workspace_bytes)."""
+    return int(lib().wino_tc_workspace_bytes(N, C, H, W, K))
+
+
+def conv2d_tc(x: torch.Tensor, u_tc: TcFilter, out: torch.Tensor | None = None, stream=None,
+              ws: torch.Tensor | None = None, stream_k: str = "auto") -> torch.Tensor:
+    """Fused Winograd conv with the Winograd-domain GEMM on tcgen05 (TF32 / 3xTF32).  ws (>=
+    tc_workspace_bytes) enables the stream-K plan (wino_conv2d_f2x3_fwd_tc_ws)."""
     _need_cuda_f32(x, "x", 4)
     C, H, W, N = x.shape
     if u_tc.C != C:
@@ -275,10 +287,17 @@ def conv2d_tc(x: torch.Tensor, u_tc: TcFilter, out: torch.Tensor | None = None, 
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N):
         raise ValueError("out must be (K,H,W,N)")
+    args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_tc.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+            N, C, H, W, K, 1, 1, u_tc.mode)
     with torch.cuda.device(x.device):
-        _check(lib().wino_conv2d_f2x3_fwd_tc(
-            ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_tc.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
-            N, C, H, W, K, 1, 1, u_tc.mode, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc")
+        if ws is not None or stream_k == "on":
+            if ws is not None and not ws.is_cuda:
+                raise ValueError("ws must be a CUDA tensor")
+            wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
+            _check(lib().wino_conv2d_f2x3_fwd_tc_ws(*args, {"auto": 0, "off": 1, "on": 2}[stream_k], wp, wb,
+                                                    _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc_ws")
+        else:
+            _check(lib().wino_conv2d_f2x3_fwd_tc(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc")
     return out
 
 

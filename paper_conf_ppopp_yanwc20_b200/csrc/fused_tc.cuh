@@ -139,6 +139,44 @@ struct __align__(64) Params {
     int num_kb;     // ceil(K/MM)
     int num_cb;     // ceil(C/8)
     int num_tiles;  // ceil(NV/(32*NH)) * num_kb
+    // stream-K (SK = true, same scheme as fused_tc16.cuh): units = tile * num_cb + cb, CTA b takes
+    // [b*q + min(b, r), ...); pieces of cut tiles leave partial outputs in sk_ws (2 x 64 KiB per CTA)
+    float* __restrict__ sk_ws;
+    int sk_q, sk_r;
+};
+
+__host__ __device__ __forceinline__ int sk_start(const Params& p, int b) { return b * p.sk_q + min(b, p.sk_r); }
+
+// The (tile, channel-block range) pieces of a CTA, identical in every warp role.
+template <bool SK>
+struct Segs {
+    int a, b, n = 0;
+    __device__ __forceinline__ explicit Segs(const Params& p) {
+        if constexpr (SK) {
+            a = sk_start(p, blockIdx.x);
+            b = sk_start(p, blockIdx.x + 1);
+        } else {
+            a = blockIdx.x;
+            b = gridDim.x;
+        }
+    }
+    __device__ __forceinline__ bool next(const Params& p, int& tile, int& lo, int& hi) {
+        if constexpr (SK) {
+            if (a >= b) return false;
+            tile = a / p.num_cb;
+            lo = a - tile * p.num_cb;
+            hi = min(p.num_cb, lo + (b - a));
+            a += hi - lo;
+        } else {
+            if (a >= p.num_tiles) return false;
+            tile = a;
+            lo = 0;
+            hi = p.num_cb;
+            a += b;
+        }
+        ++n;
+        return true;
+    }
 };
 
 template <int P, int MM, int XM>
@@ -167,7 +205,7 @@ struct Cfg {
 
 // XM: 2 = TMA x box (N % 32 == 0), 3 = 32/N TMA boxes per nu-half (N in {4, 8, 16}: the
 // per-rank batches of batch sharding), 1 = cp.async 16 B gather, 0 = cp.async 4 B gather
-template <int P, int XM, int MM>
+template <int P, int XM, int MM, bool SK = false>
 __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__ Params p) {
     using G = Cfg<P, MM, XM>;
     constexpr int NH = G::NH;
@@ -189,7 +227,6 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     uint32_t* const tmem_slot = reinterpret_cast<uint32_t*>(smem + G::OFF_TMEM);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int NCB = p.num_cb;
 
     if (tid == 0) {
         for (int s = 0; s < G::U_SLOTS; ++s) {
@@ -221,7 +258,9 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         if (warp == XPROD_WARP) {
             // --------------------------- raw-x producer ---------------------------
             int gcb = 0;  // channel blocks issued so far (all tiles)
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+            Segs<SK> segs(p);
+            int tile, lo, hi;
+            while (segs.next(p, tile, lo, hi)) {
                 const int nu0 = (tile / p.num_kb) * TN;
                 int tma_n0[NH], tma_w0[NH], tma_h0[NH];
                 if constexpr (XM == 3) {
@@ -240,7 +279,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                     }
                     // x streams from HBM (first touch): warm L2 a few blocks ahead
                     if (lane == 0)
-                        for (int cb = 0; cb < X_PREFETCH && cb < NCB; ++cb)
+                        for (int cb = lo; cb < lo + X_PREFETCH && cb < hi; ++cb)
 #pragma unroll
                             for (int h = 0; h < NH; ++h)
                                 tma_prefetch_l2_4d(&p.tmx, tma_n0[h], tma_w0[h], tma_h0[h], cb * BC);
@@ -261,7 +300,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                     }
                     __syncwarp();
                 }
-                for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                for (int cb = lo; cb < hi; ++cb, ++gcb) {
                     const int xs = gcb % G::X_SLOTS;
                     if (gcb >= G::X_SLOTS) mbar_wait(&x_empty[xs], ((gcb / G::X_SLOTS) - 1) & 1);
                     float* xdst = sx + xs * (G::X_SLOT / 4);
@@ -285,7 +324,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                             mbar_arrive_expect_tx(&x_full[xs], G::X_SLOT);
 #pragma unroll
                             for (int h = 0; h < NH; ++h) {
-                                if (cb + X_PREFETCH < NCB)
+                                if (cb + X_PREFETCH < hi)
                                     tma_prefetch_l2_4d(&p.tmx, tma_n0[h], tma_w0[h], tma_h0[h], (cb + X_PREFETCH) * BC);
                                 tma_load_4d(xdst + h * (XS_BYTES / 4), &p.tmx, &x_full[xs], tma_n0[h], tma_w0[h],
                                             tma_h0[h], cb * BC);
@@ -314,9 +353,11 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         } else if (warp == PROD_WARP) {
             // ------------------------ transformed-filter producer -----------------
             int unit = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+            Segs<SK> segs(p);
+            int tile, lo, hi;
+            while (segs.next(p, tile, lo, hi)) {
                 const int kb = tile % p.num_kb;
-                for (int cb = 0; cb < NCB; ++cb) {
+                for (int cb = lo; cb < hi; ++cb) {
                     for (int h = 0; h < G::UNITS_PER_CB; ++h, ++unit) {
                         const int us = unit % G::U_SLOTS;
                         if (unit >= G::U_SLOTS) mbar_wait(&u_empty[us], ((unit / G::U_SLOTS) - 1) & 1);
@@ -333,10 +374,12 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             // ------------------------------ MMA issuer ----------------------------
             constexpr uint32_t IDESC = umma_idesc_tf32(MM, BN);
             int unit = 0, gcb = 0, it = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+            Segs<SK> segs(p);
+            int tile, lo, hi;
+            for (; segs.next(p, tile, lo, hi); ++it) {
                 if (it > 0) mbar_wait(acc_empty, (it - 1) & 1);  // epilogue drained TMEM
                 tc_fence_after();
-                for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+                for (int cb = lo; cb < hi; ++cb, ++gcb) {
                     const int vs = gcb & 1;
                     mbar_wait(&v_full[vs], (gcb >> 1) & 1);
                     for (int half = 0; half < G::UNITS_PER_CB; ++half, ++unit) {
@@ -357,7 +400,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                                     const uint32_t d = tmem + xi * BN + ((uint32_t)(16 * h) << 16);
                                     const uint32_t b0 = vbase + ((xi * NH + h) * P) * B_TILE;
                                     const uint64_t bb = umma_desc(b0, 128, 256);
-                                    umma_tf32(d, ab, bb, IDESC, cb > 0 ? 1u : 0u);
+                                    umma_tf32(d, ab, bb, IDESC, cb > lo ? 1u : 0u);
                                     if constexpr (P == 2) {
                                         const uint64_t as = umma_desc(a0 + G::A_TILE, 128, 256);
                                         const uint64_t bs = umma_desc(b0 + B_TILE, 128, 256);
@@ -388,8 +431,10 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         const int xnb = XM == 3 ? p.N : BN;
         const int xoff = (nl / xnb) * (BC * 16 * xnb) + cl * 16 * xnb + nl % xnb;
         int gcb = 0;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-            for (int cb = 0; cb < NCB; ++cb, ++gcb) {
+        Segs<SK> segs(p);
+        int tile, lo, hi;
+        while (segs.next(p, tile, lo, hi)) {
+            for (int cb = lo; cb < hi; ++cb, ++gcb) {
                 const int xs = gcb % G::X_SLOTS, vs = gcb & 1;
                 mbar_wait(&x_full[xs], (gcb / G::X_SLOTS) & 1);
                 float t[NH][16];
@@ -429,7 +474,9 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
         const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
         const size_t dW = (size_t)p.W * p.N;
         int it = 0;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+        Segs<SK> segs(p);
+        int tile, lo, hi;
+        for (; segs.next(p, tile, lo, hi); ++it) {
             const int k = (tile % p.num_kb) * MM + kl;
             const int nu0 = (tile / p.num_kb) * TN + hsel * BN;
             mbar_wait(acc_full, it & 1);
@@ -452,6 +499,18 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(acc_empty);  // TMEM free for the next tile's MMAs
+            if (SK && hi - lo != p.num_cb) {
+                // piece of a cut tile: partial outputs -> slot 2b (the CTA's first piece) or 2b + 1
+                // (its last), [kl][output][nu of the tile]; tc_fixup_kernel adds them
+                float* wk = p.sk_ws + ((size_t)(2 * blockIdx.x + (segs.n > 1 ? 1 : 0)) * MM + kl) * (4 * TN) + hsel * BN;
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+#pragma unroll
+                    for (int j = 0; j < BN; j += 4)
+                        *reinterpret_cast<float4*>(wk + q * TN + j) =
+                            make_float4(o[j][q], o[j + 1][q], o[j + 2][q], o[j + 3][q]);
+                continue;
+            }
             if (k >= p.K || nu0 >= p.NV) continue;
             if constexpr (XM == 2) {
                 // N % 32 == 0: the 32 nu are 32 consecutive n of one image tile -> 128 B rows
@@ -506,6 +565,72 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     tc_fence_before();
     __syncthreads();
     if (warp == 0) tmem_dealloc(tmem, 512);
+}
+
+// Stream-K fixup (as tc16_fixup_kernel): blocks 16i .. 16i+15 handle the tile cut by the range
+// boundary of CTA i + 1 when it is the first boundary inside that tile; y = sum of the pieces'
+// partials in CTA order.
+constexpr int FIX_PARTS = 16;
+template <int MM>
+__global__ void __launch_bounds__(256) tc_fixup_kernel(const __grid_constant__ Params p, int G) {
+    constexpr int TN = BN * (128 / MM);
+    constexpr int PER = MM * TN / FIX_PARTS / 256;
+    __shared__ int slots[256];
+    __shared__ int nseg;
+    const int b = blockIdx.x / FIX_PARTS + 1, part = blockIdx.x % FIX_PARTS;
+    const int ub = sk_start(p, b);
+    const int tile = ub / p.num_cb;
+    const int t0 = tile * p.num_cb, t1 = t0 + p.num_cb;
+    if (ub == t0 || sk_start(p, b - 1) > t0) return;
+    if (threadIdx.x == 0) {
+        int b0 = b - 1;
+        while (b0 > 0 && sk_start(p, b0) > t0) --b0;
+        int ns = 0, c0 = sk_start(p, b0);
+        for (int c = b0; c < G && c0 < t1 && ns < 256; ++c) {
+            const int c1 = sk_start(p, c + 1);
+            if (c1 > c0) slots[ns++] = 2 * c + (c0 < t0 ? 1 : 0);
+            c0 = c1;
+        }
+        nseg = ns;
+    }
+    __syncthreads();
+    const int ns = nseg;
+    const int kb = tile % p.num_kb, nb = tile / p.num_kb;
+    const size_t HWN = (size_t)p.H * p.W * p.N, dW = (size_t)p.W * p.N;
+    constexpr size_t SLOT = (size_t)MM * 4 * TN;
+    float o[PER][4];
+#pragma unroll
+    for (int i = 0; i < PER; ++i)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) o[i][q] = 0.f;
+    for (int sidx = 0; sidx < ns; ++sidx) {
+        const float* wk = p.sk_ws + slots[sidx] * SLOT;
+        float v[PER][4];
+#pragma unroll
+        for (int i = 0; i < PER; ++i) {
+            const int e = (part * PER + i) * 256 + threadIdx.x, kl = e / TN, j = e - kl * TN;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) v[i][q] = wk[((size_t)kl * 4 + q) * TN + j];
+        }
+#pragma unroll
+        for (int i = 0; i < PER; ++i)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) o[i][q] += v[i][q];
+    }
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+        const int e = (part * PER + i) * 256 + threadIdx.x, kl = e / TN, j = e - kl * TN;
+        const int k = kb * MM + kl, nu = nb * TN + j;
+        if (k >= p.K || nu >= p.NV) continue;
+        const int t = nu / p.N, n = nu - t * p.N;
+        const int th = t / p.TW, tw = t - th * p.TW;
+        const int i0 = 2 * th, j0 = 2 * tw;
+        float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+        yk[0] = o[i][0];
+        if (j0 + 1 < p.W) yk[p.N] = o[i][1];
+        if (i0 + 1 < p.H) yk[dW] = o[i][2];
+        if (i0 + 1 < p.H && j0 + 1 < p.W) yk[dW + p.N] = o[i][3];
+    }
 }
 
 }  // namespace tc

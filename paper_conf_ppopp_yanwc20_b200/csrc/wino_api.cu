@@ -263,15 +263,20 @@ wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem,
 }  // namespace
 
 namespace {
-std::atomic<uint64_t> g_attr_tc[2][4][2];
-template <int P, int XM, int MM>
+std::atomic<uint64_t> g_attr_tc[2][4][2][2];  // [P-1][XM][MM == 64][SK]
+template <int P, int XM, int MM, bool SK = false>
 wino_status_t launch_tc(const wino::tc::Params& prm, int64_t ctas, int dev, cudaStream_t st) {
-    auto kern = wino::tc::fused_tc_kernel<P, XM, MM>;
+    auto kern = wino::tc::fused_tc_kernel<P, XM, MM, SK>;
     const int smem = wino::tc::Cfg<P, MM, XM>::BYTES;
-    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc[P - 1][XM][MM == 64]);
+    wino_status_t s = ensure_smem_attr(kern, dev, smem, g_attr_tc[P - 1][XM][MM == 64][SK]);
     if (s != WINO_OK) return s;
     kern<<<dim3(static_cast<unsigned>(ctas)), wino::tc::NT, smem, st>>>(prm);
     cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess && SK && ctas > 1) {
+        wino::tc::tc_fixup_kernel<MM><<<dim3(static_cast<unsigned>(wino::tc::FIX_PARTS * (ctas - 1))), 256, 0, st>>>(
+            prm, static_cast<int>(ctas));
+        e = cudaGetLastError();
+    }
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 }  // namespace
@@ -547,8 +552,10 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
     wino_status_t s = check_shape(N, C, H, W, K, 1, 1);
     if (s != WINO_OK) return s;
     std::memset(plan, 0, sizeof(*plan));
-    if (variant == 1 || variant == 2) {  // tcgen05 TF32 (1) / 3xTF32 (2)
+    if (variant == 1 || variant == 2 || variant == 6 || variant == 7) {  // tcgen05 TF32 / 3xTF32 (+ workspace)
         using namespace wino::tc;
+        const bool with_ws = variant >= 6;
+        variant = with_ws ? variant - 5 : variant;
         const int64_t nv = int64_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
         const int mm = tc_mm(K, variant == 2 ? 2 : 1);
         plan->variant = variant;
@@ -562,6 +569,18 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->threads = NT;
         plan->smem_bytes = variant == 1 ? (mm == 64 ? Cfg<1, 64, 2>::BYTES : Cfg<1, 128, 2>::BYTES) : Cfg<2, 128, 2>::BYTES;
         plan->launches = 1;
+        if (with_ws && plan->load_x == 2 && mm == 128) {
+            int dev = -1, sms = 148;  // host-only planning unless an sm_100 device is current
+            if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+            else cudaGetLastError();
+            sms = sms < 256 ? sms : 256;
+            if (tc16_sk_pays(plan->ctas, (C + BC - 1) / BC, sms)) {
+                plan->stream_k = 1;
+                plan->launches = 2;
+                plan->ctas = sms;
+            }
+            plan->variant = variant + 5;
+        }
         return WINO_OK;
     }
     if (variant == 3 || variant == 5) {  // tcgen05 kind::f16 (FP16 / BF16, NEXT row N4); 5: with workspace
@@ -789,14 +808,18 @@ wino_status_t wino_filter_transform_tc(const float* w_dev, float* u_tc_dev, int 
 }
 
 
-wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, int N, int C, int H,
-                                      int W, int K, int pad, int stride, wino_tc_mode_t mode,
-                                      wino_stream_t stream) {
+extern "C++" {
+namespace {
+// sk: 0 = never, 1 = planner's choice, 2 = always (TMA x paths; needs ws >= tc16_sk_bytes(SMs))
+wino_status_t conv_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, int N, int C, int H, int W, int K,
+                      int pad, int stride, wino_tc_mode_t mode, int sk, void* ws_dev, size_t ws_bytes,
+                      wino_stream_t stream) {
     if (!x_dev || !u_tc_dev || !y_dev) return WINO_ERR_INVALID_ARG;
     if (mode != WINO_TC_TF32 && mode != WINO_TC_3XTF32) return WINO_ERR_INVALID_ARG;
     wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
     if (s != WINO_OK) return s;
-    if (!aligned16(x_dev) || !aligned16(u_tc_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    if (!aligned16(x_dev) || !aligned16(u_tc_dev) || !aligned16(y_dev) || (ws_dev && !aligned16(ws_dev)))
+        return WINO_ERR_MISALIGNED;
     const size_t hwn = size_t(H) * W * N;
     const size_t yb = size_t(K) * hwn * 4;
     if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) ||
@@ -829,9 +852,31 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
         const cuuint32_t box[4] = {cuuint32_t(xm == 2 ? BN : N), 4, 4, BC};
         if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
     }
-    const int sms = sm_count(dev);
-    const int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
+    const int sms = sm_count(dev) < 256 ? sm_count(dev) : 256;
+    int64_t ctas = prm.num_tiles < sms ? prm.num_tiles : sms;  // persistent
+    if (ws_dev && (overlaps(ws_dev, ws_bytes, x_dev, size_t(C) * hwn * 4) || overlaps(ws_dev, ws_bytes, y_dev, yb) ||
+                   overlaps(ws_dev, ws_bytes, u_tc_dev, wino_filter_workspace_bytes_tc(C, K, mode))))
+        return WINO_ERR_INVALID_ARG;
+    const double units = double(prm.num_tiles) * prm.num_cb;
+    // (128-filter tiles only: the 64 x 64 tiles of K <= 64 put a cut tile's last 8 nu wrong in
+    // one parity case -- not resolved; no BASELINE shape needs stream-K there)
+    if (sk == 2 && mm == 64) return WINO_ERR_UNSUPPORTED;
+    const bool sk_ok = xm >= 2 && mm == 128 && ws_dev && ws_bytes >= tc16_sk_bytes(sms) && units < 2147483647.0;
+    if (sk == 2 && !sk_ok) return WINO_ERR_INVALID_ARG;
+    const bool use_sk = sk == 2 || (sk == 1 && sk_ok && tc16_sk_pays(prm.num_tiles, prm.num_cb, sms));
+    if (use_sk) {  // stream-K: equal (tile, channel block) ranges on every SM + fixup
+        ctas = sms;
+        prm.sk_ws = static_cast<float*>(ws_dev);
+        prm.sk_q = static_cast<int>(int64_t(units) / sms);
+        prm.sk_r = static_cast<int>(int64_t(units) % sms);
+    }
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (use_sk) {
+        if (mode == WINO_TC_TF32)
+            return xm == 3 ? launch_tc<1, 3, 128, true>(prm, ctas, dev, st)
+                           : launch_tc<1, 2, 128, true>(prm, ctas, dev, st);
+        return xm == 3 ? launch_tc<2, 3, 128, true>(prm, ctas, dev, st) : launch_tc<2, 2, 128, true>(prm, ctas, dev, st);
+    }
     if (mode == WINO_TC_TF32 && mm == 64) {
         if (xm == 3) return launch_tc<1, 3, 64>(prm, ctas, dev, st);
         if (xm == 2) return launch_tc<1, 2, 64>(prm, ctas, dev, st);
@@ -848,6 +893,24 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
     if (xm == 2) return launch_tc<2, 2, 128>(prm, ctas, dev, st);
     if (xm == 1) return launch_tc<2, 1, 128>(prm, ctas, dev, st);
     return launch_tc<2, 0, 128>(prm, ctas, dev, st);
+}
+}  // namespace
+}  // extern "C++"
+
+wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, int N, int C, int H,
+                                      int W, int K, int pad, int stride, wino_tc_mode_t mode,
+                                      wino_stream_t stream) {
+    return conv_tc(x_dev, u_tc_dev, y_dev, N, C, H, W, K, pad, stride, mode, 0, nullptr, 0, stream);
+}
+
+size_t wino_tc_workspace_bytes(int N, int C, int H, int W, int K) { return wino_half_workspace_bytes(N, C, H, W, K); }
+
+wino_status_t wino_conv2d_f2x3_fwd_tc_ws(const float* x_dev, const float* u_tc_dev, float* y_dev, int N, int C,
+                                         int H, int W, int K, int pad, int stride, wino_tc_mode_t mode, int sk,
+                                         void* ws_dev, size_t ws_bytes, wino_stream_t stream) {
+    if (sk < 0 || sk > 2 || (ws_bytes > 0 && !ws_dev)) return WINO_ERR_INVALID_ARG;
+    const int m = sk == 0 ? 1 : (sk == 1 ? 0 : 2);  // API 0 auto / 1 off / 2 force
+    return conv_tc(x_dev, u_tc_dev, y_dev, N, C, H, W, K, pad, stride, mode, m, ws_dev, ws_bytes, stream);
 }
 
 

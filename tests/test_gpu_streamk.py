@@ -141,3 +141,33 @@ def test_streamk_argument_errors(wino):
     st = L.wino_conv2d_f2x3_fwd_ws(p(x.data_ptr()), p(u.data_ptr()), p(y.data_ptr()), cfg.N, cfg.C, cfg.H, cfg.W,
                                    cfg.K, 1, 1, 1, None, 0, None)
     assert st == 0  # stream-K off needs no workspace
+
+
+# TF32 / 3xTF32 tcgen05 kernel, forced stream-K (TMA x paths: N % 32 == 0 or N in {4, 8, 16})
+TC_SK = [(4, 512, 512, 7, 7), (8, 256, 256, 14, 14), (16, 128, 128, 12, 10), (32, 64, 64, 30, 30),
+         (32, 72, 200, 5, 9)]
+
+
+@pytest.mark.parametrize("variant,tol", [("tf32", 5e-3), ("3xtf32", 1e-4)])
+@pytest.mark.parametrize("shape", TC_SK, ids=[str(s) for s in TC_SK])
+def test_tc_streamk(wino, shape, variant, tol):
+    N, C, K, H, W = shape
+    cfg = Conv3x3Config("sk", N, C, K, H, W)
+    if variant == "tf32" and K <= 64:  # 64-filter tiles: stream-K not offered (include/wino.h)
+        x, w = make_inputs(cfg)
+        u = wino.filter_transform_tc(w.to(DEV), variant)
+        ws = torch.empty(wino.tc_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+        with pytest.raises(wino.WinoError, match="UNSUPPORTED"):
+            wino.conv2d_tc(x.to(DEV), u, ws=ws, stream_k="on")
+        return
+    for kind in ("smallint", "uniform"):
+        x, w = make_inputs(cfg, kind=kind)
+        u = wino.filter_transform_tc(w.to(DEV), variant)
+        ws = torch.empty(wino.tc_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+        y = wino.conv2d_tc(x.to(DEV), u, ws=ws, stream_k="on").cpu()
+        torch.cuda.synchronize()
+        ref = oracle.direct_conv(x, w)
+        if kind == "smallint":  # exact in TF32
+            assert np.array_equal(y.double().numpy(), ref)
+        else:
+            assert oracle.max_rel_err(y.double().numpy(), ref) <= tol
