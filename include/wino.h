@@ -241,7 +241,7 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
                                       wino_tc_mode_t mode, wino_stream_t stream);
 /* The same with a caller workspace that enables a stream-K plan for tile-starved shapes (as
  * wino_conv2d_f2x3_fwd_half_ws; only the TMA x paths, N % 32 == 0 or N in {4, 8, 16}):
- *   ws_dev / ws_bytes : >= wino_tc_workspace_bytes(N,C,H,W,K) (SMs x 64 KiB), 16-byte aligned,
+ *   ws_dev / ws_bytes : >= wino_tc_workspace_bytes(N,C,H,W,K) (SMs x 128 KiB), 16-byte aligned,
  *                       not overlapping x, u_tc or y; may be NULL / 0 when sk = 1.
  *   sk                : 0 = planner's choice, 1 = never, 2 = always (short workspace or a
  *                       gather-path N -> WINO_ERR_INVALID_ARG; TF32 with K <= 64, i.e.
@@ -283,7 +283,7 @@ wino_status_t wino_conv2d_f2x3_fwd_half(const void* x_dev, const void* u_h_dev, 
 /* The same with a caller workspace that enables a stream-K plan (as wino_conv2d_f2x3_fwd_ws:
  * equal (tile, channel block) ranges on every SM; pieces of cut tiles leave FP32 partial
  * outputs in the workspace, a fixup kernel adds them in CTA order and rounds once):
- *   ws_dev / ws_bytes : >= wino_half_workspace_bytes(N,C,H,W,K) (SMs x 64 KiB), 16-byte
+ *   ws_dev / ws_bytes : >= wino_half_workspace_bytes(N,C,H,W,K) (SMs x 128 KiB), 16-byte
  *                       aligned, not overlapping x, u or y; may be NULL / 0 when sk = 1.
  *   sk                : 0 = planner's choice, 1 = never, 2 = always (a short workspace ->
  *                       WINO_ERR_INVALID_ARG). */

@@ -95,7 +95,7 @@ bool overlaps(const void* a, size_t na, const void* b, size_t nb) {
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
-// stream-K workspace of the 16-bit kernel: 2 slots of MM x 4 x TN FP32 partials per CTA (64 KiB)
+// stream-K workspace of the tensor-core kernels: 2 slots of MM x 4 x TN FP32 partials (64 KiB each) per CTA
 size_t tc16_sk_bytes(int ctas) { return size_t(ctas) * 2 * 128 * 4 * 32 * sizeof(float); }
 // stream-K pays for the 16-bit kernel only when whole tiles would leave most SMs idle: its pieces
 // run ~1.5x slower per channel block than the persistent schedule (measured: conv5 at P = 1
