@@ -315,8 +315,8 @@ def main():
         nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
         nonfused = variant == "nonfused_fp32"  # NEXT row N3: ITF -> 16 cuBLAS SGEMMs -> OTF (Sec. 9)
         half = variant in ("fp16", "bf16")  # NEXT row N4: 16-bit x, w, y on tcgen05 kind::f16 (Sec. 8.3)
-        if f4:
-            launches = sum(2 for d in per if d["n"] > 0)
+        if f4:  # FTF4 + conv (+ a stream-K fixup where the planner takes it: counted as taken)
+            launches = sum(3 for d in per if d["n"] > 0)
         elif half:  # FTF + conv (+ stream-K fixup with the workspace, variant 5 plans it)
             launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=5).launches
                            for d in per if d["n"] > 0)
@@ -334,6 +334,9 @@ def main():
             # transformed filter: computed on rank 0, broadcast once over NVLink (NCCL)
             if f4:
                 d["u"] = torch.empty((d["cfg"].C, 6, 6, d["cfg"].K), dtype=torch.float32, device=dev)
+                c = d["cfg"]
+                d["ws_f4"] = torch.empty(max(wino.f4_workspace_bytes(max(d["n"], 1), c.C, c.H, c.W, c.K), 16),
+                                         dtype=torch.uint8, device=dev)
                 if rank == 0:
                     wino.filter_transform_f4(d["w"], out=d["u"])
                 if world > 1:
@@ -404,7 +407,7 @@ def main():
                     wino.filter_transform(d["w"], out=d["u"], stream=ftf_stream)
             if conv:
                 if f4:
-                    wino.conv2d_f4(d["x"], d["u"], out=d["y"])
+                    wino.conv2d_f4(d["x"], d["u"], out=d["y"], ws=d["ws_f4"])
                 elif tc:
                     wino.conv2d_tc(d["x"], d["u"], out=d["y"], ws=d["ws_tc"])
                 elif nchw:

@@ -323,6 +323,15 @@ wino_status_t wino_filter_transform_f4(const float* w_dev, float* u4_dev, int C,
 wino_status_t wino_conv2d_f4x3_fwd(const float* x_dev, const float* u4_dev, float* y_dev,
                                    int N, int C, int H, int W, int K, int pad, int stride,
                                    wino_stream_t stream);
+/* The same with a caller workspace that enables a stream-K plan (the scheme of
+ * wino_conv2d_f2x3_fwd_ws: equal (tile, 4-channel block) ranges per SM, pieces of cut tiles
+ * leave their 16 partial outputs per (k, nu) in the workspace, a fixup kernel adds them in CTA
+ * order):  ws >= wino_f4_workspace_bytes(N,C,H,W,K) (SMs x 128 KiB), 16-byte aligned, not
+ * overlapping x, u4 or y; sk 0 = planner's choice, 1 = never, 2 = always. */
+size_t wino_f4_workspace_bytes(int N, int C, int H, int W, int K);
+wino_status_t wino_conv2d_f4x3_fwd_ws(const float* x_dev, const float* u4_dev, float* y_dev,
+                                      int N, int C, int H, int W, int K, int pad, int stride,
+                                      int sk, void* ws_dev, size_t ws_bytes, wino_stream_t stream);
 
 /*
  * Multi-layer end-to-end call on HOST buffers with copy/compute overlap: for

@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes",
+    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -137,6 +137,11 @@ def lib() -> ctypes.CDLL:
     L.wino_filter_transform_f4.argtypes = [vp, vp, i, i, vp]
     L.wino_conv2d_f4x3_fwd.restype = i
     L.wino_conv2d_f4x3_fwd.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp]
+    if hasattr(L, "wino_conv2d_f4x3_fwd_ws") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_f4_workspace_bytes.restype = st
+        L.wino_f4_workspace_bytes.argtypes = [i, i, i, i, i]
+        L.wino_conv2d_f4x3_fwd_ws.restype = i
+        L.wino_conv2d_f4x3_fwd_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp, st, vp]
     if hasattr(L, "wino_conv2d_f2x3_fwd_half") or not os.environ.get("WINO_LIB_PATH"):
         L.wino_filter_workspace_bytes_half.restype = st
         L.wino_filter_workspace_bytes_half.argtypes = [i, i]
@@ -535,9 +540,16 @@ def filter_transform_f4(w: torch.Tensor, out: torch.Tensor | None = None, stream
     return out
 
 
-def conv2d_f4(x: torch.Tensor, u4: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+def f4_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
+    """Device workspace that lets ``conv2d_f4`` use the stream-K plan (wino_f4_workspace_bytes)."""
+    return int(lib().wino_f4_workspace_bytes(N, C, H, W, K))
+
+
+def conv2d_f4(x: torch.Tensor, u4: torch.Tensor, out: torch.Tensor | None = None, stream=None,
+              ws: torch.Tensor | None = None, stream_k: str = "auto") -> torch.Tensor:
     """NEXT row N1: fused Winograd F(4x4,3x3) forward conv (FP32), pad 1 stride 1:
-    x (C,H,W,N), u4 (C,6,6,K) -> y (K,H,W,N).  Needs N % 16 == 0 and K % 4 == 0."""
+    x (C,H,W,N), u4 (C,6,6,K) -> y (K,H,W,N).  Needs N % 16 == 0 and K % 4 == 0.  ws (>=
+    f4_workspace_bytes) enables the stream-K plan (wino_conv2d_f4x3_fwd_ws)."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u4, "u4", 4)
     C, H, W, N = x.shape
@@ -551,10 +563,17 @@ def conv2d_f4(x: torch.Tensor, u4: torch.Tensor, out: torch.Tensor | None = None
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N):
         raise ValueError("out must be (K,H,W,N)")
+    args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u4.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+            N, C, H, W, K, 1, 1)
     with torch.cuda.device(x.device):
-        _check(lib().wino_conv2d_f4x3_fwd(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u4.data_ptr()),
-                                          ctypes.c_void_p(out.data_ptr()), N, C, H, W, K, 1, 1,
-                                          _stream_ptr(stream)), "wino_conv2d_f4x3_fwd")
+        if ws is not None or stream_k == "on":
+            if ws is not None and not ws.is_cuda:
+                raise ValueError("ws must be a CUDA tensor")
+            wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
+            _check(lib().wino_conv2d_f4x3_fwd_ws(*args, {"auto": 0, "off": 1, "on": 2}[stream_k], wp, wb,
+                                                 _stream_ptr(stream)), "wino_conv2d_f4x3_fwd_ws")
+        else:
+            _check(lib().wino_conv2d_f4x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f4x3_fwd")
     return out
 
 

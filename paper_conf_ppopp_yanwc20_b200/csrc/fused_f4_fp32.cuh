@@ -113,6 +113,45 @@ struct __align__(64) Params {
     int num_kb;  // ceil(K/64)
     int num_it;  // ceil(C/4)
     int num_tiles;
+    // stream-K (SK = true; the scheme of fused_fp32_ws.cuh): units = tile * num_it + g, CTA b takes
+    // [b*q + min(b, r), ...); pieces of cut tiles leave their 16 partial outputs per (k, nu) in
+    // sk_ws: 2 slots of [64 k][16 outputs][16 nu] floats (64 KiB) per CTA
+    float* __restrict__ sk_ws;
+    int sk_q, sk_r;
+};
+
+__host__ __device__ __forceinline__ int sk_start(const Params& p, int b) { return b * p.sk_q + min(b, p.sk_r); }
+
+// The (tile, channel-block range) pieces of a CTA, identical in every warp role.
+template <bool SK>
+struct Segs {
+    int a, b, n = 0;
+    __device__ __forceinline__ explicit Segs(const Params& p) {
+        if constexpr (SK) {
+            a = sk_start(p, blockIdx.x);
+            b = sk_start(p, blockIdx.x + 1);
+        } else {
+            a = blockIdx.x;
+            b = gridDim.x;
+        }
+    }
+    __device__ __forceinline__ bool next(const Params& p, int& tile, int& lo, int& hi) {
+        if constexpr (SK) {
+            if (a >= b) return false;
+            tile = a / p.num_it;
+            lo = a - tile * p.num_it;
+            hi = min(p.num_it, lo + (b - a));
+            a += hi - lo;
+        } else {
+            if (a >= p.num_tiles) return false;
+            tile = a;
+            lo = 0;
+            hi = p.num_it;
+            a += b;
+        }
+        ++n;
+        return true;
+    }
 };
 
 // FTF for F(4x4): u4 (C,6,6,K)
@@ -128,6 +167,7 @@ __global__ void __launch_bounds__(256) ftf4_kernel(const float* __restrict__ w, 
     for (int e = 0; e < 36; ++e) u[((size_t)c * 36 + e) * K + k] = t[e];
 }
 
+template <bool SK = false>
 __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(1024) float smem[];
     float* const vs = smem + S * STAGE_FLOATS;
@@ -137,7 +177,6 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
     uint64_t* const vfull = empty + S;
     uint64_t* const vempty = vfull + SV;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int NIT = p.num_it;
 
     if (tid == 0) {
         tma_prefetch_desc(&p.tmx);
@@ -161,11 +200,13 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
             if (lane == 0) {
                 constexpr uint32_t kBytes = (US_FLOATS + XS_FLOATS) * 4;
                 int G = 0;
-                for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+                Segs<SK> segs(p);
+                int tile, lo, hi;
+                while (segs.next(p, tile, lo, hi)) {
                     const int k0 = (tile % p.num_kb) * BK, nu0 = (tile / p.num_kb) * BN;
                     const int t = nu0 / p.N, n0 = nu0 - t * p.N;
                     const int th = t / p.TW, tw = t - th * p.TW;
-                    for (int g = 0; g < NIT; ++g, ++G) {
+                    for (int g = lo; g < hi; ++g, ++G) {
                         const int slot = G % S;
                         if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
                         float* us = smem + slot * STAGE_FLOATS;
@@ -183,8 +224,10 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
         const int it_thr = tid - (COMPUTE_WARPS + 1) * 32;  // 0..63
         const int c = it_thr >> 4, nl = it_thr & 15;
         int G = 0;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-            for (int g = 0; g < NIT; ++g, ++G) {
+        Segs<SK> segs(p);
+        int tile, lo, hi;
+        while (segs.next(p, tile, lo, hi)) {
+            for (int g = lo; g < hi; ++g, ++G) {
                 const int slot = G % S, vb = G % SV;
                 mbar_wait(&full[slot], (G / S) & 1);
                 if (G >= SV) mbar_wait(&vempty[vb], ((G / SV) - 1) & 1);
@@ -228,8 +271,12 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
     const size_t HWN = (size_t)p.H * p.W * p.N;
     const size_t dW = (size_t)p.W * p.N;
     int G = 0;
-    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+    Segs<SK> segs(p);
+    int tile, lo, hi;
+    while (segs.next(p, tile, lo, hi)) {
         const int k0 = (tile % p.num_kb) * BK, nu0 = (tile / p.num_kb) * BN;
+        // stream-K piece of a cut tile -> workspace slot 2b (the CTA's first piece) or 2b + 1
+        const int sk_slot = (SK && hi - lo != p.num_it) ? 2 * static_cast<int>(blockIdx.x) + (segs.n > 1 ? 1 : 0) : -1;
         float acc[3][8][4];
 #pragma unroll
         for (int q = 0; q < 3; ++q)
@@ -237,7 +284,7 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
             for (int i = 0; i < 8; ++i)
 #pragma unroll
                 for (int j = 0; j < 4; ++j) acc[q][i][j] = 0.f;
-        for (int g = 0; g < NIT; ++g, ++G) {
+        for (int g = lo; g < hi; ++g, ++G) {
             const int slot = G % S, vb = G % SV;
             mbar_wait(&full[slot], (G / S) & 1);
             mbar_wait(&vfull[vb], (G / SV) & 1);
@@ -302,17 +349,73 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
                         for (int a = 0; a < 4; ++a) tt[a][b] = o[a];
                     }
                     float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+                    float* wk = SK ? p.sk_ws + ((size_t)sk_slot * BK + kl) * (16 * BN) + nl : nullptr;
 #pragma unroll
                     for (int a = 0; a < 4; ++a) {
                         float o[4];
                         at4_vec(tt[a], o);
 #pragma unroll
-                        for (int b = 0; b < 4; ++b)
-                            if (i0 + a < p.H && j0 + b < p.W) yk[a * dW + b * p.N] = o[b];
+                        for (int b = 0; b < 4; ++b) {
+                            if (SK && sk_slot >= 0) wk[(a * 4 + b) * BN] = o[b];  // partial: [kl][a*4+b][nu]
+                            else if (i0 + a < p.H && j0 + b < p.W) yk[a * dW + b * p.N] = o[b];
+                        }
                     }
                 }
             }
         }
+    }
+}
+
+// Stream-K fixup: blocks 16i .. 16i+15 handle the tile cut by the range boundary of CTA i + 1
+// when it is the first boundary inside that tile, 1/16 of its 64 k x 16 nu x 16 outputs each:
+// y = sum of the pieces' partials in CTA order (deterministic).
+constexpr int FIX_PARTS = 16;
+__global__ void __launch_bounds__(256) f4_fixup_kernel(const __grid_constant__ Params p, int G) {
+    constexpr int PER = BK * BN * 16 / FIX_PARTS / 256;  // 4 outputs per thread
+    __shared__ int slots[256];
+    __shared__ int nseg;
+    const int b = blockIdx.x / FIX_PARTS + 1, part = blockIdx.x % FIX_PARTS;
+    const int ub = sk_start(p, b);
+    const int tile = ub / p.num_it;
+    const int t0 = tile * p.num_it, t1 = t0 + p.num_it;
+    if (ub == t0 || sk_start(p, b - 1) > t0) return;
+    if (threadIdx.x == 0) {
+        int b0 = b - 1;
+        while (b0 > 0 && sk_start(p, b0) > t0) --b0;
+        int ns = 0, c0 = sk_start(p, b0);
+        for (int c = b0; c < G && c0 < t1 && ns < 256; ++c) {
+            const int c1 = sk_start(p, c + 1);
+            if (c1 > c0) slots[ns++] = 2 * c + (c0 < t0 ? 1 : 0);
+            c0 = c1;
+        }
+        nseg = ns;
+    }
+    __syncthreads();
+    const int ns = nseg;
+    const int kb = tile % p.num_kb, nb = tile / p.num_kb;
+    const size_t HWN = (size_t)p.H * p.W * p.N, dW = (size_t)p.W * p.N;
+    constexpr size_t SLOT = (size_t)BK * 16 * BN;
+    float o[PER];
+#pragma unroll
+    for (int i = 0; i < PER; ++i) o[i] = 0.f;
+    for (int sidx = 0; sidx < ns; ++sidx) {
+        const float* wk = p.sk_ws + slots[sidx] * SLOT;
+        float v[PER];
+#pragma unroll
+        for (int i = 0; i < PER; ++i) v[i] = wk[(part * PER + i) * 256 + threadIdx.x];  // [kl][a*4+b][nu]
+#pragma unroll
+        for (int i = 0; i < PER; ++i) o[i] += v[i];
+    }
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+        const int e = (part * PER + i) * 256 + threadIdx.x;
+        const int nl = e % BN, ab = (e / BN) % 16, kl = e / (16 * BN);
+        const int k = kb * BK + kl, nu = nb * BN + nl;
+        if (k >= p.K || nu >= p.NV) continue;
+        const int t = nu / p.N, n = nu - t * p.N;
+        const int th = t / p.TW, tw = t - th * p.TW;
+        const int a = ab >> 2, bb = ab & 3, i0 = 4 * th + a, j0 = 4 * tw + bb;
+        if (i0 < p.H && j0 < p.W) p.y[(size_t)k * HWN + (size_t)i0 * dW + (size_t)j0 * p.N + n] = o[i];
     }
 }
 

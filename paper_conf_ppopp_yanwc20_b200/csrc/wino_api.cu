@@ -100,6 +100,8 @@ size_t tc16_sk_bytes(int ctas) { return size_t(ctas) * 2 * 128 * 4 * 32 * sizeof
 // stream-K pays for the 16-bit kernel only when whole tiles would leave most SMs idle: its pieces
 // run ~1.5x slower per channel block than the persistent schedule (measured: conv5 at P = 1
 // 38.9 -> 52 us, conv2 175 -> 204 us; at P = 8 conv5 with 8 tiles 325 -> 42 us)
+// stream-K workspace of the F(4x4) kernel: 2 slots of 64 k x 16 outputs x 16 nu floats per CTA
+size_t f4_sk_bytes(int ctas) { return size_t(ctas) * 2 * 64 * 16 * 16 * sizeof(float); }
 bool tc16_sk_pays(int64_t tiles, int ncb, int sms) {
     const double units = double(tiles) * ncb, reg = std::ceil(double(tiles) / sms) * ncb;
     return 2 * tiles <= sms && 1.5 * std::ceil(units / sms) + 3.0 < 0.9 * reg;
@@ -1235,14 +1237,19 @@ wino_status_t wino_filter_transform_f4(const float* w_dev, float* u4_dev, int C,
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 
-wino_status_t wino_conv2d_f4x3_fwd(const float* x_dev, const float* u4_dev, float* y_dev, int N, int C, int H,
-                                   int W, int K, int pad, int stride, wino_stream_t stream) {
+extern "C++" {
+namespace {
+std::atomic<uint64_t> g_attr_f4_sk;
+// sk: 0 = never, 1 = planner's choice, 2 = always (needs ws >= f4 workspace bytes)
+wino_status_t conv_f4(const float* x_dev, const float* u4_dev, float* y_dev, int N, int C, int H, int W, int K,
+                      int pad, int stride, int sk, void* ws_dev, size_t ws_bytes, wino_stream_t stream) {
     if (!x_dev || !u4_dev || !y_dev) return WINO_ERR_INVALID_ARG;
     wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
     if (s != WINO_OK) return s;
     if (int64_t(36) * C * K > kMaxElems) return WINO_ERR_TOO_LARGE;
     if (N % 16 != 0 || K % 4 != 0) return WINO_ERR_UNSUPPORTED;
-    if (!aligned16(x_dev) || !aligned16(u4_dev) || !aligned16(y_dev)) return WINO_ERR_MISALIGNED;
+    if (!aligned16(x_dev) || !aligned16(u4_dev) || !aligned16(y_dev) || (ws_dev && !aligned16(ws_dev)))
+        return WINO_ERR_MISALIGNED;
     const size_t hwn = size_t(H) * W * N;
     const size_t yb = size_t(K) * hwn * 4;
     if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) || overlaps(y_dev, yb, u4_dev, size_t(36) * C * K * 4))
@@ -1273,13 +1280,65 @@ wino_status_t wino_conv2d_f4x3_fwd(const float* x_dev, const float* u4_dev, floa
         const cuuint32_t box[3] = {BK, 36, BC};
         if (!encode_map(&prm.tmu, u4_dev, 3, dims, box)) return cuda_fail(cudaErrorInvalidValue);
     }
-    auto kern = fused_f4_kernel;
-    if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4)) != WINO_OK) return s;
-    const int sms = sm_count(dev);
-    const int grid = prm.num_tiles < sms ? prm.num_tiles : sms;
-    kern<<<grid, NT, Smem::bytes, reinterpret_cast<cudaStream_t>(stream)>>>(prm);
-    cudaError_t e = cudaGetLastError();
+    if (ws_dev && (overlaps(ws_dev, ws_bytes, x_dev, size_t(C) * hwn * 4) || overlaps(ws_dev, ws_bytes, y_dev, yb) ||
+                   overlaps(ws_dev, ws_bytes, u4_dev, size_t(36) * C * K * 4)))
+        return WINO_ERR_INVALID_ARG;
+    const int sms = sm_count(dev) < 256 ? sm_count(dev) : 256;
+    int grid = prm.num_tiles < sms ? prm.num_tiles : sms;
+    // stream-K (as the F(2x2) kernel): estimates in 4-channel-block times, tile epilogue ~2 blocks
+    const double units = double(prm.num_tiles) * prm.num_it;
+    const bool sk_ok = ws_dev && ws_bytes >= f4_sk_bytes(sms) && units < 2147483647.0;
+    if (sk == 2 && !sk_ok) return WINO_ERR_INVALID_ARG;
+    bool use_sk = sk == 2;
+    if (sk == 1 && sk_ok) {
+        const double reg = std::ceil(double(prm.num_tiles) / sms) * (prm.num_it + 2.0);
+        use_sk = std::ceil(units / sms) + 2.0 * (double(prm.num_tiles) / sms + 1.0) + 4.0 < 0.97 * reg;
+    }
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    cudaError_t e;
+    if (use_sk) {
+        grid = sms;
+        prm.sk_ws = static_cast<float*>(ws_dev);
+        prm.sk_q = static_cast<int>(int64_t(units) / sms);
+        prm.sk_r = static_cast<int>(int64_t(units) % sms);
+        auto kern = fused_f4_kernel<true>;
+        if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4_sk)) != WINO_OK) return s;
+        kern<<<grid, NT, Smem::bytes, st>>>(prm);
+        e = cudaGetLastError();
+        if (e == cudaSuccess && grid > 1) {
+            f4_fixup_kernel<<<FIX_PARTS * (grid - 1), 256, 0, st>>>(prm, grid);
+            e = cudaGetLastError();
+        }
+    } else {
+        auto kern = fused_f4_kernel<false>;
+        if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4)) != WINO_OK) return s;
+        kern<<<grid, NT, Smem::bytes, st>>>(prm);
+        e = cudaGetLastError();
+    }
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+}  // namespace
+}  // extern "C++"
+
+wino_status_t wino_conv2d_f4x3_fwd(const float* x_dev, const float* u4_dev, float* y_dev, int N, int C, int H,
+                                   int W, int K, int pad, int stride, wino_stream_t stream) {
+    return conv_f4(x_dev, u4_dev, y_dev, N, C, H, W, K, pad, stride, 0, nullptr, 0, stream);
+}
+
+size_t wino_f4_workspace_bytes(int N, int C, int H, int W, int K) {
+    if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
+    int dev = -1, sms = 148;
+    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+    else cudaGetLastError();
+    return f4_sk_bytes(sms < 256 ? sms : 256);
+}
+
+wino_status_t wino_conv2d_f4x3_fwd_ws(const float* x_dev, const float* u4_dev, float* y_dev, int N, int C, int H,
+                                      int W, int K, int pad, int stride, int sk, void* ws_dev, size_t ws_bytes,
+                                      wino_stream_t stream) {
+    if (sk < 0 || sk > 2 || (ws_bytes > 0 && !ws_dev)) return WINO_ERR_INVALID_ARG;
+    const int m = sk == 0 ? 1 : (sk == 1 ? 0 : 2);  // API 0 auto / 1 off / 2 force
+    return conv_f4(x_dev, u4_dev, y_dev, N, C, H, W, K, pad, stride, m, ws_dev, ws_bytes, stream);
 }
 
 }  // extern "C"

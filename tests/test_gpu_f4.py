@@ -98,3 +98,25 @@ def test_f4_unsupported_shapes_raise(wino, shape):
     u4 = torch.zeros((C, 6, 6, K), device=DEV)
     with pytest.raises(wino.WinoError, match="UNSUPPORTED"):
         wino.conv2d_f4(x, u4)
+
+
+# stream-K plan (workspace): ranges shorter than a tile, spanning tiles, tails; forced and auto
+F4_SK = [(16, 512, 512, 7, 7), (32, 256, 256, 14, 14), (16, 64, 64, 28, 28), (32, 13, 132, 6, 10),
+         (16, 3, 8, 5, 5)]
+
+
+@pytest.mark.parametrize("mode", ["on", "auto"])
+@pytest.mark.parametrize("shape", F4_SK, ids=[str(s) for s in F4_SK])
+def test_f4_stream_k(wino, shape, mode):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("f4sk", N, C, K, H, W), kind="uniform", seed_x=61, seed_w=62)
+    u4 = wino.filter_transform_f4(w.to(DEV))
+    ws = torch.empty(wino.f4_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+    y = wino.conv2d_f4(x.to(DEV), u4, ws=ws, stream_k=mode)
+    torch.cuda.synchronize()
+    yd = y.cpu().double().numpy()
+    assert np.isfinite(yd).all()
+    assert oracle.max_rel_err(yd, oracle.direct_conv(x, w)) <= F4_TOL
+    y2 = wino.conv2d_f4(x.to(DEV), u4, ws=ws, stream_k=mode)
+    torch.cuda.synchronize()
+    assert torch.equal(y.cpu(), y2.cpu())  # deterministic
