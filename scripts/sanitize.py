@@ -14,9 +14,26 @@ only = sys.argv[1] if len(sys.argv) > 1 else "all"
 for cfg in shapes:
     x, w = make_inputs(cfg)
     x, w = x.cuda(), w.cuda()
-    if only in ("all", "fp32"):
+    if only in ("all", "fp32", "sk"):
         u = wino.filter_transform(w)
         y = wino.conv2d(x, u)
+        if cfg.N % 32 == 0 or cfg.N in (4, 8, 16):  # stream-K (forced) + fixup
+            ws = torch.empty(wino.conv_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
+                             device="cuda")
+            y = wino.conv2d(x, u, ws=ws, stream_k="on")
+            if cfg.K > 64:
+                y = wino.conv2d_tc(x, wino.filter_transform_tc(w, "tf32"), ws=ws.new_empty(
+                    wino.tc_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K)), stream_k="on")
+            wsh = torch.empty(wino.half_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
+                              device="cuda")
+            y = wino.conv2d_half(x.half(), wino.filter_transform_half(w.half()), ws=wsh, stream_k="on")
+            if cfg.N % 16 == 0:
+                y = wino.conv2d_f4(x, wino.filter_transform_f4(w), stream_k="on", ws=torch.empty(
+                    wino.f4_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8, device="cuda"))
+        wsn = torch.empty(wino.nchw_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
+                          device="cuda")
+        y = wino.conv2d_nchw(x.permute(3, 0, 1, 2).contiguous(),
+                             wino.filter_transform_kcrs(w.permute(3, 0, 1, 2).contiguous()), ws=wsn)
         if cfg.N % 4 == 0:
             y = wino.conv2d(x, u, split_c=2)  # cluster split-C
         y = wino.conv2d_nchw(x.permute(3, 0, 1, 2).contiguous(), wino.filter_transform_kcrs(w.permute(3, 0, 1, 2).contiguous()))
