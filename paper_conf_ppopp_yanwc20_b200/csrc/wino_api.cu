@@ -860,10 +860,15 @@ wino_status_t conv_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, i
                    overlaps(ws_dev, ws_bytes, u_tc_dev, wino_filter_workspace_bytes_tc(C, K, mode))))
         return WINO_ERR_INVALID_ARG;
     const double units = double(prm.num_tiles) * prm.num_cb;
-    // (128-filter tiles only: the 64 x 64 tiles of K <= 64 put a cut tile's last 8 nu wrong in
-    // one parity case -- not resolved; no BASELINE shape needs stream-K there)
+    // (128-filter tiles only: with the 64 x 64 tiles of K <= 64 a cut tile's last 8 nu came out
+    // wrong in 2 of ~10 forced runs -- an intermittent hazard not yet found (scripts/dbg_tcsk64.py);
+    // no BASELINE shape needs stream-K there)
+#ifndef WINO_TC_SK_MM64  // debug builds: allow it (investigation)
     if (sk == 2 && mm == 64) return WINO_ERR_UNSUPPORTED;
     const bool sk_ok = xm >= 2 && mm == 128 && ws_dev && ws_bytes >= tc16_sk_bytes(sms) && units < 2147483647.0;
+#else
+    const bool sk_ok = xm >= 2 && ws_dev && ws_bytes >= tc16_sk_bytes(sms) && units < 2147483647.0;
+#endif
     if (sk == 2 && !sk_ok) return WINO_ERR_INVALID_ARG;
     const bool use_sk = sk == 2 || (sk == 1 && sk_ok && tc16_sk_pays(prm.num_tiles, prm.num_cb, sms));
     if (use_sk) {  // stream-K: equal (tile, channel block) ranges on every SM + fixup
@@ -874,6 +879,10 @@ wino_status_t conv_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, i
     }
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (use_sk) {
+#ifdef WINO_TC_SK_MM64
+        if (mode == WINO_TC_TF32 && mm == 64)
+            return xm == 3 ? launch_tc<1, 3, 64, true>(prm, ctas, dev, st) : launch_tc<1, 2, 64, true>(prm, ctas, dev, st);
+#endif
         if (mode == WINO_TC_TF32)
             return xm == 3 ? launch_tc<1, 3, 128, true>(prm, ctas, dev, st)
                            : launch_tc<1, 2, 128, true>(prm, ctas, dev, st);
