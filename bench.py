@@ -234,9 +234,10 @@ def _config(args, layers, world):
         "variant": args.variant,
         "inputs": f"uniform[-1,1) fp32, torch seeds x={SEED_X} w={SEED_W}",
         "l2": "flushed before every timed step by a 512 MiB write + 256 MiB read (outside the events)",
-        "step": "per layer: FTF kernel + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
-                "its own FTF; fp32: wino_conv2d_f2x3_fwd_ws with a stream-K workspace, the planner picks regular / "
-                "split-C / stream-K + fixup per layer); the whole step replayed from one CUDA graph",
+        "step": "per layer: FTF + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
+                "its own FTF; fp32: all layers' FTFs in one wino_filter_transform_multi launch, convs through "
+                "wino_conv2d_f2x3_fwd_ws with a stream-K workspace, the planner picks regular / split-C / "
+                "stream-K + fixup per layer); the whole step replayed from one CUDA graph",
     }
 
 
@@ -328,8 +329,9 @@ def main():
         else:
             # fp32: with the stream-K workspace (variant 4 plans it), which may add a fixup launch
             vid = {"fp32": 4, "tf32": 6, "3xtf32": 7}[variant]  # plans with the stream-K workspaces
-            launches = sum(1 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K,
-                                         variant=vid).launches for d in per if d["n"] > 0)
+            launches = sum((1 if variant != "fp32" else 0) +
+                           wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=vid).launches
+                           for d in per if d["n"] > 0) + (1 if variant == "fp32" else 0)  # fp32: one batched FTF
         for d in per:
             # transformed filter: computed on rank 0, broadcast once over NVLink (NCCL)
             if f4:
@@ -429,11 +431,18 @@ def main():
             fork.record(stream)
             side.wait_event(fork)
             ready = []
-            for d in per:
-                run_layer(d, conv=False, ftf_stream=side)
+            if variant == "fp32":
+                # every layer's FTF in one launch (wino_filter_transform_multi): one launch latency
+                wino.filter_transform_multi([(d["w"], d["u"]) for d in per if d["n"] > 0], stream=side)
                 ev = torch.cuda.Event()
                 ev.record(side)
-                ready.append(ev)
+                ready = [ev] * len(per)
+            else:
+                for d in per:
+                    run_layer(d, conv=False, ftf_stream=side)
+                    ev = torch.cuda.Event()
+                    ev.record(side)
+                    ready.append(ev)
             for d, ev in zip(per, ready):
                 stream.wait_event(ev)
                 run_layer(d, ftf=False)

@@ -92,6 +92,19 @@ wino_status_t wino_filter_transform(const float* w_dev, float* u_dev, int C, int
                                     wino_stream_t stream);
 
 /*
+ * Several filter transforms (Eq. 5) in one launch -- e.g. every layer of a network step, so the
+ * per-launch latency of the small FTFs is paid once.  jobs[i]: w (C,3,3,K) -> u (C,4,4,K) as
+ * wino_filter_transform; 1 <= n <= 8; the u's must not overlap each other or any w.
+ * Errors as wino_filter_transform, per job.
+ */
+typedef struct {
+    const float* w; /* (C,3,3,K) device */
+    float* u;       /* (C,4,4,K) device */
+    int C, K;
+} wino_ftf_job_t;
+wino_status_t wino_filter_transform_multi(const wino_ftf_job_t* jobs, int n, wino_stream_t stream);
+
+/*
  * Fused forward convolution on FP32 CUDA cores (FFMA), Sec. 3-4 and
  * Algorithm 1 (L351-355): for every 4x4 input tile the input transform
  * V = B^T d B (Eq. 6), the 16 Winograd-domain batched GEMMs

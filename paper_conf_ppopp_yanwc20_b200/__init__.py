@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes",
+    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes", "filter_transform_multi",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -169,6 +169,9 @@ def lib() -> ctypes.CDLL:
         L.wino_nchw_workspace_bytes.argtypes = [i, i, i, i, i]
         L.wino_conv2d_f2x3_fwd_nchw_ws.restype = i
         L.wino_conv2d_f2x3_fwd_nchw_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp, st, vp]
+    if hasattr(L, "wino_filter_transform_multi") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_filter_transform_multi.restype = i
+        L.wino_filter_transform_multi.argtypes = [ctypes.c_void_p, i, vp]
     L.wino_plan.restype = i
     L.wino_plan.argtypes = [i, i, i, i, i, i, ctypes.POINTER(_Plan)]
     _lib = L
@@ -232,6 +235,24 @@ def filter_transform(w: torch.Tensor, out: torch.Tensor | None = None, stream=No
         _check(lib().wino_filter_transform(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                            C, K, _stream_ptr(stream)), "wino_filter_transform")
     return out
+
+
+class _FtfJob(ctypes.Structure):
+    _fields_ = [("w", ctypes.c_void_p), ("u", ctypes.c_void_p), ("C", ctypes.c_int), ("K", ctypes.c_int)]
+
+
+def filter_transform_multi(pairs, stream=None) -> None:
+    """Several FTFs (Eq. 5) in one launch (wino_filter_transform_multi): pairs = [(w (C,3,3,K), u (C,4,4,K))]."""
+    jobs = (_FtfJob * len(pairs))()
+    for j, (w, u) in enumerate(pairs):
+        _need_cuda_f32(w, "w", 4)
+        _need_cuda_f32(u, "u", 4)
+        C, r, s_, K = w.shape
+        if (r, s_) != (3, 3) or tuple(u.shape) != (C, 4, 4, K):
+            raise ValueError(f"job {j}: w must be (C,3,3,K) and u (C,4,4,K)")
+        jobs[j] = _FtfJob(w.data_ptr(), u.data_ptr(), C, K)
+    with torch.cuda.device(pairs[0][0].device):
+        _check(lib().wino_filter_transform_multi(jobs, len(pairs), _stream_ptr(stream)), "wino_filter_transform_multi")
 
 
 @dataclass

@@ -44,4 +44,32 @@ __global__ void __launch_bounds__(FTF_THREADS) ftf_kcrs_kernel(const float* __re
     for (int e = 0; e < 16; ++e) uc[(size_t)e * K] = t[e];
 }
 
+// Several filter transforms in one launch (the layers of a network step): block b belongs to the
+// job whose block range [first[j], first[j+1]) holds it; the body is ftf_kernel's.
+constexpr int FTF_MAX_JOBS = 8;
+struct FtfJobs {
+    const float* w[FTF_MAX_JOBS];
+    float* u[FTF_MAX_JOBS];
+    int C[FTF_MAX_JOBS], K[FTF_MAX_JOBS];
+    unsigned first[FTF_MAX_JOBS + 1];
+    int n;
+};
+
+__global__ void __launch_bounds__(FTF_THREADS) ftf_multi_kernel(const __grid_constant__ FtfJobs jobs) {
+    int j = 0;
+    while (j + 1 < jobs.n && blockIdx.x >= jobs.first[j + 1]) ++j;
+    const int C = jobs.C[j], K = jobs.K[j];
+    const long idx = (long)(blockIdx.x - jobs.first[j]) * FTF_THREADS + threadIdx.x;
+    if (idx >= (long)C * K) return;
+    const int c = (int)(idx / K), k = (int)(idx - (long)c * K);
+    const float* wc = jobs.w[j] + (size_t)c * 9 * K + k;
+    float g[9], t[16];
+#pragma unroll
+    for (int e = 0; e < 9; ++e) g[e] = __ldg(wc + (size_t)e * K);
+    ftf_4x4(g, t);
+    float* uc = jobs.u[j] + (size_t)c * 16 * K + k;
+#pragma unroll
+    for (int e = 0; e < 16; ++e) uc[(size_t)e * K] = t[e];
+}
+
 }  // namespace wino

@@ -549,6 +549,42 @@ wino_status_t wino_filter_transform(const float* w_dev, float* u_dev, int C, int
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 
+wino_status_t wino_filter_transform_multi(const wino_ftf_job_t* jobs, int n, wino_stream_t stream) {
+    if (!jobs || n <= 0 || n > wino::FTF_MAX_JOBS) return WINO_ERR_INVALID_ARG;
+    wino::FtfJobs J;
+    std::memset(&J, 0, sizeof(J));
+    J.n = n;
+    unsigned blocks = 0;
+    for (int j = 0; j < n; ++j) {
+        const wino_ftf_job_t& b = jobs[j];
+        if (!b.w || !b.u || b.C <= 0 || b.K <= 0) return WINO_ERR_INVALID_ARG;
+        if (int64_t(16) * b.C * b.K > kMaxElems) return WINO_ERR_TOO_LARGE;
+        if (!aligned16(b.w) || !aligned16(b.u)) return WINO_ERR_MISALIGNED;
+        if (overlaps(b.w, size_t(9) * b.C * b.K * 4, b.u, size_t(16) * b.C * b.K * 4)) return WINO_ERR_INVALID_ARG;
+        for (int i = 0; i < n; ++i) {  // an output must not overlap another output or any input
+            if (i == j || !jobs[i].w || !jobs[i].u) continue;
+            if (overlaps(b.u, size_t(16) * b.C * b.K * 4, jobs[i].u, size_t(16) * jobs[i].C * jobs[i].K * 4) ||
+                overlaps(b.u, size_t(16) * b.C * b.K * 4, jobs[i].w, size_t(9) * jobs[i].C * jobs[i].K * 4))
+                return WINO_ERR_INVALID_ARG;
+        }
+        J.w[j] = b.w;
+        J.u[j] = b.u;
+        J.C[j] = b.C;
+        J.K[j] = b.K;
+        J.first[j] = blocks;
+        const int64_t nb = (int64_t(b.C) * b.K + wino::FTF_THREADS - 1) / wino::FTF_THREADS;
+        if (int64_t(blocks) + nb > 0x7fffffff) return WINO_ERR_TOO_LARGE;
+        blocks += static_cast<unsigned>(nb);
+    }
+    J.first[n] = blocks;
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    wino::ftf_multi_kernel<<<blocks, wino::FTF_THREADS, 0, reinterpret_cast<cudaStream_t>(stream)>>>(J);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+
 wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_plan_t* plan) {
     if (!plan) return WINO_ERR_INVALID_ARG;
     wino_status_t s = check_shape(N, C, H, W, K, 1, 1);

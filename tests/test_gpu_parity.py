@@ -245,3 +245,20 @@ def test_tc_full_configs_sampled(wino, name, variant):
     got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
     assert np.isfinite(y.numpy()).all()
     assert float(np.max(np.abs(got - ref))) / float(np.max(np.abs(ref))) <= TC_TOL[variant]
+
+
+def test_filter_transform_multi_matches_single(wino):
+    """One launch for several layers' FTFs (wino_filter_transform_multi) = the per-layer FTF, bit for bit."""
+    pairs, singles = [], []
+    for name in ("conv5_x", "conv4_x", "conv3_x", "conv2_x", "tiny"):
+        _, w = make_inputs(CONFIGS[name])
+        wd = w.to(DEV)
+        pairs.append((wd, torch.empty((w.shape[0], 4, 4, w.shape[3]), device=DEV)))
+        singles.append(wino.filter_transform(wd))
+    wino.filter_transform_multi(pairs)
+    torch.cuda.synchronize()
+    for (_, u), u1 in zip(pairs, singles):
+        assert torch.equal(u, u1)
+    bad_u = pairs[0][0].reshape(-1)[: pairs[1][1].numel()].view(pairs[1][1].shape)  # aliases job 0's w
+    with pytest.raises(wino.WinoError, match="INVALID_ARG"):  # an output overlapping another job's input
+        wino.filter_transform_multi([pairs[0], (pairs[1][0], bad_u)])
