@@ -249,7 +249,7 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default="resnet_3x3", choices=["resnet_3x3", *RESNET_LAYERS, "tiny"])
     ap.add_argument("--variant", default="fp32", choices=["fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw",
-                                                            "nonfused_fp32", "fp16", "bf16"])
+                                                            "nonfused_fp32", "nonfused_tf32", "fp16", "bf16"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
@@ -314,7 +314,7 @@ def main():
         f4 = variant == "f4_fp32"  # NEXT row N1: fused F(4x4,3x3), FTF4 + one fused launch per layer
         tc = variant in ("tf32", "3xtf32")
         nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
-        nonfused = variant == "nonfused_fp32"  # NEXT row N3: ITF -> 16 cuBLAS SGEMMs -> OTF (Sec. 9)
+        nonfused = variant in ("nonfused_fp32", "nonfused_tf32")  # NEXT row N3: ITF -> 16 cuBLAS GEMMs -> OTF
         half = variant in ("fp16", "bf16")  # NEXT row N4: 16-bit x, w, y on tcgen05 kind::f16 (Sec. 8.3)
         if f4:  # FTF4 + conv (+ a stream-K fixup where the planner takes it: counted as taken)
             launches = sum(3 for d in per if d["n"] > 0)
@@ -417,7 +417,7 @@ def main():
                 elif half:
                     wino.conv2d_half(d["x16"], d["u"], out=d["y16"], ws=d["ws16"])
                 elif nonfused:
-                    wino.conv2d_nonfused(d["x"], d["u"], d["ws_nf"], out=d["y"])
+                    wino.conv2d_nonfused(d["x"], d["u"], d["ws_nf"], out=d["y"], tf32=variant == "nonfused_tf32")
                 else:
                     wino.conv2d(d["x"], d["u"], out=d["y"], ws=d["ws_sk"])
 
@@ -519,7 +519,7 @@ def main():
     main_m = measure(args.variant, sample_clocks=True)
     others = {}
     if not args.no_variants:
-        for v in ("fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw", "nonfused_fp32", "fp16", "bf16"):
+        for v in ("fp32", "tf32", "3xtf32", "f4_fp32", "fp32_nchw", "nonfused_fp32", "nonfused_tf32", "fp16", "bf16"):
             if v == "f4_fp32" and any(d["n"] % 16 for d in per if d["n"]):
                 continue  # the F(4x4) kernel needs N % 16 == 0 per rank
             if v != args.variant:
@@ -616,7 +616,10 @@ def main():
                    "layers_eff_tflops": {d["cfg"].name: d["cfg"].eff_flops / (m["conv_ms"][i] * 1e-3) / 1e12
                                          for i, d in enumerate(per) if d["n"]},
                    "tolerance": {"fp32": 1e-4, "tf32": 5e-3, "3xtf32": 1e-4, "f4_fp32": 1e-4, "fp32_nchw": 1e-4,
-                                 "nonfused_fp32": 1e-4, "fp16": 5e-3, "bf16": 3e-2}[v]}
+                                 "nonfused_fp32": 1e-4, "nonfused_tf32": 5e-3, "fp16": 5e-3, "bf16": 3e-2}[v]}
+        if v == "nonfused_tf32":
+            vrep[v]["note"] = ("NEXT row N3 ablation with tensor-core GEMMs: ITF kernel -> V workspace, 16 "
+                               "strided-batched cuBLAS GEMMs in TF32 tensor-op math -> OTF kernel")
         if v == "nonfused_fp32":
             vrep[v]["note"] = ("NEXT row N3 ablation: ITF kernel -> V workspace, 16 strided-batched cuBLAS "
                                "SGEMMs (pedantic FP32) -> OTF kernel; FTF as in the fused step")

@@ -205,6 +205,12 @@ size_t wino_nonfused_workspace_bytes(int N, int C, int H, int W, int K);
 wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_dev, float* y_dev,
                                             int N, int C, int H, int W, int K, int pad, int stride,
                                             void* ws_dev, size_t ws_bytes, wino_stream_t stream);
+/* The same with the 16 Winograd-domain GEMMs on the tensor cores: cuBLAS in
+ * CUBLAS_TF32_TENSOR_OP_MATH (operands rounded to TF32 by the library; accuracy as the TF32
+ * fused kernel, <= 5e-3 of max|y|).  The ablation of SURVEY 8(f) N3 with tensor-core GEMMs. */
+wino_status_t wino_conv2d_f2x3_fwd_nonfused_tf32(const float* x_dev, const float* u_dev, float* y_dev,
+                                                 int N, int C, int H, int W, int K, int pad, int stride,
+                                                 void* ws_dev, size_t ws_bytes, wino_stream_t stream);
 
 /*
  * The fused FP32 convolution with a caller-provided device workspace, which lets the

@@ -117,6 +117,9 @@ def lib() -> ctypes.CDLL:
         L.wino_nonfused_workspace_bytes.argtypes = [i, i, i, i, i]
         L.wino_conv2d_f2x3_fwd_nonfused.restype = i
         L.wino_conv2d_f2x3_fwd_nonfused.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp, st, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_nonfused_tf32") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_conv2d_f2x3_fwd_nonfused_tf32.restype = i
+        L.wino_conv2d_f2x3_fwd_nonfused_tf32.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, vp, st, vp]
     L.wino_conv2d_f2x3_fwd_tc.restype = i
     L.wino_conv2d_f2x3_fwd_tc.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp]
     L.wino_filter_workspace_bytes_tc.restype = st
@@ -515,10 +518,10 @@ def nonfused_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
 
 
 def conv2d_nonfused(x: torch.Tensor, u: torch.Tensor, ws: torch.Tensor, out: torch.Tensor | None = None,
-                    stream=None) -> torch.Tensor:
+                    stream=None, tf32: bool = False) -> torch.Tensor:
     """NEXT row N3 (Sec. 9): NON-fused Winograd -- ITF kernel to a global workspace,
-    16 batched GEMMs (cuBLAS SGEMM), OTF kernel.  x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N);
-    ws: CUDA byte buffer of >= nonfused_workspace_bytes(N,C,H,W,K)."""
+    16 batched GEMMs (cuBLAS SGEMM; tf32=True: cuBLAS TF32 tensor-core GEMMs), OTF kernel.
+    x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N); ws: CUDA byte buffer of >= nonfused_workspace_bytes."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u, "u", 4)
     C, H, W, N = x.shape
@@ -532,11 +535,12 @@ def conv2d_nonfused(x: torch.Tensor, u: torch.Tensor, ws: torch.Tensor, out: tor
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N):
         raise ValueError("out must be (K,H,W,N)")
+    fn = "wino_conv2d_f2x3_fwd_nonfused_tf32" if tf32 else "wino_conv2d_f2x3_fwd_nonfused"
     with torch.cuda.device(x.device):
-        _check(lib().wino_conv2d_f2x3_fwd_nonfused(
+        _check(getattr(lib(), fn)(
             ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(out.data_ptr()),
             N, C, H, W, K, 1, 1, ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size(),
-            _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_nonfused")
+            _stream_ptr(stream)), fn)
     return out
 
 

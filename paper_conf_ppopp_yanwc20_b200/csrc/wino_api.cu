@@ -1405,7 +1405,7 @@ struct Cublas {
     cublasSetStream_t set_stream = nullptr;
     cublasSetMathMode_t set_math = nullptr;
     cublasSgemmStridedBatched_t sgemm_sb = nullptr;
-    void* handle[kMaxDevices] = {};
+    void* handle[kMaxDevices][2] = {};  // [device][0: pedantic FP32, 1: TF32 tensor ops]
     bool ok = false;
 };
 std::mutex g_cublas_mu;
@@ -1428,6 +1428,7 @@ bool cublas_load() {
 }
 constexpr int kCublasOpN = 0, kCublasOpT = 1;
 constexpr int kCublasPedanticMath = 2;  // CUBLAS_PEDANTIC_MATH: plain FP32, no TF32 tensor-op shortcuts
+constexpr int kCublasTf32Math = 3;      // CUBLAS_TF32_TENSOR_OP_MATH: the library's TF32 tensor-core GEMMs
 }  // namespace
 
 extern "C" {
@@ -1438,9 +1439,10 @@ size_t wino_nonfused_workspace_bytes(int N, int C, int H, int W, int K) {
     return round_up256(size_t(16) * C * nv * 4) + round_up256(size_t(16) * K * nv * 4);
 }
 
-wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_dev, float* y_dev, int N, int C,
-                                            int H, int W, int K, int pad, int stride, void* ws_dev, size_t ws_bytes,
-                                            wino_stream_t stream) {
+extern "C++" {
+namespace {
+wino_status_t conv_nonfused(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H, int W, int K,
+                            int pad, int stride, void* ws_dev, size_t ws_bytes, bool tf32, wino_stream_t stream) {
     if (!x_dev || !u_dev || !y_dev || !ws_dev) return WINO_ERR_INVALID_ARG;
     wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
     if (s != WINO_OK) return s;
@@ -1471,11 +1473,11 @@ wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_d
     {
         std::lock_guard<std::mutex> lk(g_cublas_mu);
         if (!cublas_load()) return WINO_ERR_UNSUPPORTED;
-        if (!g_cublas.handle[dev]) {
-            if (g_cublas.create(&g_cublas.handle[dev]) != 0) return WINO_ERR_CUDA;
-            g_cublas.set_math(g_cublas.handle[dev], kCublasPedanticMath);
+        if (!g_cublas.handle[dev][tf32]) {
+            if (g_cublas.create(&g_cublas.handle[dev][tf32]) != 0) return WINO_ERR_CUDA;
+            g_cublas.set_math(g_cublas.handle[dev][tf32], tf32 ? kCublasTf32Math : kCublasPedanticMath);
         }
-        void* hd = g_cublas.handle[dev];
+        void* hd = g_cublas.handle[dev][tf32];
         if (g_cublas.set_stream(hd, st) != 0) return WINO_ERR_CUDA;
         const float one = 1.f, zero = 0.f;
         if (g_cublas.sgemm_sb(hd, kCublasOpN, kCublasOpT, (int)nv, K, C, &one, v, (int)nv, (long long)C * nv, u_dev,
@@ -1487,6 +1489,20 @@ wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_d
                               st>>>(m, y_dev, N, K, H, W, TW, nv);
     e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+}  // namespace
+}  // extern "C++"
+
+wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_dev, float* y_dev, int N, int C,
+                                            int H, int W, int K, int pad, int stride, void* ws_dev, size_t ws_bytes,
+                                            wino_stream_t stream) {
+    return conv_nonfused(x_dev, u_dev, y_dev, N, C, H, W, K, pad, stride, ws_dev, ws_bytes, false, stream);
+}
+
+wino_status_t wino_conv2d_f2x3_fwd_nonfused_tf32(const float* x_dev, const float* u_dev, float* y_dev, int N, int C,
+                                                 int H, int W, int K, int pad, int stride, void* ws_dev,
+                                                 size_t ws_bytes, wino_stream_t stream) {
+    return conv_nonfused(x_dev, u_dev, y_dev, N, C, H, W, K, pad, stride, ws_dev, ws_bytes, true, stream);
 }
 
 }  // extern "C"

@@ -88,3 +88,16 @@ def test_nonfused_workspace_checks(wino):
     with pytest.raises(wino.WinoError) as e:
         wino.conv2d_nonfused(x.to(DEV), u, small)
     assert e.value.status == 1
+
+
+@pytest.mark.parametrize("shape", [(32, 64, 64, 14, 14), (5, 17, 130, 6, 10), (32, 512, 512, 7, 7)],
+                         ids=["conv2like", "ragged", "conv5"])
+def test_nonfused_tf32_tensor_core_gemms(wino, shape):
+    """N3 with cuBLAS TF32 tensor-core GEMMs: within the TF32 bar of Eq. 4."""
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nf", N, C, K, H, W), kind="uniform", seed_x=71, seed_w=72)
+    u = wino.filter_transform(w.to(DEV))
+    ws = torch.empty(wino.nonfused_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+    y = wino.conv2d_nonfused(x.to(DEV), u, ws, tf32=True)
+    torch.cuda.synchronize()
+    assert oracle.max_rel_err(y.cpu().double().numpy(), oracle.direct_conv(x, w)) <= 5e-3
