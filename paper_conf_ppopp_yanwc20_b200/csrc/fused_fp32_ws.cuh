@@ -57,7 +57,10 @@ using fp32::XS_FLOATS;
 
 constexpr int NT = 384;             // 2 compute warpgroups + 1 producer/ITF warpgroup
 constexpr int COMPUTE_THREADS = 256;
-constexpr int S = 3;                // TMA stage ring (u 32 KB + raw x 16 KB per stage)
+#ifndef WS_EPI_ROUNDS
+#define WS_EPI_ROUNDS 4  // OTF rounds of the non-split epilogue: 4 (16 filters, 3-stage ring) or 2 (A/B)
+#endif
+constexpr int S = WS_EPI_ROUNDS == 2 ? 2 : 3;  // TMA stage ring (u 32 KB + raw x 16 KB per stage)
 constexpr int SV = 2;               // V ring (16 KB each)
 constexpr int REG_COMPUTE = 208, REG_PRODUCER = 88;  // 256*208 + 128*88 = 64512 <= 65536
 constexpr int ITF_WARPS = 2;        // warps 9..10 (float4 along nu); warp 8 only issues TMA; 11 idle
@@ -81,7 +84,7 @@ __device__ unsigned long long g_ws_trace[8][64];
 // tile (a per-round exchange is latency-bound: ~8 DSMEM round trips per tile).
 template <bool SPLIT>
 struct Smem {
-    static constexpr int RR = SPLIT ? 1 : 2;
+    static constexpr int RR = SPLIT ? 1 : 8 / WS_EPI_ROUNDS;
     static constexpr int ER_KROWS = 8 * RR;
     static constexpr int ER_FLOATS = 16 * ER_KROWS * ER_LD;  // [xi][8RR k][36]
     // split receive buffer [S slots][64/S owned filters][32 nu][4 outputs] = 32 KB for any S
@@ -385,18 +388,21 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             // assignment of the accumulators (and so the FFMA bank conflicts of the main
             // loop) is sensitive to this code's shape: keep it as is.
 #pragma unroll
-            for (int rd = 0; rd < 4; ++rd) {
-                // round rd stores accumulator rows i in {2(rd&1), 2(rd&1)+1} of half rd>>1:
-                // filters kl = fo + (i&3) + 32*(i>>2); in the buffer row = (fo>>2)*2 + (i&1)
+            for (int rd = 0; rd < 8 / RR; ++rd) {
+                // round rd stores accumulator rows i = 4*rd_hi + RR*rd_lo + ii (ii < RR) of half rd_hi:
+                // filters kl = fo + (i&3) + 32*(i>>2); in the buffer row = (fo>>2)*RR + ii
+                constexpr int dummy_rr = RR;  // (RR = 2: 4 rounds of 16 filters, the paper's L499)
+                (void)dummy_rr;
+                const int rd_hi = RR == 2 ? (rd >> 1) : rd, rd_lo = RR == 2 ? (rd & 1) : 0;
 #ifndef WS_EXP_NOBAR
                 named_bar_sync(1, COMPUTE_THREADS);  // previous round's readers are done
 #endif
 #pragma unroll
                 for (int q = 0; q < 2; ++q)
 #pragma unroll
-                    for (int ii = 0; ii < 2; ++ii) {
-                        const int i = (rd >> 1) * 4 + (rd & 1) * 2 + ii;
-                        const int r = (fo >> 2) * 2 + ii;
+                    for (int ii = 0; ii < RR; ++ii) {
+                        const int i = rd_hi * 4 + rd_lo * RR + ii;
+                        const int r = (fo >> 2) * RR + ii;
                         float* row = ep + ((xi0 + q) * ER_KROWS + r) * ER_LD + io;
                         *reinterpret_cast<float4*>(row) =
                             make_float4(acc[q][i][1], acc[q][i][0], acc[q][i][3], acc[q][i][2]);
@@ -408,9 +414,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
 #endif
                 if (nu < p.NV) {
 #pragma unroll
-                    for (int h = 0; h < 2; ++h) {
-                        const int r = warp + 8 * h;  // buffer row 0..15
-                        const int kl = (r >> 1) * 4 + (rd & 1) * 2 + (r & 1) + (rd >> 1) * 32;
+                    for (int h = 0; h < RR; ++h) {
+                        const int r = warp + 8 * h;  // buffer row 0..8RR-1
+                        const int kl = (r / RR) * 4 + rd_lo * RR + (r % RR) + rd_hi * 32;
                         const int k = k0 + kl;
                         if (k < p.K) {
                             float m[16], o[4];
