@@ -391,8 +391,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             for (int rd = 0; rd < 8 / RR; ++rd) {
                 // round rd stores accumulator rows i = 4*rd_hi + RR*rd_lo + ii (ii < RR) of half rd_hi:
                 // filters kl = fo + (i&3) + 32*(i>>2); in the buffer row = (fo>>2)*RR + ii
-                constexpr int dummy_rr = RR;  // (RR = 2: 4 rounds of 16 filters, the paper's L499)
-                (void)dummy_rr;
+                // (RR = 2: 4 rounds of 16 filters, the paper's 4-round OTF, L499)
                 const int rd_hi = RR == 2 ? (rd >> 1) : rd, rd_lo = RR == 2 ? (rd & 1) : 0;
 #ifndef WS_EXP_NOBAR
                 named_bar_sync(1, COMPUTE_THREADS);  // previous round's readers are done
