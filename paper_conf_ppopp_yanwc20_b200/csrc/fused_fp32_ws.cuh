@@ -57,6 +57,9 @@ using fp32::XS_FLOATS;
 
 constexpr int NT = 384;             // 2 compute warpgroups + 1 producer/ITF warpgroup
 constexpr int COMPUTE_THREADS = 256;
+#ifndef WS_X_PREFETCH
+#define WS_X_PREFETCH 0  // channel blocks of x prefetched into L2 ahead of the TMA loads (A/B knob)
+#endif
 #ifndef WS_EPI_ROUNDS
 #define WS_EPI_ROUNDS 4  // OTF rounds of the non-split epilogue: 4 (16 filters, 3-stage ring) or 2 (A/B)
 #endif
@@ -217,12 +220,25 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                     const int t0 = nu0 / p.N;
                     const int n0 = nu0 - t0 * p.N;
                     const int nbox = BOX32 ? 1 : BN / p.xnb;
+#if WS_X_PREFETCH > 0
+                    if (BOX32) {  // x streams from HBM on first touch: warm L2 a few stages ahead
+                        const int th = t0 / p.TW, tw = t0 - th * p.TW;
+                        for (int g = g_lo; g < g_lo + WS_X_PREFETCH && g < g_hi; ++g)
+                            tma_prefetch_l2_4d(&p.tmx, n0, 2 * tw - 1, 2 * th - 1, g * BC);
+                    }
+#endif
                     for (int g = g_lo; g < g_hi; ++g, ++G) {
                         const int slot = G % S;
                         if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
                         float* us = smem + slot * STAGE_FLOATS;
                         mbar_arrive_expect_tx(&full[slot], kBytes);
                         tma_load_3d(us, &p.tmu, &full[slot], k0, 0, g * BC);
+#if WS_X_PREFETCH > 0
+                        if (BOX32 && g + WS_X_PREFETCH < g_hi) {
+                            const int th = t0 / p.TW, tw = t0 - th * p.TW;
+                            tma_prefetch_l2_4d(&p.tmx, n0, 2 * tw - 1, 2 * th - 1, (g + WS_X_PREFETCH) * BC);
+                        }
+#endif
                         for (int b = 0; b < nbox; ++b) {
                             const int t = t0 + b;
                             const int th = t / p.TW, tw = t - th * p.TW;
