@@ -60,6 +60,9 @@ constexpr int COMPUTE_THREADS = 256;
 #ifndef WS_X_PREFETCH
 #define WS_X_PREFETCH 0  // channel blocks of x prefetched into L2 ahead of the TMA loads (A/B knob)
 #endif
+#ifndef WS_XBAR
+#define WS_XBAR 0  // 1: raw x gets its own stage barrier (issued before u), so the ITF need not wait for u
+#endif
 #ifndef WS_EPI_ROUNDS
 #define WS_EPI_ROUNDS 4  // OTF rounds of the non-split epilogue: 4 (16 filters, 3-stage ring) or 2 (A/B)
 #endif
@@ -96,7 +99,7 @@ struct Smem {
     static constexpr int yp_offset = ep_offset + ER_FLOATS * 4;
     static constexpr int bar_offset = yp_offset + YP_FLOATS * 4;
     // full[S], empty[S], vfull[SV], vempty[SV], yready, yfree
-    static constexpr int bytes = bar_offset + (2 * S + 2 * SV + 2) * 8;
+    static constexpr int bytes = bar_offset + (2 * S + 2 * SV + 2 + (WS_XBAR ? S : 0)) * 8;
 };
 
 // ITF loop of warps 9..10 (Sec. 4.2): raw x of every stage -> V = B^T d B in the V ring.
@@ -154,6 +157,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
     uint64_t* const vempty = vfull + SV;
     uint64_t* const yready = vempty + SV;  // split: all S slots of this CTA's receive buffer landed (tx bytes)
     uint64_t* const yfree = yready + 1;    // split: every owner has consumed this CTA's slots of the last tile
+    uint64_t* const xfull = WS_XBAR ? yfree + 1 : full;  // raw x landed (WS_XBAR), else shares full
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     // split-C: cluster = S consecutive CTAs sharing each tile; rank r takes channel
@@ -174,6 +178,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
         tma_prefetch_desc(&p.tmu);
         for (int s = 0; s < S; ++s) {
             mbar_init(&full[s], 1);
+            if (WS_XBAR) mbar_init(&xfull[s], 1);
             mbar_init(&empty[s], 8 + ITF_WARPS);  // 8 compute warps (u) + ITF warps (raw x)
         }
         for (int s = 0; s < SV; ++s) {
@@ -231,8 +236,13 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                         const int slot = G % S;
                         if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
                         float* us = smem + slot * STAGE_FLOATS;
-                        mbar_arrive_expect_tx(&full[slot], kBytes);
-                        tma_load_3d(us, &p.tmu, &full[slot], k0, 0, g * BC);
+                        if (WS_XBAR) {
+                            mbar_arrive_expect_tx(&xfull[slot], XS_FLOATS * 4);
+                            mbar_arrive_expect_tx(&full[slot], US_FLOATS * 4);
+                        } else {
+                            mbar_arrive_expect_tx(&full[slot], kBytes);
+                            tma_load_3d(us, &p.tmu, &full[slot], k0, 0, g * BC);
+                        }
 #if WS_X_PREFETCH > 0
                         if (BOX32 && g + WS_X_PREFETCH < g_hi) {
                             const int th = t0 / p.TW, tw = t0 - th * p.TW;
@@ -246,11 +256,12 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                             // BOX32: map (n, w, h, c) -> [c][pos][n]; small N: map (n, c, w, h)
                             // -> [pos][c][n] per box (see the ITF lane map below)
                             if (BOX32)
-                                tma_load_4d(us + US_FLOATS, &p.tmx, &full[slot], n0, 2 * tw - 1, 2 * th - 1, g * BC);
+                                tma_load_4d(us + US_FLOATS, &p.tmx, &xfull[slot], n0, 2 * tw - 1, 2 * th - 1, g * BC);
                             else
-                                tma_load_4d(us + US_FLOATS + b * (BC * 16 * p.xnb), &p.tmx, &full[slot], 0, g * BC,
+                                tma_load_4d(us + US_FLOATS + b * (BC * 16 * p.xnb), &p.tmx, &xfull[slot], 0, g * BC,
                                             2 * tw - 1, 2 * th - 1);
                         }
+                        if (WS_XBAR) tma_load_3d(us, &p.tmu, &full[slot], k0, 0, g * BC);  // u after x
                     }
                     if constexpr (!SK) tile += WS_NCL;
                 }
@@ -282,14 +293,14 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             xpos = BC * p.xnb;
         }
         if (SK)  // one run of this CTA's stages (the ITF does not depend on the tile)
-            itf_loop(smem, vs, full, empty, vfull, vempty, xoff, xpos, c * BN + n4,
+            itf_loop(smem, vs, xfull, empty, vfull, vempty, xoff, xpos, c * BN + n4,
                      sk_start(p, blockIdx.x + 1) - sk_start(p, blockIdx.x),
                      0, 1, 1, lane);
         else if (BOX32)
-            itf_loop(smem, vs, full, empty, vfull, vempty, xoff, xpos, c * BN + n4, NIT, WS_CID, num_tiles, WS_NCL,
+            itf_loop(smem, vs, xfull, empty, vfull, vempty, xoff, xpos, c * BN + n4, NIT, WS_CID, num_tiles, WS_NCL,
                      lane);
         else
-            itf_loop(smem, vs, full, empty, vfull, vempty, xoff, xpos, c * BN + n4, NIT, WS_CID, num_tiles, WS_NCL,
+            itf_loop(smem, vs, xfull, empty, vfull, vempty, xoff, xpos, c * BN + n4, NIT, WS_CID, num_tiles, WS_NCL,
                      lane);
         return;
     }
