@@ -209,3 +209,18 @@ def test_tensor_core_stream_k_plans_and_workspaces():
     hwn = c4.H * c4.W * c4.N
     assert wino.nchw_workspace_bytes(c4.N, c4.C, c4.H, c4.W, c4.K) == \
         (c4.C * hwn * 4 + 255) // 256 * 256 + (c4.K * hwn * 4 + 255) // 256 * 256 + 148 * 64 * 1024
+
+
+def test_header_is_plain_c99(tmp_path):
+    """include/wino.h is a C ABI: it compiles as ISO C99 with -pedantic -Werror (no C++ or torch types)."""
+    import shutil
+    import subprocess
+    if shutil.which("gcc") is None:
+        pytest.skip("gcc not available")
+    src = tmp_path / "use_header.c"
+    src.write_text('#include "wino.h"\nint main(void) { wino_plan_t p; wino_ftf_job_t j; wino_host_layer_t l;\n'
+                   '  (void)p; (void)j; (void)l; return wino_filter_workspace_bytes(1, 1) == 64 ? 0 : 1; }\n')
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run(["gcc", "-std=c99", "-Wall", "-Wextra", "-pedantic", "-Werror", "-I", os.path.join(root, "include"),
+                        "-c", str(src), "-o", str(tmp_path / "use_header.o")], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr
