@@ -171,19 +171,22 @@ wino_status_t wino_conv2d_f2x3_fwd_nchw(const float* x_nchw_dev, const float* u_
  * results in global memory ... can utilize optimized batched matrix
  * multiplication routines. However, it needs significant amount of global
  * memory as workspace and data loading can be the new bottleneck"; Sec. 7.3
- * obs. 4-6 L1159-1241; the Sec. 8.1 break-even model L1245-1269).  Three
- * launches on `stream`:
- *   1. ITF kernel: x (C,H,W,N) -> V[16][C][NV] in ws_dev (Eq. 6),
- *   2. 16 batched GEMMs M[xi] = U[xi]^T V[xi] -> M[16][K][NV] in ws_dev (Eq. 7),
- *      one cuBLAS strided-batched SGEMM in pedantic FP32 (no TF32): the
- *      "optimized batched matrix multiplication routine" of L1291,
- *   3. OTF kernel: M -> y (K,H,W,N) (Eq. 8).
- * NV = N*ceil(H/2)*ceil(W/2).  ws_dev: caller-owned device workspace of at least
- * wino_nonfused_workspace_bytes(N,C,H,W,K) = 64*NV*(C+K) bytes (+ alignment),
- * must not overlap x, u or y.  cuBLAS (libcublas.so.12) is loaded on first use;
- * if it cannot be loaded the call returns WINO_ERR_UNSUPPORTED.  Other
- * arguments, layouts and errors as wino_conv2d_f2x3_fwd; ws_bytes too small ->
- * WINO_ERR_INVALID_ARG; V or M of >= 2^31 elements -> WINO_ERR_TOO_LARGE.
+ * obs. 4-6 L1159-1241; the Sec. 8.1 break-even model L1245-1269).  Four
+ * launches on `stream`, all of them this library's kernels:
+ *   1. u (C,4,4,K) -> Ug[16 P][K][Cp4] in ws_dev: the GEMM operand layout (channel c
+ *      contiguous, row pitch Cp4 = 4*ceil(C/4)), rounded to TF32 (RNA, reading R8),
+ *   2. ITF kernel: x (C,H,W,N) -> V[16 P][NV][Cp4] in ws_dev (Eq. 6), rounded likewise,
+ *   3. 16 batched GEMMs M[xi][k][nu] = sum_c V[xi][nu][c] Ug[xi][k][c] (Eq. 7) on the
+ *      tcgen05 tensor cores (kind::tf32, FP32 accumulation in TMEM) -> M[16][K][NV] in ws_dev,
+ *   4. OTF kernel: M -> y (K,H,W,N) (Eq. 8).
+ * This entry point is the FP32-accuracy variant: 3xTF32 with P = 2 planes per operand (big =
+ * rna(v), small = rna(v - big); D += Vb Ub + Vb Us + Vs Ub), within the FP32 bar (<= 1e-4 of
+ * max|y|) and exact on small integers.  NV = N*ceil(H/2)*ceil(W/2).  ws_dev: caller-owned
+ * device workspace of at least wino_nonfused_workspace_bytes(N,C,H,W,K) = 128*NV*Cp4 +
+ * 128*K*Cp4 + 64*K*NV bytes (each part rounded up to 256 B), 16-byte aligned, must not overlap
+ * x, u or y; clobbered.  Other arguments, layouts and errors as wino_conv2d_f2x3_fwd;
+ * ws_bytes too small -> WINO_ERR_INVALID_ARG; 32*Cp4*NV or 16*K*NV >= 2^31 ->
+ * WINO_ERR_TOO_LARGE.  wino_nonfused_launches() = 4 (kernels per call).
  */
 /*
  * NCHW with a device workspace: x is transposed to the paper's CHWN layout in the
@@ -205,9 +208,10 @@ size_t wino_nonfused_workspace_bytes(int N, int C, int H, int W, int K);
 wino_status_t wino_conv2d_f2x3_fwd_nonfused(const float* x_dev, const float* u_dev, float* y_dev,
                                             int N, int C, int H, int W, int K, int pad, int stride,
                                             void* ws_dev, size_t ws_bytes, wino_stream_t stream);
-/* The same with the 16 Winograd-domain GEMMs on the tensor cores: cuBLAS in
- * CUBLAS_TF32_TENSOR_OP_MATH (operands rounded to TF32 by the library; accuracy as the TF32
- * fused kernel, <= 5e-3 of max|y|).  The ablation of SURVEY 8(f) N3 with tensor-core GEMMs. */
+int wino_nonfused_launches(void);
+/* The same in plain TF32 (P = 1 plane per operand, half the V / Ug workspace traffic;
+ * accuracy as the TF32 fused kernel, <= 5e-3 of max|y|; exact on small integers).  Uses a
+ * prefix of the same workspace. */
 wino_status_t wino_conv2d_f2x3_fwd_nonfused_tf32(const float* x_dev, const float* u_dev, float* y_dev,
                                                  int N, int C, int H, int W, int K, int pad, int stride,
                                                  void* ws_dev, size_t ws_bytes, wino_stream_t stream);
@@ -361,7 +365,12 @@ wino_status_t wino_conv2d_f4x3_fwd_ws(const float* x_dev, const float* u4_dev, f
  * proceed concurrently over PCIe.  `stream` is joined before returning-order
  * completion: work enqueued on `stream` after this call sees all outputs.
  * The two helper streams are created once per device (cached, like the
- * attribute caches); events are created and released per call.
+ * attribute caches); every event a call needs is created before anything is
+ * queued, and released at the end of the call.  Errors: argument / shape errors
+ * return before any work is queued; an error after work was queued (a failed
+ * copy or launch) still makes `stream` wait for everything already queued on
+ * the helper streams, so the caller may free or reuse its host buffers once
+ * `stream` has drained.
  *   layers[i] : host pointers and shape of layer i (pad 1, stride 1)
  *   ws_dev    : device workspace of >= wino_host_multi_workspace_bytes() bytes
  */

@@ -68,6 +68,8 @@ def _load():
             getattr(lib, name).restype = None
         lib.oracle_num_threads.argtypes = []
         lib.oracle_num_threads.restype = ctypes.c_int
+        lib.oracle_set_num_threads.argtypes = [ctypes.c_int]
+        lib.oracle_set_num_threads.restype = None
         _lib = lib
     return _lib
 
@@ -85,6 +87,11 @@ def _ptr(a: np.ndarray):
 
 def num_threads() -> int:
     return int(_load().oracle_num_threads())
+
+
+def set_num_threads(n: int) -> None:
+    """OpenMP threads of the following oracle calls (plumbing; no arithmetic)."""
+    _load().oracle_set_num_threads(int(n))
 
 
 def direct_conv(x_chwn, w_crsk) -> np.ndarray:

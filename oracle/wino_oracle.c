@@ -51,6 +51,16 @@ int oracle_num_threads(void) {
 #endif
 }
 
+/* Thread count of the following calls (plumbing only: bench.py gives each of P ranks
+ * sharing one host cores/P threads; torchrun's OMP_NUM_THREADS=1 would serialise it). */
+void oracle_set_num_threads(int n) {
+#ifdef _OPENMP
+    if (n > 0) omp_set_num_threads(n);
+#else
+    (void)n;
+#endif
+}
+
 /* x-hat of Eq. 4 with implicit zero padding (Sec. 3.5): x inside
  * [0,H) x [0,W), 0 outside. */
 static inline double xhat(const double* x, int N, int H, int W, int c, int h, int w, int n) {

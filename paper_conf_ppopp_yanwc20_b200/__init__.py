@@ -24,7 +24,7 @@ __all__ = [
     "TcFilter", "filter_workspace_bytes_tc", "filter_transform_tc", "conv2d_tc",
     "host_multi_workspace_bytes", "conv2d_host_multi",
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
-    "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused",
+    "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused", "nonfused_launches",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
     "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes", "filter_transform_multi",
 ]
@@ -207,6 +207,26 @@ def _need_cuda_f32(t: torch.Tensor, name: str, ndim: int):
     if not t.is_contiguous():
         raise ValueError(f"{name} must be contiguous")
 
+def _same_device(ref: torch.Tensor, **tensors):
+    """Every tensor the library touches in one call must live on ref's device (a pointer into
+    another GPU's memory would fault inside the kernel and kill the CUDA context)."""
+    for name, t in tensors.items():
+        if t is None:
+            continue
+        if not t.is_cuda or t.device != ref.device:
+            raise ValueError(f"{name} must be on {ref.device}, got {t.device}")
+
+
+def _need_ws(ws: torch.Tensor | None, ref: torch.Tensor):
+    """A workspace is a contiguous CUDA byte buffer on ref's device."""
+    if ws is None:
+        return
+    if not isinstance(ws, torch.Tensor) or not ws.is_cuda:
+        raise ValueError("ws must be a CUDA tensor")
+    if not ws.is_contiguous():
+        raise ValueError("ws must be contiguous")
+    _same_device(ref, ws=ws)
+
 
 def filter_workspace_bytes(C: int, K: int) -> int:
     """16*C*K*4 bytes (L993)."""
@@ -234,6 +254,7 @@ def filter_transform(w: torch.Tensor, out: torch.Tensor | None = None, stream=No
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (C, 4, 4, K):
         raise ValueError("out must be (C,4,4,K)")
+    _same_device(w, out=out)
     with torch.cuda.device(w.device):
         _check(lib().wino_filter_transform(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                            C, K, _stream_ptr(stream)), "wino_filter_transform")
@@ -253,6 +274,7 @@ def filter_transform_multi(pairs, stream=None) -> None:
         C, r, s_, K = w.shape
         if (r, s_) != (3, 3) or tuple(u.shape) != (C, 4, 4, K):
             raise ValueError(f"job {j}: w must be (C,3,3,K) and u (C,4,4,K)")
+        _same_device(pairs[0][0], w=w, u=u)
         jobs[j] = _FtfJob(w.data_ptr(), u.data_ptr(), C, K)
     with torch.cuda.device(pairs[0][0].device):
         _check(lib().wino_filter_transform_multi(jobs, len(pairs), _stream_ptr(stream)), "wino_filter_transform_multi")
@@ -291,6 +313,8 @@ def filter_transform_tc(w: torch.Tensor, variant="tf32", out: TcFilter | None = 
         out = TcFilter(torch.empty(nbytes // 4, dtype=torch.float32, device=w.device), C, K, mode)
     if (out.C, out.K, out.mode) != (C, K, mode) or out.data.numel() * 4 < nbytes:
         raise ValueError("out TcFilter does not match w / variant")
+    _need_cuda_f32(out.data, "out.data", out.data.dim())
+    _same_device(w, out=out.data)
     with torch.cuda.device(w.device):
         _check(lib().wino_filter_transform_tc(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data.data_ptr()),
                                               C, K, mode, _stream_ptr(stream)), "wino_filter_transform_tc")
@@ -316,12 +340,13 @@ def conv2d_tc(x: torch.Tensor, u_tc: TcFilter, out: torch.Tensor | None = None, 
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N):
         raise ValueError("out must be (K,H,W,N)")
+    _need_cuda_f32(u_tc.data, "u_tc.data", u_tc.data.dim())
+    _same_device(x, u_tc=u_tc.data, out=out)
+    _need_ws(ws, x)
     args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_tc.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
             N, C, H, W, K, 1, 1, u_tc.mode)
     with torch.cuda.device(x.device):
         if ws is not None or stream_k == "on":
-            if ws is not None and not ws.is_cuda:
-                raise ValueError("ws must be a CUDA tensor")
             wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
             _check(lib().wino_conv2d_f2x3_fwd_tc_ws(*args, {"auto": 0, "off": 1, "on": 2}[stream_k], wp, wb,
                                                     _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_tc_ws")
@@ -368,6 +393,8 @@ def filter_transform_half(w: torch.Tensor, out: HalfFilter | None = None, stream
         out = HalfFilter(torch.empty(nbytes // 2, dtype=w.dtype, device=w.device), C, K, w.dtype)
     if (out.C, out.K, out.dtype) != (C, K, w.dtype) or out.data.numel() * 2 < nbytes:
         raise ValueError("out HalfFilter does not match w")
+    _need_cuda_half(out.data, "out.data", out.data.dim())
+    _same_device(w, out=out.data)
     with torch.cuda.device(w.device):
         _check(lib().wino_filter_transform_half(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data.data_ptr()),
                                                 C, K, _HALF_DTYPES[w.dtype], _stream_ptr(stream)),
@@ -395,12 +422,13 @@ def conv2d_half(x: torch.Tensor, u_h: HalfFilter, out: torch.Tensor | None = Non
     _need_cuda_half(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N) or out.dtype != x.dtype:
         raise ValueError("out must be (K,H,W,N) of x's dtype")
+    _need_cuda_half(u_h.data, "u_h.data", u_h.data.dim())
+    _same_device(x, u_h=u_h.data, out=out)
+    _need_ws(ws, x)
     args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u_h.data.data_ptr()), ctypes.c_void_p(out.data_ptr()),
             N, C, H, W, K, 1, 1, _HALF_DTYPES[x.dtype])
     with torch.cuda.device(x.device):
         if ws is not None or stream_k == "on":
-            if ws is not None and not ws.is_cuda:
-                raise ValueError("ws must be a CUDA tensor")
             wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
             _check(lib().wino_conv2d_f2x3_fwd_half_ws(*args, {"auto": 0, "off": 1, "on": 2}[stream_k], wp, wb,
                                                       _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_half_ws")
@@ -435,6 +463,8 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N):
         raise ValueError("out must be (K,H,W,N)")
+    _same_device(x, u=u, out=out)
+    _need_ws(ws, x)
     args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(out.data_ptr()),
             N, C, H, W, K, 1, 1)
     with torch.cuda.device(x.device):
@@ -445,8 +475,6 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
                 raise ValueError("split_c and a stream-K workspace are exclusive")
             mode = {"auto": 0, "off": 1, "on": 2}[stream_k]
             wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
-            if ws is not None and not ws.is_cuda:
-                raise ValueError("ws must be a CUDA tensor")
             _check(lib().wino_conv2d_f2x3_fwd_ws(*args, mode, wp, wb, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd_ws")
         elif split_c:
             _check(lib().wino_conv2d_f2x3_fwd_split(*args, int(split_c), _stream_ptr(stream)),
@@ -467,6 +495,7 @@ def filter_transform_kcrs(w_kcrs: torch.Tensor, out: torch.Tensor | None = None,
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (C, 4, 4, K):
         raise ValueError("out must be (C,4,4,K)")
+    _same_device(w_kcrs, out=out)
     with torch.cuda.device(w_kcrs.device):
         _check(lib().wino_filter_transform_kcrs(ctypes.c_void_p(w_kcrs.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                                 C, K, _stream_ptr(stream)), "wino_filter_transform_kcrs")
@@ -497,10 +526,10 @@ def conv2d_nchw(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = Non
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (N, K, H, W):
         raise ValueError("out must be (N,K,H,W)")
+    _same_device(x, u=u, out=out)
+    _need_ws(ws, x)
     with torch.cuda.device(x.device):
         if ws is not None:
-            if not ws.is_cuda:
-                raise ValueError("ws must be a CUDA tensor")
             _check(lib().wino_conv2d_f2x3_fwd_nchw_ws(
                 ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                 N, C, H, W, K, 1, 1, ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size(),
@@ -517,10 +546,16 @@ def nonfused_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
     return int(lib().wino_nonfused_workspace_bytes(N, C, H, W, K))
 
 
+def nonfused_launches() -> int:
+    """Kernels one conv2d_nonfused call launches (u arrangement, ITF, GEMM, OTF)."""
+    return int(lib().wino_nonfused_launches())
+
+
 def conv2d_nonfused(x: torch.Tensor, u: torch.Tensor, ws: torch.Tensor, out: torch.Tensor | None = None,
                     stream=None, tf32: bool = False) -> torch.Tensor:
     """NEXT row N3 (Sec. 9): NON-fused Winograd -- ITF kernel to a global workspace,
-    16 batched GEMMs (cuBLAS SGEMM; tf32=True: cuBLAS TF32 tensor-core GEMMs), OTF kernel.
+    16 batched GEMMs on the tcgen05 tensor cores (this library's kernel: 3xTF32, FP32-level accuracy;
+    tf32=True: plain TF32), OTF kernel (4 launches, nonfused_launches()).
     x (C,H,W,N), u (C,4,4,K) -> y (K,H,W,N); ws: CUDA byte buffer of >= nonfused_workspace_bytes."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u, "u", 4)
@@ -528,13 +563,13 @@ def conv2d_nonfused(x: torch.Tensor, u: torch.Tensor, ws: torch.Tensor, out: tor
     if u.shape[0] != C or tuple(u.shape[1:3]) != (4, 4):
         raise ValueError(f"u must be (C,4,4,K) with C={C}, got {tuple(u.shape)}")
     K = u.shape[3]
-    if not ws.is_cuda or not ws.is_contiguous():
-        raise ValueError("ws must be a contiguous CUDA tensor")
+    _need_ws(ws, x)
     if out is None:
         out = torch.empty((K, H, W, N), dtype=torch.float32, device=x.device)
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N):
         raise ValueError("out must be (K,H,W,N)")
+    _same_device(x, u=u, out=out)
     fn = "wino_conv2d_f2x3_fwd_nonfused_tf32" if tf32 else "wino_conv2d_f2x3_fwd_nonfused"
     with torch.cuda.device(x.device):
         _check(getattr(lib(), fn)(
@@ -559,6 +594,7 @@ def filter_transform_f4(w: torch.Tensor, out: torch.Tensor | None = None, stream
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (C, 6, 6, K):
         raise ValueError("out must be (C,6,6,K)")
+    _same_device(w, out=out)
     with torch.cuda.device(w.device):
         _check(lib().wino_filter_transform_f4(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                               C, K, _stream_ptr(stream)), "wino_filter_transform_f4")
@@ -588,12 +624,12 @@ def conv2d_f4(x: torch.Tensor, u4: torch.Tensor, out: torch.Tensor | None = None
     _need_cuda_f32(out, "out", 4)
     if tuple(out.shape) != (K, H, W, N):
         raise ValueError("out must be (K,H,W,N)")
+    _same_device(x, u4=u4, out=out)
+    _need_ws(ws, x)
     args = (ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(u4.data_ptr()), ctypes.c_void_p(out.data_ptr()),
             N, C, H, W, K, 1, 1)
     with torch.cuda.device(x.device):
         if ws is not None or stream_k == "on":
-            if ws is not None and not ws.is_cuda:
-                raise ValueError("ws must be a CUDA tensor")
             wp, wb = (ctypes.c_void_p(ws.data_ptr()), ws.numel() * ws.element_size()) if ws is not None else (None, 0)
             _check(lib().wino_conv2d_f4x3_fwd_ws(*args, {"auto": 0, "off": 1, "on": 2}[stream_k], wp, wb,
                                                  _stream_ptr(stream)), "wino_conv2d_f4x3_fwd_ws")
@@ -610,8 +646,7 @@ def conv2d_host(x_host: torch.Tensor, w_host: torch.Tensor, y_host: torch.Tensor
     for t, n in ((x_host, "x_host"), (w_host, "w_host"), (y_host, "y_host")):
         if t.is_cuda or t.dtype != torch.float32 or not t.is_contiguous() or t.dim() != 4:
             raise ValueError(f"{n} must be a contiguous 4-d float32 CPU tensor")
-    if not ws.is_cuda:
-        raise ValueError("ws must be a CUDA tensor")
+    _need_ws(ws, ws)
     C, H, W, N = x_host.shape
     K = w_host.shape[3]
     if tuple(y_host.shape) != (K, H, W, N) or tuple(w_host.shape) != (C, 3, 3, K):
@@ -647,8 +682,7 @@ def conv2d_host_multi(layers, ws: torch.Tensor, stream=None) -> None:
     """End-to-end multi-layer call on pinned host buffers with H2D / compute / D2H overlap
     (``wino_conv2d_f2x3_fwd_host_multi``); asynchronous on the stream."""
     arr = _host_layers(layers)
-    if not ws.is_cuda:
-        raise ValueError("ws must be a CUDA tensor")
+    _need_ws(ws, ws)
     with torch.cuda.device(ws.device):
         _check(lib().wino_conv2d_f2x3_fwd_host_multi(arr, len(layers), ctypes.c_void_p(ws.data_ptr()),
                                                      ws.numel() * ws.element_size(), _stream_ptr(stream)),

@@ -186,7 +186,11 @@ struct Cfg {
     static constexpr int UNITS_PER_CB = 16 / XPU;
     static constexpr int A_TILE = a_tile<MM>();
     static constexpr int UNIT = XPU * P * A_TILE;               // 64 KB (MM=128) / 32 KB (MM=64)
+#ifdef WINO_TC_DBG_U2
+    static constexpr int U_SLOTS = 2;
+#else
     static constexpr int U_SLOTS = (MM == 64 && XM >= 2) ? 3 : 2;
+#endif
     static constexpr int X_SLOTS = 2;                           // raw x boxes in flight (L2-prefetched)
     static constexpr int X_SLOT = NH * XS_BYTES;
     static constexpr int V_SLOT = 16 * NH * P * B_TILE;        // 16 / 32 KB
@@ -233,12 +237,17 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             mbar_init(&u_full[s], 1);
             mbar_init(&u_empty[s], 1);
         }
+#ifdef WINO_TC_DBG_PERLANE
+        constexpr int ARR = 32;  // debug: every ITF lane arrives itself
+#else
+        constexpr int ARR = 1;
+#endif
         for (int s = 0; s < G::X_SLOTS; ++s) {
             mbar_init(&x_full[s], 1);
-            mbar_init(&x_empty[s], ITF_WARPS);
+            mbar_init(&x_empty[s], ITF_WARPS * ARR);
         }
         for (int s = 0; s < 2; ++s) {
-            mbar_init(&v_full[s], ITF_WARPS);
+            mbar_init(&v_full[s], ITF_WARPS * ARR);
             mbar_init(&v_empty[s], 1);
         }
         mbar_init(acc_full, 1);
@@ -446,8 +455,12 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                     for (int e = 0; e < 16; ++e) d[e] = xsrc[e * xnb];
                     itf_4x4(d, t[h]);  // consumes the loads
                 }
+#ifdef WINO_TC_DBG_PERLANE
+                mbar_arrive(&x_empty[xs]);
+#else
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&x_empty[xs]);  // the x slot can be refilled
+#endif
                 if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
                 uint8_t* vdst = sv + vs * G::V_SLOT + voff;
 #pragma unroll
@@ -460,8 +473,12 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                             *reinterpret_cast<float*>(vdst + ((xi * NH + h) * P + 1) * B_TILE) = to_tf32(t[h][xi] - big);
                     }
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
+#ifdef WINO_TC_DBG_PERLANE
+                mbar_arrive(&v_full[vs]);
+#else
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&v_full[vs]);
+#endif
             }
         }
     } else {

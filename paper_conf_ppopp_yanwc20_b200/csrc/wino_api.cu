@@ -12,6 +12,7 @@
 #include <cstdint>
 #include <cstring>
 #include <mutex>
+#include <new>
 
 #include "../../include/wino.h"
 #include "ftf.cuh"
@@ -21,9 +22,9 @@
 #include "fused_tc16.cuh"
 #include "fused_f4_fp32.cuh"
 #include "nonfused.cuh"
+#include "nonfused_tc.cuh"
 #include "layout.cuh"
 
-#include <dlfcn.h>
 
 namespace {
 
@@ -233,7 +234,8 @@ PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
 // fp32 tensor map, dims innermost first; strides (bytes, dims 1..rank-1) default to dense.
 bool encode_map(CUtensorMap* m, const void* base, int rank, const cuuint64_t* dims, const cuuint32_t* box,
                 const cuuint64_t* strides_in = nullptr,
-                CUtensorMapDataType dtype = CU_TENSOR_MAP_DATA_TYPE_FLOAT32, int esize = 4) {
+                CUtensorMapDataType dtype = CU_TENSOR_MAP_DATA_TYPE_FLOAT32, int esize = 4,
+                CUtensorMapSwizzle swizzle = CU_TENSOR_MAP_SWIZZLE_NONE) {
     auto enc = tensor_map_encoder();
     if (!enc) return false;
     cuuint64_t strides[4];
@@ -244,7 +246,7 @@ bool encode_map(CUtensorMap* m, const void* base, int rank, const cuuint64_t* di
     }
     cuuint32_t estr[5] = {1, 1, 1, 1, 1};
     CUresult r = enc(m, dtype, rank, const_cast<void*>(base), dims, strides, box, estr,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);  // OOB elements read as zero
     return r == CUDA_SUCCESS;
 }
@@ -470,20 +472,25 @@ wino_status_t helper_streams(int dev, cudaStream_t* in, cudaStream_t* out) {
     return WINO_OK;
 }
 
-// Events used for cross-stream ordering within one call; destroyed at the end of
-// the call (CUDA releases them once the recorded work completes).
+// Events used for cross-stream ordering within one call, all created before anything is
+// queued (the count is known from the layer list) and destroyed at the end of the call
+// (CUDA releases an event once the work recorded on it completes).
 struct EventPool {
-    cudaEvent_t ev[256];
-    int n = 0;
-    cudaEvent_t get() {
-        if (n == 256) return nullptr;
-        cudaEvent_t e;
-        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
-        ev[n++] = e;
-        return e;
+    cudaEvent_t* ev = nullptr;
+    int n = 0, cap = 0;
+    cudaError_t reserve(int count) {
+        ev = new (std::nothrow) cudaEvent_t[count];
+        if (!ev) return cudaErrorMemoryAllocation;
+        for (; cap < count; ++cap) {
+            cudaError_t e = cudaEventCreateWithFlags(&ev[cap], cudaEventDisableTiming);
+            if (e != cudaSuccess) return e;
+        }
+        return cudaSuccess;
     }
+    cudaEvent_t get() { return n < cap ? ev[n++] : nullptr; }
     ~EventPool() {
-        for (int i = 0; i < n; ++i) cudaEventDestroy(ev[i]);
+        for (int i = 0; i < cap; ++i) cudaEventDestroy(ev[i]);
+        delete[] ev;
     }
 };
 
@@ -771,9 +778,10 @@ extern "C++" {
 namespace {
 size_t round256(size_t b) { return (b + 255) & ~size_t(255); }
 cudaError_t transpose2d(const float* in, float* out, int R, long long S, cudaStream_t st) {
-    const dim3 grid(static_cast<unsigned>((S + wino::TR_TILE - 1) / wino::TR_TILE),
-                    static_cast<unsigned>((R + wino::TR_TILE - 1) / wino::TR_TILE));
-    wino::transpose2d_kernel<<<grid, dim3(wino::TR_TILE, wino::TR_ROWS), 0, st>>>(in, out, R, S);
+    // 1-D grid over (row tile, column tile) pairs: R * S < 2^31 elements, so < 2^21 tiles
+    const long long tiles = ((S + wino::TR_TILE - 1) / wino::TR_TILE) * ((R + wino::TR_TILE - 1) / wino::TR_TILE);
+    wino::transpose2d_kernel<<<dim3(static_cast<unsigned>(tiles)), dim3(wino::TR_TILE, wino::TR_ROWS), 0, st>>>(
+        in, out, R, S);
     return cudaGetLastError();
 }
 }  // namespace
@@ -1168,12 +1176,22 @@ size_t wino_host_multi_workspace_bytes(const wino_host_layer_t* layers, int n_la
 wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, int n_layers, void* ws_dev,
                                               size_t ws_bytes, wino_stream_t stream) {
     if (!layers || n_layers <= 0 || !ws_dev) return WINO_ERR_INVALID_ARG;
+    // per layer: slice along K (contiguous copies) when K >= 128, else along the batch (2-D copies)
+    auto slices = [](const wino_host_layer_t& L, bool* kslice) {
+        *kslice = L.K >= 128;
+        return *kslice ? (L.K >= 256 ? 4 : 2) : (L.N >= 128 && L.N % 64 == 0 ? L.N / 64 : 1);
+    };
+    int64_t n_events = 1 + 1 + 2;  // fork, final join, error-path joins (s_in, s_out)
     for (int i = 0; i < n_layers; ++i) {
         const wino_host_layer_t& L = layers[i];
         if (!L.x_host || !L.w_host || !L.y_host) return WINO_ERR_INVALID_ARG;
         wino_status_t s = check_shape(L.N, L.C, L.H, L.W, L.K, 1, 1);
         if (s != WINO_OK) return s;
+        bool ks;
+        const int ns = slices(L, &ks);
+        n_events += 1 + ((ks || ns == 1) ? 1 + ns : 2 * ns);
     }
+    if (n_events > 65536) return WINO_ERR_TOO_LARGE;
     if (ws_bytes < wino_host_multi_workspace_bytes(layers, n_layers)) return WINO_ERR_INVALID_ARG;
     if (!aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
     int dev;
@@ -1182,14 +1200,22 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
     cudaStream_t s_in, s_out;
     if ((s = helper_streams(dev, &s_in, &s_out)) != WINO_OK) return s;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    EventPool ev;
-    cudaError_t e;
-#define WINO_TRY(expr)                            \
-    do {                                          \
-        if ((e = (expr)) != cudaSuccess) return cuda_fail(e); \
+    EventPool ev;  // every event this call needs, created before anything is queued
+    cudaError_t e = ev.reserve(static_cast<int>(n_events));
+    if (e != cudaSuccess) return cuda_fail(e);
+    cudaEvent_t j_in = ev.get(), j_out = ev.get();
+    // Error after work was queued: the caller's stream must still not run ahead of the copies
+    // already queued on the helper streams (they read / write the caller's host buffers).
+    auto fail = [&](wino_status_t status) {
+        if (cudaEventRecord(j_in, s_in) == cudaSuccess) cudaStreamWaitEvent(st, j_in, 0);
+        if (cudaEventRecord(j_out, s_out) == cudaSuccess) cudaStreamWaitEvent(st, j_out, 0);
+        return status;
+    };
+#define WINO_TRY(expr)                                        \
+    do {                                                      \
+        if ((e = (expr)) != cudaSuccess) return fail(cuda_fail(e)); \
     } while (0)
     cudaEvent_t e0 = ev.get();
-    if (!e0) return cuda_fail(cudaErrorMemoryAllocation);
     WINO_TRY(cudaEventRecord(e0, st));
     WINO_TRY(cudaStreamWaitEvent(s_in, e0, 0));
     WINO_TRY(cudaStreamWaitEvent(s_out, e0, 0));
@@ -1207,17 +1233,14 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
         // weights in, FTF on the compute stream
         WINO_TRY(cudaMemcpyAsync(w_dev, L.w_host, wb, cudaMemcpyHostToDevice, s_in));
         cudaEvent_t ew = ev.get();
-        if (!ew) return cuda_fail(cudaErrorMemoryAllocation);
         WINO_TRY(cudaEventRecord(ew, s_in));
         WINO_TRY(cudaStreamWaitEvent(st, ew, 0));
-        if ((s = wino_filter_transform(w_dev, u_dev, L.C, L.K, stream)) != WINO_OK) return s;
-        // slicing: along K (contiguous copies) when K >= 128, else along the batch (2-D copies)
-        const bool kslice = L.K >= 128;
-        const int nslice = kslice ? (L.K >= 256 ? 4 : 2) : (L.N >= 128 && L.N % 64 == 0 ? L.N / 64 : 1);
+        if ((s = wino_filter_transform(w_dev, u_dev, L.C, L.K, stream)) != WINO_OK) return fail(s);
+        bool kslice;
+        const int nslice = slices(L, &kslice);
         if (kslice || nslice == 1) {
             WINO_TRY(cudaMemcpyAsync(x_dev, L.x_host, xb, cudaMemcpyHostToDevice, s_in));
             cudaEvent_t ex = ev.get();
-            if (!ex) return cuda_fail(cudaErrorMemoryAllocation);
             WINO_TRY(cudaEventRecord(ex, s_in));
             WINO_TRY(cudaStreamWaitEvent(st, ex, 0));
             const int kc = ((L.K + nslice - 1) / nslice + 63) / 64 * 64;
@@ -1225,9 +1248,8 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
                 const int k1 = k0 + kc < L.K ? k0 + kc : L.K;
                 if ((s = launch_fwd_fp32(x_dev, u_dev + k0, L.K, y_dev + size_t(k0) * hwn, L.N, L.C, L.H, L.W,
                                          k1 - k0, dev, st)) != WINO_OK)
-                    return s;
+                    return fail(s);
                 cudaEvent_t ec = ev.get();
-                if (!ec) return cuda_fail(cudaErrorMemoryAllocation);
                 WINO_TRY(cudaEventRecord(ec, st));
                 WINO_TRY(cudaStreamWaitEvent(s_out, ec, 0));
                 WINO_TRY(cudaMemcpyAsync(L.y_host + size_t(k0) * hwn, y_dev + size_t(k0) * hwn,
@@ -1242,12 +1264,11 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
                 WINO_TRY(cudaMemcpy2DAsync(xj, size_t(nc) * 4, L.x_host + size_t(j) * nc, size_t(L.N) * 4,
                                            size_t(nc) * 4, size_t(L.C) * hw, cudaMemcpyHostToDevice, s_in));
                 cudaEvent_t ex = ev.get();
-                if (!ex) return cuda_fail(cudaErrorMemoryAllocation);
                 WINO_TRY(cudaEventRecord(ex, s_in));
                 WINO_TRY(cudaStreamWaitEvent(st, ex, 0));
-                if ((s = launch_fwd_fp32(xj, u_dev, L.K, yj, nc, L.C, L.H, L.W, L.K, dev, st)) != WINO_OK) return s;
+                if ((s = launch_fwd_fp32(xj, u_dev, L.K, yj, nc, L.C, L.H, L.W, L.K, dev, st)) != WINO_OK)
+                    return fail(s);
                 cudaEvent_t ec = ev.get();
-                if (!ec) return cuda_fail(cudaErrorMemoryAllocation);
                 WINO_TRY(cudaEventRecord(ec, st));
                 WINO_TRY(cudaStreamWaitEvent(s_out, ec, 0));
                 WINO_TRY(cudaMemcpy2DAsync(L.y_host + size_t(j) * nc, size_t(L.N) * 4, yj, size_t(nc) * 4,
@@ -1256,7 +1277,6 @@ wino_status_t wino_conv2d_f2x3_fwd_host_multi(const wino_host_layer_t* layers, i
         }
     }
     cudaEvent_t eo = ev.get();
-    if (!eo) return cuda_fail(cudaErrorMemoryAllocation);
     WINO_TRY(cudaEventRecord(eo, s_out));
     WINO_TRY(cudaStreamWaitEvent(st, eo, 0));  // caller's stream completes after every copy
 #undef WINO_TRY
@@ -1389,55 +1409,95 @@ wino_status_t wino_conv2d_f4x3_fwd_ws(const float* x_dev, const float* u4_dev, f
 }  // extern "C"
 
 // ---------------------------------------------------------------------------
-// NEXT row N3: non-fused Winograd (ITF kernel -> 16 library GEMMs -> OTF kernel)
+// NEXT row N3: non-fused Winograd (u arrangement, ITF kernel -> V workspace, 16 batched
+// tcgen05 GEMMs -> M workspace, OTF kernel); nonfused_tc.cuh
 // ---------------------------------------------------------------------------
 namespace {
-// cuBLAS is loaded on first use (dlopen), so libwino.so itself has no link-time
-// dependency on it; without cuBLAS the non-fused entry point returns UNSUPPORTED.
-typedef int (*cublasCreate_t)(void**);
-typedef int (*cublasSetStream_t)(void*, cudaStream_t);
-typedef int (*cublasSetMathMode_t)(void*, int);
-typedef int (*cublasSgemmStridedBatched_t)(void*, int, int, int, int, int, const float*, const float*, int,
-                                           long long, const float*, int, long long, const float*, float*, int,
-                                           long long, int);
-struct Cublas {
-    cublasCreate_t create = nullptr;
-    cublasSetStream_t set_stream = nullptr;
-    cublasSetMathMode_t set_math = nullptr;
-    cublasSgemmStridedBatched_t sgemm_sb = nullptr;
-    void* handle[kMaxDevices][2] = {};  // [device][0: pedantic FP32, 1: TF32 tensor ops]
-    bool ok = false;
+// workspace carve-up for P planes (P = 2: 3xTF32, the FP32-accuracy variant; P = 1: TF32)
+struct NfLayout {
+    size_t v_off, u_off, m_off, total;
 };
-std::mutex g_cublas_mu;
-Cublas g_cublas;
-bool g_cublas_tried = false;
-
-bool cublas_load() {
-    if (g_cublas_tried) return g_cublas.ok;
-    g_cublas_tried = true;
-    void* h = dlopen("libcublas.so.12", RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
-    if (!h) h = dlopen("libcublas.so.12", RTLD_NOW | RTLD_GLOBAL);
-    if (!h) h = dlopen("libcublas.so", RTLD_NOW | RTLD_GLOBAL);
-    if (!h) return false;
-    g_cublas.create = reinterpret_cast<cublasCreate_t>(dlsym(h, "cublasCreate_v2"));
-    g_cublas.set_stream = reinterpret_cast<cublasSetStream_t>(dlsym(h, "cublasSetStream_v2"));
-    g_cublas.set_math = reinterpret_cast<cublasSetMathMode_t>(dlsym(h, "cublasSetMathMode"));
-    g_cublas.sgemm_sb = reinterpret_cast<cublasSgemmStridedBatched_t>(dlsym(h, "cublasSgemmStridedBatched"));
-    g_cublas.ok = g_cublas.create && g_cublas.set_stream && g_cublas.set_math && g_cublas.sgemm_sb;
-    return g_cublas.ok;
+NfLayout nf_layout(int N, int C, int H, int W, int K, int P) {
+    const size_t nv = size_t(N) * ((H + 1) / 2) * ((W + 1) / 2), c4 = size_t(wino::nftc::cp4(C));
+    NfLayout L;
+    L.v_off = 0;
+    L.u_off = round_up256(size_t(16) * P * nv * c4 * 4);
+    L.m_off = L.u_off + round_up256(size_t(16) * P * K * c4 * 4);
+    L.total = L.m_off + round_up256(size_t(16) * K * nv * 4);
+    return L;
 }
-constexpr int kCublasOpN = 0, kCublasOpT = 1;
-constexpr int kCublasPedanticMath = 2;  // CUBLAS_PEDANTIC_MATH: plain FP32, no TF32 tensor-op shortcuts
-constexpr int kCublasTf32Math = 3;      // CUBLAS_TF32_TENSOR_OP_MATH: the library's TF32 tensor-core GEMMs
+std::atomic<uint64_t> g_attr_nf_gemm[2], g_attr_nf_itf[2];
+
+template <int P>
+wino_status_t nonfused_launch(const float* x_dev, const float* u_dev, float* y_dev, int N, int C, int H, int W, int K,
+                              char* ws, int dev, cudaStream_t st) {
+    using namespace wino::nftc;
+    const NfLayout L = nf_layout(N, C, H, W, K, P);
+    float* v = reinterpret_cast<float*>(ws + L.v_off);
+    float* ug = reinterpret_cast<float*>(ws + L.u_off);
+    float* m = reinterpret_cast<float*>(ws + L.m_off);
+    const int TW = (W + 1) / 2;
+    const int NV = N * ((H + 1) / 2) * TW;
+    const int C4 = cp4(C), bnk = gemm_bnk(K);
+    GemmParams gp;
+    std::memset(&gp, 0, sizeof(gp));
+    {
+        const cuuint64_t dims[3] = {cuuint64_t(C), cuuint64_t(NV), cuuint64_t(16 * P)};
+        const cuuint64_t strides[2] = {cuuint64_t(C4) * 4, cuuint64_t(NV) * C4 * 4};
+        const cuuint32_t box[3] = {BKC, BM, 1};
+        if (!encode_map(&gp.tmv, v, 3, dims, box, strides, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4,
+                        CU_TENSOR_MAP_SWIZZLE_128B))
+            return cuda_fail(cudaErrorInvalidValue);
+    }
+    {
+        const cuuint64_t dims[3] = {cuuint64_t(C), cuuint64_t(K), cuuint64_t(16 * P)};
+        const cuuint64_t strides[2] = {cuuint64_t(C4) * 4, cuuint64_t(K) * C4 * 4};
+        const cuuint32_t box[3] = {BKC, cuuint32_t(bnk), 1};
+        if (!encode_map(&gp.tmu, ug, 3, dims, box, strides, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4,
+                        CU_TENSOR_MAP_SWIZZLE_128B))
+            return cuda_fail(cudaErrorInvalidValue);
+    }
+    gp.m = m;
+    gp.K = K;
+    gp.NV = NV;
+    gp.C = C;
+    gp.bnk = bnk;
+    gp.stages = gemm_stages<P>(bnk);
+    gp.nchunks = (C + BKC - 1) / BKC;
+    wino_status_t s;
+    // 1. transformed filter -> GEMM operand layout (TF32 planes)
+    nf_arrange_u_kernel<P><<<dim3(unsigned((K + 31) / 32), unsigned((C4 + 31) / 32), 16), 256, 0, st>>>(u_dev, ug, C,
+                                                                                                       K);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e);
+    // 2. ITF -> V [16 P][NV][C4]
+    if ((s = ensure_smem_attr(nf_itf_kernel<P>, dev, ITF_SMEM, g_attr_nf_itf[P - 1])) != WINO_OK) return s;
+    nf_itf_kernel<P><<<dim3(unsigned((NV + 31) / 32), unsigned((C4 + 31) / 32)), 256, ITF_SMEM, st>>>(x_dev, v, N, C,
+                                                                                                     H, W, TW, NV);
+    if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e);
+    // 3. the 16 batched GEMMs on tcgen05: M[xi][k][nu]
+    const int smem = gemm_smem_bytes<P>(bnk);
+    if ((s = ensure_smem_attr(nf_gemm_kernel<P>, dev, gemm_smem_bytes<P>(256), g_attr_nf_gemm[P - 1])) != WINO_OK)
+        return s;
+    nf_gemm_kernel<P><<<dim3(unsigned((NV + BM - 1) / BM), unsigned((K + bnk - 1) / bnk), 16), GEMM_THREADS, smem,
+                        st>>>(gp);
+    if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e);
+    // 4. OTF -> y
+    wino::nf::otf_nf_kernel<<<unsigned((int64_t(K) * NV + wino::nf::THREADS - 1) / wino::nf::THREADS),
+                              wino::nf::THREADS, 0, st>>>(m, y_dev, N, K, H, W, TW, NV);
+    e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
 }  // namespace
 
 extern "C" {
 
 size_t wino_nonfused_workspace_bytes(int N, int C, int H, int W, int K) {
     if (check_shape(N, C, H, W, K, 1, 1) != WINO_OK) return 0;
-    const size_t nv = size_t(N) * ((H + 1) / 2) * ((W + 1) / 2);
-    return round_up256(size_t(16) * C * nv * 4) + round_up256(size_t(16) * K * nv * 4);
+    return nf_layout(N, C, H, W, K, 2).total;  // the 3xTF32 (two-plane) layout; TF32 uses a prefix of it
 }
+
+int wino_nonfused_launches(void) { return 4; }
 
 extern "C++" {
 namespace {
@@ -1447,48 +1507,22 @@ wino_status_t conv_nonfused(const float* x_dev, const float* u_dev, float* y_dev
     wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
     if (s != WINO_OK) return s;
     if (!aligned16(x_dev) || !aligned16(u_dev) || !aligned16(y_dev) || !aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
-    const size_t need = wino_nonfused_workspace_bytes(N, C, H, W, K);
-    if (ws_bytes < need) return WINO_ERR_INVALID_ARG;
+    const int P = tf32 ? 1 : 2;
+    const NfLayout L = nf_layout(N, C, H, W, K, P);
+    if (ws_bytes < L.total) return WINO_ERR_INVALID_ARG;
     const long long nv = (long long)N * ((H + 1) / 2) * ((W + 1) / 2);
-    if ((long long)16 * C * nv > kMaxElems || (long long)16 * K * nv > kMaxElems) return WINO_ERR_TOO_LARGE;
+    const long long c4 = wino::nftc::cp4(C);
+    if ((long long)16 * 2 * c4 * nv > kMaxElems || (long long)16 * K * nv > kMaxElems) return WINO_ERR_TOO_LARGE;
     const size_t hwn = size_t(H) * W * N, yb = size_t(K) * hwn * 4;
     if (overlaps(y_dev, yb, x_dev, size_t(C) * hwn * 4) || overlaps(y_dev, yb, u_dev, size_t(16) * C * K * 4) ||
-        overlaps(ws_dev, need, x_dev, size_t(C) * hwn * 4) || overlaps(ws_dev, need, u_dev, size_t(16) * C * K * 4) ||
-        overlaps(ws_dev, need, y_dev, yb))
+        overlaps(ws_dev, L.total, x_dev, size_t(C) * hwn * 4) || overlaps(ws_dev, L.total, u_dev, size_t(16) * C * K * 4) ||
+        overlaps(ws_dev, L.total, y_dev, yb))
         return WINO_ERR_INVALID_ARG;
     int dev;
     if ((s = check_device(&dev)) != WINO_OK) return s;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    float* v = static_cast<float*>(ws_dev);
-    float* m = reinterpret_cast<float*>(static_cast<char*>(ws_dev) + round_up256(size_t(16) * C * nv * 4));
-    const int TW = (W + 1) / 2;
-    // 1. ITF -> V [16][C][NV]
-    wino::nf::itf_nf_kernel<<<unsigned((C * nv + wino::nf::THREADS - 1) / wino::nf::THREADS), wino::nf::THREADS, 0,
-                              st>>>(x_dev, v, N, C, H, W, TW, nv);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_fail(e);
-    // 2. M[xi] = U[xi]^T V[xi], xi = 0..15, one strided-batched SGEMM.  Row-major M[k][nu]
-    //    is column-major M^T (NV x K): M^T = V^T (NV x C, ld NV) * U (C x K from u[c][xi][k],
-    //    column-major view K x C with ld 16K -> op T).
-    {
-        std::lock_guard<std::mutex> lk(g_cublas_mu);
-        if (!cublas_load()) return WINO_ERR_UNSUPPORTED;
-        if (!g_cublas.handle[dev][tf32]) {
-            if (g_cublas.create(&g_cublas.handle[dev][tf32]) != 0) return WINO_ERR_CUDA;
-            g_cublas.set_math(g_cublas.handle[dev][tf32], tf32 ? kCublasTf32Math : kCublasPedanticMath);
-        }
-        void* hd = g_cublas.handle[dev][tf32];
-        if (g_cublas.set_stream(hd, st) != 0) return WINO_ERR_CUDA;
-        const float one = 1.f, zero = 0.f;
-        if (g_cublas.sgemm_sb(hd, kCublasOpN, kCublasOpT, (int)nv, K, C, &one, v, (int)nv, (long long)C * nv, u_dev,
-                              16 * K, (long long)K, &zero, m, (int)nv, (long long)K * nv, 16) != 0)
-            return WINO_ERR_CUDA;
-    }
-    // 3. OTF -> y
-    wino::nf::otf_nf_kernel<<<unsigned((K * nv + wino::nf::THREADS - 1) / wino::nf::THREADS), wino::nf::THREADS, 0,
-                              st>>>(m, y_dev, N, K, H, W, TW, nv);
-    e = cudaGetLastError();
-    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+    return tf32 ? nonfused_launch<1>(x_dev, u_dev, y_dev, N, C, H, W, K, static_cast<char*>(ws_dev), dev, st)
+                : nonfused_launch<2>(x_dev, u_dev, y_dev, N, C, H, W, K, static_cast<char*>(ws_dev), dev, st);
 }
 }  // namespace
 }  // extern "C++"

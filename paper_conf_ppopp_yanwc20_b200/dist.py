@@ -52,6 +52,8 @@ class BatchShardedConv:
 
     >>> layer = BatchShardedConv(w, group=None, src=0)   # FTF on src + NCCL broadcast of u
     >>> y_local = layer(x_local)                          # fused Winograd on this rank's shard
+
+    `src` is the source rank within `group` (the default group: the global rank).
     """
 
     def __init__(self, w_crsk: Optional[torch.Tensor], C: int, K: int, *, device=None, group=None, src: int = 0,
@@ -67,7 +69,10 @@ class BatchShardedConv:
         else:
             self.u = torch.empty((C, 4, 4, K), dtype=torch.float32, device=device)
         if self.world > 1:
-            dist.broadcast(self.u, src=src, group=group)
+            # src is a rank of `group` (the comparison above uses the group-local rank);
+            # dist.broadcast takes a global rank
+            gsrc = dist.get_global_rank(group, src) if group is not None else src
+            dist.broadcast(self.u, src=gsrc, group=group)
 
     def __call__(self, x_local: torch.Tensor) -> torch.Tensor:
         return self.conv(x_local, self.u)

@@ -116,13 +116,19 @@ def test_fwd_argument_validation_host_side():
 
 
 def test_nonfused_workspace_bytes():
-    """V[16][C][NV] + M[16][K][NV] floats, each rounded up to 256 B (NEXT row N3)."""
+    """NEXT row N3 (include/wino.h): V[16*2][NV][Cp4] + Ug[16*2][K][Cp4] + M[16][K][NV] floats
+    (two TF32 planes per operand for the 3xTF32 GEMMs, Cp4 = 4*ceil(C/4)), each part rounded up
+    to 256 B; 4 launches per call."""
+    rnd = lambda b: -(-b // 256) * 256  # noqa: E731
     for name in ("conv5_x", "conv4_x", "conv3_x", "conv2_x", "tiny"):
         c = CONFIGS[name]
         nv = c.N * c.tiles
-        rnd = lambda b: -(-b // 256) * 256  # noqa: E731
-        assert wino.nonfused_workspace_bytes(c.N, c.C, c.H, c.W, c.K) == rnd(64 * c.C * nv) + rnd(64 * c.K * nv)
+        c4 = -(-c.C // 4) * 4
+        assert wino.nonfused_workspace_bytes(c.N, c.C, c.H, c.W, c.K) == \
+            rnd(128 * nv * c4) + rnd(128 * c.K * c4) + rnd(64 * c.K * nv)
+    assert wino.nonfused_workspace_bytes(3, 5, 5, 5, 4) == rnd(128 * 27 * 8) + rnd(128 * 4 * 8) + rnd(64 * 4 * 27)
     assert wino.nonfused_workspace_bytes(0, 3, 5, 5, 4) == 0
+    assert wino.nonfused_launches() == 4
 
 
 @pytest.mark.parametrize("P", [2, 4, 8])

@@ -83,3 +83,40 @@ def test_batch_sharded_matches_full(world, N):
         p.join(timeout=180)
     assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
     assert q.get(timeout=10) is True
+
+
+def _worker_subgroup(rank, world, port, q):
+    """Ranks 1 and 2 of 3 form a subgroup; src=0 names the subgroup's first rank (global 1)."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from synth_inputs import Conv3x3Config, make_inputs
+        sub = dist.new_group([1, 2])
+        if rank in (1, 2):
+            cfg = Conv3x3Config("d", 4, 5, 6, 7, 6)
+            x, w = make_inputs(cfg, kind="smallint")
+            w_holder = [w]
+            layer = BatchShardedConv(w if rank == 1 else None, cfg.C, cfg.K, group=sub, src=0, ftf=_oracle_ftf,
+                                     conv=lambda xl, u: _oracle_conv_from_u(xl, u, w_holder))
+            lr = dist.get_rank(sub)
+            y_local = layer(shard_batch(x, lr, 2))
+            y = gather_batch(y_local.double(), cfg.N, group=sub)
+            if rank == 1:
+                import oracle
+                q.put(bool(np.array_equal(y.numpy(), oracle.direct_conv(x, w))))
+        dist.barrier()
+    finally:
+        dist.destroy_process_group()
+
+
+def test_batch_sharded_subgroup_src_is_group_rank():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_subgroup, args=(r, 3, port, q)) for r in range(3)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=180)
+    assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
+    assert q.get(timeout=10) is True

@@ -12,7 +12,7 @@ import pytest
 import torch
 
 import oracle
-from synth_inputs import CONFIGS, Conv3x3Config, make_inputs, sample_points
+from synth_inputs import CONFIGS, Conv3x3Config, make_inputs
 
 pytestmark = pytest.mark.gpu
 
@@ -67,17 +67,14 @@ def test_f4_matches_oracle_f4_winograd(wino):
 
 @pytest.mark.parametrize("kind", ["uniform", "resnet"])
 @pytest.mark.parametrize("name", ["conv2_x", "conv3_x", "conv4_x", "conv5_x"])
-def test_f4_full_configs_sampled(wino, name, kind):
+def test_f4_full_configs(wino, name, kind):
+    """BASELINE configs at full size (no workspace), every output element vs Eq. 4."""
     cfg = CONFIGS[name]
     x, w = make_inputs(cfg, kind=kind)
     u4, y = _run(wino, x, w)
     assert oracle.max_rel_err(u4.double().numpy(), oracle.filter_transform_f4(w)) <= FTF4_TOL
-    idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 4000)
-    ref = oracle.direct_sample(x, w, idx)
-    ii = idx.numpy()
-    got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
     assert np.isfinite(y.numpy()).all()
-    assert float(np.max(np.abs(got - ref))) / float(np.max(np.abs(ref))) <= F4_TOL
+    assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= F4_TOL
 
 
 def test_f4_deterministic_and_overwrites(wino):

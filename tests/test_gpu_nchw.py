@@ -11,7 +11,7 @@ import pytest
 import torch
 
 import oracle
-from synth_inputs import CONFIGS, Conv3x3Config, make_inputs, sample_points
+from synth_inputs import CONFIGS, Conv3x3Config, make_inputs
 
 pytestmark = pytest.mark.gpu
 
@@ -67,23 +67,6 @@ def test_nchw_random(wino, shape):
     assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= FP32_TOL
 
 
-@pytest.mark.parametrize("name", ["conv5_x", "conv4_x", "conv3_x", "conv2_x"])
-def test_nchw_full_configs_sampled(wino, name):
-    cfg = CONFIGS[name]
-    for kind in ("smallint", "uniform"):
-        x, w = make_inputs(cfg, kind=kind)
-        _, y = _run(wino, x, w)
-        idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 2000)
-        ref = oracle.direct_sample(x, w, idx)
-        ii = idx.numpy()
-        got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
-        if kind == "smallint":
-            assert np.array_equal(got, ref)
-        else:
-            den = max(float(np.max(np.abs(ref))), 1e-30)
-            assert float(np.max(np.abs(got - ref))) / den <= FP32_TOL
-
-
 def test_nchw_matches_chwn_kernel(wino):
     """Same convolution through both layouts: the NCHW path and the CHWN path agree
     within the FP32 bound (their per-output summation orders are the same kernel's)."""
@@ -123,18 +106,6 @@ def test_nchw_ws_random(wino, shape):
     x, w = make_inputs(Conv3x3Config("nchw", N, C, K, H, W), kind="uniform", seed_x=41, seed_w=42)
     y = _run_ws(wino, x, w)
     assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= FP32_TOL
-
-
-@pytest.mark.parametrize("name", ["conv5_x", "conv4_x", "conv3_x", "conv2_x"])
-def test_nchw_ws_full_configs_sampled(wino, name):
-    cfg = CONFIGS[name]
-    x, w = make_inputs(cfg, kind="uniform")
-    y = _run_ws(wino, x, w)
-    idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 3000)
-    ref = oracle.direct_sample(x, w, idx)
-    ii = idx.numpy()
-    got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
-    assert float(np.max(np.abs(got - ref))) / float(np.max(np.abs(ref))) <= FP32_TOL
 
 
 def test_nchw_ws_short_workspace_rejected(wino):

@@ -14,7 +14,7 @@ import pytest
 import torch
 
 import oracle
-from synth_inputs import CONFIGS, Conv3x3Config, make_inputs, sample_points
+from synth_inputs import CONFIGS, Conv3x3Config, make_inputs
 
 pytestmark = pytest.mark.gpu
 
@@ -71,25 +71,6 @@ def test_streamk_random(wino, shape):
     assert oracle.max_rel_err(y.double().numpy(), oracle.direct_conv(x, w)) <= FP32_TOL
 
 
-@pytest.mark.parametrize("kind", ["smallint", "uniform"])
-@pytest.mark.parametrize("name", ["conv5_x", "conv4_x", "conv3_x", "conv2_x"])
-@pytest.mark.parametrize("mode", ["auto", "on"])
-def test_streamk_full_configs_sampled(wino, name, kind, mode):
-    """BASELINE configs at full size with the workspace (bench.py's configuration) and forced."""
-    cfg = CONFIGS[name]
-    x, w = make_inputs(cfg, kind=kind)
-    y = _run(wino, x, w, cfg, mode)
-    idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 4000)
-    ref = oracle.direct_sample(x, w, idx)
-    ii = idx.numpy()
-    got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
-    assert np.isfinite(y.numpy()).all()
-    if kind == "smallint":
-        assert np.array_equal(got, ref)
-    else:
-        assert float(np.max(np.abs(got - ref))) / float(np.max(np.abs(ref))) <= FP32_TOL
-
-
 @pytest.mark.parametrize("P", [2, 4, 8])
 def test_streamk_batch_shards(wino, P):
     """The per-rank batch shards of every BASELINE layer at P ranks (planner's choice + workspace)."""
@@ -97,10 +78,7 @@ def test_streamk_batch_shards(wino, P):
         cfg = CONFIGS[name].with_batch(CONFIGS[name].N // P)
         x, w = make_inputs(cfg, kind="smallint")
         y = _run(wino, x, w, cfg, "auto")
-        idx = sample_points(cfg.K, cfg.H, cfg.W, cfg.N, 1500)
-        ii = idx.numpy()
-        got = y.double().numpy()[ii[:, 0], ii[:, 1], ii[:, 2], ii[:, 3]]
-        assert np.array_equal(got, oracle.direct_sample(x, w, idx)), (name, cfg.N)
+        assert np.array_equal(y.double().numpy(), oracle.direct_conv(x, w)), (name, cfg.N)
 
 
 def test_streamk_deterministic_and_matches_regular(wino):
