@@ -621,7 +621,7 @@ def main():
                 x, w = d["x_cpu"], d["w_cpu"]
                 if kind != "f32":  # R18: the oracle runs on the stored 16-bit values
                     dt16 = torch.float16 if kind == "fp16" else torch.bfloat16
-                    x, w = x.to(dt16), w.to(dt16)
+                    x, w = x.to(dt16).float(), w.to(dt16).float()
                 t0 = time.perf_counter()
                 r.append(oracle.direct_conv(x, w))
                 t += time.perf_counter() - t0

@@ -267,8 +267,7 @@ wino_status_t wino_conv2d_f2x3_fwd_tc(const float* x_dev, const float* u_tc_dev,
  *   ws_dev / ws_bytes : >= wino_tc_workspace_bytes(N,C,H,W,K) (SMs x 128 KiB), 16-byte aligned,
  *                       not overlapping x, u_tc or y; may be NULL / 0 when sk = 1.
  *   sk                : 0 = planner's choice, 1 = never, 2 = always (short workspace or a
- *                       gather-path N -> WINO_ERR_INVALID_ARG; TF32 with K <= 64, i.e.
- *                       64-filter tiles -> WINO_ERR_UNSUPPORTED). */
+ *                       gather-path N -> WINO_ERR_INVALID_ARG). */
 size_t wino_tc_workspace_bytes(int N, int C, int H, int W, int K);
 wino_status_t wino_conv2d_f2x3_fwd_tc_ws(const float* x_dev, const float* u_tc_dev, float* y_dev,
                                          int N, int C, int H, int W, int K, int pad, int stride,
@@ -338,8 +337,9 @@ wino_status_t wino_conv2d_f2x3_fwd_host(const float* x_host, const float* w_host
  * 36 Winograd elements, 4x4 outputs per tile); same computation (Eq. 4).
  *   u4 : (C,6,6,K) = G4 w G4^T, element (r',s') at [c][r'][s'][k]
  *        (36*C*K floats, wino_filter_workspace_bytes_f4)
- * The fused kernel needs N % 16 == 0 and K % 4 == 0 (TMA boxes); other shapes
- * return WINO_ERR_UNSUPPORTED.  Otherwise arguments and errors as the F(2x2) calls.
+ * Any N, C, K, H, W >= 1 (L1281): N % 16 == 0 and K % 4 == 0 take TMA boxes, other
+ * shapes a cp.async gather of the same stages (generic path, same arithmetic).
+ * Arguments and errors as the F(2x2) calls.
  */
 size_t wino_filter_workspace_bytes_f4(int C, int K);
 wino_status_t wino_filter_transform_f4(const float* w_dev, float* u4_dev, int C, int K, wino_stream_t stream);

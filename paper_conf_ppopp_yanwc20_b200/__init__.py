@@ -609,7 +609,8 @@ def f4_workspace_bytes(N: int, C: int, H: int, W: int, K: int) -> int:
 def conv2d_f4(x: torch.Tensor, u4: torch.Tensor, out: torch.Tensor | None = None, stream=None,
               ws: torch.Tensor | None = None, stream_k: str = "auto") -> torch.Tensor:
     """NEXT row N1: fused Winograd F(4x4,3x3) forward conv (FP32), pad 1 stride 1:
-    x (C,H,W,N), u4 (C,6,6,K) -> y (K,H,W,N).  Needs N % 16 == 0 and K % 4 == 0.  ws (>=
+    x (C,H,W,N), u4 (C,6,6,K) -> y (K,H,W,N); any shape (N % 16 == 0 and K % 4 == 0: TMA path,
+    else a cp.async gather path).  ws (>=
     f4_workspace_bytes) enables the stream-K plan (wino_conv2d_f4x3_fwd_ws)."""
     _need_cuda_f32(x, "x", 4)
     _need_cuda_f32(u4, "u4", 4)

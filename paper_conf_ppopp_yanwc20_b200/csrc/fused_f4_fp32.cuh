@@ -17,7 +17,12 @@
 //   * producer warpgroup (56 registers): warp 12 issues TMA, warps 13-14 run
 //     the 6x6 input transform (two passes to stay within 56 registers);
 //   * OTF through a 4-round epilogue buffer (16 filters per round).
-// Used when N % 16 == 0 and K % 4 == 0 (other shapes: WINO_ERR_UNSUPPORTED).
+// TMA path when N % 16 == 0 and K % 4 == 0.  Any other shape (the paper claims generality
+// for every N, K, C, with peak speed only at the multiples, L1281) takes the generic path
+// (GEN = true): the producer warp gathers the same [c][pos][nu] x stage with 4-byte
+// cp.async from a per-tile table of window offsets (-1 = padding: zero fill, Sec. 3.5) and
+// the [c][xi][k] u stage with 16-byte (K % 4 == 0) or 4-byte cp.async, every lane arriving on
+// the stage barrier once its copies have landed (cp.async groups, one stage behind).
 #pragma once
 #include <cuda.h>
 
@@ -41,9 +46,11 @@ constexpr int STAGE_FLOATS = US_FLOATS + XS_FLOATS;
 constexpr int VS_FLOATS = NXI * BC * BN;             // [xi][c][nu]    9 KB
 constexpr int ER_KROWS = 16, ER_LD = BN + 4;
 constexpr int ER_FLOATS = NXI * ER_KROWS * ER_LD;    // [xi][16 k][20]
+constexpr int XTAB = NXI * BN;  // generic path: window offsets of a tile's 16 nu x 36 positions
 struct Smem {
     static constexpr int ep_offset = (S * STAGE_FLOATS + SV * VS_FLOATS) * 4;
-    static constexpr int bar_offset = ep_offset + ER_FLOATS * 4;
+    static constexpr int tab_offset = ep_offset + ER_FLOATS * 4;
+    static constexpr int bar_offset = tab_offset + XTAB * 4;
     static constexpr int bytes = bar_offset + (2 * S + 2 * SV) * 8;
     static_assert(bytes <= 232448, "shared memory budget");
 };
@@ -107,6 +114,9 @@ struct __align__(64) Params {
     CUtensorMap tmx;  // x (C,H,W,N) as 4-d (N, W, H, C), box (16, 6, 6, 4)
     CUtensorMap tmu;  // u4 (C,36,K) as 3-d (K, 36, C), box (64, 36, 4)
     float* __restrict__ y;
+    const float* __restrict__ x;   // generic path: gathered with cp.async
+    const float* __restrict__ u4;  // generic path
+    int u_vec;                     // generic path: K % 4 == 0 -> 16-byte u copies
     int N, C, H, W, K;
     int TW;      // ceil(W/4)
     int NV;      // N * ceil(H/4) * ceil(W/4)
@@ -167,11 +177,12 @@ __global__ void __launch_bounds__(256) ftf4_kernel(const float* __restrict__ w, 
     for (int e = 0; e < 36; ++e) u[((size_t)c * 36 + e) * K + k] = t[e];
 }
 
-template <bool SK = false>
+template <bool SK = false, bool GEN = false>
 __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(1024) float smem[];
     float* const vs = smem + S * STAGE_FLOATS;
     float* const ep = reinterpret_cast<float*>(reinterpret_cast<char*>(smem) + Smem::ep_offset);
+    int* const xtab = reinterpret_cast<int*>(reinterpret_cast<char*>(smem) + Smem::tab_offset);
     uint64_t* const full = reinterpret_cast<uint64_t*>(reinterpret_cast<char*>(smem) + Smem::bar_offset);
     uint64_t* const empty = full + S;
     uint64_t* const vfull = empty + S;
@@ -179,10 +190,12 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 
     if (tid == 0) {
-        tma_prefetch_desc(&p.tmx);
-        tma_prefetch_desc(&p.tmu);
+        if constexpr (!GEN) {
+            tma_prefetch_desc(&p.tmx);
+            tma_prefetch_desc(&p.tmu);
+        }
         for (int s = 0; s < S; ++s) {
-            mbar_init(&full[s], 1);
+            mbar_init(&full[s], GEN ? 32 : 1);
             mbar_init(&empty[s], COMPUTE_WARPS + ITF_WARPS);
         }
         for (int s = 0; s < SV; ++s) {
@@ -195,6 +208,67 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
 
     if (warp >= COMPUTE_WARPS) {
         setmaxnreg_dec<REG_PRODUCER>();
+        if (warp == COMPUTE_WARPS && GEN) {
+            // ------------------ generic gather (any N, K): all 32 lanes ------------------
+            const size_t HWN = (size_t)p.H * p.W * p.N;
+            int G = 0;
+            Segs<SK> segs(p);
+            int tile, lo, hi;
+            while (segs.next(p, tile, lo, hi)) {
+                const int k0 = (tile % p.num_kb) * BK, nu0 = (tile / p.num_kb) * BN;
+                // window offset (h*W + w)*N + n of position pos of local nu (-1: padding / past NV);
+                // only this warp reads the table, and it has issued every copy of the previous tile
+                __syncwarp();
+                for (int e = lane; e < XTAB; e += 32) {
+                    const int pos = e / BN, nl = e % BN, nu = nu0 + nl;
+                    int off = -1;
+                    if (nu < p.NV) {
+                        const int t = nu / p.N, n = nu - t * p.N;
+                        const int th = t / p.TW, tw = t - th * p.TW;
+                        const int h = 4 * th - 1 + pos / 6, w = 4 * tw - 1 + pos % 6;
+                        if (h >= 0 && h < p.H && w >= 0 && w < p.W) off = (h * p.W + w) * p.N + n;
+                    }
+                    xtab[e] = off;
+                }
+                __syncwarp();
+                for (int g = lo; g < hi; ++g, ++G) {
+                    const int slot = G % S;
+                    if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
+                    float* us = smem + slot * STAGE_FLOATS;
+                    float* xs = us + US_FLOATS;
+                    for (int e = lane; e < XS_FLOATS; e += 32) {  // [c][pos][nu]
+                        const int c = g * BC + e / XTAB, off = xtab[e % XTAB];
+                        const bool ok = c < p.C && off >= 0;
+                        cp_async4(smem_u32(xs + e), ok ? p.x + (size_t)c * HWN + off : p.x, ok);
+                    }
+                    if (p.u_vec) {
+                        for (int e = lane; e < US_FLOATS / 4; e += 32) {  // [c][xi][k], 4 k per copy
+                            const int c = g * BC + e / (NXI * BK / 4), r = e % (NXI * BK / 4);
+                            const int xi = r / (BK / 4), k = k0 + 4 * (r % (BK / 4));
+                            const bool ok = c < p.C && k < p.K;
+                            cp_async16(smem_u32(us + 4 * e), ok ? p.u4 + ((size_t)c * NXI + xi) * p.K + k : p.u4, ok);
+                        }
+                    } else {
+                        for (int e = lane; e < US_FLOATS; e += 32) {
+                            const int c = g * BC + e / (NXI * BK), r = e % (NXI * BK);
+                            const int xi = r / BK, k = k0 + r % BK;
+                            const bool ok = c < p.C && k < p.K;
+                            cp_async4(smem_u32(us + e), ok ? p.u4 + ((size_t)c * NXI + xi) * p.K + k : p.u4, ok);
+                        }
+                    }
+                    cp_async_commit();
+                    if (G > 0) {  // the previous stage's copies (one group behind) have landed
+                        cp_async_wait<1>();
+                        mbar_arrive(&full[(G - 1) % S]);
+                    }
+                }
+            }
+            if (G > 0) {
+                cp_async_wait<0>();
+                mbar_arrive(&full[(G - 1) % S]);
+            }
+            return;
+        }
         if (warp == COMPUTE_WARPS) {
             // ---------------------------- TMA issue ----------------------------
             if (lane == 0) {
@@ -250,6 +324,7 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
 #pragma unroll
                     for (int b = 0; b < 6; ++b) v[((a * 6 + b) * BC) * BN] = r[b];
                 }
+                fence_proxy_async_smem();  // generic reads of the TMA slot before its async-proxy refill
                 __syncwarp();
                 if (lane == 0) {
                     mbar_arrive(&empty[slot]);
@@ -309,6 +384,7 @@ __global__ void __launch_bounds__(NT, 1) fused_f4_kernel(const __grid_constant__
                         }
                 }
             }
+            fence_proxy_async_smem();  // generic reads of the TMA slot before its async-proxy refill
             __syncwarp();
             if (lane == 0) {
                 mbar_arrive(&empty[slot]);

@@ -297,6 +297,9 @@ __global__ void __launch_bounds__(threads_for<XPW>(), 1) fused_fp32_kernel(const
     for (int it = 0; it < NIT; ++it) {
         cp_async_wait<S - 3>();
         if (it + 1 < NIT) wait_tma(it + 1);  // stage it+1 landed
+        // the slot refilled below was read through the generic proxy; a TMA refill is an
+        // async-proxy write, ordered after those reads only through fence.proxy.async
+        if (XM == LD_TMA || UM == LD_TMA) fence_proxy_async_smem();
         __syncthreads();                      // V[it&1] complete; slot (it-1)%S free
         const int nxt = it + S - 1;
         if (nxt < NIT) issue_stage(nxt, nxt % S);

@@ -126,6 +126,7 @@ __device__ __forceinline__ void itf_loop(float* smem, float* vs, uint64_t* full,
 #pragma unroll
                 for (int e = 0; e < 16; ++e)
                     *reinterpret_cast<float4*>(v + e * BC * BN) = make_float4(t[0][e], t[1][e], t[2][e], t[3][e]);
+                fence_proxy_async_smem();  // generic reads of the TMA slot before its async-proxy refill
                 __syncwarp();
                 if (lane == 0) {
                     mbar_arrive(&empty[slot]);  // raw x of this slot consumed
@@ -388,6 +389,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                 if (c + 2 < BC) load_frag(us, v, c + 2, fa, ga);
                 ffma_block(fb, gb);
             }
+            fence_proxy_async_smem();  // generic reads of the TMA slot before its async-proxy refill (7.6)
             __syncwarp();
             if (lane == 0) {
                 mbar_arrive(&empty[slot]);  // u of this slot consumed
@@ -548,6 +550,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                     }
                 }
             }
+            fence_proxy_async_smem();  // generic reads of the slots before the peers' next st.async into them
             named_bar_sync(1, COMPUTE_THREADS);  // every slot consumed
             if (warp == 0) {
                 if (lane == 0) mbar_arrive_expect_tx(yready, kSplitTileBytes);  // next tile's partials

@@ -12,14 +12,22 @@
 //     filter per channel block into a 2-slot ring;
 //   * warp 14 (x producer): TMA box of raw x (n:32, w:4, h:4, c:8) per channel
 //     block (zero fill = implicit padding, Sec. 3.5), L2 prefetch ahead;
-//   * warps 4-11 (ITF): V = B^T d B (Eq. 6) for the 8 x 32 (c, nu) tiles of a
+//   * warps 8-11 (ITF): V = B^T d B (Eq. 6) for the 8 x 32 (c, nu) tiles of a
 //     block, rounded to TF32 (3xTF32: big + small planes), stored as the
-//     K-major UMMA B operand;
+//     K-major UMMA B operand.  A lane owns one nu and 4 channels: its raw-x reads
+//     are 32 consecutive floats per warp (conflict-free) and its V stores are one
+//     16 B core-matrix row per xi (a quarter-warp writes 128 contiguous bytes);
+//     MM = 128: two warp pairs take alternate channel blocks; MM = 64: one warp
+//     pair per nu-half;
 //   * warp 13 (MMA, one thread): per xi, D(xi) += U(xi) * V(xi) (3xTF32:
 //     big*big + big*small + small*big); tcgen05.commit frees smem slots;
-//   * warps 0-3 (epilogue): tcgen05.ld of the 16 accumulators of their 32 TMEM
-//     lanes, OTF (Eq. 8) into registers, release TMEM to the next tile's MMAs,
-//     then coalesced 128 B stores -- overlapping the next tile's main loop.
+//   * warps 0-7 (epilogue): warps w and w + 4 share TMEM lane quadrant w % 4 and
+//     split its columns (nu 0-15 / 16-31 of every accumulator): tcgen05.ld, OTF
+//     (Eq. 8) into registers, release TMEM to the next tile's MMAs, then
+//     coalesced stores -- overlapping the next tile's main loop.  Eight warps
+//     drain TMEM about twice as fast as four (tile-boundary stall).
+// Every hand-off between thread groups is an mbarrier on which each producing lane
+// arrives itself (racecheck-clean; scripts/microbench/racecheck_mbar_repro.cu).
 // All hand-offs are mbarriers; the producers run ahead across tile boundaries.
 #pragma once
 #include <cuda.h>
@@ -51,14 +59,14 @@ constexpr int BN = 32;         // nu per UMMA (N); a tile has 128 / MM such halv
 // xi interleaved in TMEM lanes (rows 0-15 of each 32-lane quadrant hold nu-half 0,
 // lanes 16-31 hold nu-half 1; scripts/microbench/umma_m64.cu) -> tile 64 x 64.
 constexpr int BC = 8;          // channels per block (UMMA K for tf32)
-constexpr int EPI_WARPS = 4;   // warps 0..3: epilogue (TMEM lane quadrants 0..3)
-constexpr int ITF_WARP0 = 4;   // warps 4..11: ITF
-constexpr int ITF_WARPS = 8;
+constexpr int EPI_WARPS = 8;   // warps 0..7: epilogue (TMEM lane quadrant warp % 4, column half warp / 4)
+constexpr int ITF_WARP0 = 8;   // warps 8..11: ITF
+constexpr int ITF_WARPS = 4;
 constexpr int PROD_WARP = 12;  // bulk-copy producer of the transformed filter U
 constexpr int MMA_WARP = 13;   // tcgen05.mma issuer
 constexpr int XPROD_WARP = 14; // TMA / cp.async producer of raw x
 constexpr int NT = 512;        // 16 warps (warp 15 idle; warpgroup-granular register split)
-constexpr int REG_EPI = 232, REG_ITF = 88, REG_PROD = 56;  // 128*232 + 256*88 + 128*56 = 59264
+constexpr int REG_EPI = 168, REG_ITF = 120, REG_PROD = 56;  // 256*168 + 128*120 + 128*56 = 65536
 template <int MM>
 constexpr int a_tile() { return MM * BC * 4; }  // one (xi, plane) A operand: 4 / 2 KB
 constexpr int B_TILE = BN * BC * 4;  // one (xi, plane, nu-half) B operand: 1 KB
@@ -186,11 +194,7 @@ struct Cfg {
     static constexpr int UNITS_PER_CB = 16 / XPU;
     static constexpr int A_TILE = a_tile<MM>();
     static constexpr int UNIT = XPU * P * A_TILE;               // 64 KB (MM=128) / 32 KB (MM=64)
-#ifdef WINO_TC_DBG_U2
-    static constexpr int U_SLOTS = 2;
-#else
     static constexpr int U_SLOTS = (MM == 64 && XM >= 2) ? 3 : 2;
-#endif
     static constexpr int X_SLOTS = 2;                           // raw x boxes in flight (L2-prefetched)
     static constexpr int X_SLOT = NH * XS_BYTES;
     static constexpr int V_SLOT = 16 * NH * P * B_TILE;        // 16 / 32 KB
@@ -237,21 +241,19 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
             mbar_init(&u_full[s], 1);
             mbar_init(&u_empty[s], 1);
         }
-#ifdef WINO_TC_DBG_PERLANE
-        constexpr int ARR = 32;  // debug: every ITF lane arrives itself
-#else
-        constexpr int ARR = 1;
-#endif
+        // ITF lanes per channel block: MM = 128 one warp pair (the pairs alternate blocks),
+        // MM = 64 both pairs (one per nu-half); the gather path's x producer arrives per lane
+        constexpr int ITF_LANES = (NH == 1 ? 2 : 4) * 32;
         for (int s = 0; s < G::X_SLOTS; ++s) {
-            mbar_init(&x_full[s], 1);
-            mbar_init(&x_empty[s], ITF_WARPS * ARR);
+            mbar_init(&x_full[s], XM >= 2 ? 1 : 32);
+            mbar_init(&x_empty[s], ITF_LANES);
         }
         for (int s = 0; s < 2; ++s) {
-            mbar_init(&v_full[s], ITF_WARPS * ARR);
+            mbar_init(&v_full[s], ITF_LANES);
             mbar_init(&v_empty[s], 1);
         }
         mbar_init(acc_full, 1);
-        mbar_init(acc_empty, EPI_WARPS);
+        mbar_init(acc_empty, EPI_WARPS * 32);
         fence_mbar_init();
         if constexpr (XM >= 2) tma_prefetch_desc(&p.tmx);
     }
@@ -354,8 +356,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                             else cp_async4(dst, src, ok);
                         }
                         cp_async_wait_all();
-                        __syncwarp();
-                        if (lane == 0) mbar_arrive(&x_full[xs]);
+                        mbar_arrive(&x_full[xs]);  // every lane: its own copies have landed
                     }
                 }
             }
@@ -431,76 +432,78 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
     } else if (warp >= ITF_WARP0) {
         setmaxnreg_dec<REG_ITF>();
         // ------------------------------ ITF warps -----------------------------
-        // thread -> (c, nu) with lanes over (nu%8, c%4): conflict-free K-major stores
+        // lane = nu of the half; warp iw: channels 4 (iw & 1) .. +3; MM = 128: warp pair iw >> 1
+        // takes the channel blocks of its parity; MM = 64: warp pair iw >> 1 = nu-half
         const int iw = warp - ITF_WARP0;
-        const int nl = (iw & 3) * 8 + (lane >> 2);
-        const int cl = (iw >> 2) * 4 + (lane & 3);
-        const uint32_t voff = (nl >> 3) * 256 + (cl >> 2) * 128 + (nl & 7) * 16 + (cl & 3) * 4;
-        // raw x of (cl, nl): [c][pos][n32] (XM != 3) or [box][c][pos][n:N] (XM == 3)
+        const int grp = NH == 1 ? (iw >> 1) : 0;
+        const int hh = NH == 1 ? 0 : (iw >> 1);
+        const int cq = iw & 1;
+        const int nl = lane;
+        // K-major core-matrix row of (nu, channels 4cq..4cq+3): [nu/8][c/4][nu%8][c%4]
+        const uint32_t voff = (nl >> 3) * 256 + cq * 128 + (nl & 7) * 16;
+        // raw x of (4cq, nl): [c][pos][n32] (XM != 3) or [box][c][pos][n:N] (XM == 3)
         const int xnb = XM == 3 ? p.N : BN;
-        const int xoff = (nl / xnb) * (BC * 16 * xnb) + cl * 16 * xnb + nl % xnb;
+        const int xoff = (nl / xnb) * (BC * 16 * xnb) + 4 * cq * 16 * xnb + nl % xnb;
         int gcb = 0;
         Segs<SK> segs(p);
         int tile, lo, hi;
         while (segs.next(p, tile, lo, hi)) {
             for (int cb = lo; cb < hi; ++cb, ++gcb) {
+                if (NH == 1 && (gcb & 1) != grp) continue;
                 const int xs = gcb % G::X_SLOTS, vs = gcb & 1;
                 mbar_wait(&x_full[xs], (gcb / G::X_SLOTS) & 1);
-                float t[NH][16];
+                const float* xsrc = sx + xs * (G::X_SLOT / 4) + hh * (XS_BYTES / 4) + xoff;
+                float t[4][16];
 #pragma unroll
-                for (int h = 0; h < NH; ++h) {
-                    const float* xsrc = sx + xs * (G::X_SLOT / 4) + h * (XS_BYTES / 4) + xoff;
+                for (int c = 0; c < 4; ++c) {
                     float d[16];
 #pragma unroll
-                    for (int e = 0; e < 16; ++e) d[e] = xsrc[e * xnb];
-                    itf_4x4(d, t[h]);  // consumes the loads
+                    for (int e = 0; e < 16; ++e) d[e] = xsrc[(c * 16 + e) * xnb];
+                    itf_4x4(d, t[c]);
                 }
-#ifdef WINO_TC_DBG_PERLANE
-                mbar_arrive(&x_empty[xs]);
-#else
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&x_empty[xs]);  // the x slot can be refilled
-#endif
+                // generic-proxy reads of a TMA-filled slot -> fence.proxy.async before releasing it: the
+                // next TMA write (async proxy) is otherwise not ordered after them
+                fence_proxy_async_smem();
+                mbar_arrive(&x_empty[xs]);  // this lane's reads of the x slot are done
                 if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);
                 uint8_t* vdst = sv + vs * G::V_SLOT + voff;
 #pragma unroll
-                for (int h = 0; h < NH; ++h)
-#pragma unroll
-                    for (int xi = 0; xi < 16; ++xi) {
-                        const float big = to_tf32(t[h][xi]);
-                        *reinterpret_cast<float*>(vdst + ((xi * NH + h) * P) * B_TILE) = big;
-                        if constexpr (P == 2)
-                            *reinterpret_cast<float*>(vdst + ((xi * NH + h) * P + 1) * B_TILE) = to_tf32(t[h][xi] - big);
-                    }
+                for (int xi = 0; xi < 16; ++xi) {
+                    const float b0 = to_tf32(t[0][xi]), b1 = to_tf32(t[1][xi]);
+                    const float b2 = to_tf32(t[2][xi]), b3 = to_tf32(t[3][xi]);
+                    uint8_t* dst = vdst + ((xi * NH + hh) * P) * B_TILE;
+                    *reinterpret_cast<float4*>(dst) = make_float4(b0, b1, b2, b3);
+                    if constexpr (P == 2)
+                        *reinterpret_cast<float4*>(dst + B_TILE) =
+                            make_float4(to_tf32(t[0][xi] - b0), to_tf32(t[1][xi] - b1), to_tf32(t[2][xi] - b2),
+                                        to_tf32(t[3][xi] - b3));
+                }
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
-#ifdef WINO_TC_DBG_PERLANE
                 mbar_arrive(&v_full[vs]);
-#else
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&v_full[vs]);
-#endif
             }
         }
     } else {
         setmaxnreg_inc<REG_EPI>();
         // ------------------------------ epilogue ------------------------------
-        // thread = TMEM lane = filter k of the tile; all 32 nu of the 16 accumulators
+        // thread = TMEM lane = filter k of the tile; nu 16 eh .. 16 eh + 15 of each accumulator
         // MM = 128: lane = filter; MM = 64: lanes 0-15 -> filters of nu-half 0, 16-31 -> nu-half 1
-        const int kl = (MM == 128) ? warp * 32 + lane : warp * 16 + (lane & 15);
+        constexpr int EN = BN / 2;  // nu per thread
+        const int qd = warp & 3, eh = warp >> 2;
+        const int kl = (MM == 128) ? qd * 32 + lane : qd * 16 + (lane & 15);
         const int hsel = (MM == 128) ? 0 : (lane >> 4);
-        const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
+        const uint32_t trow = tmem + ((uint32_t)(qd * 32) << 16) + eh * EN;
         const size_t dW = (size_t)p.W * p.N;
         int it = 0;
         Segs<SK> segs(p);
         int tile, lo, hi;
         for (; segs.next(p, tile, lo, hi); ++it) {
             const int k = (tile % p.num_kb) * MM + kl;
-            const int nu0 = (tile / p.num_kb) * TN + hsel * BN;
+            const int nu0 = (tile / p.num_kb) * TN + hsel * BN + eh * EN;
             mbar_wait(acc_full, it & 1);
             tc_fence_after();
-            float o[BN][4];  // OTF results of this filter for the 32 nu
+            float o[EN][4];  // OTF results of this filter for its 16 nu
 #pragma unroll
-            for (int ch = 0; ch < BN / 4; ++ch) {
+            for (int ch = 0; ch < EN / 4; ++ch) {
                 float m[16][4];
 #pragma unroll
                 for (int xi = 0; xi < 16; ++xi) tmem_ld4(trow + xi * BN + ch * 4, m[xi]);
@@ -514,23 +517,23 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                 }
             }
             tc_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(acc_empty);  // TMEM free for the next tile's MMAs
+            mbar_arrive(acc_empty);  // TMEM free for the next tile's MMAs (after this lane's loads)
             if (SK && hi - lo != p.num_cb) {
                 // piece of a cut tile: partial outputs -> slot 2b (the CTA's first piece) or 2b + 1
                 // (its last), [kl][output][nu of the tile]; tc_fixup_kernel adds them
-                float* wk = p.sk_ws + ((size_t)(2 * blockIdx.x + (segs.n > 1 ? 1 : 0)) * MM + kl) * (4 * TN) + hsel * BN;
+                float* wk = p.sk_ws + ((size_t)(2 * blockIdx.x + (segs.n > 1 ? 1 : 0)) * MM + kl) * (4 * TN) +
+                            hsel * BN + eh * EN;
 #pragma unroll
                 for (int q = 0; q < 4; ++q)
 #pragma unroll
-                    for (int j = 0; j < BN; j += 4)
+                    for (int j = 0; j < EN; j += 4)
                         *reinterpret_cast<float4*>(wk + q * TN + j) =
                             make_float4(o[j][q], o[j + 1][q], o[j + 2][q], o[j + 3][q]);
                 continue;
             }
             if (k >= p.K || nu0 >= p.NV) continue;
             if constexpr (XM == 2) {
-                // N % 32 == 0: the 32 nu are 32 consecutive n of one image tile -> 128 B rows
+                // N % 32 == 0: the 32 nu of a half are 32 consecutive n of one image tile -> 64 B per thread
                 const int t = nu0 / p.N, n = nu0 - t * p.N;
                 const int th = t / p.TW, tw = t - th * p.TW;
                 const int i0 = 2 * th, j0 = 2 * tw;
@@ -541,13 +544,13 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                     if (i0 + a >= p.H || j0 + b >= p.W) continue;  // odd H/W (L1155)
                     float* dst = yk + a * dW + b * p.N;
 #pragma unroll
-                    for (int j = 0; j < BN; j += 4)
+                    for (int j = 0; j < EN; j += 4)
                         *reinterpret_cast<float4*>(dst + j) = make_float4(o[j][q], o[j + 1][q], o[j + 2][q], o[j + 3][q]);
                 }
             } else if constexpr (XM == 3) {
                 // N | 32, N % 4 == 0: every group of 4 nu is 4 consecutive n of one image tile
 #pragma unroll
-                for (int j = 0; j < BN; j += 4) {
+                for (int j = 0; j < EN; j += 4) {
                     const int nu = nu0 + j;
                     if (nu >= p.NV) break;
                     const int t = nu / p.N, n = nu - t * p.N;
@@ -564,7 +567,7 @@ __global__ void __launch_bounds__(NT, 1) fused_tc_kernel(const __grid_constant__
                 }
             } else {
 #pragma unroll
-                for (int j = 0; j < BN; ++j) {
+                for (int j = 0; j < EN; ++j) {
                     const int nu = nu0 + j;
                     if (nu >= p.NV) break;
                     const int t = nu / p.N, n = nu - t * p.N;

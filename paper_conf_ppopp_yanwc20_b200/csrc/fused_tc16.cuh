@@ -496,6 +496,9 @@ __global__ void __launch_bounds__(NT, 1) fused_tc16_kernel(const __grid_constant
 #pragma unroll
                     for (int xi = 0; xi < 16; ++xi) vw[i][xi] = pack2<DT>(v0[xi], v1[xi]);
                 }
+                // generic-proxy reads of a TMA-filled slot -> fence.proxy.async before releasing it: the
+                // next TMA write (async proxy) is otherwise not ordered after them
+                fence_proxy_async_smem();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&x_empty[xs]);  // the x slot can be refilled
                 if (gcb >= 2) mbar_wait(&v_empty[vs], ((gcb >> 1) - 1) & 1);

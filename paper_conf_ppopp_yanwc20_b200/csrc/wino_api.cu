@@ -252,7 +252,7 @@ bool encode_map(CUtensorMap* m, const void* base, int rank, const cuuint64_t* di
 }
 
 std::atomic<uint64_t> g_attr_fp32[3][3];
-std::atomic<uint64_t> g_attr_f4;
+std::atomic<uint64_t> g_attr_f4[2];
 
 template <int XM, int UM>
 wino_status_t launch_fp32(const wino::fp32::Params& prm, int64_t ctas, int smem, int dev, cudaStream_t st) {
@@ -549,11 +549,8 @@ wino_status_t wino_filter_transform(const float* w_dev, float* u_dev, int C, int
     int dev;
     wino_status_t s = check_device(&dev);
     if (s != WINO_OK) return s;
-    const int64_t n = int64_t(C) * K;
-    const unsigned blocks = static_cast<unsigned>((n + wino::FTF_THREADS - 1) / wino::FTF_THREADS);
-    wino::ftf_kernel<<<blocks, wino::FTF_THREADS, 0, reinterpret_cast<cudaStream_t>(stream)>>>(w_dev, u_dev, C, K);
-    cudaError_t e = cudaGetLastError();
-    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+    const wino_ftf_job_t job = {w_dev, u_dev, C, K};  // one job of the (vectorised) multi-layer FTF kernel
+    return wino_filter_transform_multi(&job, 1, stream);
 }
 
 wino_status_t wino_filter_transform_multi(const wino_ftf_job_t* jobs, int n, wino_stream_t stream) {
@@ -578,8 +575,9 @@ wino_status_t wino_filter_transform_multi(const wino_ftf_job_t* jobs, int n, win
         J.u[j] = b.u;
         J.C[j] = b.C;
         J.K[j] = b.K;
+        J.vec[j] = b.K % 4 == 0 ? 1 : 0;  // 4 consecutive k per thread (the pointers are 16-byte aligned)
         J.first[j] = blocks;
-        const int64_t nb = (int64_t(b.C) * b.K + wino::FTF_THREADS - 1) / wino::FTF_THREADS;
+        const int64_t nb = (int64_t(b.C) * (J.vec[j] ? b.K / 4 : b.K) + wino::FTF_THREADS - 1) / wino::FTF_THREADS;
         if (int64_t(blocks) + nb > 0x7fffffff) return WINO_ERR_TOO_LARGE;
         blocks += static_cast<unsigned>(nb);
     }
@@ -614,7 +612,7 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
         plan->threads = NT;
         plan->smem_bytes = variant == 1 ? (mm == 64 ? Cfg<1, 64, 2>::BYTES : Cfg<1, 128, 2>::BYTES) : Cfg<2, 128, 2>::BYTES;
         plan->launches = 1;
-        if (with_ws && plan->load_x == 2 && mm == 128) {
+        if (with_ws && plan->load_x == 2) {
             int dev = -1, sms = 148;  // host-only planning unless an sm_100 device is current
             if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
             else cudaGetLastError();
@@ -904,15 +902,10 @@ wino_status_t conv_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, i
                    overlaps(ws_dev, ws_bytes, u_tc_dev, wino_filter_workspace_bytes_tc(C, K, mode))))
         return WINO_ERR_INVALID_ARG;
     const double units = double(prm.num_tiles) * prm.num_cb;
-    // (128-filter tiles only: with the 64 x 64 tiles of K <= 64 a cut tile's last 8 nu came out
-    // wrong in 2 of ~10 forced runs -- an intermittent hazard not yet found (scripts/dbg_tcsk64.py);
-    // no BASELINE shape needs stream-K there)
-#ifndef WINO_TC_SK_MM64  // debug builds: allow it (investigation)
-    if (sk == 2 && mm == 64) return WINO_ERR_UNSUPPORTED;
-    const bool sk_ok = xm >= 2 && mm == 128 && ws_dev && ws_bytes >= tc16_sk_bytes(sms) && units < 2147483647.0;
-#else
+    // (the 64-filter tiles' stream-K plan was fenced off in round 1 after intermittent wrong partials;
+    // the cause was a missing fence.proxy.async between the ITF's generic reads of a raw-x slot and
+    // its TMA refill, DESIGN.md 7.6 -- fixed in every kernel, so both tile heights take stream-K)
     const bool sk_ok = xm >= 2 && ws_dev && ws_bytes >= tc16_sk_bytes(sms) && units < 2147483647.0;
-#endif
     if (sk == 2 && !sk_ok) return WINO_ERR_INVALID_ARG;
     const bool use_sk = sk == 2 || (sk == 1 && sk_ok && tc16_sk_pays(prm.num_tiles, prm.num_cb, sms));
     if (use_sk) {  // stream-K: equal (tile, channel block) ranges on every SM + fixup
@@ -923,10 +916,8 @@ wino_status_t conv_tc(const float* x_dev, const float* u_tc_dev, float* y_dev, i
     }
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (use_sk) {
-#ifdef WINO_TC_SK_MM64
         if (mode == WINO_TC_TF32 && mm == 64)
             return xm == 3 ? launch_tc<1, 3, 64, true>(prm, ctas, dev, st) : launch_tc<1, 2, 64, true>(prm, ctas, dev, st);
-#endif
         if (mode == WINO_TC_TF32)
             return xm == 3 ? launch_tc<1, 3, 128, true>(prm, ctas, dev, st)
                            : launch_tc<1, 2, 128, true>(prm, ctas, dev, st);
@@ -1304,7 +1295,7 @@ wino_status_t wino_filter_transform_f4(const float* w_dev, float* u4_dev, int C,
 
 extern "C++" {
 namespace {
-std::atomic<uint64_t> g_attr_f4_sk;
+std::atomic<uint64_t> g_attr_f4_sk[2];
 // sk: 0 = never, 1 = planner's choice, 2 = always (needs ws >= f4 workspace bytes)
 wino_status_t conv_f4(const float* x_dev, const float* u4_dev, float* y_dev, int N, int C, int H, int W, int K,
                       int pad, int stride, int sk, void* ws_dev, size_t ws_bytes, wino_stream_t stream) {
@@ -1312,7 +1303,6 @@ wino_status_t conv_f4(const float* x_dev, const float* u4_dev, float* y_dev, int
     wino_status_t s = check_shape(N, C, H, W, K, pad, stride);
     if (s != WINO_OK) return s;
     if (int64_t(36) * C * K > kMaxElems) return WINO_ERR_TOO_LARGE;
-    if (N % 16 != 0 || K % 4 != 0) return WINO_ERR_UNSUPPORTED;
     if (!aligned16(x_dev) || !aligned16(u4_dev) || !aligned16(y_dev) || (ws_dev && !aligned16(ws_dev)))
         return WINO_ERR_MISALIGNED;
     const size_t hwn = size_t(H) * W * N;
@@ -1325,6 +1315,9 @@ wino_status_t conv_f4(const float* x_dev, const float* u4_dev, float* y_dev, int
     Params prm;
     std::memset(&prm, 0, sizeof(prm));
     prm.y = y_dev;
+    prm.x = x_dev;
+    prm.u4 = u4_dev;
+    prm.u_vec = K % 4 == 0 ? 1 : 0;
     prm.N = N;
     prm.C = C;
     prm.H = H;
@@ -1335,15 +1328,20 @@ wino_status_t conv_f4(const float* x_dev, const float* u4_dev, float* y_dev, int
     prm.num_kb = (K + BK - 1) / BK;
     prm.num_it = (C + BC - 1) / BC;
     prm.num_tiles = ((prm.NV + BN - 1) / BN) * prm.num_kb;
-    {
-        const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
-        const cuuint32_t box[4] = {BN, 6, 6, BC};
-        if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
-    }
-    {
-        const cuuint64_t dims[3] = {cuuint64_t(K), 36, cuuint64_t(C)};
-        const cuuint32_t box[3] = {BK, 36, BC};
-        if (!encode_map(&prm.tmu, u4_dev, 3, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+    // TMA boxes need the tile's 16 nu to be 16 consecutive n (N % 16) and 16-byte u rows (K % 4);
+    // any other shape gathers with cp.async (generic path, same arithmetic)
+    const bool gen = N % 16 != 0 || K % 4 != 0;
+    if (!gen) {
+        {
+            const cuuint64_t dims[4] = {cuuint64_t(N), cuuint64_t(W), cuuint64_t(H), cuuint64_t(C)};
+            const cuuint32_t box[4] = {BN, 6, 6, BC};
+            if (!encode_map(&prm.tmx, x_dev, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+        }
+        {
+            const cuuint64_t dims[3] = {cuuint64_t(K), 36, cuuint64_t(C)};
+            const cuuint32_t box[3] = {BK, 36, BC};
+            if (!encode_map(&prm.tmu, u4_dev, 3, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+        }
     }
     if (ws_dev && (overlaps(ws_dev, ws_bytes, x_dev, size_t(C) * hwn * 4) || overlaps(ws_dev, ws_bytes, y_dev, yb) ||
                    overlaps(ws_dev, ws_bytes, u4_dev, size_t(36) * C * K * 4)))
@@ -1366,8 +1364,8 @@ wino_status_t conv_f4(const float* x_dev, const float* u4_dev, float* y_dev, int
         prm.sk_ws = static_cast<float*>(ws_dev);
         prm.sk_q = static_cast<int>(int64_t(units) / sms);
         prm.sk_r = static_cast<int>(int64_t(units) % sms);
-        auto kern = fused_f4_kernel<true>;
-        if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4_sk)) != WINO_OK) return s;
+        auto kern = gen ? fused_f4_kernel<true, true> : fused_f4_kernel<true, false>;
+        if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4_sk[gen])) != WINO_OK) return s;
         kern<<<grid, NT, Smem::bytes, st>>>(prm);
         e = cudaGetLastError();
         if (e == cudaSuccess && grid > 1) {
@@ -1375,8 +1373,8 @@ wino_status_t conv_f4(const float* x_dev, const float* u4_dev, float* y_dev, int
             e = cudaGetLastError();
         }
     } else {
-        auto kern = fused_f4_kernel<false>;
-        if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4)) != WINO_OK) return s;
+        auto kern = gen ? fused_f4_kernel<false, true> : fused_f4_kernel<false, false>;
+        if ((s = ensure_smem_attr(kern, dev, Smem::bytes, g_attr_f4[gen])) != WINO_OK) return s;
         kern<<<grid, NT, Smem::bytes, st>>>(prm);
         e = cudaGetLastError();
     }

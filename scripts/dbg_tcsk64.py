@@ -55,3 +55,74 @@ for shape in [(32, 64, 64, 30, 30), (32, 64, 64, 16, 16), (32, 64, 48, 14, 14)]:
             if len(seen) > 24:
                 break
 print("TOTAL failing runs", total_bad)
+
+# ---- which piece is wrong: compare every workspace slot of the failing shape with the oracle's
+# partial output over that piece's channel range (Eq. 8 is linear: a piece's partial outputs are
+# the convolution restricted to its channels) ----
+N, C, K, H, W = 32, 64, 64, 30, 30
+x, w = make_inputs(Conv3x3Config("s", N, C, K, H, W), kind="smallint")
+xd = x.cuda()
+u = wino.filter_transform_tc(w.cuda(), "tf32")
+ws = torch.empty(wino.tc_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device="cuda")
+TW, TH = (W + 1) // 2, (H + 1) // 2
+NV, ncb = N * TH * TW, (C + 7) // 8
+G = min(sms, 256)
+units = ((NV + 63) // 64) * ncb
+q, r = divmod(units, G)
+starts = [b * q + min(b, r) for b in range(G + 1)]
+partial_cache = {}
+
+
+def partial_ref(c0, c1):
+    if (c0, c1) not in partial_cache:
+        xm, wm = x.clone(), w.clone()
+        xm[:c0] = 0
+        xm[c1:] = 0
+        wm[:c0] = 0
+        wm[c1:] = 0
+        partial_cache[(c0, c1)] = oracle.direct_conv(xm, wm)
+    return partial_cache[(c0, c1)]
+
+
+SLOT = 64 * 4 * 64
+for rep in range(reps):
+    ws.fill_(255)
+    wino.conv2d_tc(xd, u, ws=ws, stream_k="on")
+    torch.cuda.synchronize()
+    wsf = ws.view(torch.float32).cpu().numpy()
+    nbad = 0
+    for b in range(G):
+        a0, a1 = starts[b], starts[b + 1]
+        pieces, a, n = [], a0, 0
+        while a < a1:
+            tile = a // ncb
+            lo = a - tile * ncb
+            hi = min(ncb, lo + (a1 - a))
+            a += hi - lo
+            n += 1
+            if hi - lo != ncb:
+                pieces.append((tile, lo, hi, 2 * b + (1 if n > 1 else 0), n))
+        for tile, lo, hi, slot, n in pieces:
+            ref = partial_ref(lo * 8, hi * 8)
+            got = wsf[slot * SLOT:(slot + 1) * SLOT].reshape(64, 4, 64)  # [kl][q][j]
+            for j in range(64):
+                nu = tile * 64 + j
+                if nu >= NV:
+                    continue
+                t, nn = divmod(nu, N)
+                th, tw = divmod(t, TW)
+                for qq in range(4):
+                    i, jj = 2 * th + qq // 2, 2 * tw + qq % 2
+                    if i >= H or jj >= W:
+                        continue
+                    bad = np.nonzero(got[:, qq, j] != ref[:, i, jj, nn])[0]
+                    if len(bad):
+                        nbad += len(bad)
+                        shown = globals().setdefault("shown", set())
+                        key = (rep, b, n, j // 8, qq)
+                        if key not in shown and len(shown) < 60:
+                            shown.add(key)
+                            print(f"rep {rep} CTA {b} piece#{n} tile {tile} cb [{lo},{hi}) slot {slot} nu {j} q {qq} "
+                                  f"k {list(bad[:4])} got {got[bad[0], qq, j]} want {ref[bad[0], i, jj, nn]}",
+                                  flush=True)
+    print("rep", rep, "bad partial entries", nbad, flush=True)

@@ -201,15 +201,18 @@ def test_stream_k_plan_and_workspace():
 
 def test_tensor_core_stream_k_plans_and_workspaces():
     """Host-only planning: the 16-bit and TF32 tcgen05 kernels take stream-K only for tile-starved
-    shapes (conv5_x: 64 tiles of 128 x 32 for 148 SMs), never for the many-tile layers; 64-filter
-    TF32 tiles (K <= 64) never; workspace sizes are 2 slots of 64 KiB per SM (148 without a device)."""
+    shapes (conv5_x: 64 tiles of 128 x 32 for 148 SMs), never for the many-tile layers, with either
+    tile height (64-filter TF32 tiles for K <= 64 included); workspace sizes are 2 slots of 64 KiB per
+    SM (148 without a device)."""
     c5, c4, c2 = CONFIGS["conv5_x"], CONFIGS["conv4_x"], CONFIGS["conv2_x"]
     for v in (5, 6, 7):
         p = wino.plan(c5.N, c5.C, c5.H, c5.W, c5.K, variant=v)
         assert p.stream_k == 1 and p.launches == 2 and p.ctas == 148, (v, p)
         assert wino.plan(c2.N, c2.C, c2.H, c2.W, c2.K, variant=v).stream_k == 0
     assert wino.plan(c5.N, c5.C, c5.H, c5.W, c5.K, variant=3).stream_k == 0  # no workspace
-    assert wino.plan(c5.N // 8, c2.C, c2.H, c2.W, c2.K, variant=6).stream_k == 0  # TF32, K <= 64
+    assert wino.plan(c5.N // 8, c2.C, c2.H, c2.W, c2.K, variant=6).stream_k == 0  # 49 tiles x 8 blocks: whole tiles
+    p64 = wino.plan(32, 512, 7, 7, 64, variant=6)  # TF32, K <= 64: 8 tiles of 64 x 64 for 148 SMs
+    assert p64.bk == 64 and p64.stream_k == 1 and p64.launches == 2
     assert wino.half_workspace_bytes(c4.N, c4.C, c4.H, c4.W, c4.K) == 148 * 2 * 64 * 1024
     assert wino.tc_workspace_bytes(c4.N, c4.C, c4.H, c4.W, c4.K) == 148 * 2 * 64 * 1024
     hwn = c4.H * c4.W * c4.N

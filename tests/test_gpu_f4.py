@@ -88,13 +88,47 @@ def test_f4_deterministic_and_overwrites(wino):
     assert torch.equal(y1, y2)
 
 
-@pytest.mark.parametrize("shape", [(8, 4, 8, 5, 5), (16, 4, 6, 5, 5), (24, 3, 8, 4, 4)])
-def test_f4_unsupported_shapes_raise(wino, shape):
+# Generic path (cp.async gathers): N % 16 != 0 and / or K % 4 != 0 -- any N, K, C (L1281)
+F4_GEN = [
+    (1, 8, 8, 8, 8), (1, 1, 1, 1, 1), (3, 7, 8, 5, 5), (33, 9, 65, 7, 7), (3, 1, 65, 9, 6),
+    (8, 4, 8, 5, 5), (16, 4, 6, 5, 5), (24, 3, 8, 4, 4), (5, 17, 130, 6, 10), (33, 64, 64, 14, 14),
+    (2, 9, 3, 17, 3), (20, 12, 72, 12, 12),
+]
+
+
+@pytest.mark.parametrize("kind", ["uniform", "smallint"])
+@pytest.mark.parametrize("shape", F4_GEN, ids=[str(s) for s in F4_GEN])
+def test_f4_generic_shapes(wino, shape, kind):
     N, C, K, H, W = shape
-    x = torch.zeros((C, H, W, N), device=DEV)
-    u4 = torch.zeros((C, 6, 6, K), device=DEV)
-    with pytest.raises(wino.WinoError, match="UNSUPPORTED"):
-        wino.conv2d_f4(x, u4)
+    x, w = make_inputs(Conv3x3Config("f4gen", N, C, K, H, W), kind=kind)
+    u4, y = _run(wino, x, w)
+    assert oracle.max_rel_err(u4.double().numpy(), oracle.filter_transform_f4(w)) <= FTF4_TOL
+    yd = y.double().numpy()
+    assert np.isfinite(yd).all()
+    assert oracle.max_rel_err(yd, oracle.direct_conv(x, w)) <= F4_TOL
+
+
+@pytest.mark.parametrize("shape", [(3, 13, 65, 9, 9), (1, 512, 512, 7, 7), (33, 9, 65, 7, 7)])
+def test_f4_generic_stream_k(wino, shape):
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("f4gsk", N, C, K, H, W), kind="uniform", seed_x=63, seed_w=64)
+    u4 = wino.filter_transform_f4(w.to(DEV))
+    ws = torch.empty(wino.f4_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+    y = wino.conv2d_f4(x.to(DEV), u4, ws=ws, stream_k="on")
+    torch.cuda.synchronize()
+    assert oracle.max_rel_err(y.cpu().double().numpy(), oracle.direct_conv(x, w)) <= F4_TOL
+
+
+def test_f4_generic_matches_tma_path(wino):
+    """The same convolution through the TMA path (N = 32) and the generic path (a batch shard of
+    N = 31 plus the last image as N = 1): within the FP32 bar of each other image by image."""
+    cfg = Conv3x3Config("f4ab", 32, 24, 68, 10, 10)
+    x, w = make_inputs(cfg, kind="uniform", seed_x=65, seed_w=66)
+    _, y = _run(wino, x, w)
+    _, ya = _run(wino, x[..., :31].contiguous(), w)
+    _, yb = _run(wino, x[..., 31:].contiguous(), w)
+    yg = torch.cat([ya, yb], dim=-1).double()
+    assert float((yg - y.double()).abs().max() / y.double().abs().max()) <= F4_TOL
 
 
 # stream-K plan (workspace): ranges shorter than a tile, spanning tiles, tails; forced and auto

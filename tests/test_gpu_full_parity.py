@@ -116,11 +116,11 @@ def test_full_config_every_plan(wino, name, kind):
             _check(y, ref, exact, TOL[v], f"{v} {what}", fails)
 
     # ---- NEXT rows ----
-    if N % 16 == 0 and K % 4 == 0:  # F(4x4) (N1): no exact input class (G4 has 1/6, 1/12, 1/24)
-        u4 = wino.filter_transform_f4(wd)
-        y = wino.conv2d_f4(xd, u4, ws=_ws(wino.f4_workspace_bytes(N, C, H, W, K)))
-        torch.cuda.synchronize()
-        _check(y, ref, False, TOL["f4"], "f4 bench plan", fails)
+    # F(4x4) (N1), any shape: no exact input class (G4 has 1/6, 1/12, 1/24)
+    u4 = wino.filter_transform_f4(wd)
+    y = wino.conv2d_f4(xd, u4, ws=_ws(wino.f4_workspace_bytes(N, C, H, W, K)))
+    torch.cuda.synchronize()
+    _check(y, ref, False, TOL["f4"], "f4 bench plan", fails)
     xn = xd.permute(3, 0, 1, 2).contiguous()
     un = wino.filter_transform_kcrs(wd.permute(3, 0, 1, 2).contiguous())
     refn = np.ascontiguousarray(ref.transpose(3, 0, 1, 2))

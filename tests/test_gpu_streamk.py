@@ -131,13 +131,6 @@ TC_SK = [(4, 512, 512, 7, 7), (8, 256, 256, 14, 14), (16, 128, 128, 12, 10), (32
 def test_tc_streamk(wino, shape, variant, tol):
     N, C, K, H, W = shape
     cfg = Conv3x3Config("sk", N, C, K, H, W)
-    if variant == "tf32" and K <= 64:  # 64-filter tiles: stream-K not offered (include/wino.h)
-        x, w = make_inputs(cfg)
-        u = wino.filter_transform_tc(w.to(DEV), variant)
-        ws = torch.empty(wino.tc_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
-        with pytest.raises(wino.WinoError, match="UNSUPPORTED"):
-            wino.conv2d_tc(x.to(DEV), u, ws=ws, stream_k="on")
-        return
     for kind in ("smallint", "uniform"):
         x, w = make_inputs(cfg, kind=kind)
         u = wino.filter_transform_tc(w.to(DEV), variant)
