@@ -195,12 +195,27 @@ def _ewmm_flops(c, variant):
     return 32 * c.K * c.C * c.N * c.tiles
 
 
+def _coll_device(device):
+    """Scalars for the timing / error reductions live on the GPU for NCCL, on the host for gloo."""
+    return device if dist.get_backend() == "nccl" else torch.device("cpu")
+
+
 def _reduce(v: float, world: int, device, op=None) -> float:
     if world == 1:
         return v
-    t = torch.tensor([v], dtype=torch.float64, device=device)
+    t = torch.tensor([v], dtype=torch.float64, device=_coll_device(device))
     dist.all_reduce(t, op=op or dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def _gather_scalar(v: float, world: int, device) -> list:
+    """Every rank's value (for the line: the max over ranks is what `value` uses)."""
+    if world == 1:
+        return [v]
+    t = torch.tensor([v], dtype=torch.float64, device=_coll_device(device))
+    out = [torch.empty_like(t) for _ in range(world)]
+    dist.all_gather(out, t)
+    return [float(o.item()) for o in out]
 
 
 def _max_over_ranks(v: float, world: int, device) -> float:
@@ -365,9 +380,10 @@ def main():
         for d in per:
             c = d["cfg"]
             u_own = wino.filter_transform(d["w"])
-            u0 = u_own.clone() if rank == 0 else torch.empty_like(u_own)
+            cd = _coll_device(dev)  # NCCL: over NVLink; gloo (tests): through the host
+            u0 = u_own.to(cd) if rank == 0 else torch.empty(u_own.shape, dtype=u_own.dtype, device=cd)
             dist.broadcast(u0, src=0)
-            ok = ok and bool(torch.equal(u0, u_own))
+            ok = ok and bool(torch.equal(u0.to(dev), u_own))
         u_bcast_ok = _reduce(0.0 if ok else 1.0, world, dev) == 0.0
         if not u_bcast_ok:
             raise SystemExit("bench.py: a rank's FTF output differs from rank 0's broadcast u")
@@ -401,9 +417,9 @@ def main():
             launches = sum(3 + wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=4).launches
                            for d in live)
         elif nonfused:
-            launches = sum(3 for d in live)  # FTF, ITF, OTF (the 16 GEMMs: library kernels, not counted)
+            launches = sum(1 + wino.nonfused_launches() for d in live)  # FTF + u arrangement, ITF, GEMM, OTF
         else:
-            # fp32: with the stream-K workspace (variant 4 plans it), which may add a fixup launch
+            # fp32: the stream-K workspace plan (variant 4) is one launch; tf32: + a fixup launch
             vid = {"fp32": 4, "tf32": 6, "3xtf32": 7}[variant]  # plans with the stream-K workspaces
             launches = sum((1 if variant != "fp32" else 0) +
                            wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=vid).launches
@@ -438,12 +454,12 @@ def main():
                 d["y_nchw"] = torch.empty((n1, c.K, c.H, c.W), dtype=torch.float32, device=dev)
                 d["u"] = torch.empty((c.C, 4, 4, c.K), dtype=torch.float32, device=dev)
                 # workspace of the transpose -> CHWN fused kernel -> transpose path (DESIGN 7.8)
-                d["ws_nchw"] = torch.empty(wino.nchw_workspace_bytes(n1, c.C, c.H, c.W, c.K),
+                d["ws_nchw"] = torch.zeros(wino.nchw_workspace_bytes(n1, c.C, c.H, c.W, c.K),
                                            dtype=torch.uint8, device=dev)
             else:
                 d["u"] = torch.empty((c.C, 4, 4, c.K), dtype=torch.float32, device=dev)
                 # device workspace of the stream-K plan (wino_conv2d_f2x3_fwd_ws; the planner decides)
-                d["ws_sk"] = torch.empty(max(wino.conv_workspace_bytes(n1, c.C, c.H, c.W, c.K), 16),
+                d["ws_sk"] = torch.zeros(max(wino.conv_workspace_bytes(n1, c.C, c.H, c.W, c.K), 16),
                                          dtype=torch.uint8, device=dev)
 
         def run_layer(d, ftf=True, conv=True, ftf_stream=None):
@@ -599,6 +615,7 @@ def main():
             else:
                 outs.append(d["y"])
         return {"ms_step": _max_over_ranks(ms_step, world, dev),
+                "ms_step_ranks": _gather_scalar(ms_step, world, dev),
                 "conv_ms": [_max_over_ranks(v, world, dev) for v in conv_ms],
                 "ftf_ms_step": _max_over_ranks(ftf_ms_step, world, dev),
                 "hot_ms_step": _max_over_ranks(hot_step, world, dev),
@@ -760,6 +777,7 @@ def main():
                      "achieved_def": "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) per launch summed over layers / "
                                      "summed conv durations from timing events inside the timed step graph",
                      "peak_def": FP32_PEAK_NOTE},
+        "ms_per_step_ranks": main_m["ms_step_ranks"],
         "gpu_launches": launches_per_step * args.steps,
         "clocks": clocks, "wall_s_timed_region": wall,
     }

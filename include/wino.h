@@ -196,7 +196,8 @@ wino_status_t wino_conv2d_f2x3_fwd_nchw(const float* x_nchw_dev, const float* u_
  * strided gather of wino_conv2d_f2x3_fwd_nchw on every BASELINE layer.
  *   ws_dev / ws_bytes : >= wino_nchw_workspace_bytes(N,C,H,W,K) bytes = |x| + |y| (fp32,
  *                       each rounded up to 256 B) + wino_conv_workspace_bytes; 16-byte
- *                       aligned, not overlapping x, u or y; clobbered.
+ *                       aligned, not overlapping x, u or y; zero-filled before its first
+ *                       use (the stream-K flags, as wino_conv2d_f2x3_fwd_ws), clobbered.
  * Arguments and errors as wino_conv2d_f2x3_fwd_nchw, plus WINO_ERR_INVALID_ARG for a
  * NULL or short workspace.
  */
@@ -225,10 +226,18 @@ wino_status_t wino_conv2d_f2x3_fwd_nonfused_tf32(const float* x_dev, const float
  * linear) in a fixed order -- deterministic, no atomics.  It removes the wave
  * quantisation of tiles over SMs (e.g. 392 tiles on 148 SMs) and keeps small per-rank
  * batches (batch sharding) on every SM.
- *   ws_dev / ws_bytes : >= wino_conv_workspace_bytes(N,C,H,W,K) bytes (SM count x 64 KiB;
+ *   ws_dev / ws_bytes : >= wino_conv_workspace_bytes(N,C,H,W,K) bytes (SM count x 64 KiB of
+ *                       partial tiles + one 4-byte arrival counter per SM, rounded to 256 B;
  *                       the current device's SM count, 148 when no device is current),
  *                       16-byte aligned, not overlapping x, u or y; may be NULL / 0 when
- *                       sk = 1.  Contents need no initialisation and are clobbered.
+ *                       sk = 1.  The stream-K plan reduces the tiles cut between CTAs inside
+ *                       the kernel: every piece of a cut tile leaves its partial outputs in the
+ *                       workspace and counts itself on a GPU-scope arrival counter; the last
+ *                       piece to arrive sums them (in CTA order) and stores y.  The counters
+ *                       must be ZERO before the first use of a workspace (zero-fill it, e.g.
+ *                       cudaMemset); every call leaves them zero again, so one initialisation
+ *                       serves any number of calls on one stream (concurrent calls must not
+ *                       share a workspace).
  *   sk                : 0 = the planner's choice (stream-K where its estimate beats the
  *                       regular / split-C plans and the workspace suffices), 1 = never,
  *                       2 = always when the warp-specialised kernel applies

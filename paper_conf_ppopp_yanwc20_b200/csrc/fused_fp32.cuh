@@ -80,6 +80,7 @@ struct __align__(64) Params {
     // cut into gridDim.x equal contiguous ranges; partial tiles go to sk_ws (2 slots of
     // 64 k x 4 outputs x 32 nu per CTA) and are summed by sk_fixup_kernel.
     float* __restrict__ sk_ws;
+    unsigned* __restrict__ sk_flags;  // arrival counter per CTA holding a cut tile's block 0 (zero between launches)
     long long sk_total;  // tiles * num_it  (< 2^31)
     int sk_q, sk_r;      // sk_total = gridDim * sk_q + sk_r: CTA b's range starts at b*q + min(b, r)
 };

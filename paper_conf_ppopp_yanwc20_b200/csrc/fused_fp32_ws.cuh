@@ -82,6 +82,18 @@ __device__ unsigned long long g_ws_trace[8][64];
 #else
 #define WS_TR(e, T) do { } while (0)
 #endif
+#ifdef WINO_WS_CTATRACE
+// debug builds only: %globaltimer (ns) per CTA: entry, first stage landed, last main loop done, exit
+__device__ unsigned long long g_cta_trace[256][4];
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+#define WS_CT(e) do { if (blockIdx.x < 256) g_cta_trace[blockIdx.x][e] = gtimer(); } while (0)
+#else
+#define WS_CT(e) do { } while (0)
+#endif
 
 // Epilogue geometry: RR accumulator rows per thread per round -> 8*RR filters per
 // round, 8/RR rounds.  Without split RR = 2 (4 rounds of 16 filters, L499).  With
@@ -98,8 +110,9 @@ struct Smem {
     static constexpr int ep_offset = (S * STAGE_FLOATS + SV * VS_FLOATS) * 4;
     static constexpr int yp_offset = ep_offset + ER_FLOATS * 4;
     static constexpr int bar_offset = yp_offset + YP_FLOATS * 4;
-    // full[S], empty[S], vfull[SV], vempty[SV], yready, yfree
-    static constexpr int bytes = bar_offset + (2 * S + 2 * SV + 2 + (WS_XBAR ? S : 0)) * 8;
+    // full[S], empty[S], vfull[SV], vempty[SV], yready, yfree; then 2 ints (stream-K reduction)
+    static constexpr int sk_offset = bar_offset + (2 * S + 2 * SV + 2 + (WS_XBAR ? S : 0)) * 8;
+    static constexpr int bytes = sk_offset + 16;
 };
 
 // ITF loop of warps 9..10 (Sec. 4.2): raw x of every stage -> V = B^T d B in the V ring.
@@ -137,11 +150,117 @@ __device__ __forceinline__ void itf_loop(float* smem, float* vs, uint64_t* full,
 }
 // Stream-K (SK = true): CTA b of G takes units [b*total/G, (b+1)*total/G) of the flattened
 // (tile, channel block) space, unit = tile * NIT + g.  A tile is cut into segments at CTA
-// boundaries; a segment covering the whole tile stores y, a partial one stores its partial OTF
-// outputs (Eq. 8 is linear) in slot 2b (the CTA's first segment) or 2b+1 (its last) of sk_ws,
-// and sk_fixup_kernel adds the segments of each cut tile in CTA order (deterministic).
+// boundaries; a segment covering the whole tile stores y.  A segment of a cut tile stores its
+// partial OTF outputs (Eq. 8 is linear) in sk_ws: slot 2b if it starts inside the tile (it is
+// then CTA b's first segment), slot 2b + 1 if it holds the tile's channel block 0 (CTA b's last
+// segment, or its only one).  Each segment then counts itself on the tile's arrival counter
+// (indexed by the CTA holding block 0); the LAST segment to arrive sums all the tile's partials in
+// CTA order (deterministic) with every compute thread and stores y, and resets the counter --
+// no fixup launch, no CTA ever waits for another.
 // (the first total % G CTAs get one unit more; no division on the device)
 __host__ __device__ __forceinline__ int sk_start(const Params& p, int b) { return b * p.sk_q + min(b, p.sk_r); }
+// The pi-th segment of CTA b's range in PROCESSING order: its first segment, then its last, then the
+// whole tiles in between.  Both ends of a range are (possibly) cut tiles, so every CTA handles its
+// cut segments first: all pieces of a cut tile arrive early, and the reduction by the last one to
+// arrive overlaps the other CTAs' whole tiles instead of adding a tail to the launch.
+__device__ __forceinline__ bool sk_piece(const Params& p, int b, int pi, int& tile, int& g_lo, int& nst) {
+    const int s = sk_start(p, b), e = sk_start(p, b + 1);
+    if (s >= e) return false;
+    const int tf = s / p.num_it, tl = (e - 1) / p.num_it;
+    int t;
+    if (pi == 0) {
+        t = tf;
+    } else if (pi == 1) {
+        if (tl == tf) return false;
+        t = tl;
+    } else {
+        t = tf + pi - 1;
+        if (t >= tl) return false;
+    }
+    const int u0 = max(s, t * p.num_it), u1 = min(e, (t + 1) * p.num_it);
+    tile = t;
+    g_lo = u0 - t * p.num_it;
+    nst = u1 - u0;
+    return true;
+}
+// Stream-K cut tile: this segment's partials are in the workspace; count the segment on the tile's
+// arrival counter; the last of the tile's segments sums them in CTA order and stores y.  Called by
+// the 256 compute threads (named barrier 1).  sh: 2 ints of shared memory.
+__device__ __noinline__ void sk_arrive(const Params& p, int tile, int k0, int nu0, int* sh, int tid) {
+    // The 256 threads' partial outputs are ordered before thread 0's acq_rel atomic by the barrier
+    // (release is cumulative over what thread 0 has observed); on the reducing side thread 0's
+    // acquire is carried to the other threads by the second barrier.
+    named_bar_sync(1, COMPUTE_THREADS);
+    if (tid == 0) {
+        const int t0 = tile * p.num_it, t1 = t0 + p.num_it;
+        int b0 = static_cast<int>(blockIdx.x);
+        while (sk_start(p, b0) > t0) --b0;  // the CTA holding channel block 0 (slot 2 b0 + 1)
+        int nc = 0;                         // CTAs starting inside the tile (slots 2c)
+        while (b0 + nc + 1 < static_cast<int>(gridDim.x) && sk_start(p, b0 + nc + 1) < t1) ++nc;
+        const unsigned seen = atom_add_acq_rel_gpu(p.sk_flags + b0, 1u);
+        const bool last = seen == static_cast<unsigned>(nc);
+        if (last) p.sk_flags[b0] = 0u;  // every segment has arrived: reset for the next launch
+        sh[0] = last ? b0 : -1;
+        sh[1] = nc;
+    }
+    named_bar_sync(1, COMPUTE_THREADS);
+    const int b0 = sh[0], nc = sh[1];
+    if (b0 < 0) return;
+    // 64 k x 32 nu (k, nu) pairs, 8 per thread, nu = lane: coalesced [slot][kl][output][nu] rows
+    constexpr int PER = BK * BN / COMPUTE_THREADS;
+    const int nl = tid & 31, kr = tid >> 5;
+    float o[PER][4];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        const float* w = p.sk_ws + ((size_t)(2 * b0 + 1) * BK + kr + 8 * j) * (4 * BN) + nl;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) o[j][q] = __ldcg(w + q * BN);
+    }
+    int c = 1;
+    for (; c + 1 <= nc; c += 2) {  // two pieces' loads in flight per step; adds in CTA order (deterministic)
+        float v0[PER][4], v1[PER][4];
+#pragma unroll
+        for (int j = 0; j < PER; ++j) {
+            const float* w0 = p.sk_ws + ((size_t)(2 * (b0 + c)) * BK + kr + 8 * j) * (4 * BN) + nl;
+            const float* w1 = w0 + (size_t)2 * BK * 4 * BN;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                v0[j][q] = __ldcg(w0 + q * BN);
+                v1[j][q] = __ldcg(w1 + q * BN);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < PER; ++j)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) o[j][q] = (o[j][q] + v0[j][q]) + v1[j][q];
+    }
+    if (c == nc) {
+#pragma unroll
+        for (int j = 0; j < PER; ++j) {
+            const float* w = p.sk_ws + ((size_t)(2 * (b0 + c)) * BK + kr + 8 * j) * (4 * BN) + nl;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) o[j][q] += __ldcg(w + q * BN);
+        }
+    }
+    const int nu = nu0 + nl;
+    if (nu >= p.NV) return;
+    const int t = nu / p.N, n = nu - t * p.N;
+    const int th = t / p.TW, tw = t - th * p.TW;
+    const int i0 = 2 * th, j0 = 2 * tw;
+    const bool okr = i0 + 1 < p.H, okc = j0 + 1 < p.W;  // odd H/W (L1155)
+    const size_t HWN = (size_t)p.H * p.W * p.N, dW = (size_t)p.W * p.N;
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        const int k = k0 + kr + 8 * j;
+        if (k >= p.K) continue;
+        float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
+        yk[0] = o[j][0];
+        if (okc) yk[p.N] = o[j][1];
+        if (okr) yk[dW] = o[j][2];
+        if (okr && okc) yk[dW + p.N] = o[j][3];
+    }
+}
+
 // BOX32: N % 32 == 0 (one x box per stage, compile-time ITF strides); else N | 32
 // (32/N boxes, runtime strides -- costs the 88-register ITF warps one spill).
 template <bool SPLIT, bool BOX32, bool SK = false>
@@ -159,8 +278,10 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
     uint64_t* const yready = vempty + SV;  // split: all S slots of this CTA's receive buffer landed (tx bytes)
     uint64_t* const yfree = yready + 1;    // split: every owner has consumed this CTA's slots of the last tile
     uint64_t* const xfull = WS_XBAR ? yfree + 1 : full;  // raw x landed (WS_XBAR), else shares full
+    int* const sk_sh = reinterpret_cast<int*>(reinterpret_cast<char*>(smem) + SM::sk_offset);
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) WS_CT(0);
     // split-C: cluster = S consecutive CTAs sharing each tile; rank r takes channel
     // blocks [it_lo, it_hi).  Without split every CTA is its own "cluster".
     const int nsplit = SPLIT ? p.split : 1;
@@ -206,16 +327,13 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             if (lane == 0) {
                 constexpr uint32_t kBytes = (US_FLOATS + XS_FLOATS) * 4;
                 int G = 0;  // global stage counter across tiles
-                int su = SK ? sk_start(p, blockIdx.x) : 0;
-                const int su_end = SK ? sk_start(p, blockIdx.x + 1) : 0;
+                int pi = 0;  // stream-K: segment index in processing order (sk_piece)
                 for (int tile = SK ? 0 : WS_CID;;) {
                     int g_lo = it_lo, g_hi = it_hi;
                     if constexpr (SK) {
-                        if (su >= su_end) break;
-                        tile = su / p.num_it;
-                        g_lo = su - tile * p.num_it;
-                        g_hi = min(p.num_it, g_lo + (su_end - su));
-                        su += g_hi - g_lo;
+                        int nst;
+                        if (!sk_piece(p, blockIdx.x, pi++, tile, g_lo, nst)) break;
+                        g_hi = g_lo + nst;
                     } else if (tile >= num_tiles) {
                         break;
                     }
@@ -329,23 +447,15 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
     };
 
     int G = 0;
-    int su = SK ? sk_start(p, blockIdx.x) : 0;
+    int pi = 0;  // stream-K: segment index in processing order (sk_piece), live across the main loop
     for (int tile = SK ? 0 : WS_CID;; tile += SK ? 0 : WS_NCL) {
         int nst = NIT;     // channel blocks of this tile handled here
-        int sk_slot = -1;  // stream-K partial tile -> workspace slot 2b (the CTA's first segment) or
-                           // 2b + 1 (its last); whole tile -> y (-1)
+        int sk_slot = -1;  // stream-K: -1 whole tile -> y; else the workspace slot of this cut segment:
+                           // 2b (starts inside the tile) or 2b + 1 (holds the tile's channel block 0)
         if constexpr (SK) {
-            // (su is kept live across the main loop on purpose: re-deriving it from G changes
-            // ptxas' accumulator assignment, 1.20 -> 1.55 register reads per FFMA, sass_bank.py)
-            const int su_end = sk_start(p, blockIdx.x + 1);
-            if (su >= su_end) break;
-            tile = su / p.num_it;
-            const int g_lo = su - tile * p.num_it;
-            nst = min(p.num_it - g_lo, su_end - su);
-            if (nst != p.num_it)
-                sk_slot = 2 * static_cast<int>(blockIdx.x) +
-                          (su == sk_start(p, blockIdx.x) ? 0 : 1);
-            su += nst;
+            int g_lo;
+            if (!sk_piece(p, blockIdx.x, pi++, tile, g_lo, nst)) break;
+            if (nst != p.num_it) sk_slot = 2 * static_cast<int>(blockIdx.x) + (g_lo > 0 ? 0 : 1);
         } else if (tile >= num_tiles) {
             break;
         }
@@ -378,6 +488,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             const int slot = G % S, vb = G % SV;
             mbar_wait(&full[slot], (G / S) & 1);
             mbar_wait(&vfull[vb], (G / SV) & 1);
+#ifdef WINO_WS_CTATRACE
+            if (tid == 0 && G == 0) WS_CT(1);
+#endif
             const float* us = smem + slot * STAGE_FLOATS + xi0 * BK + fo;
             const float* v = vs + vb * VS_FLOATS + xi0 * BC * BN + io;
             float fa[2][8], ga[2][8], fb[2][8], gb[2][8];
@@ -397,6 +510,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
             }
         }
 
+        if (tid == 0) WS_CT(2);
         // ---- OTF (Sec. 4.4) through the epilogue buffer ----
         const int nu = nu0 + lane;
         int t = 0, n = 0, i0 = 0, j0 = 0;
@@ -422,9 +536,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                 // filters kl = fo + (i&3) + 32*(i>>2); in the buffer row = (fo>>2)*RR + ii
                 // (RR = 2: 4 rounds of 16 filters, the paper's 4-round OTF, L499)
                 const int rd_hi = RR == 2 ? (rd >> 1) : rd, rd_lo = RR == 2 ? (rd & 1) : 0;
-#ifndef WS_EXP_NOBAR
                 named_bar_sync(1, COMPUTE_THREADS);  // previous round's readers are done
-#endif
 #pragma unroll
                 for (int q = 0; q < 2; ++q)
 #pragma unroll
@@ -437,9 +549,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                         *reinterpret_cast<float4*>(row + 16) =
                             make_float4(acc[q][i][5], acc[q][i][4], acc[q][i][7], acc[q][i][6]);
                     }
-#ifndef WS_EXP_NOBAR
                 named_bar_sync(1, COMPUTE_THREADS);
-#endif
                 if (nu < p.NV) {
 #pragma unroll
                     for (int h = 0; h < RR; ++h) {
@@ -452,7 +562,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                             for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + r) * ER_LD + (lane ^ 1)];
                             otf_2x2(m, o);
                             if (SK && sk_slot >= 0) {
-                                // partial tile: [slot][kl][output][nu] for sk_fixup_kernel
+                                // cut segment: [slot][kl][output][nu], summed by the tile's last arrival
                                 float* wk = p.sk_ws + ((size_t)sk_slot * BK + kl) * (4 * BN) + lane;
                                 wk[0] = o[0];
                                 wk[BN] = o[1];
@@ -460,19 +570,16 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                                 wk[3 * BN] = o[3];
                             } else {
                             float* yk = p.y + (size_t)k * HWN + base;
-#ifdef WS_EXP_NOSTG
-                            if (o[0] == 1234.5f && o[1] == o[2] && o[3] == 7.f) yk[0] = o[0];
-#else
                             yk[0] = o[0];
                             if (okc) yk[p.N] = o[1];
                             if (okr) yk[dW] = o[2];
                             if (okr && okc) yk[dW + p.N] = o[3];
-#endif
                             }
                         }
                     }
                 }
             }
+            if (SK && sk_slot >= 0) sk_arrive(p, tile, k0, nu0, sk_sh, tid);
 #ifdef WINO_WS_TRACE
             if (tid == 0) WS_TR(3, (tile - WS_CID) / WS_NCL);
 #endif
@@ -562,6 +669,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
 #endif
         }
     }
+    if (tid == 0) WS_CT(3);
     if constexpr (SPLIT) {
         // peers may still be reading this CTA's yp: exit only after they all signalled
         const int T = num_tiles > WS_CID ? (num_tiles - WS_CID + WS_NCL - 1) / WS_NCL : 0;  // tiles done
@@ -572,67 +680,5 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
 #undef WS_CID
 #undef WS_NCL
 
-// Stream-K fixup: blocks 8i .. 8i+7 handle the tile cut by the range boundary of CTA b = i + 1
-// (when it is the first boundary inside that tile), 8 filters each: y = sum of the tile's
-// segments' partial outputs, added in CTA order (deterministic).  256 threads = 8 filters x
-// 32 nu; each thread issues the loads of 8 segments before adding them (latency-bound otherwise).
-__global__ void __launch_bounds__(256) sk_fixup_kernel(const __grid_constant__ Params p, int G) {
-    __shared__ int slots[256];  // workspace slots of the tile's segments, CTA order (G <= 256)
-    __shared__ int nseg;
-    const int b = blockIdx.x / 8 + 1, kr = blockIdx.x % 8;
-    const int ub = sk_start(p, b);
-    const int tile = ub / p.num_it;
-    const int t0 = tile * p.num_it, t1 = t0 + p.num_it;
-    if (ub == t0 || sk_start(p, b - 1) > t0) return;  // no cut, or an earlier boundary owns it
-    if (threadIdx.x == 0) {
-        int b0 = b - 1;  // the CTA whose range holds unit t0
-        while (b0 > 0 && sk_start(p, b0) > t0) --b0;
-        int ns = 0;
-        int c0 = sk_start(p, b0);
-        for (int c = b0; c < G && c0 < t1 && ns < 256; ++c) {
-            const int c1 = sk_start(p, c + 1);
-            if (c1 > c0) slots[ns++] = 2 * c + (c0 < t0 ? 1 : 0);  // first segment of CTA c -> 2c, else its last
-            c0 = c1;
-        }
-        nseg = ns;
-    }
-    __syncthreads();
-    const int kb = tile % p.num_kb, nb = tile / p.num_kb;
-    const int lane = threadIdx.x & 31;
-    const int kl = kr * 8 + (threadIdx.x >> 5), k = kb * BK + kl;
-    const int nu = nb * BN + lane;
-    if (nu >= p.NV || k >= p.K) return;
-    const int t = nu / p.N, n = nu - t * p.N;
-    const int th = t / p.TW, tw = t - th * p.TW;
-    const int i0 = 2 * th, j0 = 2 * tw;
-    const bool okr = i0 + 1 < p.H, okc = j0 + 1 < p.W;
-    const size_t HWN = (size_t)p.H * p.W * p.N, dW = (size_t)p.W * p.N;
-    const float* wbase = p.sk_ws + (size_t)kl * (4 * BN) + lane;
-    constexpr size_t SLOT = (size_t)BK * 4 * BN;
-    const int ns = nseg;
-    float o[4] = {0.f, 0.f, 0.f, 0.f};
-    for (int i0s = 0; i0s < ns; i0s += 8) {
-        float v[8][4];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            if (i0s + i < ns) {
-                const float* wk = wbase + (size_t)slots[i0s + i] * SLOT;
-#pragma unroll
-                for (int q = 0; q < 4; ++q) v[i][q] = wk[q * BN];
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-            if (i0s + i < ns) {
-#pragma unroll
-                for (int q = 0; q < 4; ++q) o[q] += v[i][q];
-            }
-    }
-    float* yk = p.y + (size_t)k * HWN + ((size_t)i0 * p.W + j0) * p.N + n;
-    yk[0] = o[0];
-    if (okc) yk[p.N] = o[1];
-    if (okr) yk[dW] = o[2];
-    if (okr && okc) yk[dW + p.N] = o[3];
-}
 }  // namespace fp32ws
 }  // namespace wino

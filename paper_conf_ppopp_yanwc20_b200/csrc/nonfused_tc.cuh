@@ -46,9 +46,20 @@ __host__ __device__ inline int gemm_stages(int bnk) {
     const int s = (200 * 1024) / stage;
     return s > 6 ? 6 : s;
 }
+// stages actually used: no more than the K loop has chunks (short K loops -> smaller CTAs, more
+// of them per SM to overlap one tile's epilogue with another's loads)
 template <int P>
-__host__ __device__ inline int gemm_smem_bytes(int bnk) {
-    return 1024 /* alignment slack */ + gemm_stages<P>(bnk) * P * (A_TILE + bnk * BKC * 4) + 256;
+__host__ __device__ inline int gemm_stages_for(int bnk, int nchunks) {
+    if (nchunks <= 4) {  // short K loop (C <= 128): <= 75 KB per CTA so that >= 3 CTAs share an SM
+        const int per = (75 * 1024) / (P * (A_TILE + bnk * BKC * 4));
+        const int s = nchunks < per ? nchunks : per;
+        return s < 2 ? 2 : s;
+    }
+    return gemm_stages<P>(bnk);
+}
+template <int P>
+__host__ __device__ inline int gemm_smem_bytes(int bnk, int stages) {
+    return 1024 /* alignment slack */ + stages * P * (A_TILE + bnk * BKC * 4) + 256;
 }
 
 // SWIZZLE_128B K-major shared-memory matrix descriptor (sm_100): start >> 4, LBO unused (1),
@@ -65,10 +76,6 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t r[16]) {
         : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
           "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
         : "r"(taddr));
-}
-
-__device__ __forceinline__ void tma_load_3d_hint(void* dst, const void* map, uint64_t* bar, int c0, int c1, int c2) {
-    tma_load_3d(dst, map, bar, c0, c1, c2);
 }
 
 struct __align__(64) GemmParams {

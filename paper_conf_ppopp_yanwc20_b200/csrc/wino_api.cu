@@ -96,6 +96,8 @@ bool overlaps(const void* a, size_t na, const void* b, size_t nb) {
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
+size_t round_up256(size_t b) { return (b + 255) & ~size_t(255); }
+
 // stream-K workspace of the tensor-core kernels: 2 slots of MM x 4 x TN FP32 partials (64 KiB each) per CTA
 size_t tc16_sk_bytes(int ctas) { return size_t(ctas) * 2 * 128 * 4 * 32 * sizeof(float); }
 // stream-K pays for the 16-bit kernel only when whole tiles would leave most SMs idle: its pieces
@@ -138,12 +140,15 @@ struct Fp32Plan {
     bool sk = false;     // stream-K WS kernel (+ fixup kernel); needs the workspace
 };
 
-// Stream-K workspace: 2 partial-tile slots (64 k x 4 outputs x 32 nu fp32) per CTA.
-size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * wino::fp32::BK * 4 * wino::fp32::BN * sizeof(float); }
+// Stream-K workspace: 2 partial-tile slots (64 k x 4 outputs x 32 nu fp32) per CTA, then one
+// arrival counter per CTA (zero between launches; see fused_fp32_ws.cuh).
+size_t sk_slot_bytes() { return size_t(wino::fp32::BK) * 4 * wino::fp32::BN * sizeof(float); }
+size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * sk_slot_bytes() + round_up256(size_t(ctas) * 4); }
 
 int log2_small(int s) { return s == 1 ? 0 : s == 2 ? 1 : s == 4 ? 2 : 3; }
-// planner cost of the stream-K fixup launch, in channel-block times (~1 us each)
-constexpr double kSkFixupBlocks = 2.0;
+// planner cost of the stream-K cut-tile reduction (owners add their contributors' partials in the
+// kernel's epilogue), in channel-block times
+constexpr double kSkFixupBlocks = 0.5;
 
 // Shape -> kernel / tiling / split-C.  force_split: 0 = choose, else 1, 2, 4 or 8.
 // The split model: a cluster of S CTAs shares a tile, each CTA runs ceil(NIT/S)
@@ -402,6 +407,8 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
     const bool box32 = prm.xnb == BN;
     if (pl.ws && pl.sk) {  // stream-K: equal unit ranges on every SM + fixup of the cut tiles
         prm.sk_ws = static_cast<float*>(ws);
+        // 2 partial-tile slots per CTA, then one arrival counter per CTA (zero between launches)
+        prm.sk_flags = reinterpret_cast<unsigned*>(static_cast<char*>(ws) + 2 * sk_slot_bytes() * pl.grid);
         prm.sk_total = pl.tiles * prm.num_it;  // < 2^31 (planner)
         prm.sk_q = static_cast<int>(prm.sk_total / pl.grid);
         prm.sk_r = static_cast<int>(prm.sk_total % pl.grid);
@@ -410,11 +417,7 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
         wino_status_t s = ensure_smem_attr(kern, dev, sm, g_attr_ws_sk[box32]);
         if (s != WINO_OK) return s;
         kern<<<dim3(static_cast<unsigned>(pl.grid)), wino::fp32ws::NT, sm, st>>>(prm, static_cast<int>(g));
-        cudaError_t e = cudaGetLastError();
-        if (e == cudaSuccess && pl.grid > 1)
-            wino::fp32ws::sk_fixup_kernel<<<dim3(static_cast<unsigned>(8 * (pl.grid - 1))), 256, 0, st>>>(
-                prm, static_cast<int>(pl.grid));
-        if (e == cudaSuccess) e = cudaGetLastError();
+        cudaError_t e = cudaGetLastError();  // the cut tiles are summed inside the kernel (no fixup launch)
         return e == cudaSuccess ? WINO_OK : cuda_fail(e);
     }
     if (pl.ws && pl.split == 1) {  // warp-specialised persistent kernel, one CTA per SM
@@ -494,7 +497,6 @@ struct EventPool {
     }
 };
 
-size_t round_up256(size_t b) { return (b + 255) & ~size_t(255); }
 
 extern "C" {
 
@@ -522,6 +524,11 @@ int wino_debug_cluster_slots(int split) {
 }
 int wino_debug_ws_trace(unsigned long long* host, int n) {
     return (int)cudaMemcpyFromSymbol(host, wino::fp32ws::g_ws_trace, sizeof(unsigned long long) * n);
+}
+#endif
+#ifdef WINO_WS_CTATRACE
+int wino_debug_cta_trace(unsigned long long* host, int n) {
+    return (int)cudaMemcpyFromSymbol(host, wino::fp32ws::g_cta_trace, sizeof(unsigned long long) * n);
 }
 #endif
 #ifdef WINO_TC16_TRACE
@@ -671,7 +678,7 @@ wino_status_t wino_plan(int N, int C, int H, int W, int K, int variant, wino_pla
     plan->ctas = p.sk ? p.grid : p.tiles * p.split;
     plan->threads = p.threads;
     plan->smem_bytes = p.smem;
-    plan->launches = p.sk ? 2 : 1;
+    plan->launches = 1;  // the FP32 stream-K plan reduces its cut tiles in the kernel
     plan->stream_k = p.sk ? 1 : 0;
     return WINO_OK;
 }
@@ -1460,8 +1467,8 @@ wino_status_t nonfused_launch(const float* x_dev, const float* u_dev, float* y_d
     gp.NV = NV;
     gp.C = C;
     gp.bnk = bnk;
-    gp.stages = gemm_stages<P>(bnk);
     gp.nchunks = (C + BKC - 1) / BKC;
+    gp.stages = gemm_stages_for<P>(bnk, gp.nchunks);
     wino_status_t s;
     // 1. transformed filter -> GEMM operand layout (TF32 planes)
     nf_arrange_u_kernel<P><<<dim3(unsigned((K + 31) / 32), unsigned((C4 + 31) / 32), 16), 256, 0, st>>>(u_dev, ug, C,
@@ -1474,8 +1481,9 @@ wino_status_t nonfused_launch(const float* x_dev, const float* u_dev, float* y_d
                                                                                                      H, W, TW, NV);
     if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e);
     // 3. the 16 batched GEMMs on tcgen05: M[xi][k][nu]
-    const int smem = gemm_smem_bytes<P>(bnk);
-    if ((s = ensure_smem_attr(nf_gemm_kernel<P>, dev, gemm_smem_bytes<P>(256), g_attr_nf_gemm[P - 1])) != WINO_OK)
+    const int smem = gemm_smem_bytes<P>(bnk, gp.stages);
+    if ((s = ensure_smem_attr(nf_gemm_kernel<P>, dev, gemm_smem_bytes<P>(256, gemm_stages<P>(256)),
+                              g_attr_nf_gemm[P - 1])) != WINO_OK)
         return s;
     nf_gemm_kernel<P><<<dim3(unsigned((NV + BM - 1) / BM), unsigned((K + bnk - 1) / bnk), 16), GEMM_THREADS, smem,
                         st>>>(gp);

@@ -252,6 +252,12 @@ __device__ __forceinline__ float4 ld_dsmem4(uint32_t cluster_addr) {
 }  // namespace wino
 
 namespace wino {
+// GPU-scope acquire-release atomic add on a counter word (cross-CTA hand-off in global memory)
+__device__ __forceinline__ unsigned atom_add_acq_rel_gpu(unsigned* p, unsigned v) {
+    unsigned old;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;\n" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
 // Asynchronous 16 B store into (possibly another CTA's) shared memory; completion is
 // counted in bytes on an mbarrier of the destination CTA (complete_tx).
 __device__ __forceinline__ void st_async4(uint32_t cluster_addr, float a, float b, float c, float d,

@@ -18,7 +18,7 @@ for cfg in shapes:
         u = wino.filter_transform(w)
         y = wino.conv2d(x, u)
         if cfg.N % 32 == 0 or cfg.N in (4, 8, 16):  # stream-K (forced) + fixup
-            ws = torch.empty(wino.conv_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
+            ws = torch.zeros(wino.conv_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
                              device="cuda")
             y = wino.conv2d(x, u, ws=ws, stream_k="on")
             if cfg.K > 64:
@@ -30,7 +30,7 @@ for cfg in shapes:
             if cfg.N % 16 == 0:
                 y = wino.conv2d_f4(x, wino.filter_transform_f4(w), stream_k="on", ws=torch.empty(
                     wino.f4_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8, device="cuda"))
-        wsn = torch.empty(wino.nchw_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
+        wsn = torch.zeros(wino.nchw_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8,
                           device="cuda")
         y = wino.conv2d_nchw(x.permute(3, 0, 1, 2).contiguous(),
                              wino.filter_transform_kcrs(w.permute(3, 0, 1, 2).contiguous()), ws=wsn)

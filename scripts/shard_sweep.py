@@ -75,7 +75,7 @@ def main():
                 if var == "fp32":
                     u = wino.filter_transform(wd)
                     if a.sk != "none":
-                        wsb = torch.empty(wino.conv_workspace_bytes(hi - lo, cfg.C, cfg.H, cfg.W, cfg.K),
+                        wsb = torch.zeros(wino.conv_workspace_bytes(hi - lo, cfg.C, cfg.H, cfg.W, cfg.K),
                                           dtype=torch.uint8, device=dev)
                         conv = lambda: wino.conv2d(xs, u, out=y, ws=wsb, stream_k=a.sk)  # noqa: E731
                     elif a.split:

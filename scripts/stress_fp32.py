@@ -16,7 +16,7 @@ for P in (1, 2, 4, 8):
         ref = oracle.direct_sample(x, w, idx)
         ii = idx.cuda()
         xd, u = x.cuda(), wino.filter_transform(w.cuda())
-        ws = torch.empty(wino.conv_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8, device="cuda")
+        ws = torch.zeros(wino.conv_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8, device="cuda")
         modes = {"plain": lambda: wino.conv2d(xd, u), "sk-on": lambda: wino.conv2d(xd, u, ws=ws, stream_k="on"),
                  "split2": lambda: wino.conv2d(xd, u, split_c=2)}
         for m, fn in modes.items():

@@ -61,7 +61,7 @@ def _check(y, ref, exact, tol, what, failures):
 
 
 def _ws(nbytes):
-    return torch.empty(max(int(nbytes), 16), dtype=torch.uint8, device=DEV)
+    return torch.zeros(max(int(nbytes), 16), dtype=torch.uint8, device=DEV)  # stream-K flags: zero
 
 
 @pytest.mark.parametrize("kind", ["smallint", "uniform", "resnet"])

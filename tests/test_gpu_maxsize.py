@@ -59,7 +59,7 @@ def test_maxsize_fp32_regular_and_stream_k(big):
     y = wino.conv2d(x, u)
     torch.cuda.synchronize()
     _check(y, pts, ref)
-    ws = torch.empty(wino.conv_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+    ws = torch.zeros(wino.conv_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
     y.fill_(float("nan"))
     wino.conv2d(x, u, out=y, ws=ws, stream_k="on")
     torch.cuda.synchronize()

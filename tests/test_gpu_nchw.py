@@ -83,7 +83,7 @@ def test_nchw_matches_chwn_kernel(wino):
 def _run_ws(wino, x, w):
     u = wino.filter_transform_kcrs(_kcrs(w).to(DEV))
     N, C, H, W = x.shape[3], x.shape[0], x.shape[1], x.shape[2]
-    ws = torch.empty(wino.nchw_workspace_bytes(N, C, H, W, w.shape[3]), dtype=torch.uint8, device=DEV)
+    ws = torch.zeros(wino.nchw_workspace_bytes(N, C, H, W, w.shape[3]), dtype=torch.uint8, device=DEV)
     y = wino.conv2d_nchw(_nchw(x).to(DEV), u, ws=ws)
     torch.cuda.synchronize()
     return y.cpu().permute(1, 2, 3, 0).contiguous()
@@ -113,3 +113,13 @@ def test_nchw_ws_short_workspace_rejected(wino):
     u = torch.zeros((8, 4, 4, 16), device=DEV)
     with pytest.raises(wino.WinoError, match="INVALID_ARG"):
         wino.conv2d_nchw(x, u, ws=torch.empty(1024, dtype=torch.uint8, device=DEV))
+
+
+@pytest.mark.parametrize("shape", [(2, 4, 64, 192, 192), (1, 3, 130, 131, 129)], ids=["KHW=2.36M", "KHW=2.20M"])
+def test_nchw_ws_large_plane_transposes(wino, shape):
+    """K*H*W (and C*H*W rows) beyond 65535 transpose tiles in one grid dimension: the 2-D
+    transposes use a 1-D tile grid (the round-1 grid.y = K*H*W/32 broke above 2,097,120)."""
+    N, C, K, H, W = shape
+    x, w = make_inputs(Conv3x3Config("nchw-big", N, C, K, H, W), kind="smallint")
+    y = _run_ws(wino, x, w)
+    assert np.array_equal(y.double().numpy(), oracle.direct_conv(x, w))

@@ -32,7 +32,7 @@ def wino():
 
 
 def _ws(wino, cfg):
-    return torch.empty(wino.conv_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8, device=DEV)
+    return torch.zeros(wino.conv_workspace_bytes(cfg.N, cfg.C, cfg.H, cfg.W, cfg.K), dtype=torch.uint8, device=DEV)
 
 
 def _run(wino, x, w, cfg, mode):
@@ -142,3 +142,21 @@ def test_tc_streamk(wino, shape, variant, tol):
             assert np.array_equal(y.double().numpy(), ref)
         else:
             assert oracle.max_rel_err(y.double().numpy(), ref) <= tol
+
+
+def test_streamk_leaves_flags_zero(wino):
+    """The in-kernel reduction of cut tiles clears every flag word it consumed (include/wino.h:
+    one zero-fill of the workspace serves any number of calls)."""
+    cfg = CONFIGS["conv5_x"].with_batch(8)
+    x, w = make_inputs(cfg, kind="smallint")
+    ws = _ws(wino, cfg)
+    u = wino.filter_transform(w.to(DEV))
+    ref = oracle.direct_conv(x, w)
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    slot = 64 * 4 * 32 * 4
+    for _ in range(3):
+        y = wino.conv2d(x.to(DEV), u, ws=ws, stream_k="on")
+        torch.cuda.synchronize()
+        assert np.array_equal(y.cpu().double().numpy(), ref)
+        counters = ws[2 * sms * slot: 2 * sms * slot + 4 * sms]  # after the 2 slots per CTA
+        assert int(counters.count_nonzero()) == 0

@@ -63,7 +63,7 @@ def test_repeated_runs_exact(wino, variant, shape, sk):
         assert oracle.max_rel_err(ref, oracle.direct_conv(x, w)) <= 1e-4
     else:
         u = wino.filter_transform(wd)
-        ws = torch.empty(wino.conv_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
+        ws = torch.zeros(wino.conv_workspace_bytes(N, C, H, W, K), dtype=torch.uint8, device=DEV)
         run = lambda: wino.conv2d(xd, u, ws=ws, stream_k=sk)  # noqa: E731
     bad_runs = []
     for r in range(REPS):
