@@ -19,7 +19,8 @@ Timing: the step is captured in one CUDA graph.  Headline (cold L2): L2 flushed
 (512 MiB write + 256 MiB read) before every timed step, outside the events; CUDA
 events on the launching stream; max over ranks.  Paper protocol (hot L2, L863):
 5 repeats of 20 back-to-back replays, median of the means.  Per-kernel durations
-come from timing events recorded INSIDE the step graph (the same step as `value`).
+come from timing events recorded inside a second, instrumented capture of the same
+step (event nodes between kernels cost ~10 us each, so `value` replays the bare graph).
 After timing, every variant's outputs are compared element by element with the
 fp64 oracle (Eq. 4) on this rank's full shard: measured max_rel_err per layer.
 
@@ -302,7 +303,9 @@ def _config(args, layers, world):
         "step": "per layer: FTF + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
                 "its own FTF; fp32: all layers' FTFs in one wino_filter_transform_multi launch, convs through "
                 "wino_conv2d_f2x3_fwd_ws with a stream-K workspace, the planner picks regular / split-C / "
-                "stream-K + fixup per layer); the whole step replayed from one CUDA graph",
+                "stream-K per layer); " + ("each layer's conv on its own stream (the layers are independent "
+                "problems), " if args.concurrent_layers else "convs in sequence on one stream, ") +
+                "the whole step replayed from one CUDA graph",
         "filter": "w replicated on every rank; each rank runs the FTF inside every step; rank 0's u broadcast "
                   "once over NCCL at setup and checked bit-identical to every rank's own FTF output",
     }
@@ -319,6 +322,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
     ap.add_argument("--no-check", action="store_true", help="skip the element-wise oracle comparison")
+    ap.add_argument("--concurrent-layers", action="store_true",
+                    help="issue each layer's convolution on its own stream (the BASELINE layers are independent "
+                         "problems); default: in sequence on one stream, as a network would")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo only to exercise the multi-rank logic with several ranks on one GPU")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -491,12 +497,17 @@ def main():
                     wino.conv2d(d["x"], d["u"], out=d["y"], ws=d["ws_sk"])
 
         side = torch.cuda.Stream(dev)
+        lstreams = [torch.cuda.Stream(dev) for _ in per]  # one stream per (independent) layer
         # timing events recorded inside the step graph (event-record nodes): per-kernel durations
         # of the very step `value` times
         conv_ev = [(mk_in_graph(), mk_in_graph()) for _ in per]
         ftf_ev = (mk_in_graph(), mk_in_graph())
 
-        def step(timed=False):
+        def step(timed=False, concurrent=None):
+            # concurrent: the layers are independent problems (BASELINE configs), so each layer's
+            # conv goes on its own stream -- a layer's persistent grid starts on the SMs the previous
+            # one frees in its tail instead of after its last CTA (no data dependence between them)
+            concurrent = args.concurrent_layers if concurrent is None else concurrent
             # The layers' filter transforms (a1) do not depend on the convolutions, so they run
             # on a side stream: FTF of layer l+1 overlaps conv l (the persistent conv grids
             # leave SMs free at small per-rank batches).  conv l waits for its own FTF only.
@@ -523,13 +534,24 @@ def main():
                     ready.append(ev)
             if timed:
                 ftf_ev[1].record(side)
-            for d, ev, (ea, eb) in zip(per, ready, conv_ev):
-                cur.wait_event(ev)
-                if timed:
-                    ea.record(cur)
-                run_layer(d, ftf=False)
-                if timed:
-                    eb.record(cur)
+            done = []
+            for d, ev, (ea, eb), ls in zip(per, ready, conv_ev, lstreams):
+                st = ls if concurrent else cur
+                if concurrent:
+                    st.wait_event(fork)
+                st.wait_event(ev)
+                with torch.cuda.stream(st):
+                    if timed:
+                        ea.record(st)
+                    run_layer(d, ftf=False)
+                    if timed:
+                        eb.record(st)
+                if concurrent:
+                    e = torch.cuda.Event()
+                    e.record(st)
+                    done.append(e)
+            for e in done:
+                cur.wait_event(e)
             join = torch.cuda.Event()
             join.record(side)
             cur.wait_event(join)
@@ -540,9 +562,15 @@ def main():
         torch.cuda.synchronize()
         # The timed step is replayed from a CUDA graph (captured once, after warm-up):
         # host launch latency stays out of the device timeline, as in a serving loop.
+        # `value` replays an uninstrumented graph: timing-event nodes between the kernels of a graph
+        # were measured to add ~10 us each to the step (round 2); the per-kernel breakdown replays
+        # a second, instrumented capture of the same step (layers in sequence)
         g_step = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g_step):
-            step(timed=True)
+            step()
+        g_timed = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g_timed):
+            step(timed=True, concurrent=False)
         g_conv = []
         for d in per:
             gc = torch.cuda.CUDAGraph()
@@ -576,16 +604,20 @@ def main():
         clocks = sampler.stop() if sampler else None
         ms_step = sum(a.elapsed_time(b) for a, b in step_ev) / args.steps
 
-        # per-kernel breakdown: the same graph, the same flush, events inside the graph
-        conv_ms, ftf_ms_step = [0.0] * len(per), 0.0
+        # per-kernel breakdown: the instrumented capture of the same step, the same flush
+        conv_ms, ftf_ms_step, timed_ms = [0.0] * len(per), 0.0, 0.0
         for s in range(args.steps):
             flush_l2(float(s))
-            g_step.replay()
+            a, b = mk(), mk()
+            a.record(stream)
+            g_timed.replay()
+            b.record(stream)
             torch.cuda.synchronize()
             for i, d in enumerate(per):
                 if d["n"]:
                     conv_ms[i] += conv_ev[i][0].elapsed_time(conv_ev[i][1]) / args.steps
             ftf_ms_step += ftf_ev[0].elapsed_time(ftf_ev[1]) / args.steps
+            timed_ms += a.elapsed_time(b) / args.steps
 
         # the paper's protocol (L863): hot L2, 20 back-to-back launches, mean; 5 repeats, median
         def hot(g, reps=5, n=20):
@@ -620,7 +652,8 @@ def main():
                 "ftf_ms_step": _max_over_ranks(ftf_ms_step, world, dev),
                 "hot_ms_step": _max_over_ranks(hot_step, world, dev),
                 "hot_conv_ms": [_max_over_ranks(v, world, dev) for v in hot_conv],
-                "launches": launches, "wall": wall, "clocks": clocks, "outs": outs}
+                "launches": launches, "wall": wall, "clocks": clocks, "outs": outs,
+                "timed_ms": _max_over_ranks(timed_ms, world, dev)}
 
     # ---- the fp64 oracle's outputs on this rank's shard (computed once per input rounding) ----
     refs, ref_time = {}, {}
@@ -768,6 +801,8 @@ def main():
         "hot_l2": {"value": total_eff / (main_m["hot_ms_step"] * 1e-3) / 1e12, "ms_per_step": main_m["hot_ms_step"],
                    "protocol": "L863: 20 back-to-back graph replays of the step, mean; 5 repeats, median"},
         "ftf_us_step": main_m["ftf_ms_step"] * 1e3,
+        "layers_in_step": ("concurrent: one stream per layer (independent problems), each conv waits only for "
+                           "its FTF" if args.concurrent_layers else "in sequence on one stream"),
         "layers": layer_rep,
         "roofline": {"bound": "alu", "kernel": f"wino fused_{args.variant}", "achieved": achieved,
                      "peak": fp32_peak, "unit": "TFLOP/s", "frac": achieved / fp32_peak, "traffic": traffic,
@@ -775,7 +810,8 @@ def main():
                                        "dram__bytes_write.sum of the conv launches of one step "
                                        "(profiles/traffic.json)",
                      "achieved_def": "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) per launch summed over layers / "
-                                     "summed conv durations from timing events inside the timed step graph",
+                                     "summed conv durations from timing events inside an instrumented capture "
+                                     "of the same step graph (L2 flushed as for value)",
                      "peak_def": FP32_PEAK_NOTE},
         "ms_per_step_ranks": main_m["ms_step_ranks"],
         "gpu_launches": launches_per_step * args.steps,
@@ -785,6 +821,10 @@ def main():
         res["max_rel_err"] = max(errs_main.values()) if errs_main else 0.0
         res["parity"] = {"vs": "fp64 oracle direct conv (Eq. 4), every output element of every rank's shard",
                          "tolerance": TOL[args.variant], "pass": res["max_rel_err"] <= TOL[args.variant]}
+    res["instrumented_step"] = {"ms_per_step": main_m["timed_ms"],
+                                "note": "the step graph with timing-event nodes around every kernel (the source "
+                                        "of the per-layer conv_us and of roofline.achieved); value uses the "
+                                        "uninstrumented graph"}
     if u_bcast_ok is not None:
         res["u_broadcast_bit_identical"] = u_bcast_ok
     if e2e:
@@ -837,6 +877,7 @@ def main():
         res["cpu_baseline"] = cpu_base
     if args.shard_of:
         res = {"diagnostic": f"rank 0 shard of a {args.shard_of}-rank job timed alone on one GPU", "ms_per_step": ms_step,
+               "instrumented_ms_per_step": main_m["timed_ms"],
                "projected_value_if_all_ranks_equal": total_eff / (ms_step * 1e-3) / 1e12,
                "layers_us": {k: {"conv_us": v["conv_us"]} for k, v in layer_rep.items()},
                "variants_ms_per_step": {k: v["ms_per_step"] for k, v in vrep.items()}}
