@@ -40,11 +40,15 @@ while [ $# -gt 0 ]; do
         --csv --log-file ${O}_launches.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline \
         --no-variants --no-check > /dev/null 2>&1; step launches $? ;;
     profile)
+      # the .ncu-rep stays in /tmp (gpurun copies back at most 64 MiB); summaries come back
       V=$2; R=$3; shift 2
-      timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$R" -s 0 -c 8 -o ${O}_prof_$V \
+      REP=/tmp/${TAG}_prof_$V
+      timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$R" -s 0 -c 8 -o $REP \
         python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline --no-check --no-variants --variant $V \
         > ${O}_prof_$V.log 2>&1; step profile-$V $?
-      python scripts/ncu_summary.py ${O}_prof_$V.ncu-rep --json ${O}_prof_$V.json > /dev/null 2>&1 ;;
+      python scripts/ncu_summary.py $REP.ncu-rep --json ${O}_prof_$V.json > ${O}_prof_$V.txt 2>&1
+      for L in 0 1 2 3; do python scripts/ncu_line_stalls.py $REP.ncu-rep $L > ${O}_prof_${V}_lines$L.txt 2>&1; done
+      [ "${KEEP_REP:-0}" = "1" ] && cp $REP.ncu-rep ${O}_prof_$V.ncu-rep ;;
     sanitize)
       for tool in memcheck synccheck; do
         timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python scripts/sanitize.py > ${O}_$tool.log 2>&1
