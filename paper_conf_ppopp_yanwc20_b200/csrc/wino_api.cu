@@ -146,9 +146,9 @@ size_t sk_slot_bytes() { return size_t(wino::fp32::BK) * 4 * wino::fp32::BN * si
 size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * sk_slot_bytes() + round_up256(size_t(ctas) * 4); }
 
 int log2_small(int s) { return s == 1 ? 0 : s == 2 ? 1 : s == 4 ? 2 : 3; }
-// planner cost of the stream-K cut-tile reduction (owners add their contributors' partials in the
-// kernel's epilogue), in channel-block times
-constexpr double kSkFixupBlocks = 0.5;
+// planner cost of the stream-K plan beyond its units, in channel-block times: up to two partial
+// epilogues per CTA plus the last-arrival reductions (fitted to scripts/sk_ab.py)
+constexpr double kSkFixupBlocks = 4.0;
 
 // Shape -> kernel / tiling / split-C.  force_split: 0 = choose, else 1, 2, 4 or 8.
 // The split model: a cluster of S CTAs shares a tile, each CTA runs ceil(NIT/S)
@@ -191,7 +191,9 @@ Fp32Plan plan_fp32(int N, int C, int H, int W, int K, bool u_tma_ok, int dev, in
             const int cl = cluster_slots(s, dev);
             if (cl <= 0) continue;
             const double waves = double((p.tiles + cl - 1) / cl);
-            const double est = waves * (double((nit + s - 1) / s) + (s == 1 ? 0.5 : 1.5));
+            // epilogue in channel-block times: plain 0.5; the cluster reduction 1.5 for S = 2, 4 and
+            // 5 for S = 8 (8 partials per output; fitted to scripts/sk_ab.py)
+            const double est = waves * (double((nit + s - 1) / s) + (s == 1 ? 0.5 : (s == 8 ? 5.0 : 1.5)));
             if (s == 1 || est < best * 0.97) {
                 best = est;
                 p.split = s;
