@@ -300,11 +300,15 @@ def _config(args, layers, world):
         "inputs": f"uniform[-1,1) fp32, torch seeds x={SEED_X} w={SEED_W}",
         "l2": "headline: flushed before every timed step by a 512 MiB write + 256 MiB read (outside the events); "
               "hot_l2: the paper's protocol (L863), 5 repeats x 20 back-to-back replays, median of the means",
-        "step": "per layer: FTF + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
-                "its own FTF; fp32: all layers' FTFs in one wino_filter_transform_multi launch, convs through "
-                "wino_conv2d_f2x3_fwd_ws with a stream-K workspace, the planner picks regular / split-C / "
-                "stream-K per layer); " + ("each layer's conv on its own stream (the layers are independent "
-                "problems), " if args.concurrent_layers else "convs in sequence on one stream, ") +
+        "step": ("fp32: all layers' FTFs in one wino_filter_transform_multi launch, then every conv through "
+                 "ONE wino_conv2d_f2x3_fwd_multi call (layers with < 32 tiles per SM share one persistent "
+                 "stream-K launch, larger ones run alone through the planner); "
+                 if args.variant == "fp32" and not args.per_layer_launches else
+                 "per layer: FTF + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
+                 "its own FTF; fp32: all layers' FTFs in one wino_filter_transform_multi launch, convs through "
+                 "wino_conv2d_f2x3_fwd_ws with a stream-K workspace, the planner picks regular / split-C / "
+                 "stream-K per layer); " + ("each layer's conv on its own stream (the layers are independent "
+                 "problems), " if args.concurrent_layers else "convs in sequence on one stream, ")) +
                 "the whole step replayed from one CUDA graph",
         "filter": "w replicated on every rank; each rank runs the FTF inside every step; rank 0's u broadcast "
                   "once over NCCL at setup and checked bit-identical to every rank's own FTF output",
@@ -322,6 +326,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip timing the other kernel variants")
     ap.add_argument("--no-check", action="store_true", help="skip the element-wise oracle comparison")
+    ap.add_argument("--per-layer-launches", action="store_true",
+                    help="fp32: one conv launch per layer (wino_conv2d_f2x3_fwd_ws) instead of one "
+                         "wino_conv2d_f2x3_fwd_multi call for all layers (shared persistent stream-K launch)")
     ap.add_argument("--concurrent-layers", action="store_true",
                     help="issue each layer's convolution on its own stream (the BASELINE layers are independent "
                          "problems); default: in sequence on one stream, as a network would")
@@ -414,6 +421,8 @@ def main():
         nchw = variant == "fp32_nchw"  # NEXT row N2: NCHW / KCRS front end (Sec. 8.4)
         nonfused = variant in ("nonfused_fp32", "nonfused_tf32")  # NEXT row N3: ITF -> 16 GEMMs -> OTF
         half = variant in ("fp16", "bf16")  # NEXT row N4: 16-bit x, w, y on tcgen05 kind::f16 (Sec. 8.3)
+        # fp32: every layer through one wino_conv2d_f2x3_fwd_multi call (shared persistent launch)
+        multi = variant == "fp32" and not args.per_layer_launches
         if f4:  # FTF4 + conv (+ a stream-K fixup where the planner takes it: counted as taken)
             launches = sum(3 for d in live)
         elif half:  # FTF + conv (+ stream-K fixup with the workspace, variant 5 plans it)
@@ -424,8 +433,11 @@ def main():
                            for d in live)
         elif nonfused:
             launches = sum(1 + wino.nonfused_launches() for d in live)  # FTF + u arrangement, ITF, GEMM, OTF
+        elif multi:  # one batched FTF + the conv launches of wino_conv2d_f2x3_fwd_multi
+            launches = 1 + wino.conv_multi_launches([(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K)
+                                                     for d in live])
         else:
-            # fp32: the stream-K workspace plan (variant 4) is one launch; tf32: + a fixup launch
+            # fp32 per layer: the stream-K workspace plan (variant 4) is one launch; tf32: + a fixup launch
             vid = {"fp32": 4, "tf32": 6, "3xtf32": 7}[variant]  # plans with the stream-K workspaces
             launches = sum((1 if variant != "fp32" else 0) +
                            wino.plan(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K, variant=vid).launches
@@ -496,11 +508,16 @@ def main():
                 else:
                     wino.conv2d(d["x"], d["u"], out=d["y"], ws=d["ws_sk"])
 
+        if multi:
+            ws_ml = torch.zeros(max(wino.conv_multi_workspace_bytes(
+                [(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K) for d in live]), 16),
+                dtype=torch.uint8, device=dev)
         side = torch.cuda.Stream(dev)
         lstreams = [torch.cuda.Stream(dev) for _ in per]  # one stream per (independent) layer
         # timing events recorded inside the step graph (event-record nodes): per-kernel durations
         # of the very step `value` times
         conv_ev = [(mk_in_graph(), mk_in_graph()) for _ in per]
+        multi_ev = (mk_in_graph(), mk_in_graph())
         ftf_ev = (mk_in_graph(), mk_in_graph())
 
         def step(timed=False, concurrent=None):
@@ -535,7 +552,15 @@ def main():
             if timed:
                 ftf_ev[1].record(side)
             done = []
-            for d, ev, (ea, eb), ls in zip(per, ready, conv_ev, lstreams):
+            if multi:  # all layers' convolutions in one launch, after all FTFs
+                for ev in set(ready):
+                    cur.wait_event(ev)
+                if timed:
+                    multi_ev[0].record(cur)
+                wino.conv2d_multi([(d["x"], d["u"], d["y"]) for d in live], ws_ml)
+                if timed:
+                    multi_ev[1].record(cur)
+            for d, ev, (ea, eb), ls in zip(per, ready if not multi else [], conv_ev, lstreams):
                 st = ls if concurrent else cur
                 if concurrent:
                     st.wait_event(fork)
@@ -605,7 +630,7 @@ def main():
         ms_step = sum(a.elapsed_time(b) for a, b in step_ev) / args.steps
 
         # per-kernel breakdown: the instrumented capture of the same step, the same flush
-        conv_ms, ftf_ms_step, timed_ms = [0.0] * len(per), 0.0, 0.0
+        conv_ms, ftf_ms_step, timed_ms, multi_ms = [0.0] * len(per), 0.0, 0.0, 0.0
         for s in range(args.steps):
             flush_l2(float(s))
             a, b = mk(), mk()
@@ -613,8 +638,10 @@ def main():
             g_timed.replay()
             b.record(stream)
             torch.cuda.synchronize()
+            if multi:
+                multi_ms += multi_ev[0].elapsed_time(multi_ev[1]) / args.steps
             for i, d in enumerate(per):
-                if d["n"]:
+                if d["n"] and not multi:
                     conv_ms[i] += conv_ev[i][0].elapsed_time(conv_ev[i][1]) / args.steps
             ftf_ms_step += ftf_ev[0].elapsed_time(ftf_ev[1]) / args.steps
             timed_ms += a.elapsed_time(b) / args.steps
@@ -633,6 +660,18 @@ def main():
             return _median(means)
         hot_step = hot(g_step)
         hot_conv = [hot(gc) if d["n"] else 0.0 for gc, d in zip(g_conv, per)]
+        if multi:  # per-layer breakdown: each layer alone through wino_conv2d_f2x3_fwd_ws, L2 flushed
+            for s in range(args.steps):
+                for i, (gc, d) in enumerate(zip(g_conv, per)):
+                    if not d["n"]:
+                        continue
+                    flush_l2(float(s))
+                    a, b = mk(), mk()
+                    a.record(stream)
+                    gc.replay()
+                    b.record(stream)
+                    torch.cuda.synchronize()
+                    conv_ms[i] += a.elapsed_time(b) / args.steps
         torch.cuda.synchronize()
 
         # outputs of the last replay (deterministic) vs the fp64 oracle, element by element
@@ -653,7 +692,8 @@ def main():
                 "hot_ms_step": _max_over_ranks(hot_step, world, dev),
                 "hot_conv_ms": [_max_over_ranks(v, world, dev) for v in hot_conv],
                 "launches": launches, "wall": wall, "clocks": clocks, "outs": outs,
-                "timed_ms": _max_over_ranks(timed_ms, world, dev)}
+                "timed_ms": _max_over_ranks(timed_ms, world, dev),
+                "multi_ms": _max_over_ranks(multi_ms, world, dev) if multi else None}
 
     # ---- the fp64 oracle's outputs on this rank's shard (computed once per input rounding) ----
     refs, ref_time = {}, {}
@@ -780,7 +820,11 @@ def main():
         }
         if errs_main is not None:
             layer_rep[c.name]["max_rel_err"] = errs_main[c.name]
-    achieved = ewmm_flops / (conv_total_ms * 1e-3) / 1e12
+    multi_ms = main_m.get("multi_ms")
+    # the dominant kernel's duration inside the step: the multi-layer launch (fp32 default) or the
+    # summed per-layer conv launches
+    conv_step_ms = multi_ms if multi_ms else conv_total_ms
+    achieved = ewmm_flops / (conv_step_ms * 1e-3) / 1e12
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
@@ -801,6 +845,9 @@ def main():
         "hot_l2": {"value": total_eff / (main_m["hot_ms_step"] * 1e-3) / 1e12, "ms_per_step": main_m["hot_ms_step"],
                    "protocol": "L863: 20 back-to-back graph replays of the step, mean; 5 repeats, median"},
         "ftf_us_step": main_m["ftf_ms_step"] * 1e3,
+        "conv_launch": ("all layers through one wino_conv2d_f2x3_fwd_multi call: " + f"{multi_ms * 1e3:.1f} us in "
+                        "the instrumented step; layers.*.conv_us time each layer alone (wino_conv2d_f2x3_fwd_ws, "
+                        "L2 flushed)") if multi_ms else "one launch per layer (layers.*.conv_us from the step)",
         "layers_in_step": ("concurrent: one stream per layer (independent problems), each conv waits only for "
                            "its FTF" if args.concurrent_layers else "in sequence on one stream"),
         "layers": layer_rep,
@@ -809,9 +856,13 @@ def main():
                      "traffic_source": "stored, not measured in this run: ncu dram__bytes_read.sum + "
                                        "dram__bytes_write.sum of the conv launches of one step "
                                        "(profiles/traffic.json)",
-                     "achieved_def": "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) per launch summed over layers / "
-                                     "summed conv durations from timing events inside an instrumented capture "
-                                     "of the same step graph (L2 flushed as for value)",
+                     "achieved_def": ("EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) summed over layers / the duration of "
+                                      "the wino_conv2d_f2x3_fwd_multi call (its shared persistent stream-K launch + any layer run alone) "
+                                      if multi_ms else
+                                      "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) per launch summed over layers / "
+                                      "summed conv durations") +
+                                     " from timing events inside an instrumented capture of the same step graph "
+                                     "(L2 flushed as for value)",
                      "peak_def": FP32_PEAK_NOTE},
         "ms_per_step_ranks": main_m["ms_step_ranks"],
         "gpu_launches": launches_per_step * args.steps,
@@ -878,6 +929,7 @@ def main():
     if args.shard_of:
         res = {"diagnostic": f"rank 0 shard of a {args.shard_of}-rank job timed alone on one GPU", "ms_per_step": ms_step,
                "instrumented_ms_per_step": main_m["timed_ms"],
+               "multi_conv_us": main_m["multi_ms"] * 1e3 if main_m.get("multi_ms") else None,
                "projected_value_if_all_ranks_equal": total_eff / (ms_step * 1e-3) / 1e12,
                "layers_us": {k: {"conv_us": v["conv_us"]} for k, v in layer_rep.items()},
                "variants_ms_per_step": {k: v["ms_per_step"] for k, v in vrep.items()}}

@@ -251,6 +251,40 @@ wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, fl
                                       int sk, void* ws_dev, size_t ws_bytes, wino_stream_t stream);
 
 /*
+ * Several INDEPENDENT layers (a network step's convolutions, each with its own x, u, y and
+ * shape; pad 1, stride 1) through as few launches as pay (Sec. 3-4 method per layer, Eq. 4-8;
+ * the batching across layers is this library's, not the paper's).  Layers that the
+ * warp-specialised FP32 kernel takes (N % 32 == 0 or N in {4, 8, 16}; K % 4 == 0) and that have
+ * fewer than 32 output tiles (64 filters x 32 positions) per SM share ONE persistent launch per
+ * group of up to 4: the (tile, channel block) units of the group are concatenated and cut into one
+ * contiguous range per SM, balanced on a work model (unit cost per x box mode, one output
+ * transform per tile), so the group pays one pipeline fill and one tail instead of one per layer,
+ * and each CTA has at most two cut tiles (reduced inside the kernel as in
+ * wino_conv2d_f2x3_fwd_ws).  Any other layer runs alone through wino_conv2d_f2x3_fwd_ws's
+ * planner (sk = 0).  Same arithmetic per output as wino_conv2d_f2x3_fwd_ws (equal up to FP32
+ * summation order of cut tiles; bit-identical on small-integer inputs).  Launches go to `stream`
+ * in job order.
+ *   jobs[i]          : device pointers and shape of layer i; y of a job must not overlap any
+ *                      job's x, u or y; 1 <= n.
+ *   ws_dev / ws_bytes: >= wino_conv_multi_workspace_bytes(jobs, n) (= wino_conv_workspace_bytes),
+ *                      16-byte aligned, not overlapping any tensor, ZERO-FILLED before its first
+ *                      use (the arrival counters; every call leaves them zero).
+ * Errors as wino_conv2d_f2x3_fwd_ws, per job, all checked before anything is launched;
+ * n <= 0 or jobs == NULL -> WINO_ERR_INVALID_ARG.
+ * wino_conv_multi_launches: kernel launches one such call makes (host only; -1 on bad input).
+ */
+typedef struct {
+    const float* x; /* (C,H,W,N) device */
+    const float* u; /* (C,4,4,K) device (wino_filter_transform) */
+    float* y;       /* (K,H,W,N) device */
+    int N, C, H, W, K;
+} wino_conv_job_t;
+size_t wino_conv_multi_workspace_bytes(const wino_conv_job_t* jobs, int n);
+wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, size_t ws_bytes,
+                                         wino_stream_t stream);
+int wino_conv_multi_launches(const wino_conv_job_t* jobs, int n);
+
+/*
  * Tensor-core variant (a5' of SURVEY 8(a)): the Winograd-domain GEMM (Eq. 7)
  * on the 5th-generation tensor cores (tcgen05.mma kind::tf32, accumulators in
  * TMEM).  The paper has no tensor-core path ("the data layout needs a

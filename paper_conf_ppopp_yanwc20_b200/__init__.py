@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused", "nonfused_launches",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half", "conv_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes", "filter_transform_multi",
+    "conv2d_half", "conv_workspace_bytes", "conv2d_multi", "conv_multi_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes", "filter_transform_multi",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -79,6 +79,12 @@ class Plan:
     smem_bytes: int
     launches: int
     stream_k: int = 0
+
+
+class _ConvJob(ctypes.Structure):
+    _fields_ = [("x", ctypes.c_void_p), ("u", ctypes.c_void_p), ("y", ctypes.c_void_p),
+                ("N", ctypes.c_int), ("C", ctypes.c_int), ("H", ctypes.c_int), ("W", ctypes.c_int),
+                ("K", ctypes.c_int)]
 
 
 def lib() -> ctypes.CDLL:
@@ -167,6 +173,13 @@ def lib() -> ctypes.CDLL:
         L.wino_conv_workspace_bytes.argtypes = [i, i, i, i, i]
         L.wino_conv2d_f2x3_fwd_ws.restype = i
         L.wino_conv2d_f2x3_fwd_ws.argtypes = [vp, vp, vp, i, i, i, i, i, i, i, i, vp, st, vp]
+    if hasattr(L, "wino_conv2d_f2x3_fwd_multi") or not os.environ.get("WINO_LIB_PATH"):
+        L.wino_conv_multi_workspace_bytes.restype = st
+        L.wino_conv_multi_workspace_bytes.argtypes = [ctypes.POINTER(_ConvJob), i]
+        L.wino_conv_multi_launches.restype = i
+        L.wino_conv_multi_launches.argtypes = [ctypes.POINTER(_ConvJob), i]
+        L.wino_conv2d_f2x3_fwd_multi.restype = i
+        L.wino_conv2d_f2x3_fwd_multi.argtypes = [ctypes.POINTER(_ConvJob), i, vp, st, vp]
     if hasattr(L, "wino_conv2d_f2x3_fwd_nchw_ws") or not os.environ.get("WINO_LIB_PATH"):
         L.wino_nchw_workspace_bytes.restype = st
         L.wino_nchw_workspace_bytes.argtypes = [i, i, i, i, i]
@@ -482,6 +495,53 @@ def conv2d(x: torch.Tensor, u: torch.Tensor, out: torch.Tensor | None = None, va
         else:
             _check(lib().wino_conv2d_f2x3_fwd(*args, _stream_ptr(stream)), "wino_conv2d_f2x3_fwd")
     return out
+
+
+def _conv_jobs(layers):
+    arr = (_ConvJob * len(layers))()
+    for i, (x, u, y) in enumerate(layers):
+        _need_cuda_f32(x, f"layer {i} x", 4)
+        _need_cuda_f32(u, f"layer {i} u", 4)
+        _need_cuda_f32(y, f"layer {i} y", 4)
+        _same_device(layers[0][0], x=x, u=u, y=y)
+        C, H, W, N = x.shape
+        K = u.shape[3]
+        if tuple(u.shape) != (C, 4, 4, K) or tuple(y.shape) != (K, H, W, N):
+            raise ValueError(f"layer {i}: x (C,H,W,N), u (C,4,4,K), y (K,H,W,N) expected")
+        arr[i] = _ConvJob(x.data_ptr(), u.data_ptr(), y.data_ptr(), N, C, H, W, K)
+    return arr
+
+
+def conv_multi_workspace_bytes(shapes) -> int:
+    """Workspace of conv2d_multi for [(N, C, H, W, K), ...] (wino_conv_multi_workspace_bytes)."""
+    arr = (_ConvJob * len(shapes))()
+    for i, (N, C, H, W, K) in enumerate(shapes):
+        arr[i] = _ConvJob(None, None, None, N, C, H, W, K)
+    return int(lib().wino_conv_multi_workspace_bytes(arr, len(shapes)))
+
+
+def conv_multi_launches(shapes) -> int:
+    """Kernel launches of one conv2d_multi call on [(N, C, H, W, K), ...] (wino_conv_multi_launches)."""
+    arr = (_ConvJob * len(shapes))()
+    for i, (N, C, H, W, K) in enumerate(shapes):
+        arr[i] = _ConvJob(None, None, None, N, C, H, W, K)
+    n = int(lib().wino_conv_multi_launches(arr, len(shapes)))
+    if n < 0:
+        raise WinoError(1, f"wino_conv_multi_launches {shapes}")
+    return n
+
+
+def conv2d_multi(layers, ws: torch.Tensor, stream=None) -> None:
+    """Several independent layers [(x (C,H,W,N), u (C,4,4,K), y (K,H,W,N)), ...]: the layers with
+    fewer than 32 tiles per SM share one persistent stream-K launch of the warp-specialised FP32
+    kernel per group of <= 4, the others run alone through the planner (wino_conv2d_f2x3_fwd_multi).
+    ws: a ZERO-FILLED CUDA byte buffer of >= conv_multi_workspace_bytes (calls leave it zeroed)."""
+    arr = _conv_jobs(layers)
+    _need_ws(ws, layers[0][0])
+    with torch.cuda.device(layers[0][0].device):
+        _check(lib().wino_conv2d_f2x3_fwd_multi(arr, len(layers), ctypes.c_void_p(ws.data_ptr()),
+                                                ws.numel() * ws.element_size(), _stream_ptr(stream)),
+               "wino_conv2d_f2x3_fwd_multi")
 
 
 def filter_transform_kcrs(w_kcrs: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:

@@ -18,6 +18,7 @@
 #include "ftf.cuh"
 #include "fused_fp32.cuh"
 #include "fused_fp32_ws.cuh"
+#include "fused_fp32_ml.cuh"
 #include "fused_tc.cuh"
 #include "fused_tc16.cuh"
 #include "fused_f4_fp32.cuh"
@@ -144,6 +145,12 @@ struct Fp32Plan {
 // arrival counter per CTA (zero between launches; see fused_fp32_ws.cuh).
 size_t sk_slot_bytes() { return size_t(wino::fp32::BK) * 4 * wino::fp32::BN * sizeof(float); }
 size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * sk_slot_bytes() + round_up256(size_t(ctas) * 4); }
+// The arrival counters sit after the slots of a FULL grid (one CTA per SM) whatever the grid of a
+// launch: a smaller grid's counters would otherwise land on slots that an earlier launch on the
+// same workspace left non-zero.
+unsigned* sk_flags_of(void* ws, int dev) {
+    return reinterpret_cast<unsigned*>(static_cast<char*>(ws) + 2 * sk_slot_bytes() * size_t(sm_count(dev)));
+}
 
 int log2_small(int s) { return s == 1 ? 0 : s == 2 ? 1 : s == 4 ? 2 : 3; }
 // planner cost of the stream-K plan beyond its units, in channel-block times: up to two partial
@@ -212,7 +219,7 @@ Fp32Plan plan_fp32(int N, int C, int H, int W, int K, bool u_tma_ok, int dev, in
     }
     if (p.sk) {
         p.split = 1;
-        p.grid = sms < 256 ? sms : 256;  // sk_fixup_kernel lists <= 256 segments per tile
+        p.grid = sms;  // one CTA per SM (the workspace holds 2 slots + a counter per SM)
         p.threads = wino::fp32ws::NT;
         p.smem = wino::fp32ws::Smem<false>::bytes;
         return p;
@@ -410,7 +417,7 @@ wino_status_t launch_fwd_fp32(const float* x_dev, const float* u_dev, int ldu, f
     if (pl.ws && pl.sk) {  // stream-K: equal unit ranges on every SM + fixup of the cut tiles
         prm.sk_ws = static_cast<float*>(ws);
         // 2 partial-tile slots per CTA, then one arrival counter per CTA (zero between launches)
-        prm.sk_flags = reinterpret_cast<unsigned*>(static_cast<char*>(ws) + 2 * sk_slot_bytes() * pl.grid);
+        prm.sk_flags = sk_flags_of(ws, dev);
         prm.sk_total = pl.tiles * prm.num_it;  // < 2^31 (planner)
         prm.sk_q = static_cast<int>(prm.sk_total / pl.grid);
         prm.sk_r = static_cast<int>(prm.sk_total % pl.grid);
@@ -746,6 +753,198 @@ wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, fl
     const int mode = sk == 0 ? 1 : (sk == 1 ? 0 : 2);  // API 0 auto / 1 off / 2 force -> planner 1 / 0 / 2
     return launch_fwd_fp32(x_dev, u_dev, K, y_dev, N, C, H, W, K, dev, reinterpret_cast<cudaStream_t>(stream), 0,
                            false, mode, ws_dev, ws_bytes);
+}
+
+size_t wino_conv_multi_workspace_bytes(const wino_conv_job_t* jobs, int n) {
+    if (!jobs || n <= 0) return 0;
+    for (int i = 0; i < n; ++i)
+        if (check_shape(jobs[i].N, jobs[i].C, jobs[i].H, jobs[i].W, jobs[i].K, 1, 1) != WINO_OK) return 0;
+    int dev = -1, sms = 148;
+    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+    else cudaGetLastError();
+    return sk_workspace_bytes(sms);
+}
+
+}  // extern "C"
+
+namespace {
+std::atomic<uint64_t> g_attr_ml;
+// Work model of the multi-layer cut, in units of one N % 32 == 0 channel block (~1.5 us of one
+// SM), fitted to per-CTA timelines of the ResNet step and its batch shards (scripts/ml_trace.py,
+// DESIGN.md 7.8): small-N box modes move x in 32/N boxes of N-float rows (N = 16 / 8 / 4: 1.07 /
+// 1.31 / 1.65 blocks), and each tile's 4-round OTF epilogue costs ~2 blocks (~3 us).
+constexpr double kMlEpiCost = 2.0;
+double ml_unit_cost(int xnb) { return xnb >= 32 ? 1.0 : (xnb == 16 ? 1.07 : (xnb == 8 ? 1.31 : 1.65)); }
+// A job joins the shared persistent launch when the warp-specialised kernel takes it (N % 32 == 0
+// or N in {4, 8, 16}; K % 4 == 0) and it has fewer than 32 tiles per SM; a layer that big fills
+// the GPU on its own and runs faster through the planner's one-tile-per-CTA grid (ResNet conv2 at
+// N = 256: 1136 vs 1162 us for the step, scripts/ml_ab.py).
+bool ml_shares_launch(const wino_conv_job_t& J, int sms) {
+    using namespace wino::fp32ml;
+    if (J.K % 4 != 0 || !(J.N % 32 == 0 || J.N == 4 || J.N == 8 || J.N == 16)) return false;
+    const long long nv = static_cast<long long>(J.N) * ((J.H + 1) / 2) * ((J.W + 1) / 2);
+    const long long tiles = ((nv + BN - 1) / BN) * ((J.K + BK - 1) / BK);
+    return tiles < 32LL * sms;
+}
+// Layers [0, n) of jobs (n <= 4, all warp-specialised eligible) in one multi-layer stream-K launch.
+wino_status_t launch_multi_fp32(const wino_conv_job_t* jobs, int n, void* ws, int dev, cudaStream_t st) {
+    using namespace wino::fp32ml;
+    Params prm;
+    std::memset(&prm, 0, sizeof(prm));
+    prm.nl = n;
+    long long units = 0;
+    double cu[MAX_LAYERS], per_tile[MAX_LAYERS], work0[MAX_LAYERS + 1];
+    work0[0] = 0.0;
+    for (int i = 0; i < n; ++i) {
+        const wino_conv_job_t& J = jobs[i];
+        Layer& L = prm.L[i];
+        L.y = J.y;
+        L.N = J.N;
+        L.C = J.C;
+        L.H = J.H;
+        L.W = J.W;
+        L.K = J.K;
+        L.TW = (J.W + 1) / 2;
+        L.NV = J.N * ((J.H + 1) / 2) * L.TW;
+        L.num_kb = (J.K + BK - 1) / BK;
+        L.num_it = (J.C + BC - 1) / BC;
+        const long long tiles = static_cast<long long>((L.NV + BN - 1) / BN) * L.num_kb;
+        L.xnb = J.N % 32 == 0 ? BN : J.N;
+        L.unit0 = static_cast<int>(units < 2147483647LL ? units : 0);
+        units += tiles * L.num_it;
+        cu[i] = ml_unit_cost(L.xnb);
+        per_tile[i] = L.num_it * cu[i] + kMlEpiCost;
+        work0[i + 1] = work0[i] + tiles * per_tile[i];
+        if (L.xnb < BN) {  // small N: (n, c, w, h) boxes + the conflict-free ITF map (as launch_fwd_fp32)
+            const int Q = L.xnb / 4;
+            for (int t = 0; t < 64; ++t) {
+                const int j = t / 8, ii = t % 8, b = ii / Q, h = ii % Q;
+                const int c = (b + j) % 8, n4 = b * L.xnb + 4 * h;
+                const int xoff = b * (BC * 16 * L.xnb) + c * L.xnb + 4 * h;
+                L.itf_map[t] = c | (n4 << 3) | (xoff << 8);
+            }
+            const cuuint64_t dims[4] = {cuuint64_t(J.N), cuuint64_t(J.C), cuuint64_t(J.W), cuuint64_t(J.H)};
+            const cuuint64_t strides[3] = {cuuint64_t(J.H) * J.W * J.N * 4, cuuint64_t(J.N) * 4,
+                                           cuuint64_t(J.W) * J.N * 4};
+            const cuuint32_t box[4] = {cuuint32_t(L.xnb), BC, 4, 4};
+            if (!encode_map(&L.tmx, J.x, 4, dims, box, strides)) return cuda_fail(cudaErrorInvalidValue);
+        } else {
+            const cuuint64_t dims[4] = {cuuint64_t(J.N), cuuint64_t(J.W), cuuint64_t(J.H), cuuint64_t(J.C)};
+            const cuuint32_t box[4] = {BN, 4, 4, BC};
+            if (!encode_map(&L.tmx, J.x, 4, dims, box)) return cuda_fail(cudaErrorInvalidValue);
+        }
+        const cuuint64_t udims[3] = {cuuint64_t(J.K), 16, cuuint64_t(J.C)};
+        const cuuint64_t ustrides[2] = {cuuint64_t(J.K) * 4, cuuint64_t(16) * J.K * 4};
+        const cuuint32_t ubox[3] = {BK, 16, BC};
+        if (!encode_map(&L.tmu, J.u, 3, udims, ubox, ustrides)) return cuda_fail(cudaErrorInvalidValue);
+    }
+    if (units >= 2147483647LL) return WINO_ERR_TOO_LARGE;
+    // one CTA per SM; CTA b starts at the first unit whose work position reaches b / grid of the
+    // total, then pushed up so that every range is non-empty
+    const int sms = sm_count(dev) < MAX_GRID ? sm_count(dev) : MAX_GRID;
+    const int grid = units < sms ? static_cast<int>(units) : sms;
+    const double total = work0[n];
+    for (int b = 0; b <= grid; ++b) {
+        long long u = static_cast<long long>(units);
+        if (b < grid) {
+            const double w = total * b / grid;
+            int i = 0;
+            while (i + 1 < n && work0[i + 1] <= w) ++i;
+            const Layer& L = prm.L[i];
+            const double local = w - work0[i];
+            const long long tile = static_cast<long long>(local / per_tile[i]);
+            long long g = static_cast<long long>(std::ceil((local - tile * per_tile[i]) / cu[i] - 1e-9));
+            if (g > L.num_it) g = L.num_it;
+            if (g < 0) g = 0;
+            u = L.unit0 + tile * L.num_it + g;
+        }
+        if (b > 0 && u <= prm.start[b - 1]) u = prm.start[b - 1] + 1;  // non-empty ranges
+        if (u > static_cast<long long>(units) - (grid - b)) u = static_cast<long long>(units) - (grid - b);
+        prm.start[b] = static_cast<int>(u);
+    }
+    prm.sk_ws = static_cast<float*>(ws);
+    prm.sk_flags = sk_flags_of(ws, dev);
+    const int smem = wino::fp32ml::SMEM_BYTES;
+    wino_status_t s = ensure_smem_attr(fused_fp32_ml_kernel, dev, smem, g_attr_ml);
+    if (s != WINO_OK) return s;
+    fused_fp32_ml_kernel<<<dim3(static_cast<unsigned>(grid)), wino::fp32ws::NT, smem, st>>>(prm);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+}  // namespace
+
+extern "C" {
+
+wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, size_t ws_bytes,
+                                         wino_stream_t stream) {
+    if (!jobs || n <= 0 || !ws_dev) return WINO_ERR_INVALID_ARG;
+    if (!aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
+    for (int i = 0; i < n; ++i) {
+        const wino_conv_job_t& J = jobs[i];
+        if (!J.x || !J.u || !J.y) return WINO_ERR_INVALID_ARG;
+        wino_status_t s = check_shape(J.N, J.C, J.H, J.W, J.K, 1, 1);
+        if (s != WINO_OK) return s;
+        if (!aligned16(J.x) || !aligned16(J.u) || !aligned16(J.y)) return WINO_ERR_MISALIGNED;
+    }
+    for (int i = 0; i < n; ++i) {  // outputs overlap nothing else; the workspace overlaps nothing
+        const wino_conv_job_t& A = jobs[i];
+        const size_t hwn = size_t(A.H) * A.W * A.N;
+        const size_t yb = size_t(A.K) * hwn * 4, xb = size_t(A.C) * hwn * 4, ub = size_t(16) * A.C * A.K * 4;
+        if (overlaps(ws_dev, ws_bytes, A.x, xb) || overlaps(ws_dev, ws_bytes, A.u, ub) ||
+            overlaps(ws_dev, ws_bytes, A.y, yb))
+            return WINO_ERR_INVALID_ARG;
+        for (int j = 0; j < n; ++j) {
+            const wino_conv_job_t& B = jobs[j];
+            const size_t hwn_b = size_t(B.H) * B.W * B.N;
+            if (overlaps(A.y, yb, B.x, size_t(B.C) * hwn_b * 4) || overlaps(A.y, yb, B.u, size_t(16) * B.C * B.K * 4))
+                return WINO_ERR_INVALID_ARG;
+            if (j != i && overlaps(A.y, yb, B.y, size_t(B.K) * hwn_b * 4)) return WINO_ERR_INVALID_ARG;
+        }
+    }
+    int dev;
+    wino_status_t s = check_device(&dev);
+    if (s != WINO_OK) return s;
+    if (ws_bytes < sk_workspace_bytes(sm_count(dev))) return WINO_ERR_INVALID_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const int sms = sm_count(dev);
+    wino_conv_job_t group[wino::fp32ml::MAX_LAYERS];
+    int m = 0;
+    for (int i = 0; i <= n; ++i) {
+        const bool flush = i == n || (m == wino::fp32ml::MAX_LAYERS);
+        if (flush && m > 0) {  // one persistent launch for the collected layers
+            if ((s = launch_multi_fp32(group, m, ws_dev, dev, st)) != WINO_OK) return s;
+            m = 0;
+        }
+        if (i == n) break;
+        const wino_conv_job_t& J = jobs[i];
+        if (ml_shares_launch(J, sms)) {
+            group[m++] = J;
+        } else if ((s = launch_fwd_fp32(J.x, J.u, J.K, J.y, J.N, J.C, J.H, J.W, J.K, dev, st, 0, false, 1, ws_dev,
+                                        ws_bytes)) != WINO_OK) {
+            return s;
+        }
+    }
+    return WINO_OK;
+}
+
+int wino_conv_multi_launches(const wino_conv_job_t* jobs, int n) {
+    if (!jobs || n <= 0) return -1;
+    int dev = -1, sms = 148;
+    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+    else cudaGetLastError();
+    int launches = 0, m = 0;
+    for (int i = 0; i < n; ++i) {
+        const wino_conv_job_t& J = jobs[i];
+        if (ml_shares_launch(J, sms)) {
+            if (m == 0) ++launches;
+            m = (m + 1) % wino::fp32ml::MAX_LAYERS;
+        } else {
+            wino_plan_t pl;
+            if (wino_plan(J.N, J.C, J.H, J.W, J.K, 4, &pl) != WINO_OK) return -1;
+            launches += pl.launches;
+        }
+    }
+    return launches;
 }
 
 wino_status_t wino_filter_transform_kcrs(const float* w_kcrs_dev, float* u_dev, int C, int K, wino_stream_t stream) {

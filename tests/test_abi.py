@@ -200,6 +200,26 @@ def test_stream_k_plan_and_workspace():
     assert wino.conv_workspace_bytes(0, 1, 1, 1, 1) == 0
 
 
+def test_multi_layer_launch_grouping():
+    """Host-only (148 SMs without a device): wino_conv2d_f2x3_fwd_multi puts the layers with fewer
+    than 32 tiles per SM into one shared persistent launch per group of <= 4 and runs the others
+    alone through the planner.  ResNet step: conv2_x at N = 256 (6272 tiles = 42 per SM) alone, the
+    other three shared -> 2 launches; any batch shard (P >= 2) -> all four shared, 1 launch."""
+    names = ("conv5_x", "conv4_x", "conv3_x", "conv2_x")
+    for P, want in ((1, 2), (2, 1), (4, 1), (8, 1)):
+        shapes = [(CONFIGS[n].N // P, CONFIGS[n].C, CONFIGS[n].H, CONFIGS[n].W, CONFIGS[n].K) for n in names]
+        assert wino.conv_multi_launches(shapes) == want, P
+        assert wino.conv_multi_workspace_bytes(shapes) == 148 * 2 * 64 * 4 * 32 * 4 + 768
+    small = (32, 64, 9, 9, 64)
+    assert wino.conv_multi_launches([small] * 4) == 1
+    assert wino.conv_multi_launches([small] * 5) == 2  # groups of at most 4
+    odd = (3, 16, 8, 8, 16)  # N = 3: not warp-specialised -> its own plan (one launch)
+    assert wino.conv_multi_launches([small, odd, small]) == 1 + wino.plan(*odd[:4], odd[4], variant=4).launches
+    assert wino.conv_multi_launches([(8, 16, 8, 8, 18)]) == 1  # K % 4 != 0: planner, 1 launch
+    with pytest.raises(wino.WinoError):
+        wino.conv_multi_launches([(0, 1, 1, 1, 1)])
+
+
 def test_tensor_core_stream_k_plans_and_workspaces():
     """Host-only planning: the 16-bit and TF32 tcgen05 kernels take stream-K only for tile-starved
     shapes (conv5_x: 64 tiles of 128 x 32 for 148 SMs), never for the many-tile layers, with either
