@@ -262,13 +262,20 @@ wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, fl
  * and each CTA has at most two cut tiles (reduced inside the kernel as in
  * wino_conv2d_f2x3_fwd_ws).  Any other layer runs alone through wino_conv2d_f2x3_fwd_ws's
  * planner (sk = 0).  Same arithmetic per output as wino_conv2d_f2x3_fwd_ws (equal up to FP32
- * summation order of cut tiles; bit-identical on small-integer inputs).  Launches go to `stream`
- * in job order.
+ * summation order of cut tiles; bit-identical on small-integer inputs).  Batch shards with N = 4
+ * or 8 do not load x through 32/N TMA boxes of N-float rows: a separate input-transform kernel writes
+ * their V = B^T d B (Eq. 6, same arithmetic as the fused ITF, so bit-identical) into the workspace
+ * and the fused kernel loads V tiles directly ("vmode").  Launches go to `stream`: first the
+ * input transforms (they read x only), then -- when `u_ready` is not NULL -- a wait on that
+ * cudaEvent_t (e.g. recorded after the filter transform on another stream, so both overlap),
+ * then the convolutions.
  *   jobs[i]          : device pointers and shape of layer i; y of a job must not overlap any
  *                      job's x, u or y; 1 <= n.
- *   ws_dev / ws_bytes: >= wino_conv_multi_workspace_bytes(jobs, n) (= wino_conv_workspace_bytes),
- *                      16-byte aligned, not overlapping any tensor, ZERO-FILLED before its first
- *                      use (the arrival counters; every call leaves them zero).
+ *   ws_dev / ws_bytes: >= wino_conv_multi_workspace_bytes(jobs, n) (the stream-K slots and
+ *                      counters of wino_conv_workspace_bytes, plus 16 x C x NV floats per vmode
+ *                      layer), 16-byte aligned, not overlapping any tensor, ZERO-FILLED before
+ *                      its first use (the arrival counters; every call leaves them zero).
+ *   u_ready          : NULL, or a cudaEvent_t the convolutions wait for (not the input transforms).
  * Errors as wino_conv2d_f2x3_fwd_ws, per job, all checked before anything is launched;
  * n <= 0 or jobs == NULL -> WINO_ERR_INVALID_ARG.
  * wino_conv_multi_launches: kernel launches one such call makes (host only; -1 on bad input).
@@ -281,7 +288,7 @@ typedef struct {
 } wino_conv_job_t;
 size_t wino_conv_multi_workspace_bytes(const wino_conv_job_t* jobs, int n);
 wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, size_t ws_bytes,
-                                         wino_stream_t stream);
+                                         void* u_ready, wino_stream_t stream);
 int wino_conv_multi_launches(const wino_conv_job_t* jobs, int n);
 
 /*

@@ -179,7 +179,7 @@ def lib() -> ctypes.CDLL:
         L.wino_conv_multi_launches.restype = i
         L.wino_conv_multi_launches.argtypes = [ctypes.POINTER(_ConvJob), i]
         L.wino_conv2d_f2x3_fwd_multi.restype = i
-        L.wino_conv2d_f2x3_fwd_multi.argtypes = [ctypes.POINTER(_ConvJob), i, vp, st, vp]
+        L.wino_conv2d_f2x3_fwd_multi.argtypes = [ctypes.POINTER(_ConvJob), i, vp, st, vp, vp]
     if hasattr(L, "wino_conv2d_f2x3_fwd_nchw_ws") or not os.environ.get("WINO_LIB_PATH"):
         L.wino_nchw_workspace_bytes.restype = st
         L.wino_nchw_workspace_bytes.argtypes = [i, i, i, i, i]
@@ -531,16 +531,19 @@ def conv_multi_launches(shapes) -> int:
     return n
 
 
-def conv2d_multi(layers, ws: torch.Tensor, stream=None) -> None:
+def conv2d_multi(layers, ws: torch.Tensor, stream=None, u_ready: torch.cuda.Event | None = None) -> None:
     """Several independent layers [(x (C,H,W,N), u (C,4,4,K), y (K,H,W,N)), ...]: the layers with
     fewer than 32 tiles per SM share one persistent stream-K launch of the warp-specialised FP32
     kernel per group of <= 4, the others run alone through the planner (wino_conv2d_f2x3_fwd_multi).
-    ws: a ZERO-FILLED CUDA byte buffer of >= conv_multi_workspace_bytes (calls leave it zeroed)."""
+    ws: a ZERO-FILLED CUDA byte buffer of >= conv_multi_workspace_bytes (calls leave it zeroed).
+    u_ready: an event the convolutions wait for (the x-only input transforms of N = 4 / 8 layers
+    are queued before the wait), e.g. recorded after filter_transform_multi on another stream."""
     arr = _conv_jobs(layers)
     _need_ws(ws, layers[0][0])
+    ev = ctypes.c_void_p(u_ready.cuda_event) if u_ready is not None else None
     with torch.cuda.device(layers[0][0].device):
         _check(lib().wino_conv2d_f2x3_fwd_multi(arr, len(layers), ctypes.c_void_p(ws.data_ptr()),
-                                                ws.numel() * ws.element_size(), _stream_ptr(stream)),
+                                                ws.numel() * ws.element_size(), ev, _stream_ptr(stream)),
                "wino_conv2d_f2x3_fwd_multi")
 
 

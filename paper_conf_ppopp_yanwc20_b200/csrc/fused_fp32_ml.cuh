@@ -62,10 +62,12 @@ constexpr int MAX_GRID = 160;  // CTAs of one launch (B200: 148 SMs, one CTA eac
 struct __align__(64) Layer {
     CUtensorMap tmx;  // x: (N, W, H, C) box (32, 4, 4, 8) when N % 32 == 0, else (n, c, w, h) box (N, 8, 4, 4)
     CUtensorMap tmu;  // u: (K, 16, C) box (64, 16, 8)
+    CUtensorMap tmv;  // vmode: V = B^T d B of every tile, (NV, C, 16) box (32, 8, 16) -> the V ring as is
     float* __restrict__ y;
     int N, C, H, W, K;
     int TW, NV, num_kb, num_it, xnb;
     int unit0;         // global index of the layer's first unit (tile * num_it + g)
+    int vmode;         // 1: V comes transformed from ml_itf_kernel (small N), the ITF warps idle
     int itf_map[64];   // N | 32: ITF task map of the 64 ITF lanes (as fp32::Params::itf_map)
 };
 
@@ -201,6 +203,59 @@ __device__ __noinline__ void ml_arrive(const Params& p, int l, int t0, int k0, i
     }
 }
 
+// Input transform of the vmode layers ahead of the fused launch (Sec. 4.2's ITF, Eq. 6, with the
+// expression tree of itf_4x4 so V is bit-identical to the ITF warps'): thread (row r of V, c, 4
+// consecutive nu) reads the two rows of its 4x4 patch that row r of B^T combines, as float4 along n
+// (N % 4 == 0; zero outside the image = the implicit padding of Sec. 3.5), and writes
+// V[4r..4r+3][c][nu..nu+3] as float4 -- a warp stores 512 contiguous bytes per xi.
+struct ItfJob {
+    const float* __restrict__ x;
+    float* __restrict__ v;
+    int N, C, H, W, TW, NV;
+    int first;  // first thread index of this job (C * NV / 4 threads per V row, blockIdx.y = row)
+};
+struct ItfJobs {
+    ItfJob j[MAX_LAYERS];
+    int n;
+    int total;
+};
+
+__global__ void __launch_bounds__(256) ml_itf_kernel(const __grid_constant__ ItfJobs p) {
+    const int row = blockIdx.y;  // row of V = B^T row: (d[i0] - d[i1]) for rows 0, 2, 3, (d[i0] + d[i1]) for row 1
+    const int i0 = row == 0 ? 0 : (row == 2 ? 2 : 1), i1 = row == 0 ? 2 : (row == 2 ? 1 : (row == 1 ? 2 : 3));
+    for (int i = blockIdx.x * 256 + threadIdx.x; i < p.total; i += gridDim.x * 256) {
+        int a = 0;
+        while (a + 1 < p.n && p.j[a + 1].first <= i) ++a;
+        const ItfJob& J = p.j[a];
+        const int nq = J.NV >> 2, r = i - J.first;
+        const int c = r / nq, nu = 4 * (r - c * nq);
+        const int t = nu / J.N, n = nu - t * J.N;
+        const int th = t / J.TW, tw = t - th * J.TW;
+        const int ha = 2 * th - 1 + i0, hb = 2 * th - 1 + i1, w0 = 2 * tw - 1;
+        const float* xa = J.x + ((c * J.H + ha) * J.W + w0) * J.N + n;  // < 2^31 floats (kMaxElems)
+        const float* xb = xa + (i1 - i0) * J.W * J.N;
+        const bool oka = ha >= 0 && ha < J.H, okb = hb >= 0 && hb < J.H;
+        float4 tr[4];  // row `row` of B^T d
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const bool okw = w0 + j >= 0 && w0 + j < J.W;
+            float4 d0 = make_float4(0.f, 0.f, 0.f, 0.f), d1 = d0;
+            if (okw && oka) d0 = __ldg(reinterpret_cast<const float4*>(xa + j * J.N));
+            if (okw && okb) d1 = __ldg(reinterpret_cast<const float4*>(xb + j * J.N));
+            tr[j] = row == 1 ? make_float4(d0.x + d1.x, d0.y + d1.y, d0.z + d1.z, d0.w + d1.w)
+                             : make_float4(d0.x - d1.x, d0.y - d1.y, d0.z - d1.z, d0.w - d1.w);
+        }
+        auto sub = [](float4 u, float4 w) { return make_float4(u.x - w.x, u.y - w.y, u.z - w.z, u.w - w.w); };
+        auto add = [](float4 u, float4 w) { return make_float4(u.x + w.x, u.y + w.y, u.z + w.z, u.w + w.w); };
+        const size_t plane = static_cast<size_t>(J.C) * J.NV;
+        float* vo = J.v + 4 * row * plane + static_cast<size_t>(c) * J.NV + nu;
+        __stcg(reinterpret_cast<float4*>(vo), sub(tr[0], tr[2]));
+        __stcg(reinterpret_cast<float4*>(vo + plane), add(tr[1], tr[2]));
+        __stcg(reinterpret_cast<float4*>(vo + 2 * plane), sub(tr[2], tr[1]));
+        __stcg(reinterpret_cast<float4*>(vo + 3 * plane), sub(tr[1], tr[3]));
+    }
+}
+
 #ifdef WINO_WS_CTATRACE
 #define ML_CT(e, v) do { if (blockIdx.x < 256) fp32ws::g_cta_trace[blockIdx.x][e] = (v); } while (0)
 #else
@@ -225,7 +280,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
 
     if (tid == 0) {
         for (int l = 0; l < p.nl; ++l) {
-            tma_prefetch_desc(&p.L[l].tmx);
+            tma_prefetch_desc(p.L[l].vmode ? &p.L[l].tmv : &p.L[l].tmx);
             tma_prefetch_desc(&p.L[l].tmu);
         }
         for (int s = 0; s < S; ++s) {
@@ -260,6 +315,20 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                     const int t0 = nu0 / L.N, n0 = nu0 - t0 * L.N;
                     const bool box32 = L.xnb == BN;
                     const int nbox = box32 ? 1 : BN / L.xnb;
+                    if (L.vmode) {  // u into the stage, V (16 KB, 128 B rows) straight into the V ring
+                        for (int g = g_lo; g < g_hi; ++g, ++G) {
+                            const int slot = G % S, vb = G % SV;
+                            if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
+                            float* us = smem + slot * STAGE_FLOATS;
+                            mbar_arrive_expect_tx(&full[slot], US_FLOATS * 4);
+                            tma_load_3d(us, &L.tmu, &full[slot], k0, 0, g * BC);
+                            if (G >= SV) mbar_wait(&vempty[vb], ((G / SV) - 1) & 1);
+                            mbar_arrive_expect_tx(&vfull[vb], VS_FLOATS * 4);
+                            tma_load_3d(vs + vb * VS_FLOATS, &L.tmv, &vfull[vb], nu0, g * BC, 0);
+                            mbar_arrive(&vfull[vb]);  // vfull counts ITF_WARPS = 2 arrivals
+                        }
+                        continue;
+                    }
                     for (int g = g_lo; g < g_hi; ++g, ++G) {
                         const int slot = G % S;
                         if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
@@ -292,6 +361,14 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
             const int4 r = rec[pi % PR];
             const int u0 = r.x, u1 = r.y;
             const Layer& L = p.L[r.z];
+            if (L.vmode) {  // no raw x: only keep the stage hand-off (the producer waits on our arrival)
+                for (int g = u0; g < u1; ++g, ++G) {
+                    mbar_wait(&full[G % S], (G / S) & 1);
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&empty[G % S]);
+                }
+                continue;
+            }
             int c, n4, xoff, xpos;
             if (L.xnb == BN) {
                 c = 4 * (warp - 9) + (lane >> 3);

@@ -13,6 +13,7 @@
 #include <cstring>
 #include <mutex>
 #include <new>
+#include <vector>
 
 #include "../../include/wino.h"
 #include "ftf.cuh"
@@ -755,16 +756,6 @@ wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, fl
                            false, mode, ws_dev, ws_bytes);
 }
 
-size_t wino_conv_multi_workspace_bytes(const wino_conv_job_t* jobs, int n) {
-    if (!jobs || n <= 0) return 0;
-    for (int i = 0; i < n; ++i)
-        if (check_shape(jobs[i].N, jobs[i].C, jobs[i].H, jobs[i].W, jobs[i].K, 1, 1) != WINO_OK) return 0;
-    int dev = -1, sms = 148;
-    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
-    else cudaGetLastError();
-    return sk_workspace_bytes(sms);
-}
-
 }  // extern "C"
 
 namespace {
@@ -774,7 +765,9 @@ std::atomic<uint64_t> g_attr_ml;
 // DESIGN.md 7.8): small-N box modes move x in 32/N boxes of N-float rows (N = 16 / 8 / 4: 1.07 /
 // 1.31 / 1.65 blocks), and each tile's 4-round OTF epilogue costs ~2 blocks (~3 us).
 constexpr double kMlEpiCost = 2.0;
-double ml_unit_cost(int xnb) { return xnb >= 32 ? 1.0 : (xnb == 16 ? 1.07 : (xnb == 8 ? 1.31 : 1.65)); }
+double ml_unit_cost(int xnb, bool vmode) {
+    return vmode ? 0.92 : (xnb >= 32 ? 1.0 : (xnb == 16 ? 1.07 : (xnb == 8 ? 1.31 : 1.65)));
+}
 // A job joins the shared persistent launch when the warp-specialised kernel takes it (N % 32 == 0
 // or N in {4, 8, 16}; K % 4 == 0) and it has fewer than 32 tiles per SM; a layer that big fills
 // the GPU on its own and runs faster through the planner's one-tile-per-CTA grid (ResNet conv2 at
@@ -786,12 +779,57 @@ bool ml_shares_launch(const wino_conv_job_t& J, int sms) {
     const long long tiles = ((nv + BN - 1) / BN) * ((J.K + BK - 1) / BK);
     return tiles < 32LL * sms;
 }
-// Layers [0, n) of jobs (n <= 4, all warp-specialised eligible) in one multi-layer stream-K launch.
-wino_status_t launch_multi_fp32(const wino_conv_job_t* jobs, int n, void* ws, int dev, cudaStream_t st) {
+// vmode (N = 4, 8): the small-N x boxes (rows of 16 / 32 B, 8 / 4 TMA boxes per stage) cost a
+// shared layer 1.65 / 1.31 channel-block times; instead ml_itf_kernel transforms the (small) x into
+// V once per call and the fused kernel loads V tiles with one 16 KB box of 128 B rows per stage.
+#ifndef WINO_ML_VMODE_MAX_N  // A/B builds only (scripts/ml_ab.py)
+#define WINO_ML_VMODE_MAX_N 8
+#endif
+constexpr int kMlVModeMaxN = WINO_ML_VMODE_MAX_N;
+bool ml_vmode(const wino_conv_job_t& J) { return J.N % 32 != 0 && J.N <= kMlVModeMaxN; }
+size_t ml_v_bytes(const wino_conv_job_t& J) {
+    const size_t nv = size_t(J.N) * ((J.H + 1) / 2) * ((J.W + 1) / 2);
+    return round_up256(size_t(16) * J.C * nv * 4);
+}
+size_t ml_multi_ws_bytes(const wino_conv_job_t* jobs, int n, int sms) {
+    size_t b = sk_workspace_bytes(sms);
+    for (int i = 0; i < n; ++i)
+        if (ml_shares_launch(jobs[i], sms) && ml_vmode(jobs[i])) b += ml_v_bytes(jobs[i]);
+    return b;
+}
+}  // namespace
+
+extern "C" {
+
+size_t wino_conv_multi_workspace_bytes(const wino_conv_job_t* jobs, int n) {
+    if (!jobs || n <= 0) return 0;
+    for (int i = 0; i < n; ++i)
+        if (check_shape(jobs[i].N, jobs[i].C, jobs[i].H, jobs[i].W, jobs[i].K, 1, 1) != WINO_OK) return 0;
+    int dev = -1, sms = 148;
+    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
+    else cudaGetLastError();
+    return ml_multi_ws_bytes(jobs, n, sms);
+}
+
+}  // extern "C"
+
+namespace {
+// One multi-layer stream-K launch (and its vmode input transform), prepared on the host.
+struct MlLaunch {
+    wino::fp32ml::Params prm;
+    wino::fp32ml::ItfJobs itf;
+    int grid;
+};
+// Layers [0, n) of jobs (n <= 4, all warp-specialised eligible) as one multi-layer launch; vbuf[i]:
+// the V buffer of a vmode layer (else unused).  Nothing is queued.
+wino_status_t prepare_multi_fp32(const wino_conv_job_t* jobs, float* const* vbuf, int n, void* ws, int dev,
+                                 MlLaunch& out) {
     using namespace wino::fp32ml;
-    Params prm;
+    Params& prm = out.prm;
     std::memset(&prm, 0, sizeof(prm));
     prm.nl = n;
+    ItfJobs& itf = out.itf;
+    std::memset(&itf, 0, sizeof(itf));
     long long units = 0;
     double cu[MAX_LAYERS], per_tile[MAX_LAYERS], work0[MAX_LAYERS + 1];
     work0[0] = 0.0;
@@ -812,10 +850,27 @@ wino_status_t launch_multi_fp32(const wino_conv_job_t* jobs, int n, void* ws, in
         L.xnb = J.N % 32 == 0 ? BN : J.N;
         L.unit0 = static_cast<int>(units < 2147483647LL ? units : 0);
         units += tiles * L.num_it;
-        cu[i] = ml_unit_cost(L.xnb);
+        L.vmode = ml_vmode(J) ? 1 : 0;
+        cu[i] = ml_unit_cost(L.xnb, L.vmode);
         per_tile[i] = L.num_it * cu[i] + kMlEpiCost;
         work0[i + 1] = work0[i] + tiles * per_tile[i];
-        if (L.xnb < BN) {  // small N: (n, c, w, h) boxes + the conflict-free ITF map (as launch_fwd_fp32)
+        if (L.vmode) {  // V[xi][c][nu] from ml_itf_kernel: (NV, C, 16) box (32, 8, 16) = the V ring slot
+            ItfJob& T = itf.j[itf.n++];
+            T.x = J.x;
+            T.v = vbuf[i];
+            T.N = J.N;
+            T.C = J.C;
+            T.H = J.H;
+            T.W = J.W;
+            T.TW = L.TW;
+            T.NV = L.NV;
+            T.first = itf.total;
+            itf.total += J.C * (L.NV / 4);  // < 2^31: C * NV <= C * H * W * N <= kMaxElems
+            const cuuint64_t dims[3] = {cuuint64_t(L.NV), cuuint64_t(J.C), 16};
+            const cuuint64_t strides[2] = {cuuint64_t(L.NV) * 4, cuuint64_t(J.C) * L.NV * 4};
+            const cuuint32_t box[3] = {BN, BC, 16};
+            if (!encode_map(&L.tmv, vbuf[i], 3, dims, box, strides)) return cuda_fail(cudaErrorInvalidValue);
+        } else if (L.xnb < BN) {  // small N: (n, c, w, h) boxes + the conflict-free ITF map (as launch_fwd_fp32)
             const int Q = L.xnb / 4;
             for (int t = 0; t < 64; ++t) {
                 const int j = t / 8, ii = t % 8, b = ii / Q, h = ii % Q;
@@ -864,10 +919,23 @@ wino_status_t launch_multi_fp32(const wino_conv_job_t* jobs, int n, void* ws, in
     }
     prm.sk_ws = static_cast<float*>(ws);
     prm.sk_flags = sk_flags_of(ws, dev);
+    out.grid = grid;
+    return WINO_OK;
+}
+// the vmode input transform of a prepared launch (reads x only)
+wino_status_t launch_ml_itf(const MlLaunch& L, int dev, cudaStream_t st) {
+    if (L.itf.n == 0) return WINO_OK;
+    int blocks = (L.itf.total + 255) / 256;
+    if (blocks > 2 * sm_count(dev)) blocks = 2 * sm_count(dev);
+    wino::fp32ml::ml_itf_kernel<<<dim3(static_cast<unsigned>(blocks), 4), 256, 0, st>>>(L.itf);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? WINO_OK : cuda_fail(e);
+}
+wino_status_t launch_ml(const MlLaunch& L, int dev, cudaStream_t st) {
     const int smem = wino::fp32ml::SMEM_BYTES;
-    wino_status_t s = ensure_smem_attr(fused_fp32_ml_kernel, dev, smem, g_attr_ml);
+    wino_status_t s = ensure_smem_attr(wino::fp32ml::fused_fp32_ml_kernel, dev, smem, g_attr_ml);
     if (s != WINO_OK) return s;
-    fused_fp32_ml_kernel<<<dim3(static_cast<unsigned>(grid)), wino::fp32ws::NT, smem, st>>>(prm);
+    wino::fp32ml::fused_fp32_ml_kernel<<<dim3(static_cast<unsigned>(L.grid)), wino::fp32ws::NT, smem, st>>>(L.prm);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
@@ -876,7 +944,7 @@ wino_status_t launch_multi_fp32(const wino_conv_job_t* jobs, int n, void* ws, in
 extern "C" {
 
 wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, size_t ws_bytes,
-                                         wino_stream_t stream) {
+                                         void* u_ready, wino_stream_t stream) {
     if (!jobs || n <= 0 || !ws_dev) return WINO_ERR_INVALID_ARG;
     if (!aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
     for (int i = 0; i < n; ++i) {
@@ -904,25 +972,49 @@ wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, voi
     int dev;
     wino_status_t s = check_device(&dev);
     if (s != WINO_OK) return s;
-    if (ws_bytes < sk_workspace_bytes(sm_count(dev))) return WINO_ERR_INVALID_ARG;
-    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     const int sms = sm_count(dev);
+    if (ws_bytes < ml_multi_ws_bytes(jobs, n, sms)) return WINO_ERR_INVALID_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    // 1. plan every shared launch (groups of <= 4 in job order); the other jobs run alone
     wino_conv_job_t group[wino::fp32ml::MAX_LAYERS];
+    float* vbuf[wino::fp32ml::MAX_LAYERS];
+    char* vnext = static_cast<char*>(ws_dev) + sk_workspace_bytes(sms);  // V buffers of vmode layers
+    std::vector<MlLaunch> ml;
+    std::vector<int> alone;
     int m = 0;
     for (int i = 0; i <= n; ++i) {
-        const bool flush = i == n || (m == wino::fp32ml::MAX_LAYERS);
-        if (flush && m > 0) {  // one persistent launch for the collected layers
-            if ((s = launch_multi_fp32(group, m, ws_dev, dev, st)) != WINO_OK) return s;
+        if ((i == n || m == wino::fp32ml::MAX_LAYERS) && m > 0) {
+            ml.emplace_back();
+            if ((s = prepare_multi_fp32(group, vbuf, m, ws_dev, dev, ml.back())) != WINO_OK) return s;
             m = 0;
         }
         if (i == n) break;
         const wino_conv_job_t& J = jobs[i];
         if (ml_shares_launch(J, sms)) {
+            vbuf[m] = nullptr;
+            if (ml_vmode(J)) {
+                vbuf[m] = reinterpret_cast<float*>(vnext);
+                vnext += ml_v_bytes(J);
+            }
             group[m++] = J;
-        } else if ((s = launch_fwd_fp32(J.x, J.u, J.K, J.y, J.N, J.C, J.H, J.W, J.K, dev, st, 0, false, 1, ws_dev,
-                                        ws_bytes)) != WINO_OK) {
-            return s;
+        } else {
+            alone.push_back(i);
         }
+    }
+    // 2. work that reads x only (the vmode input transforms), then wait for u, then the convolutions
+    for (const MlLaunch& L : ml)
+        if ((s = launch_ml_itf(L, dev, st)) != WINO_OK) return s;
+    if (u_ready) {
+        cudaError_t e = cudaStreamWaitEvent(st, static_cast<cudaEvent_t>(u_ready), 0);
+        if (e != cudaSuccess) return cuda_fail(e);
+    }
+    for (const MlLaunch& L : ml)
+        if ((s = launch_ml(L, dev, st)) != WINO_OK) return s;
+    for (int i : alone) {
+        const wino_conv_job_t& J = jobs[i];
+        if ((s = launch_fwd_fp32(J.x, J.u, J.K, J.y, J.N, J.C, J.H, J.W, J.K, dev, st, 0, false, 1, ws_dev,
+                                 ws_bytes)) != WINO_OK)
+            return s;
     }
     return WINO_OK;
 }
@@ -933,10 +1025,18 @@ int wino_conv_multi_launches(const wino_conv_job_t* jobs, int n) {
     if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
     else cudaGetLastError();
     int launches = 0, m = 0;
+    bool group_v = false;  // the current group has a vmode layer (+ one ml_itf_kernel launch)
     for (int i = 0; i < n; ++i) {
         const wino_conv_job_t& J = jobs[i];
         if (ml_shares_launch(J, sms)) {
-            if (m == 0) ++launches;
+            if (m == 0) {
+                launches += 1;
+                group_v = false;
+            }
+            if (ml_vmode(J) && !group_v) {
+                launches += 1;
+                group_v = true;
+            }
             m = (m + 1) % wino::fp32ml::MAX_LAYERS;
         } else {
             wino_plan_t pl;

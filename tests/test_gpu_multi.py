@@ -134,6 +134,29 @@ def test_argument_errors(wino):
     with pytest.raises(wino.WinoError, match="INVALID_ARG"):  # y of one job is another job's x
         wino.conv2d_multi([(x, u, y), (y[:cfg.C], u, y2)], ws)
     L = wino.lib()
-    assert L.wino_conv2d_f2x3_fwd_multi(None, 1, ctypes.c_void_p(ws.data_ptr()), ws.numel(), None) == 1
+    assert L.wino_conv2d_f2x3_fwd_multi(None, 1, ctypes.c_void_p(ws.data_ptr()), ws.numel(), None, None) == 1
     wino.conv2d_multi([(x, u, y), (x, u, y2)], ws)  # shared inputs are fine
     torch.cuda.synchronize()
+
+
+def test_u_ready_event_orders_the_convolutions(wino):
+    """FTF on a side stream, convolutions on the main stream ordered only by the u_ready event
+    (the N = 4 / 8 input transforms are queued before the wait): every element as the oracle."""
+    cfgs = [c.with_batch(c.N // 8) for c in RESNET]  # N = 4, 8, 16, 32: two vmode layers
+    main, side = torch.cuda.current_stream(), torch.cuda.Stream()
+    data, layers, ws_list = [], [], []
+    for i, cfg in enumerate(cfgs):
+        x, w = make_inputs(cfg, kind="smallint", seed_x=500 + i, seed_w=600 + i)
+        data.append((x, w))
+        layers.append((x.to(DEV), torch.full((cfg.C, 4, 4, cfg.K), float("nan"), device=DEV),
+                       torch.full((cfg.K, cfg.H, cfg.W, cfg.N), float("nan"), device=DEV), w.to(DEV)))
+    ws = torch.zeros(wino.conv_multi_workspace_bytes([(c.N, c.C, c.H, c.W, c.K) for c in cfgs]),
+                     dtype=torch.uint8, device=DEV)
+    torch.cuda.synchronize()
+    side.wait_stream(main)
+    wino.filter_transform_multi([(wd, u) for _, u, _, wd in layers], stream=side)
+    ev = torch.cuda.Event()
+    ev.record(side)
+    wino.conv2d_multi([(x, u, y) for x, u, y, _ in layers], ws, u_ready=ev)
+    torch.cuda.synchronize()
+    _check(data, [y.cpu().double().numpy() for _, _, y, _ in layers], "smallint")
