@@ -301,7 +301,7 @@ def _config(args, layers, world):
         "l2": "headline: flushed before every timed step by a 512 MiB write + 256 MiB read (outside the events); "
               "hot_l2: the paper's protocol (L863), 5 repeats x 20 back-to-back replays, median of the means",
         "step": ("fp32: all layers' FTFs in one wino_filter_transform_multi launch, then every conv through "
-                 "ONE wino_conv2d_f2x3_fwd_multi call (layers with < 32 tiles per SM share one persistent "
+                 "ONE wino_conv2d_f2x3_fwd_multi call (layers with < 64 tiles per SM share one persistent "
                  "stream-K launch, larger ones run alone through the planner); "
                  if args.variant == "fp32" and not args.per_layer_launches else
                  "per layer: FTF + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "

@@ -255,7 +255,7 @@ wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, fl
  * shape; pad 1, stride 1) through as few launches as pay (Sec. 3-4 method per layer, Eq. 4-8;
  * the batching across layers is this library's, not the paper's).  Layers that the
  * warp-specialised FP32 kernel takes (N % 32 == 0 or N in {4, 8, 16}; K % 4 == 0) and that have
- * fewer than 32 output tiles (64 filters x 32 positions) per SM share ONE persistent launch per
+ * fewer than 64 output tiles (64 filters x 32 positions) per SM share ONE persistent launch per
  * group of up to 4: the (tile, channel block) units of the group are concatenated and cut into one
  * contiguous range per SM, balanced on a work model (unit cost per x box mode, one output
  * transform per tile), so the group pays one pipeline fill and one tail instead of one per layer,

@@ -533,7 +533,7 @@ def conv_multi_launches(shapes) -> int:
 
 def conv2d_multi(layers, ws: torch.Tensor, stream=None, u_ready: torch.cuda.Event | None = None) -> None:
     """Several independent layers [(x (C,H,W,N), u (C,4,4,K), y (K,H,W,N)), ...]: the layers with
-    fewer than 32 tiles per SM share one persistent stream-K launch of the warp-specialised FP32
+    fewer than 64 tiles per SM share one persistent stream-K launch of the warp-specialised FP32
     kernel per group of <= 4, the others run alone through the planner (wino_conv2d_f2x3_fwd_multi).
     ws: a ZERO-FILLED CUDA byte buffer of >= conv_multi_workspace_bytes (calls leave it zeroed).
     u_ready: an event the convolutions wait for (the x-only input transforms of N = 4 / 8 layers

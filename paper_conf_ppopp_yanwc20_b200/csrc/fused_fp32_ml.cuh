@@ -53,8 +53,18 @@ using SM = fp32ws::Smem<false>;
 // the slowest consumer, so a record is rewritten only after its segment is finished.
 constexpr int PR = 4;
 static_assert(PR > fp32ws::S, "piece ring must outlive the TMA ring");
+// The record also carries what the epilogue needs of the layer, so the compute warps never index
+// the parameter block with a run-time layer number (dependent constant-cache loads, ~12 % of a
+// shared tile's epilogue samples).
+struct __align__(16) PieceRec {
+    int u0, u1, l, sk_slot;  // global units [u0, u1) of layer l; cut-segment workspace slot or -1
+    int k0, nu0, K, NV;      // tile origin, layer K and NV
+    int N, TW, H, W;
+    float* y;
+    int pad[2];
+};
 constexpr int REC_OFFSET = (SM::bytes + 15) / 16 * 16;
-constexpr int SMEM_BYTES = REC_OFFSET + PR * 16;
+constexpr int SMEM_BYTES = REC_OFFSET + PR * static_cast<int>(sizeof(PieceRec));
 
 constexpr int MAX_LAYERS = 4;
 constexpr int MAX_GRID = 160;  // CTAs of one launch (B200: 148 SMs, one CTA each)
@@ -257,8 +267,12 @@ __global__ void __launch_bounds__(256) ml_itf_kernel(const __grid_constant__ Itf
 }
 
 #ifdef WINO_WS_CTATRACE
+__device__ unsigned long long g_ml_piece_trace[4][96][4];  // CTAs 0, 40, 80, 120: per piece t0, loop end, epi end, nst
+#define ML_PT(pi, e, v) do { const int cs_ = blockIdx.x % 40 == 0 ? blockIdx.x / 40 : -1; \
+    if (cs_ >= 0 && cs_ < 4 && (pi) < 96) g_ml_piece_trace[cs_][pi][e] = (v); } while (0)
 #define ML_CT(e, v) do { if (blockIdx.x < 256) fp32ws::g_cta_trace[blockIdx.x][e] = (v); } while (0)
 #else
+#define ML_PT(pi, e, v) do { } while (0)
 #define ML_CT(e, v) do { } while (0)
 #endif
 
@@ -272,7 +286,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
     uint64_t* const vfull = empty + S;
     uint64_t* const vempty = vfull + SV;
     int* const sk_sh = reinterpret_cast<int*>(reinterpret_cast<char*>(smem) + SM::sk_offset);
-    int4* const rec = reinterpret_cast<int4*>(reinterpret_cast<char*>(smem) + REC_OFFSET);
+    PieceRec* const rec = reinterpret_cast<PieceRec*>(reinterpret_cast<char*>(smem) + REC_OFFSET);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 #ifdef WINO_WS_CTATRACE
     if (tid == 0) ML_CT(0, fp32ws::gtimer());
@@ -306,12 +320,25 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                 int l, u0, u1;
                 for (int pi = 0; ml_piece(p, blockIdx.x, pi, l, u0, u1); ++pi) {
                     const Layer& L = p.L[l];
-                    if (G >= S) mbar_wait(&empty[G % S], ((G / S) - 1) & 1);  // (re-checked below: free)
-                    rec[pi % PR] = make_int4(u0, u1, l, 0);
                     const int lu = u0 - L.unit0;
                     const int tile = lu / L.num_it, g_lo = lu - tile * L.num_it, g_hi = g_lo + (u1 - u0);
                     const int kb = tile % L.num_kb, nb = tile / L.num_kb;
                     const int k0 = kb * BK, nu0 = nb * BN;
+                    if (G >= S) mbar_wait(&empty[G % S], ((G / S) - 1) & 1);  // (re-checked below: free)
+                    PieceRec& R = rec[pi % PR];
+                    R.u0 = u0;
+                    R.u1 = u1;
+                    R.l = l;
+                    R.sk_slot = u1 - u0 == L.num_it ? -1 : 2 * static_cast<int>(blockIdx.x) + (g_lo > 0 ? 0 : 1);
+                    R.k0 = k0;
+                    R.nu0 = nu0;
+                    R.K = L.K;
+                    R.NV = L.NV;
+                    R.N = L.N;
+                    R.TW = L.TW;
+                    R.H = L.H;
+                    R.W = L.W;
+                    R.y = L.y;
                     const int t0 = nu0 / L.N, n0 = nu0 - t0 * L.N;
                     const bool box32 = L.xnb == BN;
                     const int nbox = box32 ? 1 : BN / L.xnb;
@@ -358,9 +385,8 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
         const int total = p.start[blockIdx.x + 1] - p.start[blockIdx.x];
         for (int pi = 0; G < total; ++pi) {
             mbar_wait(&full[G % S], (G / S) & 1);  // the segment's first stage: its record is published
-            const int4 r = rec[pi % PR];
-            const int u0 = r.x, u1 = r.y;
-            const Layer& L = p.L[r.z];
+            const int u0 = rec[pi % PR].u0, u1 = rec[pi % PR].u1;
+            const Layer& L = p.L[rec[pi % PR].l];
             if (L.vmode) {  // no raw x: only keep the stage hand-off (the producer waits on our arrival)
                 for (int g = u0; g < u1; ++g, ++G) {
                     mbar_wait(&full[G % S], (G / S) & 1);
@@ -438,7 +464,10 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
     int G = 0;
     for (int pi = 0; G < p.start[blockIdx.x + 1] - p.start[blockIdx.x]; ++pi) {
         mbar_wait(&full[G % S], (G / S) & 1);  // the segment's first stage: its record is published
-        const int nst = rec[pi % PR].y - rec[pi % PR].x;
+        const int nst = rec[pi % PR].u1 - rec[pi % PR].u0;
+#ifdef WINO_WS_CTATRACE
+        if (tid == 0) { ML_PT(pi, 0, fp32ws::gtimer()); ML_PT(pi, 3, nst); }
+#endif
         float acc[2][8][8];
 #pragma unroll
         for (int q = 0; q < 2; ++q)
@@ -481,29 +510,36 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
             }
         }
 
+#ifdef WINO_WS_CTATRACE
+        if (tid == 0) ML_PT(pi, 1, fp32ws::gtimer());
+#endif
         // ---- OTF (Sec. 4.4): 4 rounds of 16 filters through the epilogue buffer (L499) ----
-        const int4 r4 = rec[pi % PR];
-        const int l = r4.z;
-        const Layer& L = p.L[l];
-        const int lu = r4.x - L.unit0;
-        const int tile = lu / L.num_it, g_lo = lu - tile * L.num_it;
+        const PieceRec& R = rec[pi % PR];
         // -1: whole tile -> y; else this cut segment's workspace slot: 2b (starts inside the
         // tile) or 2b + 1 (holds the tile's channel block 0)
-        const int sk_slot = nst == L.num_it ? -1 : 2 * static_cast<int>(blockIdx.x) + (g_lo > 0 ? 0 : 1);
-        const int kb = tile % L.num_kb, nb = tile / L.num_kb;
-        const int k0 = kb * BK, nu0 = nb * BN;
+        const int sk_slot = R.sk_slot;
+        const int k0 = R.k0, nu0 = R.nu0, LK = R.K, LN = R.N, LNV = R.NV, LH = R.H, LW = R.W;
+        float* const Ly = R.y;
         const int nu = nu0 + lane;
         int t = 0, n = 0, i0 = 0, j0 = 0;
-        if (nu < L.NV) {
-            t = nu / L.N;
-            n = nu - t * L.N;
-            const int th = t / L.TW, tw = t - th * L.TW;
+        if (nu < LNV) {
+            t = nu / LN;
+            n = nu - t * LN;
+            const int th = t / R.TW, tw = t - th * R.TW;
             i0 = 2 * th;
             j0 = 2 * tw;
         }
-        const bool okr = i0 + 1 < L.H, okc = j0 + 1 < L.W;  // odd H/W: drop extra outputs (L1155)
-        const size_t base = ((size_t)i0 * L.W + j0) * L.N + n;
-        const size_t HWN = (size_t)L.H * L.W * L.N, dW = (size_t)L.W * L.N;
+        const bool okr = i0 + 1 < LH, okc = j0 + 1 < LW;  // odd H/W: drop extra outputs (L1155)
+        const size_t base = ((size_t)i0 * LW + j0) * LN + n;
+        const size_t HWN = (size_t)LH * LW * LN, dW = (size_t)LW * LN;
+        // one store pattern for both destinations (y, or this cut segment's workspace slot
+        // [slot][kl][output][nu]); the round's reads are branch-free so the 2 RR x 16 LDS issue back to
+        // back and only the stores are predicated
+        const bool cut = sk_slot >= 0, nu_ok = nu < LNV;
+        const size_t o1 = cut ? BN : LN, o2 = cut ? 2 * BN : dW, o3 = cut ? 3 * BN : dW + LN;
+        const bool p1 = cut || okc, p2 = cut || okr, p3 = cut || (okr && okc);
+        float* const dst0 = cut ? p.sk_ws + (size_t)sk_slot * BK * (4 * BN) + lane : Ly + (size_t)k0 * HWN + base;
+        const size_t dk = cut ? 4 * BN : HWN;  // per filter
 #pragma unroll
         for (int rd = 0; rd < 8 / RR; ++rd) {
             const int rd_hi = RR == 2 ? (rd >> 1) : rd, rd_lo = RR == 2 ? (rd & 1) : 0;
@@ -520,35 +556,33 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                         make_float4(acc[q][i][5], acc[q][i][4], acc[q][i][7], acc[q][i][6]);
                 }
             named_bar_sync(1, COMPUTE_THREADS);
-            if (nu < L.NV) {
+            float m[RR][16], o[RR][4];
 #pragma unroll
-                for (int h = 0; h < RR; ++h) {
-                    const int r = warp + 8 * h;
-                    const int kl = (r / RR) * 4 + rd_lo * RR + (r % RR) + rd_hi * 32;
-                    const int k = k0 + kl;
-                    if (k < L.K) {
-                        float m[16], o[4];
+            for (int h = 0; h < RR; ++h)
 #pragma unroll
-                        for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + r) * ER_LD + (lane ^ 1)];
-                        otf_2x2(m, o);
-                        if (sk_slot >= 0) {  // cut segment: [slot][kl][output][nu]
-                            float* wk = p.sk_ws + ((size_t)sk_slot * BK + kl) * (4 * BN) + lane;
-                            wk[0] = o[0];
-                            wk[BN] = o[1];
-                            wk[2 * BN] = o[2];
-                            wk[3 * BN] = o[3];
-                        } else {
-                            float* yk = L.y + (size_t)k * HWN + base;
-                            yk[0] = o[0];
-                            if (okc) yk[L.N] = o[1];
-                            if (okr) yk[dW] = o[2];
-                            if (okr && okc) yk[dW + L.N] = o[3];
-                        }
-                    }
+                for (int e = 0; e < 16; ++e) m[h][e] = ep[(e * ER_KROWS + warp + 8 * h) * ER_LD + (lane ^ 1)];
+#pragma unroll
+            for (int h = 0; h < RR; ++h) otf_2x2(m[h], o[h]);
+#pragma unroll
+            for (int h = 0; h < RR; ++h) {
+                const int r = warp + 8 * h;
+                const int kl = (r / RR) * 4 + rd_lo * RR + (r % RR) + rd_hi * 32;
+                if (nu_ok && k0 + kl < LK) {
+                    float* d = dst0 + (size_t)kl * dk;
+                    d[0] = o[h][0];
+                    if (p1) d[o1] = o[h][1];
+                    if (p2) d[o2] = o[h][2];
+                    if (p3) d[o3] = o[h][3];
                 }
             }
         }
-        if (sk_slot >= 0) ml_arrive(p, l, L.unit0 + tile * L.num_it, k0, nu0, sk_sh, tid);
+        if (sk_slot >= 0) {
+            const Layer& L = p.L[R.l];
+            ml_arrive(p, R.l, L.unit0 + ((R.u0 - L.unit0) / L.num_it) * L.num_it, k0, nu0, sk_sh, tid);
+        }
+#ifdef WINO_WS_CTATRACE
+        if (tid == 0) ML_PT(pi, 2, fp32ws::gtimer());
+#endif
     }
 #ifdef WINO_WS_CTATRACE
     if (tid == 0) {

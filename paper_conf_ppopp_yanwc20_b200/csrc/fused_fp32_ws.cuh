@@ -550,32 +550,27 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ws_kernel(const __grid_const
                             make_float4(acc[q][i][5], acc[q][i][4], acc[q][i][7], acc[q][i][6]);
                     }
                 named_bar_sync(1, COMPUTE_THREADS);
-                if (nu < p.NV) {
+                // branch-free reads (all 2 RR x 16 LDS issue back to back), predicated stores; one
+                // store pattern for y and for a cut segment's workspace slot [slot][kl][output][nu]
+                float m[RR][16], o[RR][4];
 #pragma unroll
-                    for (int h = 0; h < RR; ++h) {
-                        const int r = warp + 8 * h;  // buffer row 0..8RR-1
-                        const int kl = (r / RR) * 4 + rd_lo * RR + (r % RR) + rd_hi * 32;
-                        const int k = k0 + kl;
-                        if (k < p.K) {
-                            float m[16], o[4];
+                for (int h = 0; h < RR; ++h)
 #pragma unroll
-                            for (int e = 0; e < 16; ++e) m[e] = ep[(e * ER_KROWS + r) * ER_LD + (lane ^ 1)];
-                            otf_2x2(m, o);
-                            if (SK && sk_slot >= 0) {
-                                // cut segment: [slot][kl][output][nu], summed by the tile's last arrival
-                                float* wk = p.sk_ws + ((size_t)sk_slot * BK + kl) * (4 * BN) + lane;
-                                wk[0] = o[0];
-                                wk[BN] = o[1];
-                                wk[2 * BN] = o[2];
-                                wk[3 * BN] = o[3];
-                            } else {
-                            float* yk = p.y + (size_t)k * HWN + base;
-                            yk[0] = o[0];
-                            if (okc) yk[p.N] = o[1];
-                            if (okr) yk[dW] = o[2];
-                            if (okr && okc) yk[dW + p.N] = o[3];
-                            }
-                        }
+                    for (int e = 0; e < 16; ++e) m[h][e] = ep[(e * ER_KROWS + warp + 8 * h) * ER_LD + (lane ^ 1)];
+#pragma unroll
+                for (int h = 0; h < RR; ++h) otf_2x2(m[h], o[h]);
+                const bool cut = SK && sk_slot >= 0;
+#pragma unroll
+                for (int h = 0; h < RR; ++h) {
+                    const int r = warp + 8 * h;  // buffer row 0..8RR-1
+                    const int kl = (r / RR) * 4 + rd_lo * RR + (r % RR) + rd_hi * 32;
+                    if (nu < p.NV && k0 + kl < p.K) {
+                        float* d = cut ? p.sk_ws + ((size_t)sk_slot * BK + kl) * (4 * BN) + lane
+                                       : p.y + (size_t)(k0 + kl) * HWN + base;
+                        d[0] = o[h][0];
+                        if (cut || okc) d[cut ? BN : p.N] = o[h][1];
+                        if (cut || okr) d[cut ? 2 * BN : dW] = o[h][2];
+                        if (cut || (okr && okc)) d[cut ? 3 * BN : dW + p.N] = o[h][3];
                     }
                 }
             }

@@ -540,6 +540,9 @@ int wino_debug_ws_trace(unsigned long long* host, int n) {
 int wino_debug_cta_trace(unsigned long long* host, int n) {
     return (int)cudaMemcpyFromSymbol(host, wino::fp32ws::g_cta_trace, sizeof(unsigned long long) * n);
 }
+int wino_debug_ml_piece_trace(unsigned long long* host, int n) {
+    return (int)cudaMemcpyFromSymbol(host, wino::fp32ml::g_ml_piece_trace, sizeof(unsigned long long) * n);
+}
 #endif
 #ifdef WINO_TC16_TRACE
 int wino_debug_tc16_trace(unsigned long long* host, int n) {
@@ -761,23 +764,27 @@ wino_status_t wino_conv2d_f2x3_fwd_ws(const float* x_dev, const float* u_dev, fl
 namespace {
 std::atomic<uint64_t> g_attr_ml;
 // Work model of the multi-layer cut, in units of one N % 32 == 0 channel block (~1.5 us of one
-// SM), fitted to per-CTA timelines of the ResNet step and its batch shards (scripts/ml_trace.py,
-// DESIGN.md 7.8): small-N box modes move x in 32/N boxes of N-float rows (N = 16 / 8 / 4: 1.07 /
-// 1.31 / 1.65 blocks), and each tile's 4-round OTF epilogue costs ~2 blocks (~3 us).
-constexpr double kMlEpiCost = 2.0;
+// SM), fitted to per-CTA / per-piece timelines of the ResNet step and its batch shards
+// (scripts/ml_trace.py): small-N box modes move x in 32/N boxes of N-float rows
+// (N = 16 / 8 / 4: 1.07 / 1.31 / 1.65 blocks), vmode layers skip the raw-x staging and the ITF
+// (0.93), and each tile's 4-round OTF epilogue costs ~1.65 blocks (~2.5 us).
+constexpr double kMlEpiCost = 1.65;
 double ml_unit_cost(int xnb, bool vmode) {
-    return vmode ? 0.92 : (xnb >= 32 ? 1.0 : (xnb == 16 ? 1.07 : (xnb == 8 ? 1.31 : 1.65)));
+    return vmode ? 0.93 : (xnb >= 32 ? 1.0 : (xnb == 16 ? 1.07 : (xnb == 8 ? 1.31 : 1.65)));
 }
 // A job joins the shared persistent launch when the warp-specialised kernel takes it (N % 32 == 0
-// or N in {4, 8, 16}; K % 4 == 0) and it has fewer than 32 tiles per SM; a layer that big fills
-// the GPU on its own and runs faster through the planner's one-tile-per-CTA grid (ResNet conv2 at
-// N = 256: 1136 vs 1162 us for the step, scripts/ml_ab.py).
+// or N in {4, 8, 16}; K % 4 == 0) and it has fewer than 64 tiles per SM; a layer that big fills
+// the GPU on its own and gains nothing from sharing (ResNet conv2 at N = 256, 42 tiles per SM:
+// shared 1129.5 vs alone 1131.5 us for the step, scripts/ml_ab.py).
+#ifndef WINO_ML_ALONE_TILES_PER_SM  // A/B builds only (scripts/ml_ab.py)
+#define WINO_ML_ALONE_TILES_PER_SM 64
+#endif
 bool ml_shares_launch(const wino_conv_job_t& J, int sms) {
     using namespace wino::fp32ml;
     if (J.K % 4 != 0 || !(J.N % 32 == 0 || J.N == 4 || J.N == 8 || J.N == 16)) return false;
     const long long nv = static_cast<long long>(J.N) * ((J.H + 1) / 2) * ((J.W + 1) / 2);
     const long long tiles = ((nv + BN - 1) / BN) * ((J.K + BK - 1) / BK);
-    return tiles < 32LL * sms;
+    return tiles < static_cast<long long>(WINO_ML_ALONE_TILES_PER_SM) * sms;
 }
 // vmode (N = 4, 8): the small-N x boxes (rows of 16 / 32 B, 8 / 4 TMA boxes per stage) cost a
 // shared layer 1.65 / 1.31 channel-block times; instead ml_itf_kernel transforms the (small) x into

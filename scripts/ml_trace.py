@@ -50,3 +50,21 @@ for l, c in enumerate(cfgs):
     if m.any():
         print(f"  start in {c.name:8s} N={c.N:3d}: CTAs {m.sum():3d} units/CTA {units[m].mean():6.1f} "
               f"exit median {np.median(dur[m]):6.1f} max {dur[m].max():6.1f} us -> us/unit {np.median(dur[m] / units[m]):.3f}")
+
+# per-piece timeline of CTAs 0, 40, 80, 120: main-loop time per channel block and epilogue time per tile
+L.wino_debug_ml_piece_trace.argtypes = [ctypes.c_void_p, ctypes.c_int]
+pb = (ctypes.c_ulonglong * (4 * 96 * 4))()
+L.wino_debug_ml_piece_trace(ctypes.cast(pb, ctypes.c_void_p), 4 * 96 * 4)
+pt = np.array(list(pb), dtype=np.int64).reshape(4, 96, 4)
+for ci in range(4):
+    rows = [r for r in pt[ci] if r[0] > 0]
+    if not rows:
+        continue
+    rows = np.array(rows)
+    loop = (rows[:, 1] - rows[:, 0]) / 1000.0
+    epi = (rows[:, 2] - rows[:, 1]) / 1000.0
+    gap = (rows[1:, 0] - rows[:-1, 2]) / 1000.0
+    nst = rows[:, 3]
+    whole = nst == nst.max()
+    print(f"  CTA {40 * ci:3d}: pieces {len(rows)}, main loop {np.median(loop[whole] / nst[whole]):.3f} us/block "
+          f"(nst {int(nst.max())}), epilogue median {np.median(epi):.2f} us, gap to next piece {np.median(gap) if len(gap) else 0:.2f} us")

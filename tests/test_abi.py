@@ -202,19 +202,22 @@ def test_stream_k_plan_and_workspace():
 
 def test_multi_layer_launch_grouping():
     """Host-only (148 SMs without a device): wino_conv2d_f2x3_fwd_multi puts the layers with fewer
-    than 32 tiles per SM into one shared persistent launch per group of <= 4 and runs the others
-    alone through the planner.  ResNet step: conv2_x at N = 256 (6272 tiles = 42 per SM) alone, the
-    other three shared -> 2 launches; any batch shard (P >= 2) -> all four shared, 1 launch, plus
-    one ml_itf_kernel launch when a shard has N = 4 or 8 (P = 4: conv5_x; P = 8: conv5_x, conv4_x)."""
+    than 64 tiles per SM into one shared persistent launch per group of <= 4 and runs the others
+    alone through the planner.  ResNet step: all four layers shared (conv2_x at N = 256: 6272 tiles
+    = 42 per SM) -> 1 launch, plus one ml_itf_kernel launch when a shard has N = 4 or 8 (P = 4:
+    conv5_x; P = 8: conv5_x, conv4_x); a 64-tiles-per-SM layer runs alone."""
     names = ("conv5_x", "conv4_x", "conv3_x", "conv2_x")
     sk = 148 * 2 * 64 * 4 * 32 * 4 + 768
-    for P, want in ((1, 2), (2, 1), (4, 2), (8, 2)):
+    for P, want in ((1, 1), (2, 1), (4, 2), (8, 2)):
         shapes = [(CONFIGS[n].N // P, CONFIGS[n].C, CONFIGS[n].H, CONFIGS[n].W, CONFIGS[n].K) for n in names]
         assert wino.conv_multi_launches(shapes) == want, P
         # N = 4 / 8 layers (vmode): + one input-transform launch and a V buffer of 16 x C x NV floats
         vbytes = sum(-(-16 * C * N * ((H + 1) // 2) * ((W + 1) // 2) * 4 // 256) * 256
                      for N, C, H, W, K in shapes if N in (4, 8))
         assert wino.conv_multi_workspace_bytes(shapes) == sk + vbytes, P
+    big = (512, 64, 56, 56, 64)  # 25088 tiles = 169.5 per SM: alone (the planner's one launch)
+    assert wino.conv_multi_launches([big]) == wino.plan(*big[:4], big[4], variant=4).launches == 1
+    assert wino.conv_multi_launches([big, (32, 64, 9, 9, 64)]) == 2
     small = (32, 64, 9, 9, 64)
     assert wino.conv_multi_launches([small] * 4) == 1
     assert wino.conv_multi_launches([small] * 5) == 2  # groups of at most 4

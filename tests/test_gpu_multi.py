@@ -1,6 +1,6 @@
 """Several independent layers through wino_conv2d_f2x3_fwd_multi (shared persistent stream-K launch,
-csrc/fused_fp32_ml.cuh; layers with >= 32 tiles per SM, e.g. conv2_x at N = 256, run alone through
-the planner) against the fp64 oracle, every output element of every layer.
+csrc/fused_fp32_ml.cuh; layers with >= 64 tiles per SM run alone through the planner) against the
+fp64 oracle, every output element of every layer.
 
 Bars as tests/test_gpu_parity.py: bit-exact vs Eq. 4 on small integers, <= 1e-4 of max|y| on
 random inputs (per layer).  Covered: the four BASELINE ResNet layers at their global batch and
@@ -160,3 +160,15 @@ def test_u_ready_event_orders_the_convolutions(wino):
     wino.conv2d_multi([(x, u, y) for x, u, y, _ in layers], ws, u_ready=ev)
     torch.cuda.synchronize()
     _check(data, [y.cpu().double().numpy() for _, _, y, _ in layers], "smallint")
+
+
+def test_big_layer_runs_alone_next_to_shared_ones(wino):
+    """A layer with >= 64 tiles per SM (10240 tiles of 64 x 32 here) is launched alone through the
+    planner in the same call as a shared group: both bit-exact on small integers."""
+    big = Conv3x3Config("big", 32, 1, 640, 64, 64)
+    cfgs = [Conv3x3Config("s1", 8, 40, 72, 7, 7), big, Conv3x3Config("s2", 32, 16, 36, 5, 5)]
+    shapes = [(c.N, c.C, c.H, c.W, c.K) for c in cfgs]
+    # the shared launch (+ its input transform for N = 8) and the planner's launch for the big layer
+    assert wino.conv_multi_launches(shapes) == 2 + wino.plan(*shapes[1][:4], shapes[1][4], variant=4).launches
+    data, outs, _ = _run_multi(wino, cfgs, "smallint", seed0=700)
+    _check(data, outs[0], "smallint")
