@@ -76,6 +76,7 @@ struct __align__(64) Layer {
     float* __restrict__ y;
     int N, C, H, W, K;
     int TW, NV, num_kb, num_it, xnb;
+    int vg, vr, vlc;   // nu-tile order (ml_nu_tile): ~vg CTAs share the layer, vr nu-tiles each
     int unit0;         // global index of the layer's first unit (tile * num_it + g)
     int vmode;         // 1: V comes transformed from ml_itf_kernel (small N), the ITF warps idle
     int itf_map[64];   // N | 32: ITF task map of the 64 ITF lanes (as fp32::Params::itf_map)
@@ -95,6 +96,19 @@ __device__ __forceinline__ int layer_of(const Params& p, int u) {
     int l = 0;
     while (l + 1 < p.nl && p.L[l + 1].unit0 <= u) ++l;
     return l;
+}
+
+// Order of a layer's nu-tiles along its unit sequence.  Each CTA of the persistent launch walks its
+// own contiguous range, so in natural order the ~vg CTAs sharing a layer would stream vg distant
+// regions of x at once, and the Winograd tiles' overlap (Sec. 3.5: neighbouring 4x4 input patches
+// share 2 rows / columns) would be re-read from DRAM after eviction (whole ResNet step in one launch:
+// 1.21 GB of DRAM reads for 310 MB of x and u).  Instead sequence position s (column s / vr ~ one
+// CTA's share, row s % vr ~ its step) maps to nu-tile row * vg + column, so that at each step the
+// CTAs work on ~vg neighbouring nu-tiles, as a one-tile-per-CTA grid would (step reads 0.57 GB;
+// DESIGN.md 7.8).  A bijection on [0, ng) with ng = (vg - 1) * vr + vlc, 1 <= vlc <= vr.
+__device__ __forceinline__ int ml_nu_tile(const Layer& L, int s) {
+    const int c = s / L.vr, r = s - c * L.vr;
+    return r < L.vlc ? r * L.vg + c : L.vlc * L.vg + (r - L.vlc) * (L.vg - 1) + c;
 }
 
 // The pi-th segment of CTA b's range in processing order: its first segment, its last, then the
@@ -316,6 +330,8 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
             // ---------------- TMA issue (one elected lane) ----------------
             if (lane == 0) {
                 constexpr uint32_t kBytes = (US_FLOATS + XS_FLOATS) * 4;
+                // L2 priority: u is re-read by every tile of its layer (y is stored with .cs)
+                const uint64_t pol_keep = l2_policy_evict_last();
                 int G = 0;
                 int l, u0, u1;
                 for (int pi = 0; ml_piece(p, blockIdx.x, pi, l, u0, u1); ++pi) {
@@ -323,7 +339,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                     const int lu = u0 - L.unit0;
                     const int tile = lu / L.num_it, g_lo = lu - tile * L.num_it, g_hi = g_lo + (u1 - u0);
                     const int kb = tile % L.num_kb, nb = tile / L.num_kb;
-                    const int k0 = kb * BK, nu0 = nb * BN;
+                    const int k0 = kb * BK, nu0 = ml_nu_tile(L, nb) * BN;
                     if (G >= S) mbar_wait(&empty[G % S], ((G / S) - 1) & 1);  // (re-checked below: free)
                     PieceRec& R = rec[pi % PR];
                     R.u0 = u0;
@@ -348,7 +364,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                             if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
                             float* us = smem + slot * STAGE_FLOATS;
                             mbar_arrive_expect_tx(&full[slot], US_FLOATS * 4);
-                            tma_load_3d(us, &L.tmu, &full[slot], k0, 0, g * BC);
+                            tma_load_3d_hint(us, &L.tmu, &full[slot], k0, 0, g * BC, pol_keep);
                             if (G >= SV) mbar_wait(&vempty[vb], ((G / SV) - 1) & 1);
                             mbar_arrive_expect_tx(&vfull[vb], VS_FLOATS * 4);
                             tma_load_3d(vs + vb * VS_FLOATS, &L.tmv, &vfull[vb], nu0, g * BC, 0);
@@ -361,16 +377,15 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                         if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
                         float* us = smem + slot * STAGE_FLOATS;
                         mbar_arrive_expect_tx(&full[slot], kBytes);
-                        tma_load_3d(us, &L.tmu, &full[slot], k0, 0, g * BC);
+                        tma_load_3d_hint(us, &L.tmu, &full[slot], k0, 0, g * BC, pol_keep);
                         for (int b = 0; b < nbox; ++b) {
                             const int t = t0 + b;
                             const int th = t / L.TW, tw = t - th * L.TW;
                             // -1 / past the end: TMA zero fill = implicit padding (Sec. 3.5)
-                            if (box32)
-                                tma_load_4d(us + US_FLOATS, &L.tmx, &full[slot], n0, 2 * tw - 1, 2 * th - 1, g * BC);
-                            else
-                                tma_load_4d(us + US_FLOATS + b * (BC * 16 * L.xnb), &L.tmx, &full[slot], 0, g * BC,
-                                            2 * tw - 1, 2 * th - 1);
+                            float* dst = us + US_FLOATS + (box32 ? 0 : b * (BC * 16 * L.xnb));
+                            const int c0 = box32 ? n0 : 0, c1 = box32 ? 2 * tw - 1 : g * BC;
+                            const int c2 = box32 ? 2 * th - 1 : 2 * tw - 1, c3 = box32 ? g * BC : 2 * th - 1;
+                            tma_load_4d(dst, &L.tmx, &full[slot], c0, c1, c2, c3);
                         }
                     }
                 }
@@ -521,9 +536,10 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
         const int k0 = R.k0, nu0 = R.nu0, LK = R.K, LN = R.N, LNV = R.NV, LH = R.H, LW = R.W;
         float* const Ly = R.y;
         const int nu = nu0 + lane;
-        int t = 0, n = 0, i0 = 0, j0 = 0;
-        if (nu < LNV) {
-            t = nu / LN;
+        const bool nu_ok = nu < LNV;
+        int n = 0, i0 = 0, j0 = 0;
+        if (nu_ok) {
+            const int t = nu / LN;
             n = nu - t * LN;
             const int th = t / R.TW, tw = t - th * R.TW;
             i0 = 2 * th;
@@ -535,7 +551,7 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
         // one store pattern for both destinations (y, or this cut segment's workspace slot
         // [slot][kl][output][nu]); the round's reads are branch-free so the 2 RR x 16 LDS issue back to
         // back and only the stores are predicated
-        const bool cut = sk_slot >= 0, nu_ok = nu < LNV;
+        const bool cut = sk_slot >= 0;
         const size_t o1 = cut ? BN : LN, o2 = cut ? 2 * BN : dW, o3 = cut ? 3 * BN : dW + LN;
         const bool p1 = cut || okc, p2 = cut || okr, p3 = cut || (okr && okc);
         float* const dst0 = cut ? p.sk_ws + (size_t)sk_slot * BK * (4 * BN) + lane : Ly + (size_t)k0 * HWN + base;
@@ -567,12 +583,12 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
             for (int h = 0; h < RR; ++h) {
                 const int r = warp + 8 * h;
                 const int kl = (r / RR) * 4 + rd_lo * RR + (r % RR) + rd_hi * 32;
-                if (nu_ok && k0 + kl < LK) {
+                if (nu_ok && k0 + kl < LK) {  // y is never re-read here: stream it past L2 (st.global.cs)
                     float* d = dst0 + (size_t)kl * dk;
-                    d[0] = o[h][0];
-                    if (p1) d[o1] = o[h][1];
-                    if (p2) d[o2] = o[h][2];
-                    if (p3) d[o3] = o[h][3];
+                    __stcs(d, o[h][0]);
+                    if (p1) __stcs(d + o1, o[h][1]);
+                    if (p2) __stcs(d + o2, o[h][2]);
+                    if (p3) __stcs(d + o3, o[h][3]);
                 }
             }
         }

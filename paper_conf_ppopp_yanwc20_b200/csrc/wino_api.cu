@@ -906,6 +906,15 @@ wino_status_t prepare_multi_fp32(const wino_conv_job_t* jobs, float* const* vbuf
     const int sms = sm_count(dev) < MAX_GRID ? sm_count(dev) : MAX_GRID;
     const int grid = units < sms ? static_cast<int>(units) : sms;
     const double total = work0[n];
+    for (int i = 0; i < n; ++i) {  // nu-tile order (ml_nu_tile): the CTAs' shares of each layer
+        Layer& L = prm.L[i];
+        const int ng = (L.NV + BN - 1) / BN;
+        long long g = std::llround((work0[i + 1] - work0[i]) * grid / total);
+        g = g < 1 ? 1 : (g > ng ? ng : g);
+        L.vr = static_cast<int>((ng + g - 1) / g);
+        L.vg = (ng + L.vr - 1) / L.vr;
+        L.vlc = ng - (L.vg - 1) * L.vr;
+    }
     for (int b = 0; b <= grid; ++b) {
         long long u = static_cast<long long>(units);
         if (b < grid) {
