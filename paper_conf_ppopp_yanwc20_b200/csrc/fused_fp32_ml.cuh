@@ -105,7 +105,7 @@ __device__ __forceinline__ int layer_of(const Params& p, int u) {
 // 1.21 GB of DRAM reads for 310 MB of x and u).  Instead sequence position s (column s / vr ~ one
 // CTA's share, row s % vr ~ its step) maps to nu-tile row * vg + column, so that at each step the
 // CTAs work on ~vg neighbouring nu-tiles, as a one-tile-per-CTA grid would (step reads 0.57 GB;
-// DESIGN.md 7.8).  A bijection on [0, ng) with ng = (vg - 1) * vr + vlc, 1 <= vlc <= vr.
+// DESIGN.md 7.11).  A bijection on [0, ng) with ng = (vg - 1) * vr + vlc, 1 <= vlc <= vr.
 __device__ __forceinline__ int ml_nu_tile(const Layer& L, int s) {
     const int c = s / L.vr, r = s - c * L.vr;
     return r < L.vlc ? r * L.vg + c : L.vlc * L.vg + (r - L.vlc) * (L.vg - 1) + c;

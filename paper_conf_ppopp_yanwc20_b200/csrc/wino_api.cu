@@ -765,7 +765,7 @@ namespace {
 std::atomic<uint64_t> g_attr_ml;
 // Work model of the multi-layer cut, in units of one N % 32 == 0 channel block (~1.5 us of one
 // SM), fitted to per-CTA / per-piece timelines of the ResNet step and its batch shards
-// (scripts/ml_trace.py, DESIGN.md 7.8): small-N box modes move x in 32/N boxes of N-float rows
+// (scripts/ml_trace.py, DESIGN.md 7.11): small-N box modes move x in 32/N boxes of N-float rows
 // (N = 16 / 8 / 4: 1.07 / 1.31 / 1.65 blocks), vmode layers skip the raw-x staging and the ITF
 // (0.93), and each tile's 4-round OTF epilogue costs ~1.65 blocks (~2.5 us).
 constexpr double kMlEpiCost = 1.65;
@@ -775,7 +775,7 @@ double ml_unit_cost(int xnb, bool vmode) {
 // A job joins the shared persistent launch when the warp-specialised kernel takes it (N % 32 == 0
 // or N in {4, 8, 16}; K % 4 == 0) and it has fewer than 64 tiles per SM; a layer that big fills
 // the GPU on its own and gains nothing from sharing (ResNet conv2 at N = 256, 42 tiles per SM:
-// shared 1129.5 vs alone 1131.5 us for the step, scripts/ml_ab.py, DESIGN.md 7.8).
+// shared 1129.5 vs alone 1131.5 us for the step, scripts/ml_ab.py, DESIGN.md 7.11).
 #ifndef WINO_ML_ALONE_TILES_PER_SM  // A/B builds only (scripts/ml_ab.py)
 #define WINO_ML_ALONE_TILES_PER_SM 64
 #endif
