@@ -543,9 +543,6 @@ int wino_debug_cta_trace(unsigned long long* host, int n) {
 int wino_debug_ml_piece_trace(unsigned long long* host, int n) {
     return (int)cudaMemcpyFromSymbol(host, wino::fp32ml::g_ml_piece_trace, sizeof(unsigned long long) * n);
 }
-int wino_debug_ml_epi_rounds(unsigned long long* host, int n) {
-    return (int)cudaMemcpyFromSymbol(host, wino::fp32ml::g_ml_epi_rounds, sizeof(unsigned long long) * n);
-}
 #endif
 #ifdef WINO_TC16_TRACE
 int wino_debug_tc16_trace(unsigned long long* host, int n) {
@@ -771,12 +768,9 @@ std::atomic<uint64_t> g_attr_ml;
 // (scripts/ml_trace.py): small-N box modes move x in 32/N boxes of N-float rows
 // (N = 16 / 8 / 4: 1.07 / 1.31 / 1.65 blocks), vmode layers skip the raw-x staging and the ITF
 // (0.93), and each tile's 4-round OTF epilogue costs ~1.65 blocks (~2.5 us).
-// TEPI (epilogue in its own warpgroup, fused_fp32_ml.cuh): a tile's epilogue costs the compute warps only
-// the TMEM hand-off, but the epilogue warps slow the FFMA stream of short tiles; fitted to per-CTA exit
-// times of the P = 1 and P = 8 ResNet steps (scripts/ml_trace.py): 1.25 blocks per tile, N = 16 units 1.03.
-constexpr double kMlEpiCost = wino::fp32ml::TEPI ? 1.25 : 1.65;
+constexpr double kMlEpiCost = 1.65;
 double ml_unit_cost(int xnb, bool vmode) {
-    return vmode ? 0.93 : (xnb >= 32 ? 1.0 : (xnb == 16 ? (wino::fp32ml::TEPI ? 1.03 : 1.07) : (xnb == 8 ? 1.31 : 1.65)));
+    return vmode ? 0.93 : (xnb >= 32 ? 1.0 : (xnb == 16 ? 1.07 : (xnb == 8 ? 1.31 : 1.65)));
 }
 // A job joins the shared persistent launch when the warp-specialised kernel takes it (N % 32 == 0
 // or N in {4, 8, 16}; K % 4 == 0) and it has fewer than 64 tiles per SM; a layer that big fills
@@ -954,10 +948,10 @@ wino_status_t launch_ml_itf(const MlLaunch& L, int dev, cudaStream_t st) {
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }
 wino_status_t launch_ml(const MlLaunch& L, int dev, cudaStream_t st) {
-    const int smem = wino::fp32ml::SMEM_BYTES_ML;
+    const int smem = wino::fp32ml::SMEM_BYTES;
     wino_status_t s = ensure_smem_attr(wino::fp32ml::fused_fp32_ml_kernel, dev, smem, g_attr_ml);
     if (s != WINO_OK) return s;
-    wino::fp32ml::fused_fp32_ml_kernel<<<dim3(static_cast<unsigned>(L.grid)), wino::fp32ml::NT_ML, smem, st>>>(L.prm);
+    wino::fp32ml::fused_fp32_ml_kernel<<<dim3(static_cast<unsigned>(L.grid)), wino::fp32ws::NT, smem, st>>>(L.prm);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
 }

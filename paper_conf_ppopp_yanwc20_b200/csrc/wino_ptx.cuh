@@ -176,12 +176,6 @@ __device__ __forceinline__ void tmem_ld8(uint32_t taddr, float v[8]) {
 #pragma unroll
     for (int j = 0; j < 8; ++j) v[j] = __uint_as_float(r[j]);
 }
-__device__ __forceinline__ void tmem_ld2(uint32_t taddr, float v[2]) {
-    uint32_t r[2];
-    asm volatile("tcgen05.ld.sync.aligned.32x32b.x2.b32 {%0,%1}, [%2];\n" : "=r"(r[0]), "=r"(r[1]) : "r"(taddr));
-    v[0] = __uint_as_float(r[0]);
-    v[1] = __uint_as_float(r[1]);
-}
 __device__ __forceinline__ void tmem_ld4(uint32_t taddr, float v[4]) {
     uint32_t r[4];
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0,%1,%2,%3}, [%4];\n"
@@ -191,13 +185,6 @@ __device__ __forceinline__ void tmem_ld4(uint32_t taddr, float v[4]) {
     for (int j = 0; j < 4; ++j) v[j] = __uint_as_float(r[j]);
 }
 __device__ __forceinline__ void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory"); }
-// registers -> TMEM: 32 lanes x 32 bit, 4 consecutive columns per thread (a register quad, like STS.128)
-__device__ __forceinline__ void tmem_st4(uint32_t taddr, float a, float b, float c, float d) {
-    asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};\n" ::"r"(taddr), "r"(__float_as_uint(a)),
-                 "r"(__float_as_uint(b)), "r"(__float_as_uint(c)), "r"(__float_as_uint(d))
-                 : "memory");
-}
-__device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory"); }
 
 // TF32 rounding, round-to-nearest ties-away (reading R8)
 __device__ __forceinline__ float to_tf32(float x) {

@@ -53,9 +53,9 @@ for l, c in enumerate(cfgs):
 
 # per-piece timeline of CTAs 0, 40, 80, 120: main-loop time per channel block and epilogue time per tile
 L.wino_debug_ml_piece_trace.argtypes = [ctypes.c_void_p, ctypes.c_int]
-pb = (ctypes.c_ulonglong * (4 * 96 * 8))()
-L.wino_debug_ml_piece_trace(ctypes.cast(pb, ctypes.c_void_p), 4 * 96 * 8)
-pt = np.array(list(pb), dtype=np.int64).reshape(4, 96, 8)
+pb = (ctypes.c_ulonglong * (4 * 96 * 4))()
+L.wino_debug_ml_piece_trace(ctypes.cast(pb, ctypes.c_void_p), 4 * 96 * 4)
+pt = np.array(list(pb), dtype=np.int64).reshape(4, 96, 4)
 for ci in range(4):
     rows = [r for r in pt[ci] if r[0] > 0]
     if not rows:
@@ -68,22 +68,3 @@ for ci in range(4):
     whole = nst == nst.max()
     print(f"  CTA {40 * ci:3d}: pieces {len(rows)}, main loop {np.median(loop[whole] / nst[whole]):.3f} us/block "
           f"(nst {int(nst.max())}), epilogue median {np.median(epi):.2f} us, gap to next piece {np.median(gap) if len(gap) else 0:.2f} us")
-    if (rows[:, 4] > 0).any():  # TEPI epilogue warps
-        e = rows[rows[:, 4] > 0]
-        print(f"           epilogue warps: per tile {np.median((e[:, 6] - e[:, 4]) / 1000.0):.2f} us (TMEM held "
-              f"{np.median((e[:, 5] - e[:, 4]) / 1000.0):.2f}), lag behind hand-off {np.median((e[:, 4] - e[:, 2]) / 1000.0):.2f} us, "
-              f"last piece done {(e[-1, 6] - rows[-1, 2]) / 1000.0:.2f} us after the compute warps")
-
-# TEPI epilogue warps of CTA 0, per round: barrier wait, TMEM reads + column sums, exchange barrier, combine + stores
-if hasattr(L, "wino_debug_ml_epi_rounds"):
-    L.wino_debug_ml_epi_rounds.argtypes = [ctypes.c_void_p, ctypes.c_int]
-    eb = (ctypes.c_ulonglong * (96 * 4 * 4))()
-    L.wino_debug_ml_epi_rounds(ctypes.cast(eb, ctypes.c_void_p), 96 * 4 * 4)
-    er = np.array(list(eb), dtype=np.int64).reshape(96, 4, 4)
-    er = er[er[:, 0, 0] > 0]
-    if len(er):
-        nxt = np.concatenate([er[:, 1:, 0], np.full((len(er), 1), 0)], axis=1)
-        d = np.stack([er[:, :, 1] - er[:, :, 0], er[:, :, 2] - er[:, :, 1], er[:, :, 3] - er[:, :, 2]], axis=2) / 1000.0
-        comb = (er[:, :3, 0].astype(float) * 0 + (er[:, 1:, 0] - er[:, :3, 3])) / 1000.0
-        print("  CTA 0 epilogue rounds (median us): bar-in %.2f, TMEM+sums %.2f, bar %.2f, combine(rd0-2) %.2f" %
-              (np.median(d[:, :, 0]), np.median(d[:, :, 1]), np.median(d[:, :, 2]), np.median(comb)))
