@@ -300,13 +300,9 @@ def _config(args, layers, world):
         "inputs": f"uniform[-1,1) fp32, torch seeds x={SEED_X} w={SEED_W}",
         "l2": "headline: flushed before every timed step by a 512 MiB write + 256 MiB read (outside the events); "
               "hot_l2: the paper's protocol (L863), 5 repeats x 20 back-to-back replays, median of the means",
-        "step": ("fp32: ONE wino_conv2d_f2x3_fwd_multi_ftf call: when every layer has < 64 tiles per SM "
-                 "(the ResNet step at every P) one cooperative persistent stream-K launch whose prologue runs "
-                 "every layer's FTF (and the N = 4 / 8 shards' input transforms), then all convolutions; "
-                 "otherwise all layers' FTFs in one wino_filter_transform_multi launch + wino_conv2d_f2x3_fwd_multi; "
-                 if args.variant == "fp32" and not args.per_layer_launches and not args.separate_ftf else
-                 "fp32: all layers' FTFs in one wino_filter_transform_multi launch on a side stream, then every "
-                 "conv through ONE wino_conv2d_f2x3_fwd_multi call; "
+        "step": ("fp32: all layers' FTFs in one wino_filter_transform_multi launch, then every conv through "
+                 "ONE wino_conv2d_f2x3_fwd_multi call (layers with < 64 tiles per SM share one persistent "
+                 "stream-K launch, larger ones run alone through the planner); "
                  if args.variant == "fp32" and not args.per_layer_launches else
                  "per layer: FTF + fused ITF/16xGEMM/OTF kernel (FTFs on a side stream, each conv waits for "
                  "its own FTF; fp32: all layers' FTFs in one wino_filter_transform_multi launch, convs through "
@@ -333,9 +329,6 @@ def main():
     ap.add_argument("--per-layer-launches", action="store_true",
                     help="fp32: one conv launch per layer (wino_conv2d_f2x3_fwd_ws) instead of one "
                          "wino_conv2d_f2x3_fwd_multi call for all layers (shared persistent stream-K launch)")
-    ap.add_argument("--separate-ftf", action="store_true",
-                    help="fp32: the FTFs as their own launch on a side stream (wino_filter_transform_multi) "
-                         "instead of the prologue of the shared conv launch (wino_conv2d_f2x3_fwd_multi_ftf)")
     ap.add_argument("--concurrent-layers", action="store_true",
                     help="issue each layer's convolution on its own stream (the BASELINE layers are independent "
                          "problems); default: in sequence on one stream, as a network would")
@@ -430,10 +423,6 @@ def main():
         half = variant in ("fp16", "bf16")  # NEXT row N4: 16-bit x, w, y on tcgen05 kind::f16 (Sec. 8.3)
         # fp32: every layer through one wino_conv2d_f2x3_fwd_multi call (shared persistent launch)
         multi = variant == "fp32" and not args.per_layer_launches
-        shapes_ml = [(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K) for d in live]
-        # fp32 default: FTFs + convolutions through ONE wino_conv2d_f2x3_fwd_multi_ftf call; when all
-        # layers share one persistent launch the FTFs are its prologue (one cooperative launch per step)
-        fused_ftf = multi and not args.separate_ftf and wino.conv_multi_ftf_launches(shapes_ml) == 1
         if f4:  # FTF4 + conv (+ a stream-K fixup where the planner takes it: counted as taken)
             launches = sum(3 for d in live)
         elif half:  # FTF + conv (+ stream-K fixup with the workspace, variant 5 plans it)
@@ -444,10 +433,9 @@ def main():
                            for d in live)
         elif nonfused:
             launches = sum(1 + wino.nonfused_launches() for d in live)  # FTF + u arrangement, ITF, GEMM, OTF
-        elif fused_ftf:  # FTF prologue + convolutions: one launch
-            launches = wino.conv_multi_ftf_launches(shapes_ml)
         elif multi:  # one batched FTF + the conv launches of wino_conv2d_f2x3_fwd_multi
-            launches = 1 + wino.conv_multi_launches(shapes_ml)
+            launches = 1 + wino.conv_multi_launches([(d["n"], d["cfg"].C, d["cfg"].H, d["cfg"].W, d["cfg"].K)
+                                                     for d in live])
         else:
             # fp32 per layer: the stream-K workspace plan (variant 4) is one launch; tf32: + a fixup launch
             vid = {"fp32": 4, "tf32": 6, "3xtf32": 7}[variant]  # plans with the stream-K workspaces
@@ -549,9 +537,7 @@ def main():
             if timed:
                 ftf_ev[0].record(side)
             ready = []
-            if fused_ftf:
-                ready = [None] * len(per)  # the FTFs run inside the conv launch (below)
-            elif variant == "fp32":
+            if variant == "fp32":
                 # every layer's FTF in one launch (wino_filter_transform_multi): one launch latency
                 wino.filter_transform_multi([(d["w"], d["u"]) for d in live], stream=side)
                 ev = torch.cuda.Event()
@@ -570,10 +556,7 @@ def main():
                 # shards) are queued before its wait for the FTF event, so they overlap the FTF
                 if timed:
                     multi_ev[0].record(cur)
-                if fused_ftf:
-                    wino.conv2d_multi_ftf([(d["x"], d["w"], d["u"], d["y"]) for d in live], ws_ml)
-                else:
-                    wino.conv2d_multi([(d["x"], d["u"], d["y"]) for d in live], ws_ml, u_ready=ready[0])
+                wino.conv2d_multi([(d["x"], d["u"], d["y"]) for d in live], ws_ml, u_ready=ready[0])
                 if timed:
                     multi_ev[1].record(cur)
             for d, ev, (ea, eb), ls in zip(per, ready if not multi else [], conv_ev, lstreams):
@@ -705,7 +688,6 @@ def main():
                 "ms_step_ranks": _gather_scalar(ms_step, world, dev),
                 "conv_ms": [_max_over_ranks(v, world, dev) for v in conv_ms],
                 "ftf_ms_step": _max_over_ranks(ftf_ms_step, world, dev),
-                "fused_ftf": fused_ftf,
                 "hot_ms_step": _max_over_ranks(hot_step, world, dev),
                 "hot_conv_ms": [_max_over_ranks(v, world, dev) for v in hot_conv],
                 "launches": launches, "wall": wall, "clocks": clocks, "outs": outs,
@@ -861,11 +843,8 @@ def main():
         "fp32_peak_tflops": fp32_peak, "fp32_peak_source": f"{FP32_PEAK_NOTE}; {peak_src}",
         "hot_l2": {"value": total_eff / (main_m["hot_ms_step"] * 1e-3) / 1e12, "ms_per_step": main_m["hot_ms_step"],
                    "protocol": "L863: 20 back-to-back graph replays of the step, mean; 5 repeats, median"},
-        "ftf_us_step": (main_m["ftf_ms_step"] * 1e3 if not main_m.get("fused_ftf") else
-                        "inside conv_launch: the FTFs are the prologue of the shared launch"),
-        "conv_launch": (("FTFs + all layers through one wino_conv2d_f2x3_fwd_multi_ftf call (one cooperative launch): "
-                         if main_m.get("fused_ftf") else "all layers through one wino_conv2d_f2x3_fwd_multi call: ") +
-                        f"{multi_ms * 1e3:.1f} us in "
+        "ftf_us_step": main_m["ftf_ms_step"] * 1e3,
+        "conv_launch": ("all layers through one wino_conv2d_f2x3_fwd_multi call: " + f"{multi_ms * 1e3:.1f} us in "
                         "the instrumented step; layers.*.conv_us time each layer alone (wino_conv2d_f2x3_fwd_ws, "
                         "L2 flushed)") if multi_ms else "one launch per layer (layers.*.conv_us from the step)",
         "layers_in_step": ("concurrent: one stream per layer (independent problems), each conv waits only for "
@@ -877,10 +856,6 @@ def main():
                                        "dram__bytes_write.sum of the conv launches of one step "
                                        "(profiles/traffic.json)",
                      "achieved_def": ("EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) summed over layers / the duration of "
-                                      "the wino_conv2d_f2x3_fwd_multi_ftf call (ONE cooperative launch: the FTF and "
-                                      "N = 4 / 8 input-transform prologue, then the shared persistent stream-K convolutions) "
-                                      if multi_ms and main_m.get("fused_ftf") else
-                                      "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2) summed over layers / the duration of "
                                       "the wino_conv2d_f2x3_fwd_multi call (input transforms of N = 4 / 8 shards, the wait for the FTF, "
                                       "the shared persistent stream-K launch, any layer run alone) "
                                       if multi_ms else

@@ -292,26 +292,6 @@ wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, voi
 int wino_conv_multi_launches(const wino_conv_job_t* jobs, int n);
 
 /*
- * The filter transform (Eq. 5, Sec. 3.1) and the convolutions of several layers in one
- * call: a1-a6 of a network step.  jobs[i].u is the OUTPUT here (16 x C x K floats, (C,4,4,K), as
- * wino_filter_transform writes it, bit-identical) and w[i] the layer's filter (C,3,3,K) ("CRSK",
- * Table 4), 16-byte aligned.  When every job joins ONE shared persistent launch (see
- * wino_conv2d_f2x3_fwd_multi), the filter transforms -- and the vmode input transforms -- run as a
- * prologue of that launch: each CTA transforms its share, then a grid-wide count (the launch is
- * cooperative, all CTAs resident) gates the first TMA load of u, so there is no separate FTF or
- * input-transform launch and no launch gap between them.  Otherwise it is exactly
- * wino_filter_transform_multi followed by wino_conv2d_f2x3_fwd_multi on `stream`.
- *   ws_dev / ws_bytes: as wino_conv2d_f2x3_fwd_multi (zero-filled before first use; every call
- *                      leaves its counters zero).
- * Errors as wino_conv2d_f2x3_fwd_multi, plus: w[i] NULL -> WINO_ERR_INVALID_ARG; w[i] not 16-byte
- * aligned -> WINO_ERR_MISALIGNED; u[i] overlapping any w, x, y or the workspace -> INVALID_ARG.
- * wino_conv_multi_ftf_launches: kernel launches one such call makes (1 when fused; host only).
- */
-wino_status_t wino_conv2d_f2x3_fwd_multi_ftf(const wino_conv_job_t* jobs, const float* const* w, int n, void* ws_dev,
-                                             size_t ws_bytes, wino_stream_t stream);
-int wino_conv_multi_ftf_launches(const wino_conv_job_t* jobs, int n);
-
-/*
  * Tensor-core variant (a5' of SURVEY 8(a)): the Winograd-domain GEMM (Eq. 7)
  * on the 5th-generation tensor cores (tcgen05.mma kind::tf32, accumulators in
  * TMEM).  The paper has no tensor-core path ("the data layout needs a

@@ -26,7 +26,7 @@ __all__ = [
     "filter_workspace_bytes_f4", "filter_transform_f4", "conv2d_f4",
     "filter_transform_kcrs", "conv2d_nchw", "nonfused_workspace_bytes", "conv2d_nonfused", "nonfused_launches",
     "HALF_FP16", "HALF_BF16", "HalfFilter", "filter_workspace_bytes_half", "filter_transform_half",
-    "conv2d_half", "conv_workspace_bytes", "conv2d_multi", "conv2d_multi_ftf", "conv_multi_ftf_launches", "conv_multi_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes", "filter_transform_multi",
+    "conv2d_half", "conv_workspace_bytes", "conv2d_multi", "conv_multi_workspace_bytes", "nchw_workspace_bytes", "half_workspace_bytes", "tc_workspace_bytes", "f4_workspace_bytes", "filter_transform_multi",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -180,11 +180,6 @@ def lib() -> ctypes.CDLL:
         L.wino_conv_multi_launches.argtypes = [ctypes.POINTER(_ConvJob), i]
         L.wino_conv2d_f2x3_fwd_multi.restype = i
         L.wino_conv2d_f2x3_fwd_multi.argtypes = [ctypes.POINTER(_ConvJob), i, vp, st, vp, vp]
-    if hasattr(L, "wino_conv2d_f2x3_fwd_multi_ftf") or not os.environ.get("WINO_LIB_PATH"):
-        L.wino_conv2d_f2x3_fwd_multi_ftf.restype = i
-        L.wino_conv2d_f2x3_fwd_multi_ftf.argtypes = [ctypes.POINTER(_ConvJob), ctypes.POINTER(vp), i, vp, st, vp]
-        L.wino_conv_multi_ftf_launches.restype = i
-        L.wino_conv_multi_ftf_launches.argtypes = [ctypes.POINTER(_ConvJob), i]
     if hasattr(L, "wino_conv2d_f2x3_fwd_nchw_ws") or not os.environ.get("WINO_LIB_PATH"):
         L.wino_nchw_workspace_bytes.restype = st
         L.wino_nchw_workspace_bytes.argtypes = [i, i, i, i, i]
@@ -550,37 +545,6 @@ def conv2d_multi(layers, ws: torch.Tensor, stream=None, u_ready: torch.cuda.Even
         _check(lib().wino_conv2d_f2x3_fwd_multi(arr, len(layers), ctypes.c_void_p(ws.data_ptr()),
                                                 ws.numel() * ws.element_size(), ev, _stream_ptr(stream)),
                "wino_conv2d_f2x3_fwd_multi")
-
-
-def conv_multi_ftf_launches(shapes) -> int:
-    """Kernel launches of one conv2d_multi_ftf call on [(N, C, H, W, K), ...] (1 when fused)."""
-    arr = (_ConvJob * len(shapes))()
-    for i, (N, C, H, W, K) in enumerate(shapes):
-        arr[i] = _ConvJob(None, None, None, N, C, H, W, K)
-    n = int(lib().wino_conv_multi_ftf_launches(arr, len(shapes)))
-    if n < 0:
-        raise WinoError(1, f"wino_conv_multi_ftf_launches {shapes}")
-    return n
-
-
-def conv2d_multi_ftf(layers, ws: torch.Tensor, stream=None) -> None:
-    """Filter transforms + convolutions of several layers [(x (C,H,W,N), w (C,3,3,K), u (C,4,4,K) out,
-    y (K,H,W,N) out), ...] in one call (wino_conv2d_f2x3_fwd_multi_ftf): when all layers share one
-    persistent launch, the FTFs run as its prologue (one cooperative launch); else FTF launch + conv2d_multi.
-    ws: a ZERO-FILLED CUDA byte buffer of >= conv_multi_workspace_bytes (calls leave it zeroed)."""
-    for i, (x, w, u, y) in enumerate(layers):
-        _need_cuda_f32(w, f"layer {i} w", 4)
-        C, K = w.shape[0], w.shape[3]
-        if tuple(w.shape) != (C, 3, 3, K) or tuple(u.shape) != (C, 4, 4, K):
-            raise ValueError(f"layer {i}: w (C,3,3,K), u (C,4,4,K) expected")
-        _same_device(x, w=w)
-    arr = _conv_jobs([(x, u, y) for (x, w, u, y) in layers])
-    wp = (ctypes.c_void_p * len(layers))(*[w.data_ptr() for (_, w, _, _) in layers])
-    _need_ws(ws, layers[0][0])
-    with torch.cuda.device(layers[0][0].device):
-        _check(lib().wino_conv2d_f2x3_fwd_multi_ftf(arr, wp, len(layers), ctypes.c_void_p(ws.data_ptr()),
-                                                    ws.numel() * ws.element_size(), _stream_ptr(stream)),
-               "wino_conv2d_f2x3_fwd_multi_ftf")
 
 
 def filter_transform_kcrs(w_kcrs: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:

@@ -43,9 +43,11 @@ struct FtfJobs {
     int n;
 };
 
-// Item idx of job j: 4 consecutive k (jobs.vec[j]: 9 LDG.128 + 16 STG.128) or one (c, k).
-__device__ __forceinline__ void ftf_item(const FtfJobs& jobs, int j, long idx) {
+__global__ void __launch_bounds__(FTF_THREADS) ftf_multi_kernel(const __grid_constant__ FtfJobs jobs) {
+    int j = 0;
+    while (j + 1 < jobs.n && blockIdx.x >= jobs.first[j + 1]) ++j;
     const int C = jobs.C[j], K = jobs.K[j];
+    const long idx = (long)(blockIdx.x - jobs.first[j]) * FTF_THREADS + threadIdx.x;
     if (jobs.vec[j]) {
         const int K4 = K >> 2;
         if (idx >= (long)C * K4) return;
@@ -78,38 +80,6 @@ __device__ __forceinline__ void ftf_item(const FtfJobs& jobs, int j, long idx) {
     float* uc = jobs.u[j] + (size_t)c * 16 * K + k;
 #pragma unroll
     for (int e = 0; e < 16; ++e) uc[(size_t)e * K] = t[e];
-}
-
-// The vec item split in its loads and its transform + stores, so a caller can keep several items'
-// loads in flight (the multi-layer kernel's prologue).  idx < C * K / 4 of job j (K % 4 == 0).
-__device__ __forceinline__ void ftf_load4(const FtfJobs& jobs, int j, long idx, float4 g4[9]) {
-    const int K = jobs.K[j], K4 = K >> 2;
-    const int c = (int)(idx / K4), k = 4 * (int)(idx - (long)c * K4);
-    const float* wc = jobs.w[j] + (size_t)c * 9 * K + k;
-#pragma unroll
-    for (int e = 0; e < 9; ++e) g4[e] = __ldg(reinterpret_cast<const float4*>(wc + (size_t)e * K));
-}
-__device__ __forceinline__ void ftf_store4(const FtfJobs& jobs, int j, long idx, const float4 g4[9]) {
-    const int K = jobs.K[j], K4 = K >> 2;
-    const int c = (int)(idx / K4), k = 4 * (int)(idx - (long)c * K4);
-    float t[4][16];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        float g[9];
-#pragma unroll
-        for (int e = 0; e < 9; ++e) g[e] = q == 0 ? g4[e].x : q == 1 ? g4[e].y : q == 2 ? g4[e].z : g4[e].w;
-        ftf_4x4(g, t[q]);
-    }
-    float* uc = jobs.u[j] + (size_t)c * 16 * K + k;
-#pragma unroll
-    for (int e = 0; e < 16; ++e)
-        *reinterpret_cast<float4*>(uc + (size_t)e * K) = make_float4(t[0][e], t[1][e], t[2][e], t[3][e]);
-}
-
-__global__ void __launch_bounds__(FTF_THREADS) ftf_multi_kernel(const __grid_constant__ FtfJobs jobs) {
-    int j = 0;
-    while (j + 1 < jobs.n && blockIdx.x >= jobs.first[j + 1]) ++j;
-    ftf_item(jobs, j, (long)(blockIdx.x - jobs.first[j]) * FTF_THREADS + threadIdx.x);
 }
 
 }  // namespace wino

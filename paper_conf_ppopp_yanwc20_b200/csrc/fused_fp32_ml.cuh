@@ -21,7 +21,6 @@
 
 #include <cstdint>
 
-#include "ftf.cuh"
 #include "fused_fp32_ws.cuh"
 #include "wino_ptx.cuh"
 #include "wino_transforms.cuh"
@@ -83,18 +82,6 @@ struct __align__(64) Layer {
     int itf_map[64];   // N | 32: ITF task map of the 64 ITF lanes (as fp32::Params::itf_map)
 };
 
-struct ItfJob {
-    const float* __restrict__ x;
-    float* __restrict__ v;
-    int N, C, H, W, TW, NV;
-    int first;  // first thread index of this job (C * NV / 4 threads per V row, blockIdx.y = row)
-};
-struct ItfJobs {
-    ItfJob j[MAX_LAYERS];
-    int n;
-    int total;
-};
-
 struct __align__(64) Params {
     Layer L[MAX_LAYERS];
     int nl;
@@ -103,17 +90,6 @@ struct __align__(64) Params {
     int start[MAX_GRID + 1];
     float* __restrict__ sk_ws;          // 2 partial-tile slots per CTA
     unsigned* __restrict__ sk_flags;    // one arrival counter per CTA (zero between launches)
-    // Prologue (wino_conv2d_f2x3_fwd_multi_ftf): every CTA first transforms its share of the layers'
-    // filters (Eq. 5, ftf_item) and of the vmode layers' inputs (Eq. 6, ml_itf_item), then a grid-wide
-    // count on `sync` (2 words after the arrival counters, zero between launches; the launch is
-    // cooperative, so every CTA is resident) gates the first TMA load of u / V.
-    int pro;                            // 1: run the prologue
-    int pro_ftf_total;                  // filter items (4 consecutive k, or 1 k when K % 4 != 0) of all jobs
-    int pro_vec;                        // every job has K % 4 == 0 (items of 4 k: batched loads)
-    unsigned pro_first[MAX_LAYERS + 1]; // first item of each job
-    FtfJobs ftf;
-    ItfJobs itf;                        // vmode input transforms (rows x items: 4 * itf.total)
-    unsigned* __restrict__ sync;
 };
 
 __device__ __forceinline__ int layer_of(const Params& p, int u) {
@@ -256,43 +232,52 @@ __device__ __noinline__ void ml_arrive(const Params& p, int l, int t0, int k0, i
 // consecutive nu) reads the two rows of its 4x4 patch that row r of B^T combines, as float4 along n
 // (N % 4 == 0; zero outside the image = the implicit padding of Sec. 3.5), and writes
 // V[4r..4r+3][c][nu..nu+3] as float4 -- a warp stores 512 contiguous bytes per xi.
-// V row `row` (= B^T row) of item i of the vmode input transforms (one thread's 4 consecutive nu of one c)
-__device__ __forceinline__ void ml_itf_item(const ItfJobs& p, int row, int i) {
-    const int i0 = row == 0 ? 0 : (row == 2 ? 2 : 1), i1 = row == 0 ? 2 : (row == 2 ? 1 : (row == 1 ? 2 : 3));
-    int a = 0;
-    while (a + 1 < p.n && p.j[a + 1].first <= i) ++a;
-    const ItfJob& J = p.j[a];
-    const int nq = J.NV >> 2, r = i - J.first;
-    const int c = r / nq, nu = 4 * (r - c * nq);
-    const int t = nu / J.N, n = nu - t * J.N;
-    const int th = t / J.TW, tw = t - th * J.TW;
-    const int ha = 2 * th - 1 + i0, hb = 2 * th - 1 + i1, w0 = 2 * tw - 1;
-    const float* xa = J.x + ((c * J.H + ha) * J.W + w0) * J.N + n;  // < 2^31 floats (kMaxElems)
-    const float* xb = xa + (i1 - i0) * J.W * J.N;
-    const bool oka = ha >= 0 && ha < J.H, okb = hb >= 0 && hb < J.H;
-    float4 tr[4];  // row `row` of B^T d
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const bool okw = w0 + j >= 0 && w0 + j < J.W;
-        float4 d0 = make_float4(0.f, 0.f, 0.f, 0.f), d1 = d0;
-        if (okw && oka) d0 = __ldg(reinterpret_cast<const float4*>(xa + j * J.N));
-        if (okw && okb) d1 = __ldg(reinterpret_cast<const float4*>(xb + j * J.N));
-        tr[j] = row == 1 ? make_float4(d0.x + d1.x, d0.y + d1.y, d0.z + d1.z, d0.w + d1.w)
-                         : make_float4(d0.x - d1.x, d0.y - d1.y, d0.z - d1.z, d0.w - d1.w);
-    }
-    auto sub = [](float4 u, float4 w) { return make_float4(u.x - w.x, u.y - w.y, u.z - w.z, u.w - w.w); };
-    auto add = [](float4 u, float4 w) { return make_float4(u.x + w.x, u.y + w.y, u.z + w.z, u.w + w.w); };
-    const size_t plane = static_cast<size_t>(J.C) * J.NV;
-    float* vo = J.v + 4 * row * plane + static_cast<size_t>(c) * J.NV + nu;
-    __stcg(reinterpret_cast<float4*>(vo), sub(tr[0], tr[2]));
-    __stcg(reinterpret_cast<float4*>(vo + plane), add(tr[1], tr[2]));
-    __stcg(reinterpret_cast<float4*>(vo + 2 * plane), sub(tr[2], tr[1]));
-    __stcg(reinterpret_cast<float4*>(vo + 3 * plane), sub(tr[1], tr[3]));
-}
+struct ItfJob {
+    const float* __restrict__ x;
+    float* __restrict__ v;
+    int N, C, H, W, TW, NV;
+    int first;  // first thread index of this job (C * NV / 4 threads per V row, blockIdx.y = row)
+};
+struct ItfJobs {
+    ItfJob j[MAX_LAYERS];
+    int n;
+    int total;
+};
 
 __global__ void __launch_bounds__(256) ml_itf_kernel(const __grid_constant__ ItfJobs p) {
     const int row = blockIdx.y;  // row of V = B^T row: (d[i0] - d[i1]) for rows 0, 2, 3, (d[i0] + d[i1]) for row 1
-    for (int i = blockIdx.x * 256 + threadIdx.x; i < p.total; i += gridDim.x * 256) ml_itf_item(p, row, i);
+    const int i0 = row == 0 ? 0 : (row == 2 ? 2 : 1), i1 = row == 0 ? 2 : (row == 2 ? 1 : (row == 1 ? 2 : 3));
+    for (int i = blockIdx.x * 256 + threadIdx.x; i < p.total; i += gridDim.x * 256) {
+        int a = 0;
+        while (a + 1 < p.n && p.j[a + 1].first <= i) ++a;
+        const ItfJob& J = p.j[a];
+        const int nq = J.NV >> 2, r = i - J.first;
+        const int c = r / nq, nu = 4 * (r - c * nq);
+        const int t = nu / J.N, n = nu - t * J.N;
+        const int th = t / J.TW, tw = t - th * J.TW;
+        const int ha = 2 * th - 1 + i0, hb = 2 * th - 1 + i1, w0 = 2 * tw - 1;
+        const float* xa = J.x + ((c * J.H + ha) * J.W + w0) * J.N + n;  // < 2^31 floats (kMaxElems)
+        const float* xb = xa + (i1 - i0) * J.W * J.N;
+        const bool oka = ha >= 0 && ha < J.H, okb = hb >= 0 && hb < J.H;
+        float4 tr[4];  // row `row` of B^T d
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const bool okw = w0 + j >= 0 && w0 + j < J.W;
+            float4 d0 = make_float4(0.f, 0.f, 0.f, 0.f), d1 = d0;
+            if (okw && oka) d0 = __ldg(reinterpret_cast<const float4*>(xa + j * J.N));
+            if (okw && okb) d1 = __ldg(reinterpret_cast<const float4*>(xb + j * J.N));
+            tr[j] = row == 1 ? make_float4(d0.x + d1.x, d0.y + d1.y, d0.z + d1.z, d0.w + d1.w)
+                             : make_float4(d0.x - d1.x, d0.y - d1.y, d0.z - d1.z, d0.w - d1.w);
+        }
+        auto sub = [](float4 u, float4 w) { return make_float4(u.x - w.x, u.y - w.y, u.z - w.z, u.w - w.w); };
+        auto add = [](float4 u, float4 w) { return make_float4(u.x + w.x, u.y + w.y, u.z + w.z, u.w + w.w); };
+        const size_t plane = static_cast<size_t>(J.C) * J.NV;
+        float* vo = J.v + 4 * row * plane + static_cast<size_t>(c) * J.NV + nu;
+        __stcg(reinterpret_cast<float4*>(vo), sub(tr[0], tr[2]));
+        __stcg(reinterpret_cast<float4*>(vo + plane), add(tr[1], tr[2]));
+        __stcg(reinterpret_cast<float4*>(vo + 2 * plane), sub(tr[2], tr[1]));
+        __stcg(reinterpret_cast<float4*>(vo + 3 * plane), sub(tr[1], tr[3]));
+    }
 }
 
 #ifdef WINO_WS_CTATRACE
@@ -337,47 +322,6 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
         fence_mbar_init();
     }
     __syncthreads();
-    if (p.pro) {
-        // ---- prologue (wino_conv2d_f2x3_fwd_multi_ftf): this CTA's share of every layer's filter
-        // transform (Eq. 5; the items of ftf_multi_kernel, bit-identical) and of the vmode layers'
-        // input transforms (Eq. 6), then count the CTA on the grid-wide barrier word ----
-        const int gstride = static_cast<int>(gridDim.x) * NT, g0 = static_cast<int>(blockIdx.x) * NT + tid;
-        auto job_of = [&](int i) {
-            int j = 0;
-            while (j + 1 < p.ftf.n && static_cast<unsigned>(i) >= p.pro_first[j + 1]) ++j;
-            return j;
-        };
-        if (p.pro_vec) {  // every job has K % 4 == 0: PRO_B items' loads in flight per thread
-            constexpr int PRO_B = 3;
-            for (int i0 = g0; i0 < p.pro_ftf_total; i0 += PRO_B * gstride) {
-                float4 g4[PRO_B][9];
-                int jb[PRO_B];
-#pragma unroll
-                for (int b = 0; b < PRO_B; ++b) {
-                    const int i = i0 + b * gstride;
-                    jb[b] = job_of(i);
-                    if (i < p.pro_ftf_total) ftf_load4(p.ftf, jb[b], static_cast<long>(i) - p.pro_first[jb[b]], g4[b]);
-                }
-#pragma unroll
-                for (int b = 0; b < PRO_B; ++b) {
-                    const int i = i0 + b * gstride;
-                    if (i < p.pro_ftf_total) ftf_store4(p.ftf, jb[b], static_cast<long>(i) - p.pro_first[jb[b]], g4[b]);
-                }
-            }
-        } else {
-            for (int i = g0; i < p.pro_ftf_total; i += gstride) {
-                const int j = job_of(i);
-                ftf_item(p.ftf, j, static_cast<long>(i) - static_cast<long>(p.pro_first[j]));
-            }
-        }
-        for (int i = g0; i < 4 * p.itf.total; i += gstride) {
-            const int row = i / p.itf.total;
-            ml_itf_item(p.itf, row, i - row * p.itf.total);
-        }
-        fence_proxy_async_global();  // these generic stores before the async-proxy (TMA) reads of u / V
-        __syncthreads();
-        if (tid == 0) red_add_release_gpu(p.sync, 1u);
-    }
 
     if (warp >= 8) {
         // ============================ producer / ITF ============================
@@ -388,15 +332,6 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                 constexpr uint32_t kBytes = (US_FLOATS + XS_FLOATS) * 4;
                 // L2 priority: u is re-read by every tile of its layer (y is stored with .cs)
                 const uint64_t pol_keep = l2_policy_evict_last();
-                if (p.pro) {  // every CTA's prologue is done: u (and V) are complete in global memory
-                    while (ld_acquire_gpu(p.sync) < gridDim.x) {
-                    }
-                    fence_proxy_async_global();
-                    if (atom_add_relaxed_gpu(p.sync + 1, 1u) == gridDim.x - 1) {  // the last CTA past the wait
-                        p.sync[0] = 0u;                                           // resets both words
-                        p.sync[1] = 0u;
-                    }
-                }
                 int G = 0;
                 int l, u0, u1;
                 for (int pi = 0; ml_piece(p, blockIdx.x, pi, l, u0, u1); ++pi) {

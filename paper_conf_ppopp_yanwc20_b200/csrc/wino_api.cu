@@ -145,8 +145,7 @@ struct Fp32Plan {
 // Stream-K workspace: 2 partial-tile slots (64 k x 4 outputs x 32 nu fp32) per CTA, then one
 // arrival counter per CTA (zero between launches; see fused_fp32_ws.cuh).
 size_t sk_slot_bytes() { return size_t(wino::fp32::BK) * 4 * wino::fp32::BN * sizeof(float); }
-// slots, one arrival counter per CTA, and 2 words for the multi-layer prologue's grid-wide count
-size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * sk_slot_bytes() + round_up256(size_t(ctas) * 4 + 8); }
+size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * sk_slot_bytes() + round_up256(size_t(ctas) * 4); }
 // The arrival counters sit after the slots of a FULL grid (one CTA per SM) whatever the grid of a
 // launch: a smaller grid's counters would otherwise land on slots that an earlier launch on the
 // same workspace left non-zero.
@@ -952,59 +951,16 @@ wino_status_t launch_ml(const MlLaunch& L, int dev, cudaStream_t st) {
     const int smem = wino::fp32ml::SMEM_BYTES;
     wino_status_t s = ensure_smem_attr(wino::fp32ml::fused_fp32_ml_kernel, dev, smem, g_attr_ml);
     if (s != WINO_OK) return s;
-    if (!L.prm.pro) {
-        wino::fp32ml::fused_fp32_ml_kernel<<<dim3(static_cast<unsigned>(L.grid)), wino::fp32ws::NT, smem, st>>>(L.prm);
-    } else {  // the prologue's grid-wide count needs every CTA resident: cooperative launch
-        cudaLaunchConfig_t cfg = {};
-        cfg.gridDim = dim3(static_cast<unsigned>(L.grid));
-        cfg.blockDim = dim3(wino::fp32ws::NT);
-        cfg.dynamicSmemBytes = static_cast<size_t>(smem);
-        cfg.stream = st;
-        cudaLaunchAttribute attr[1];
-        attr[0].id = cudaLaunchAttributeCooperative;
-        attr[0].val.cooperative = 1;
-        cfg.attrs = attr;
-        cfg.numAttrs = 1;
-        cudaError_t e = cudaLaunchKernelEx(&cfg, wino::fp32ml::fused_fp32_ml_kernel, L.prm);
-        if (e != cudaSuccess) return cuda_fail(e);
-    }
+    wino::fp32ml::fused_fp32_ml_kernel<<<dim3(static_cast<unsigned>(L.grid)), wino::fp32ws::NT, smem, st>>>(L.prm);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? WINO_OK : cuda_fail(e);
-}
-// The fused form of wino_conv2d_f2x3_fwd_multi_ftf: every job in one shared launch, whose prologue
-// runs the filter transforms (and the vmode input transforms, instead of ml_itf_kernel).
-bool ml_fuse_prologue(MlLaunch& L, const wino_conv_job_t* jobs, const float* const* w, int n, void* ws, int dev) {
-    using namespace wino::fp32ml;
-    Params& prm = L.prm;
-    long long items = 0;
-    prm.ftf.n = n;
-    for (int i = 0; i < n; ++i) {
-        prm.ftf.w[i] = w[i];
-        prm.ftf.u[i] = const_cast<float*>(jobs[i].u);
-        prm.ftf.C[i] = jobs[i].C;
-        prm.ftf.K[i] = jobs[i].K;
-        prm.ftf.vec[i] = jobs[i].K % 4 == 0 ? 1 : 0;
-        prm.pro_first[i] = static_cast<unsigned>(items);
-        items += int64_t(jobs[i].C) * (prm.ftf.vec[i] ? jobs[i].K / 4 : jobs[i].K);
-    }
-    if (items + 4LL * L.itf.total > 0x7fffffffLL - int64_t(L.grid) * wino::fp32ws::NT) return false;
-    prm.pro_first[n] = static_cast<unsigned>(items);
-    prm.pro_vec = 1;
-    for (int i = 0; i < n; ++i) prm.pro_vec &= prm.ftf.vec[i];
-    prm.pro_ftf_total = static_cast<int>(items);
-    prm.itf = L.itf;
-    prm.sync = sk_flags_of(ws, dev) + sm_count(dev);
-    prm.pro = 1;
-    return true;
 }
 }  // namespace
 
 extern "C" {
 
-}  // extern "C"
-namespace {
-// argument checks of wino_conv2d_f2x3_fwd_multi (and _ftf); the device on success
-wino_status_t validate_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, size_t ws_bytes, int* dev_out) {
+wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, size_t ws_bytes,
+                                         void* u_ready, wino_stream_t stream) {
     if (!jobs || n <= 0 || !ws_dev) return WINO_ERR_INVALID_ARG;
     if (!aligned16(ws_dev)) return WINO_ERR_MISALIGNED;
     for (int i = 0; i < n; ++i) {
@@ -1034,18 +990,6 @@ wino_status_t validate_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, s
     if (s != WINO_OK) return s;
     const int sms = sm_count(dev);
     if (ws_bytes < ml_multi_ws_bytes(jobs, n, sms)) return WINO_ERR_INVALID_ARG;
-    *dev_out = dev;
-    return WINO_OK;
-}
-}  // namespace
-extern "C" {
-
-wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, void* ws_dev, size_t ws_bytes,
-                                         void* u_ready, wino_stream_t stream) {
-    int dev;
-    wino_status_t s = validate_multi(jobs, n, ws_dev, ws_bytes, &dev);
-    if (s != WINO_OK) return s;
-    const int sms = sm_count(dev);
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     // 1. plan every shared launch (groups of <= 4 in job order); the other jobs run alone
     wino_conv_job_t group[wino::fp32ml::MAX_LAYERS];
@@ -1089,74 +1033,6 @@ wino_status_t wino_conv2d_f2x3_fwd_multi(const wino_conv_job_t* jobs, int n, voi
             return s;
     }
     return WINO_OK;
-}
-
-namespace {
-// every job of a _ftf call joins one shared launch (then its prologue runs the transforms)
-bool ml_ftf_fusable(const wino_conv_job_t* jobs, int n, int sms) {
-    if (n > wino::fp32ml::MAX_LAYERS) return false;
-    for (int i = 0; i < n; ++i)
-        if (!ml_shares_launch(jobs[i], sms)) return false;
-    return true;
-}
-}  // namespace
-
-wino_status_t wino_conv2d_f2x3_fwd_multi_ftf(const wino_conv_job_t* jobs, const float* const* w, int n, void* ws_dev,
-                                             size_t ws_bytes, wino_stream_t stream) {
-    if (!jobs || !w || n <= 0) return WINO_ERR_INVALID_ARG;
-    for (int i = 0; i < n; ++i) {  // w[i] in, u[i] out: u overlaps no input, no other output, no workspace
-        const wino_conv_job_t& A = jobs[i];
-        if (!w[i] || !A.u) return WINO_ERR_INVALID_ARG;
-        if (A.C <= 0 || A.K <= 0) return WINO_ERR_INVALID_ARG;
-        if (int64_t(16) * A.C * A.K > kMaxElems) return WINO_ERR_TOO_LARGE;
-        if (!aligned16(w[i])) return WINO_ERR_MISALIGNED;
-        const size_t ub = size_t(16) * A.C * A.K * 4;
-        if (overlaps(A.u, ub, ws_dev, ws_bytes)) return WINO_ERR_INVALID_ARG;
-        for (int j = 0; j < n; ++j) {
-            const wino_conv_job_t& B = jobs[j];
-            if (B.C <= 0 || B.K <= 0 || B.N <= 0 || B.H <= 0 || B.W <= 0) continue;  // reported below
-            const size_t hwn_b = size_t(B.H) * B.W * B.N;
-            if (overlaps(A.u, ub, w[j], size_t(9) * B.C * B.K * 4) || (B.x && overlaps(A.u, ub, B.x, size_t(B.C) * hwn_b * 4)))
-                return WINO_ERR_INVALID_ARG;
-            if (j != i && B.u && overlaps(A.u, ub, B.u, size_t(16) * B.C * B.K * 4)) return WINO_ERR_INVALID_ARG;
-        }
-    }
-    int dev;
-    wino_status_t s = validate_multi(jobs, n, ws_dev, ws_bytes, &dev);
-    if (s != WINO_OK) return s;
-    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    if (!ml_ftf_fusable(jobs, n, sm_count(dev))) {  // wino_filter_transform_multi + wino_conv2d_f2x3_fwd_multi
-        for (int i0 = 0; i0 < n; i0 += wino::FTF_MAX_JOBS) {
-            wino_ftf_job_t fj[wino::FTF_MAX_JOBS];
-            const int m = n - i0 < wino::FTF_MAX_JOBS ? n - i0 : wino::FTF_MAX_JOBS;
-            for (int k = 0; k < m; ++k) fj[k] = wino_ftf_job_t{w[i0 + k], const_cast<float*>(jobs[i0 + k].u), jobs[i0 + k].C, jobs[i0 + k].K};
-            if ((s = wino_filter_transform_multi(fj, m, stream)) != WINO_OK) return s;
-        }
-        return wino_conv2d_f2x3_fwd_multi(jobs, n, ws_dev, ws_bytes, nullptr, stream);
-    }
-    float* vbuf[wino::fp32ml::MAX_LAYERS];
-    char* vnext = static_cast<char*>(ws_dev) + sk_workspace_bytes(sm_count(dev));
-    for (int i = 0; i < n; ++i) {
-        vbuf[i] = nullptr;
-        if (ml_vmode(jobs[i])) {
-            vbuf[i] = reinterpret_cast<float*>(vnext);
-            vnext += ml_v_bytes(jobs[i]);
-        }
-    }
-    MlLaunch L;
-    if ((s = prepare_multi_fp32(jobs, vbuf, n, ws_dev, dev, L)) != WINO_OK) return s;
-    if (!ml_fuse_prologue(L, jobs, w, n, ws_dev, dev)) return WINO_ERR_TOO_LARGE;
-    return launch_ml(L, dev, st);
-}
-
-int wino_conv_multi_ftf_launches(const wino_conv_job_t* jobs, int n) {
-    if (!jobs || n <= 0) return -1;
-    int dev = -1, sms = 148;
-    if (check_device(&dev) == WINO_OK) sms = sm_count(dev);
-    else cudaGetLastError();
-    if (ml_ftf_fusable(jobs, n, sms)) return 1;
-    const int m = wino_conv_multi_launches(jobs, n);
-    return m < 0 ? -1 : m + (n + wino::FTF_MAX_JOBS - 1) / wino::FTF_MAX_JOBS;
 }
 
 int wino_conv_multi_launches(const wino_conv_job_t* jobs, int n) {

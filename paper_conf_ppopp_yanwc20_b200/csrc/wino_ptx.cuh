@@ -285,22 +285,6 @@ __device__ __forceinline__ unsigned atom_add_acq_rel_gpu(unsigned* p, unsigned v
     asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;\n" : "=r"(old) : "l"(p), "r"(v) : "memory");
     return old;
 }
-// grid-wide hand-off of data written with generic stores and read by TMA on other SMs: writer side
-// fence.proxy.async (generic -> async proxy) + release add, reader side acquire load + fence.proxy.async
-__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;\n" ::: "memory"); }
-__device__ __forceinline__ void red_add_release_gpu(unsigned* p, unsigned v) {
-    asm volatile("red.release.gpu.global.add.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
-    unsigned v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ unsigned atom_add_relaxed_gpu(unsigned* p, unsigned v) {
-    unsigned old;
-    asm volatile("atom.relaxed.gpu.global.add.u32 %0, [%1], %2;\n" : "=r"(old) : "l"(p), "r"(v) : "memory");
-    return old;
-}
 // Asynchronous 16 B store into (possibly another CTA's) shared memory; completion is
 // counted in bytes on an mbarrier of the destination CTA (complete_tx).
 __device__ __forceinline__ void st_async4(uint32_t cluster_addr, float a, float b, float c, float d,

@@ -48,19 +48,16 @@ for cfg in shapes:
         for dt in (torch.float16, torch.bfloat16):
             y = wino.conv2d_half(x.to(dt), wino.filter_transform_half(w.to(dt)))
 if only in ("all", "fp32", "ml"):
-    # multi-layer persistent launch (fused_fp32_ml.cuh): N % 32 == 0, N = 16 boxes and vmode N = 4 / 8 in one
-    # launch, with and without the cooperative FTF / input-transform prologue (wino_conv2d_f2x3_fwd_multi_ftf)
+    # multi-layer persistent launch (fused_fp32_ml.cuh): N % 32 == 0, N = 16 boxes and vmode N = 4 / 8 in one launch
     cfgs = [Conv3x3Config("m1", 32, 16, 64, 6, 6), Conv3x3Config("m2", 16, 24, 40, 7, 9),
             Conv3x3Config("m3", 4, 40, 72, 7, 7), Conv3x3Config("m4", 8, 8, 16, 5, 5)]
-    lay, lay_w = [], []
+    lay = []
     for c in cfgs:
         x, w = make_inputs(c)
         x, w = x.cuda(), w.cuda()
         lay.append((x, wino.filter_transform(w), torch.empty((c.K, c.H, c.W, c.N), device="cuda")))
-        lay_w.append((x, w, torch.empty((c.C, 4, 4, c.K), device="cuda"), torch.empty((c.K, c.H, c.W, c.N), device="cuda")))
     ws = torch.zeros(wino.conv_multi_workspace_bytes([(c.N, c.C, c.H, c.W, c.K) for c in cfgs]), dtype=torch.uint8,
                      device="cuda")
     wino.conv2d_multi(lay, ws)
-    wino.conv2d_multi_ftf(lay_w, ws)
 torch.cuda.synchronize()
 print("ok")
