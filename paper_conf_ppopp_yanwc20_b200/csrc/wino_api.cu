@@ -10,6 +10,8 @@
 #include <atomic>
 #include <cmath>
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -768,9 +770,23 @@ std::atomic<uint64_t> g_attr_ml;
 // (scripts/ml_trace.py): small-N box modes move x in 32/N boxes of N-float rows
 // (N = 16 / 8 / 4: 1.07 / 1.31 / 1.65 blocks), vmode layers skip the raw-x staging and the ITF
 // (0.93), and each tile's 4-round OTF epilogue costs ~1.65 blocks (~2.5 us).
-constexpr double kMlEpiCost = 1.65;
+// Costs in channel-block times: [0] epilogue per tile, [1] vmode unit, [2..4] N = 16 / 8 / 4 x-box units.
+// WINO_ML_COSTS="e,v,n16,n8,n4" overrides them (A/B of the work model only, scripts/gpu.sh; read once).
+struct MlCosts {
+    double c[5] = {1.65, 0.93, 1.07, 1.31, 1.65};
+    MlCosts() {
+        if (const char* e = std::getenv("WINO_ML_COSTS"))
+            std::sscanf(e, "%lf,%lf,%lf,%lf,%lf", &c[0], &c[1], &c[2], &c[3], &c[4]);
+    }
+};
+const MlCosts& ml_costs() {
+    static const MlCosts m;
+    return m;
+}
+double ml_epi_cost() { return ml_costs().c[0]; }
 double ml_unit_cost(int xnb, bool vmode) {
-    return vmode ? 0.93 : (xnb >= 32 ? 1.0 : (xnb == 16 ? 1.07 : (xnb == 8 ? 1.31 : 1.65)));
+    const double* c = ml_costs().c;
+    return vmode ? c[1] : (xnb >= 32 ? 1.0 : (xnb == 16 ? c[2] : (xnb == 8 ? c[3] : c[4])));
 }
 // A job joins the shared persistent launch when the warp-specialised kernel takes it (N % 32 == 0
 // or N in {4, 8, 16}; K % 4 == 0) and it has fewer than 64 tiles per SM; a layer that big fills
@@ -859,7 +875,7 @@ wino_status_t prepare_multi_fp32(const wino_conv_job_t* jobs, float* const* vbuf
         units += tiles * L.num_it;
         L.vmode = ml_vmode(J) ? 1 : 0;
         cu[i] = ml_unit_cost(L.xnb, L.vmode);
-        per_tile[i] = L.num_it * cu[i] + kMlEpiCost;
+        per_tile[i] = L.num_it * cu[i] + ml_epi_cost();
         work0[i + 1] = work0[i] + tiles * per_tile[i];
         if (L.vmode) {  // V[xi][c][nu] from ml_itf_kernel: (NV, C, 16) box (32, 8, 16) = the V ring slot
             ItfJob& T = itf.j[itf.n++];
