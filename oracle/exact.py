@@ -82,23 +82,57 @@ def count_otf_adds():
     return 4 * count_adds_linear_map(AT) + 2 * count_adds_linear_map(AT)
 
 
-def count_ftf_instructions():
-    """G g G^T: G applied to 3 column vectors of g, then to 4 row vectors of (G g).
+class _Counted:
+    """A Fraction that counts the float instructions (FADD / FMUL / FFMA) spent on it."""
+    ops = 0
 
-    Per 3-vector (a, b, c) the rows of G need: row 0 -> a (0 instr), row 3 -> c
-    (0 instr), rows 1,2 -> 0.5(a+c) +- 0.5 b = t +- 0.5 b with t = 0.5*(a+c):
-    one FADD, one FMUL, two FFMA = 4 instructions whenever G has exactly two
-    dense rows whose coefficients share |0.5| and the same a/c part.  The count
-    is derived from G's structure below, not hard-coded.
-    """
-    dense_rows = [row for row in G if sum(1 for x in row if x != 0) == 3]
-    # rows 1 and 2 must share the outer coefficients and differ only by the sign
-    # of the middle one for the 4-instruction schedule to exist
-    assert len(dense_rows) == 2
-    r1, r2 = dense_rows
-    assert r1[0] == r2[0] and r1[2] == r2[2] and r1[0] == r1[2] and r1[1] == -r2[1]
-    per_vector = 4  # t=a+c; t*=|g|; r1=fma(+g1,b,t); r2=fma(-g1,b,t)
-    return per_vector * (3 + 4)
+    def __init__(self, v):
+        self.v = Fr(v)
+
+    def __add__(self, o):
+        _Counted.ops += 1
+        return _Counted(self.v + o.v)
+
+    def __sub__(self, o):
+        _Counted.ops += 1
+        return _Counted(self.v - o.v)
+
+    def scale(self, k):  # FMUL by a constant
+        _Counted.ops += 1
+        return _Counted(k * self.v)
+
+    def fma(self, k, c):  # FFMA: k * self + c in one instruction
+        _Counted.ops += 1
+        return _Counted(k * self.v + c.v)
+
+
+def _g_vector_schedule(a, b, c):
+    """G applied to one 3-vector (a, b, c) with the cheapest schedule G's structure allows: rows 0 and 3
+    of G copy a and c (0 instructions); rows 1 and 2 are 0.5 (a + c) +- 0.5 b = h +- 0.5 b with
+    h = 0.5 (a + c): FADD, FMUL, 2 FFMA."""
+    h = (a + c).scale(Fr(1, 2))
+    return [a, b.fma(Fr(1, 2), h), b.fma(Fr(-1, 2), h), c]
+
+
+def ftf_counted(g):
+    """G g G^T (Eq. 5) through _g_vector_schedule on the 3 columns of g, then on the 4 rows of G g;
+    returns (u as Fractions, float instructions used)."""
+    _Counted.ops = 0
+    gc = [[_Counted(g[r][s]) for s in range(3)] for r in range(3)]
+    cols = [_g_vector_schedule(gc[0][s], gc[1][s], gc[2][s]) for s in range(3)]  # (G g)[:, s]
+    t = [[cols[s][r] for s in range(3)] for r in range(4)]                          # G g, 4 x 3
+    u = [_g_vector_schedule(*t[r]) for r in range(4)]                                # (G g) G^T
+    return [[u[r][s].v for s in range(4)] for r in range(4)], _Counted.ops
+
+
+def count_ftf_instructions():
+    """Float instructions of the FTF (L115 prints 28): counted by executing the schedule on a tile and
+    checking that the schedule really computes G g G^T (an exact product with G from Eq. 3), so that a
+    wrong or more expensive schedule fails the pin."""
+    g = [[Fr(3, 7), Fr(-2), Fr(5, 3)], [Fr(1, 9), Fr(4), Fr(-6, 5)], [Fr(7), Fr(-1, 4), Fr(2, 11)]]
+    u, ops = ftf_counted(g)
+    assert u == ftf(g), "counted FTF schedule does not compute G g G^T"
+    return ops
 
 
 def correlate_tile(d, g):
