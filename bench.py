@@ -196,6 +196,20 @@ def _ewmm_flops(c, variant):
     return 32 * c.K * c.C * c.N * c.tiles
 
 
+def _nonfused_bytes(c, n, planes):
+    """Bytes the non-fused method must move for one layer of batch n (Sec. 9): x read, the
+    Winograd-domain input V = 16 x C x NV written by the ITF and read by the GEMMs, U (16 x K x C) read,
+    the Winograd-domain output M = 16 x K x NV written by the GEMMs and read by the OTF, y written."""
+    nv = n * ((c.H + 1) // 2) * ((c.W + 1) // 2)
+    c4 = (c.C + 3) // 4 * 4
+    x = c.C * c.H * c.W * n * 4
+    y = c.K * c.H * c.W * n * 4
+    v = planes * 16 * c4 * nv * 4
+    u = planes * 16 * c.K * c4 * 4
+    m_ = 16 * c.K * nv * 4
+    return x + 2 * v + u + 2 * m_ + y
+
+
 def _coll_device(device):
     """Scalars for the timing / error reductions live on the GPU for NCCL, on the host for gloo."""
     return device if dist.get_backend() == "nccl" else torch.device("cpu")
@@ -905,7 +919,22 @@ def main():
                                    "frac": ach / fp32_peak,
                                    "achieved_def": ("F(4x4) EWMM flops 72*K*C*N*ceil(H/4)*ceil(W/4)" if v == "f4_fp32"
                                                     else "EWMM flops 32*K*C*N*ceil(H/2)*ceil(W/2)") + " / conv time"}
-        if v in ("tf32", "3xtf32", "nonfused_tf32", "nonfused_fp32"):
+        if v in ("nonfused_tf32", "nonfused_fp32"):
+            # the non-fused method moves its Winograd-domain operands through HBM (Sec. 9, Sec. 8.1
+            # cost model): its roofline is the bytes it must move, not the tensor pipe (its GEMM runs at
+            # the HBM rate, profiles/r02_nonfused_launches.csv)
+            pp = 2 if v == "nonfused_fp32" else 1  # 3xTF32: big + small planes of V and U
+            byt = sum(_nonfused_bytes(d["cfg"], d["n"], pp) for d in live)
+            ach_b = byt / (sum(m["conv_ms"]) * 1e-3) / 1e9
+            ach = sum(_ewmm_flops(d["cfg"], v) for d in live) / (sum(m["conv_ms"]) * 1e-3) / 1e12
+            vrep[v]["roofline"] = {"bound": "hbm", "achieved": ach_b, "peak": hbm_peak, "unit": "GB/s",
+                                   "frac": ach_b / hbm_peak,
+                                   "achieved_def": "algorithmic bytes of the non-fused method per step: x read, V "
+                                                   "written and read, U read, M written and read, y written "
+                                                   "(V, U with 2 planes for 3xTF32) / conv time (ITF + GEMM + OTF)",
+                                   "peak_def": "MEASURED_PEAKS hbm_gbs",
+                                   "tensor_frac": ach * (3 if pp == 2 else 1) / tf32_peak}
+        if v in ("tf32", "3xtf32"):
             ach = sum(_ewmm_flops(d["cfg"], v) for d in live) / (sum(m["conv_ms"]) * 1e-3) / 1e12
             mult = 3 if v in ("3xtf32", "nonfused_fp32") else 1
             vrep[v]["roofline"] = {"bound": "tensor", "achieved": ach * mult, "peak": tf32_peak,
