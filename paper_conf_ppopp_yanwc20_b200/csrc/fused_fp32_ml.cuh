@@ -90,6 +90,12 @@ struct __align__(64) Params {
     int start[MAX_GRID + 1];
     float* __restrict__ sk_ws;          // 2 partial-tile slots per CTA
     unsigned* __restrict__ sk_flags;    // one arrival counter per CTA (zero between launches)
+    // Dynamic tail: units [start[grid], start[grid] + dyn_n * dyn_nu) are dyn_n whole tiles of the last
+    // layer that the producers grab one at a time from dyn_ctr[0] after their static range (per-CTA
+    // speed differences -- DRAM latency, cut tiles -- no longer set the launch's tail); dyn_ctr[1]
+    // counts the producers done, the last one resets both words (zero between launches).
+    int dyn_n, dyn_nu;
+    unsigned* __restrict__ dyn_ctr;
 };
 
 __device__ __forceinline__ int layer_of(const Params& p, int u) {
@@ -334,7 +340,27 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
                 const uint64_t pol_keep = l2_policy_evict_last();
                 int G = 0;
                 int l, u0, u1;
-                for (int pi = 0; ml_piece(p, blockIdx.x, pi, l, u0, u1); ++pi) {
+                bool dyn = false;  // past the static range: grabbing whole tiles of the dynamic tail
+                for (int pi = 0;; ++pi) {
+                    if (!dyn && !ml_piece(p, blockIdx.x, pi, l, u0, u1)) dyn = true;
+                    if (dyn) {
+                        const unsigned t = p.dyn_n > 0 ? atomicAdd(p.dyn_ctr, 1u) : 0u;
+                        if (static_cast<int>(t) >= p.dyn_n) {
+                            if (p.dyn_n > 0 && atomicAdd(p.dyn_ctr + 1, 1u) == gridDim.x - 1) {
+                                p.dyn_ctr[0] = 0u;  // every producer made its last grab: reset for the next call
+                                p.dyn_ctr[1] = 0u;
+                            }
+                            // terminal record, published through one empty stage: the consumers stop
+                            const int slot = G % S;
+                            if (G >= S) mbar_wait(&empty[slot], ((G / S) - 1) & 1);
+                            rec[pi % PR].l = -1;
+                            mbar_arrive(&full[slot]);
+                            break;
+                        }
+                        l = p.nl - 1;
+                        u0 = p.start[gridDim.x] + static_cast<int>(t) * p.dyn_nu;
+                        u1 = u0 + p.dyn_nu;
+                    }
                     const Layer& L = p.L[l];
                     const int lu = u0 - L.unit0;
                     const int tile = lu / L.num_it, g_lo = lu - tile * L.num_it, g_hi = g_lo + (u1 - u0);
@@ -397,9 +423,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
         // lane map per layer: N % 32 == 0 -> (c = 4 (w - 9) + lane / 8, nu4 = lane % 8) on [c][pos][n];
         // N | 32 -> the host-computed conflict-free map of fp32::Params::itf_map on [box][pos][c][n]
         int G = 0;
-        const int total = p.start[blockIdx.x + 1] - p.start[blockIdx.x];
-        for (int pi = 0; G < total; ++pi) {
+        for (int pi = 0;; ++pi) {
             mbar_wait(&full[G % S], (G / S) & 1);  // the segment's first stage: its record is published
+            if (rec[pi % PR].l < 0) break;         // terminal record (no stage behind it)
             const int u0 = rec[pi % PR].u0, u1 = rec[pi % PR].u1;
             const Layer& L = p.L[rec[pi % PR].l];
             if (L.vmode) {  // no raw x: only keep the stage hand-off (the producer waits on our arrival)
@@ -477,8 +503,9 @@ __global__ void __launch_bounds__(NT, 1) fused_fp32_ml_kernel(const __grid_const
     };
 
     int G = 0;
-    for (int pi = 0; G < p.start[blockIdx.x + 1] - p.start[blockIdx.x]; ++pi) {
+    for (int pi = 0;; ++pi) {
         mbar_wait(&full[G % S], (G / S) & 1);  // the segment's first stage: its record is published
+        if (rec[pi % PR].l < 0) break;         // terminal record (no stage behind it)
         const int nst = rec[pi % PR].u1 - rec[pi % PR].u0;
 #ifdef WINO_WS_CTATRACE
         if (tid == 0) { ML_PT(pi, 0, fp32ws::gtimer()); ML_PT(pi, 3, nst); }

@@ -147,7 +147,8 @@ struct Fp32Plan {
 // Stream-K workspace: 2 partial-tile slots (64 k x 4 outputs x 32 nu fp32) per CTA, then one
 // arrival counter per CTA (zero between launches; see fused_fp32_ws.cuh).
 size_t sk_slot_bytes() { return size_t(wino::fp32::BK) * 4 * wino::fp32::BN * sizeof(float); }
-size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * sk_slot_bytes() + round_up256(size_t(ctas) * 4); }
+// slots, one arrival counter per CTA, and 2 words for the multi-layer launch's dynamic tail (dyn_ctr)
+size_t sk_workspace_bytes(int ctas) { return size_t(ctas) * 2 * sk_slot_bytes() + round_up256(size_t(ctas) * 4 + 8); }
 // The arrival counters sit after the slots of a FULL grid (one CTA per SM) whatever the grid of a
 // launch: a smaller grid's counters would otherwise land on slots that an earlier launch on the
 // same workspace left non-zero.
@@ -918,10 +919,27 @@ wino_status_t prepare_multi_fp32(const wino_conv_job_t* jobs, float* const* vbuf
     }
     if (units >= 2147483647LL) return WINO_ERR_TOO_LARGE;
     // one CTA per SM; CTA b starts at the first unit whose work position reaches b / grid of the
-    // total, then pushed up so that every range is non-empty
+    // static total, then pushed up so that every range is non-empty.  The last ~6 % of the work --
+    // whole tiles of the last layer -- is the dynamic tail the CTAs grab after their static ranges.
     const int sms = sm_count(dev) < MAX_GRID ? sm_count(dev) : MAX_GRID;
     const int grid = units < sms ? static_cast<int>(units) : sms;
-    const double total = work0[n];
+    long long dyn = 0;
+    {
+        static const double frac = [] {
+            const char* e = std::getenv("WINO_ML_DYN");  // A/B of the tail fraction (0: off)
+            return e ? std::atof(e) : 0.08;
+        }();
+        const Layer& Lz = prm.L[n - 1];
+        const long long tiles_z = static_cast<long long>((Lz.NV + BN - 1) / BN) * Lz.num_kb;
+        dyn = static_cast<long long>(frac * work0[n] / per_tile[n - 1]);
+        if (dyn > tiles_z - 1) dyn = tiles_z - 1;
+        if (units - dyn * Lz.num_it < 2LL * grid) dyn = 0;  // keep every static range at >= 2 units
+        // a tail pays only when each CTA can grab a few tiles of it (P = 8 shard, 0.6 tile per CTA at
+        // 6 %: 176 vs 171 us; the P = 1 step with ~6 tiles per CTA: 1128 vs 1139 us, scripts: DESIGN 7.11)
+        if (dyn < 3LL * grid) dyn = 0;
+    }
+    const long long units_static = units - dyn * prm.L[n - 1].num_it;
+    const double total = work0[n] - dyn * per_tile[n - 1];
     for (int i = 0; i < n; ++i) {  // nu-tile order (ml_nu_tile): the CTAs' shares of each layer
         Layer& L = prm.L[i];
         const int ng = (L.NV + BN - 1) / BN;
@@ -932,7 +950,7 @@ wino_status_t prepare_multi_fp32(const wino_conv_job_t* jobs, float* const* vbuf
         L.vlc = ng - (L.vg - 1) * L.vr;
     }
     for (int b = 0; b <= grid; ++b) {
-        long long u = static_cast<long long>(units);
+        long long u = units_static;
         if (b < grid) {
             const double w = total * b / grid;
             int i = 0;
@@ -946,11 +964,14 @@ wino_status_t prepare_multi_fp32(const wino_conv_job_t* jobs, float* const* vbuf
             u = L.unit0 + tile * L.num_it + g;
         }
         if (b > 0 && u <= prm.start[b - 1]) u = prm.start[b - 1] + 1;  // non-empty ranges
-        if (u > static_cast<long long>(units) - (grid - b)) u = static_cast<long long>(units) - (grid - b);
+        if (u > units_static - (grid - b)) u = units_static - (grid - b);
         prm.start[b] = static_cast<int>(u);
     }
     prm.sk_ws = static_cast<float*>(ws);
     prm.sk_flags = sk_flags_of(ws, dev);
+    prm.dyn_n = static_cast<int>(dyn);
+    prm.dyn_nu = prm.L[n - 1].num_it;
+    prm.dyn_ctr = sk_flags_of(ws, dev) + sm_count(dev);
     out.grid = grid;
     return WINO_OK;
 }

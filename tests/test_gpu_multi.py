@@ -105,6 +105,8 @@ def test_deterministic_and_counters_zero(wino):
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     slot = 64 * 4 * 32 * 4
     assert int(ws[2 * sms * slot: 2 * sms * slot + 4 * sms].count_nonzero()) == 0
+    # the dynamic tail's grab / done counters (2 words after the arrival counters) are reset too
+    assert int(ws[2 * sms * slot + 4 * sms: 2 * sms * slot + 4 * sms + 8].count_nonzero()) == 0
 
 
 def test_matches_single_layer_calls(wino):
