@@ -77,6 +77,7 @@ struct __align__(64) Layer {
     int N, C, H, W, K;
     int TW, NV, num_kb, num_it, xnb;
     int vg, vr, vlc;   // nu-tile order (ml_nu_tile): ~vg CTAs share the layer, vr nu-tiles each
+    int ng_s;          // nu-tiles in that order; the dynamic tail's nu-tiles [ng_s, ng) keep their own index
     int unit0;         // global index of the layer's first unit (tile * num_it + g)
     int vmode;         // 1: V comes transformed from ml_itf_kernel (small N), the ITF warps idle
     int itf_map[64];   // N | 32: ITF task map of the 64 ITF lanes (as fp32::Params::itf_map)
@@ -111,8 +112,9 @@ __device__ __forceinline__ int layer_of(const Params& p, int u) {
 // 1.21 GB of DRAM reads for 310 MB of x and u).  Instead sequence position s (column s / vr ~ one
 // CTA's share, row s % vr ~ its step) maps to nu-tile row * vg + column, so that at each step the
 // CTAs work on ~vg neighbouring nu-tiles, as a one-tile-per-CTA grid would (step reads 0.57 GB;
-// DESIGN.md 7.11).  A bijection on [0, ng) with ng = (vg - 1) * vr + vlc, 1 <= vlc <= vr.
+// DESIGN.md 7.11).  A bijection on [0, ng_s) with ng_s = (vg - 1) * vr + vlc, 1 <= vlc <= vr.
 __device__ __forceinline__ int ml_nu_tile(const Layer& L, int s) {
+    if (s >= L.ng_s) return s;  // dynamic tail: consecutive grabs take neighbouring nu-tiles
     const int c = s / L.vr, r = s - c * L.vr;
     return r < L.vlc ? r * L.vg + c : L.vlc * L.vg + (r - L.vlc) * (L.vg - 1) + c;
 }

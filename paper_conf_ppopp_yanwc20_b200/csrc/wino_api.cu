@@ -937,13 +937,17 @@ wino_status_t prepare_multi_fp32(const wino_conv_job_t* jobs, float* const* vbuf
         // a tail pays only when each CTA can grab a few tiles of it (P = 8 shard, 0.6 tile per CTA at
         // 6 %: 176 vs 171 us; the P = 1 step with ~6 tiles per CTA: 1128 vs 1139 us, scripts: DESIGN 7.11)
         if (dyn < 3LL * grid) dyn = 0;
+        dyn = dyn / Lz.num_kb * Lz.num_kb;  // whole nu-tiles (all their filter blocks)
     }
     const long long units_static = units - dyn * prm.L[n - 1].num_it;
     const double total = work0[n] - dyn * per_tile[n - 1];
     for (int i = 0; i < n; ++i) {  // nu-tile order (ml_nu_tile): the CTAs' shares of each layer
         Layer& L = prm.L[i];
-        const int ng = (L.NV + BN - 1) / BN;
-        long long g = std::llround((work0[i + 1] - work0[i]) * grid / total);
+        // the last layer's dynamic tail (whole nu-tiles at the end) keeps the identity order
+        const int ng = (L.NV + BN - 1) / BN - (i == n - 1 ? static_cast<int>(dyn / L.num_kb) : 0);
+        L.ng_s = ng;
+        const double wl = work0[i + 1] - work0[i] - (i == n - 1 ? dyn * per_tile[i] : 0.0);
+        long long g = std::llround(wl * grid / total);
         g = g < 1 ? 1 : (g > ng ? ng : g);
         L.vr = static_cast<int>((ng + g - 1) / g);
         L.vg = (ng + L.vr - 1) / L.vr;
